@@ -1,0 +1,302 @@
+"""Seeded synthetic inputs: scheduling regions, the machine model and parameters.
+
+This module is the ONLY code shared by the oracle side (oracle/, tests/) and the
+CUDA side (the C-ABI library).  It generates DATA -- DDGs with latency-labelled
+edges and Def/Use sets of typed virtual registers -- and
+holds the default configuration values; it contains none of the method's
+arithmetic (no RP, no cost, no selection, no pheromone math).
+
+Workload recipe:
+  * instruction mix shaped like a GPU basic block: VALU 55 %, SALU 15 %,
+    VMEM load 12 %, SMEM load 8 %, LDS load 5 %, store 5 %;
+  * operands pick recent values of the needed class with geometric recency
+    (p = 0.3) or, for SGPR operands, a long-lived live-in base (20 %);
+  * memory ordering: every load and store depends on the last store (lat 1);
+  * 4 SGPR + 2 VGPR live-in registers; unused defs are live-out with p = 0.7;
+  * latency profiles "mixed" (VMEM 20-80, SMEM 8-20, LDS 4-8, transcendental
+    VALU 4, else 1) and "unit" (all 1);
+  * region sizes for the rocPRIM-shaped batch follow Table 3.a's bucket counts
+    (728 : 643 : 363 of 1,734 pass-1 regions).
+"""
+from __future__ import annotations
+
+import dataclasses
+from typing import List, Optional, Sequence
+
+import numpy as np
+
+LIVE_IN = 1
+LIVE_OUT = 2
+VGPR = 0
+SGPR = 1
+
+
+@dataclasses.dataclass
+class Region:
+    """One scheduling region (a basic block)."""
+
+    n_insts: int
+    edge_src: np.ndarray  # uint32 [E]
+    edge_dst: np.ndarray  # uint32 [E]
+    edge_lat: np.ndarray  # uint32 [E]
+    reg_class: np.ndarray  # uint8 [R]
+    reg_flags: np.ndarray  # uint8 [R] bit0 LIVE_IN, bit1 LIVE_OUT
+    def_ptr: np.ndarray  # uint32 [n+1]
+    def_reg: np.ndarray  # uint32
+    use_ptr: np.ndarray  # uint32 [n+1]
+    use_reg: np.ndarray  # uint32
+    name: str = ""
+
+    @property
+    def n_edges(self) -> int:
+        return int(self.edge_src.shape[0])
+
+    @property
+    def n_regs(self) -> int:
+        return int(self.reg_class.shape[0])
+
+    @staticmethod
+    def from_lists(n, edges, reg_class, reg_flags, defs, uses, name=""):
+        """edges: [(src, dst, lat)], defs/uses: per-instruction lists of reg ids."""
+        e = np.asarray(edges, dtype=np.uint32).reshape(-1, 3)
+        dptr = np.zeros(n + 1, np.uint32)
+        uptr = np.zeros(n + 1, np.uint32)
+        for j in range(n):
+            dptr[j + 1] = dptr[j] + len(defs[j])
+            uptr[j + 1] = uptr[j] + len(uses[j])
+        dreg = np.asarray([g for d in defs for g in d], np.uint32)
+        ureg = np.asarray([g for u in uses for g in u], np.uint32)
+        return Region(
+            n_insts=n,
+            edge_src=np.ascontiguousarray(e[:, 0]),
+            edge_dst=np.ascontiguousarray(e[:, 1]),
+            edge_lat=np.ascontiguousarray(e[:, 2]),
+            reg_class=np.asarray(reg_class, np.uint8),
+            reg_flags=np.asarray(reg_flags, np.uint8),
+            def_ptr=dptr,
+            def_reg=dreg,
+            use_ptr=uptr,
+            use_reg=ureg,
+            name=name,
+        )
+
+    def defs(self, j: int) -> List[int]:
+        return [int(g) for g in self.def_reg[self.def_ptr[j]:self.def_ptr[j + 1]]]
+
+    def uses(self, j: int) -> List[int]:
+        return [int(g) for g in self.use_reg[self.use_ptr[j]:self.use_ptr[j + 1]]]
+
+    def edges(self):
+        return [(int(s), int(d), int(l)) for s, d, l in zip(self.edge_src, self.edge_dst, self.edge_lat)]
+
+
+# --------------------------------------------------------------------------
+# Machine model: gfx906 occupancy tables (PAPER.md L70-L72 for the VGPR points;
+# the rest of the VGPR table and the SGPR table are AMDGPU facts, not the paper).
+# --------------------------------------------------------------------------
+@dataclasses.dataclass
+class Machine:
+    n_classes: int = 2
+    occ_max: int = 10
+    steps: Sequence[Sequence[int]] = (
+        (24, 28, 32, 36, 40, 48, 64, 84, 128, 256),  # VGPR: occupancy 10..1
+        (80, 88, 100, 102),  # SGPR: occupancy 10..7
+    )
+    perp_limit: Sequence[int] = (24, 80, 0, 0)
+
+
+GFX906 = Machine()
+
+# --------------------------------------------------------------------------
+# Parameters (defaults: DESIGN.md section 3).  Integers only.
+# --------------------------------------------------------------------------
+COST_PRP_SUM, COST_APRP_SUM, COST_OCC, COST_PERP = 0, 1, 2, 3
+STOP_PAPER_CLASSES = 0xFFFFFFFF
+
+
+@dataclasses.dataclass
+class Params:
+    ants: int = 1024
+    iterations: int = 10
+    seed: int = 0
+    passes: int = 3  # 1 RP pass, 2 ILP pass (pass-1 best = heuristic), 3 both
+    cost_mode: int = COST_APRP_SUM
+    q0_t: int = 3865470566  # floor(0.9 * 2^32)
+    group_size: int = 64  # the paper's wavefront (L82, L198)
+    stall_mod: int = 4  # a quarter of the wavefronts may stall (L204)
+    stall_rem: int = 0
+    tau0: int = 4096  # 1.0 in units of 2^-12
+    rho_q16: int = 52429  # decay factor 0.8 (L120) in Q0.16
+    delta: int = 4096
+    tau_min: int = 256
+    tau_max: int = 32768
+    stop_no_improve: int = 0
+    stop_at_lb: int = 0
+
+
+# --------------------------------------------------------------------------
+# Synthetic generator.
+# --------------------------------------------------------------------------
+_KINDS = ("valu", "salu", "vmem", "smem", "lds", "store")
+_MIX = np.array([0.55, 0.15, 0.12, 0.08, 0.05, 0.05])
+
+
+def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "") -> Region:
+    """A synthetic GPU-basic-block-like region of n instructions (2 classes)."""
+    rng = np.random.default_rng(np.uint64(seed))
+    reg_class: List[int] = []
+    reg_flags: List[int] = []
+    pools = {VGPR: [], SGPR: []}
+
+    def new_reg(c, flags=0):
+        reg_class.append(c)
+        reg_flags.append(flags)
+        return len(reg_class) - 1
+
+    for _ in range(4):
+        pools[SGPR].append(new_reg(SGPR, LIVE_IN))
+    for _ in range(2):
+        pools[VGPR].append(new_reg(VGPR, LIVE_IN))
+    base = pools[SGPR][0]
+
+    def pick(c):
+        if c == SGPR and rng.random() < 0.2:
+            return base
+        pool = pools[c]
+        back = int(rng.geometric(0.3)) - 1
+        return pool[max(0, len(pool) - 1 - back)]
+
+    def lat_of(kind):
+        if profile == "unit":
+            return 1
+        if kind == "vmem":
+            return int(rng.integers(20, 81))
+        if kind == "smem":
+            return int(rng.integers(8, 21))
+        if kind == "lds":
+            return int(rng.integers(4, 9))
+        if kind == "valu" and rng.random() < 0.1:
+            return 4
+        return 1
+
+    kinds = rng.choice(len(_KINDS), size=n, p=_MIX)
+    defs: List[List[int]] = []
+    uses: List[List[int]] = []
+    lat = np.zeros(n, np.int64)
+    def_by = {}
+    last_store = -1
+    edge_lat = {}
+
+    def add_edge(s, d, l):
+        key = (s, d)
+        if edge_lat.get(key, -1) < l:
+            edge_lat[key] = l
+
+    for i in range(n):
+        kind = _KINDS[int(kinds[i])]
+        u: List[int] = []
+        d: List[int] = []
+        if kind == "valu":
+            k = int(rng.choice([1, 2, 3], p=[0.3, 0.5, 0.2]))
+            for _ in range(k):
+                u.append(pick(VGPR if rng.random() < 0.8 else SGPR))
+            d.append(new_reg(VGPR))
+        elif kind == "salu":
+            for _ in range(int(rng.integers(1, 3))):
+                u.append(pick(SGPR))
+            d.append(new_reg(SGPR))
+        elif kind == "vmem":
+            u.append(pick(VGPR))
+            u.append(pick(SGPR))
+            for _ in range(int(rng.choice([1, 2, 3, 4], p=[0.4, 0.2, 0.1, 0.3]))):
+                d.append(new_reg(VGPR))
+        elif kind == "smem":
+            u.append(pick(SGPR))
+            for _ in range(int(rng.integers(1, 3))):
+                d.append(new_reg(SGPR))
+        elif kind == "lds":
+            u.append(pick(VGPR))
+            d.append(new_reg(VGPR))
+        else:  # store
+            u.append(pick(VGPR))
+            u.append(pick(VGPR))
+            u.append(pick(SGPR))
+        # de-duplicate uses, keep first occurrence order
+        seen = set()
+        u = [g for g in u if not (g in seen or seen.add(g))]
+        lat[i] = lat_of(kind)
+        for g in u:
+            if g in def_by:
+                add_edge(def_by[g], i, int(lat[def_by[g]]))
+        if kind in ("vmem", "smem", "lds", "store") and last_store >= 0:
+            add_edge(last_store, i, 1)
+        if kind == "store":
+            last_store = i
+        for g in d:
+            def_by[g] = i
+            pools[reg_class[g]].append(g)
+        defs.append(d)
+        uses.append(u)
+
+    used = set(g for ul in uses for g in ul)
+    for g in range(len(reg_class)):
+        if reg_flags[g] & LIVE_IN:
+            continue
+        if g not in used:
+            if rng.random() < 0.7:
+                reg_flags[g] |= LIVE_OUT
+        elif rng.random() < 0.03:
+            reg_flags[g] |= LIVE_OUT
+    edges = sorted((s, d, l) for (s, d), l in edge_lat.items())
+    return Region.from_lists(n, edges, reg_class, reg_flags, defs, uses, name=name or f"synth-n{n}-s{seed}")
+
+
+def region_seed(base: int, region_id: int) -> int:
+    """Per-region generator seed = base XOR region id (SplitMix-style mixing)."""
+    z = (base ^ (region_id * 0x9E3779B97F4A7C15)) & 0xFFFFFFFFFFFFFFFF
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & 0xFFFFFFFFFFFFFFFF
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & 0xFFFFFFFFFFFFFFFF
+    return z ^ (z >> 31)
+
+
+def c3_sizes(count: int, base_seed: int = 3) -> np.ndarray:
+    """Region sizes for the rocPRIM-shaped batch (config 3)."""
+    rng = np.random.default_rng(np.uint64(base_seed))
+    bucket = rng.choice(3, size=count, p=[728 / 1734, 643 / 1734, 363 / 1734])
+    small = rng.integers(20, 50, size=count)
+    mid = rng.integers(50, 100, size=count)
+    big = np.floor(np.exp(rng.uniform(np.log(100), np.log(501), size=count))).astype(np.int64)
+    big = np.clip(big, 100, 500)
+    return np.where(bucket == 0, small, np.where(bucket == 1, mid, big)).astype(np.int64)
+
+
+def gen_batch(count: int, base_seed: int = 3, profile: str = "mixed", first_id: int = 0,
+              sizes: Optional[np.ndarray] = None) -> List[Region]:
+    """Regions first_id .. first_id+count-1 of the config-3 batch."""
+    if sizes is None:
+        sizes = c3_sizes(first_id + count, base_seed)[first_id:]
+    return [gen_region(int(sizes[i]), region_seed(base_seed, first_id + i), profile,
+                       name=f"c3-{first_id + i}") for i in range(count)]
+
+
+# --------------------------------------------------------------------------
+# Hand-built fixtures (data only).  FIG1-R reconstructs PAPER.md Fig. 1 from
+# its text (L143-L155, L184, L200); FIX10-A is config 1.
+# --------------------------------------------------------------------------
+def fig1r() -> Region:
+    A, B, C, D, E, F, G = range(7)
+    edges = [(A, E, 4), (B, E, 4), (C, F, 2), (D, F, 2), (E, G, 1), (F, G, 1)]
+    defs = [[0], [1], [2], [3], [4], [5], [6]]
+    uses = [[], [], [], [], [0, 1], [2, 3], [4, 5]]
+    return Region.from_lists(7, edges, [VGPR] * 7, [0] * 7, defs, uses, name="FIG1-R")
+
+
+def fix10a() -> Region:
+    # registers: Sa0 Vb1 Vc2 Vd3 Sg4 Ve5 Vf6 Vh7 Vi8
+    cls = [SGPR, VGPR, VGPR, VGPR, SGPR, VGPR, VGPR, VGPR, VGPR]
+    defs = [[0], [1], [2], [3], [4], [5], [6], [7], [8], []]
+    uses = [[], [0], [0], [0], [0], [1, 4], [2, 4], [3, 4], [5, 6], [8, 7, 0]]
+    lat = [4, 6, 6, 6, 1, 2, 2, 2, 1, 1]
+    def_by = {g: j for j, d in enumerate(defs) for g in d}
+    edges = sorted({(def_by[g], j, lat[def_by[g]]) for j, u in enumerate(uses) for g in u})
+    return Region.from_lists(10, edges, cls, [0] * 9, defs, uses, name="FIX10-A")
