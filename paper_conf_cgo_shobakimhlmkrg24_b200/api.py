@@ -1,0 +1,208 @@
+"""Python API over the C ABI (argument marshalling only; every step of the
+hot path runs in the CUDA library).  PyTorch provides device memory and streams.
+
+    sched = Scheduler(inputs.GFX906, device=0)
+    sched.load(regions)                    # aco_load_regions (host preprocessing + 1 H2D)
+    sched.run(inputs.Params(ants=1024))    # aco_schedule_batch (all kernels, async)
+    res = sched.results()                  # aco_get_results (sync + D2H)
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import List, Optional, Sequence
+
+import numpy as np
+import torch
+
+from . import _lib
+from .inputs import GFX906, Machine, Params, Region
+
+
+def _stream_handle(stream: Optional[torch.cuda.Stream]) -> C.c_void_p:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return C.c_void_p(s.cuda_stream)
+
+
+def machine_struct(m: Machine) -> _lib.Machine:
+    s = _lib.Machine()
+    s.n_classes = m.n_classes
+    s.occ_max = m.occ_max
+    for c, steps in enumerate(m.steps):
+        s.step_count[c] = len(steps)
+        for i, v in enumerate(steps):
+            s.step_max[c][i] = v
+    for c in range(4):
+        s.perp_limit[c] = m.perp_limit[c] if c < len(m.perp_limit) else 0
+    return s
+
+
+def params_struct(p: Params, flags: int = 0) -> _lib.Params:
+    return _lib.Params(p.ants, p.iterations, p.seed, p.passes, p.cost_mode, p.q0_t, p.group_size,
+                       p.stall_mod, p.stall_rem, p.tau0, p.rho_q16, p.delta, p.tau_min, p.tau_max,
+                       p.stop_no_improve, p.stop_at_lb, flags)
+
+
+class HostBatch:
+    """Region descriptors pointing at contiguous host arrays (kept alive here)."""
+
+    def __init__(self, regions: Sequence[Region], region_ids: Sequence[int]):
+        self.keep = []
+        self.descs = (_lib.RegionDesc * len(regions))()
+        for i, (r, rid) in enumerate(zip(regions, region_ids)):
+            arrs = []
+            for x, dt in ((r.edge_src, np.uint32), (r.edge_dst, np.uint32), (r.edge_lat, np.uint32),
+                          (r.reg_class, np.uint8), (r.reg_flags, np.uint8), (r.def_ptr, np.uint32),
+                          (r.def_reg, np.uint32), (r.use_ptr, np.uint32), (r.use_reg, np.uint32)):
+                a = np.ascontiguousarray(x, dtype=dt)
+                if a.size == 0:
+                    a = np.zeros(1, dt)
+                arrs.append(a)
+            self.keep.append(arrs)
+            self.descs[i] = _lib.RegionDesc(int(rid), int(r.n_insts), int(r.n_edges), int(r.n_regs),
+                                            *[a.ctypes.data for a in arrs])
+        self.sizes = np.array([r.n_insts for r in regions], np.int64)
+        self.offsets = np.concatenate([[0], np.cumsum(self.sizes)]).astype(np.int64)
+
+
+class Scheduler:
+    def __init__(self, machine: Machine = GFX906, device: int = 0):
+        self.lib = _lib.load()
+        self.device = device
+        torch.cuda.set_device(device)
+        self.ctx = C.c_void_p()
+        self._m = machine_struct(machine)
+        _lib.check(self.lib.aco_create(device, C.byref(self._m), C.byref(self.ctx)), "aco_create")
+        self.arena: Optional[torch.Tensor] = None
+        self.ws: Optional[torch.Tensor] = None
+        self.batch: Optional[HostBatch] = None
+        self.count = 0
+        self.params: Optional[Params] = None
+        self.dump = None
+
+    def __del__(self):
+        try:
+            if self.ctx:
+                self.lib.aco_destroy(self.ctx)
+                self.ctx = C.c_void_p()
+        except Exception:
+            pass
+
+    # ---------------------------------------------------------------- load
+    def load(self, regions: Sequence[Region], region_ids: Optional[Sequence[int]] = None,
+             stream: Optional[torch.cuda.Stream] = None, batch: Optional[HostBatch] = None):
+        if region_ids is None:
+            region_ids = list(range(len(regions)))
+        b = batch if batch is not None else HostBatch(regions, region_ids)
+        need = C.c_size_t(0)
+        sh = _stream_handle(stream)
+        _lib.check(self.lib.aco_load_regions(self.ctx, b.descs, len(regions), None, 0, C.byref(need), sh),
+                   "aco_load_regions(size)")
+        if self.arena is None or self.arena.numel() < need.value:
+            self.arena = torch.empty(max(256, need.value), dtype=torch.uint8, device=f"cuda:{self.device}")
+        _lib.check(self.lib.aco_load_regions(self.ctx, b.descs, len(regions), C.c_void_p(self.arena.data_ptr()),
+                                             self.arena.numel(), C.byref(need), sh), "aco_load_regions")
+        self.batch = b
+        self.count = len(regions)
+        return self
+
+    # ---------------------------------------------------------------- run
+    def workspace_bytes(self, p: Params, flags: int = 0) -> int:
+        need = C.c_size_t(0)
+        ps = params_struct(p, flags)
+        _lib.check(self.lib.aco_schedule_batch(self.ctx, C.byref(ps), None, 0, C.byref(need), None),
+                   "aco_schedule_batch(size)")
+        return need.value
+
+    def set_dump(self, p: Params, orders: bool = True):
+        """Allocate dump buffers (test/debug): costs of every ant of every
+        iteration, and optionally every ant's order and pass-2 cycles."""
+        dev = f"cuda:{self.device}"
+        costs = torch.full((2, p.iterations, self.count, p.ants), -1, dtype=torch.int32, device=dev)
+        sum_n = int(self.batch.offsets[-1])
+        od = cy = None
+        if orders:
+            od = torch.zeros((2, p.iterations, p.ants * sum_n + 1), dtype=torch.int16, device=dev)
+            cy = torch.zeros((2, p.iterations, p.ants * sum_n + 1), dtype=torch.int32, device=dev)
+        self.dump = (costs, od, cy)
+        _lib.check(self.lib.aco_set_dump(self.ctx, C.c_void_p(costs.data_ptr()),
+                                         C.c_void_p(od.data_ptr()) if od is not None else None,
+                                         C.c_void_p(cy.data_ptr()) if cy is not None else None),
+                   "aco_set_dump")
+
+    def run(self, p: Params, stream: Optional[torch.cuda.Stream] = None, no_prune: bool = False,
+            dump: bool = False, timing: bool = False):
+        flags = ((_lib.ACO_FLAG_NO_PRUNE if no_prune else 0) | (_lib.ACO_FLAG_DUMP if dump else 0)
+                 | (_lib.ACO_FLAG_TIMING if timing else 0))
+        if dump and self.dump is None:
+            self.set_dump(p)
+        need = self.workspace_bytes(p, flags)
+        if self.ws is None or self.ws.numel() < need:
+            self.ws = torch.empty(max(256, need), dtype=torch.uint8, device=f"cuda:{self.device}")
+        ps = params_struct(p, flags)
+        n = C.c_size_t(0)
+        _lib.check(self.lib.aco_schedule_batch(self.ctx, C.byref(ps), C.c_void_p(self.ws.data_ptr()),
+                                               self.ws.numel(), C.byref(n), _stream_handle(stream)),
+                   "aco_schedule_batch")
+        self.params = p
+        return self
+
+    def timing(self):
+        """(ms[construct, finalize, init], launches[...]) of the last timed run."""
+        ms = (C.c_double * 3)()
+        ln = (C.c_uint64 * 3)()
+        _lib.check(self.lib.aco_get_timing(self.ctx, ms, ln), "aco_get_timing")
+        return [float(x) for x in ms], [int(x) for x in ln]
+
+    def launch_count(self) -> int:
+        v = C.c_uint64(0)
+        _lib.check(self.lib.aco_last_launch_count(self.ctx, C.byref(v)), "aco_last_launch_count")
+        return int(v.value)
+
+    # ---------------------------------------------------------------- results
+    def results_raw(self, first: int = 0, count: Optional[int] = None, orders=None, cycles=None):
+        """Fill caller-provided host arrays (for the e2e path); returns the Result array."""
+        if count is None:
+            count = self.count - first
+        out = (_lib.Result * max(1, count))()
+        _lib.check(self.lib.aco_get_results(self.ctx, first, count, out,
+                                            None if orders is None else orders.ctypes.data,
+                                            None if cycles is None else cycles.ctypes.data),
+                   "aco_get_results")
+        return out
+
+    def results(self, first: int = 0, count: Optional[int] = None) -> List[dict]:
+        if count is None:
+            count = self.count - first
+        off = self.batch.offsets
+        tot = int(off[first + count] - off[first])
+        orders = np.zeros(max(1, tot), np.uint32)
+        cycles = np.zeros(max(1, tot), np.uint32)
+        out = self.results_raw(first, count, orders, cycles)
+        res = []
+        for k in range(count):
+            r = out[k]
+            a, b = int(off[first + k] - off[first]), int(off[first + k + 1] - off[first])
+            res.append(dict(
+                n=r.n_insts, cost_rp=r.cost_rp, length=r.length, prp=list(r.prp),
+                iters1=r.iters_run[0], iters2=r.iters_run[1], best1=r.best_cost[0], best2=r.best_cost[1],
+                init1=r.init_cost[0], init2=r.init_cost[1], lb1=r.lb_cost, lblen=r.lb_len,
+                target=list(r.target), trace_hash=int(r.trace_hash),
+                order=orders[a:b].copy(), cycle=cycles[a:b].copy()))
+        return res
+
+    def dump_arrays(self):
+        """(costs[2][I][count][A] u32, orders[2][I][A*sum_n] u16, cycles ...) as numpy."""
+        torch.cuda.synchronize(self.device)
+        costs, od, cy = self.dump
+        c = costs.cpu().numpy().view(np.uint32)
+        o = od.cpu().numpy().view(np.uint16) if od is not None else None
+        y = cy.cpu().numpy().view(np.uint32) if cy is not None else None
+        return c, o, y
+
+    def dump_ant(self, region: int, pass_: int, it: int, ant: int):
+        c, o, y = self.dump_arrays()
+        A = self.params.ants
+        n = int(self.batch.sizes[region])
+        base = A * int(self.batch.offsets[region]) + ant * n
+        return (int(c[pass_ - 1, it, region, ant]), o[pass_ - 1, it, base:base + n].astype(np.uint32),
+                y[pass_ - 1, it, base:base + n].copy())

@@ -1,0 +1,699 @@
+// aco_host.cpp -- host side of the C ABI (include/aco.h): validation and
+// preprocessing of regions into the device arena (row a1 of SURVEY 8),
+// the workspace plan, the launch sequence of L135-L139, and results.
+//
+// This is product code: it shares nothing with oracle/.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <map>
+#include <new>
+#include <tuple>
+#include <vector>
+
+#include "aco_internal.h"
+
+using namespace aco;
+
+struct aco_ctx_s {
+  int device = 0;
+  MachineDev mach{};
+  bool machine_uploaded = false;
+  // loaded batch
+  uint32_t count = 0;
+  std::vector<RegionDev> regions;  // host copy (offsets valid in the arena)
+  std::vector<uint64_t> inst_off;  // prefix sums of n
+  unsigned char *arena = nullptr;
+  size_t arena_bytes = 0;
+  // last run
+  unsigned char *ws = nullptr;
+  size_t ws_bytes = 0;
+  void *stream = nullptr;
+  RunCfg cfg{};
+  uint64_t o_state = 0, o_rws = 0, o_gb2 = 0, o_gb2c = 0;
+  bool have_run = false;
+  uint64_t launches = 0;
+  uint32_t *dump_cost = nullptr;
+  uint16_t *dump_order = nullptr;
+  uint32_t *dump_cycle = nullptr;
+  std::vector<unsigned char> plan_blob;  // host staging of RegionWs + BlockItems
+  // ACO_FLAG_TIMING: event pairs per phase
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  std::vector<std::pair<size_t, size_t>> ev_pairs[3];
+  uint64_t phase_launches[3] = {0, 0, 0};
+  ~aco_ctx_s() {
+    for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+  }
+  cudaEvent_t next_event() {
+    if (ev_used == ev_pool.size()) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+      ev_pool.push_back(e);
+    }
+    return ev_pool[ev_used++];
+  }
+};
+
+namespace {
+
+struct Prepped {
+  RegionDev rd{};
+  std::vector<uint32_t> succ_ptr, succ, muse, rb0, cnt0, rem0;
+  std::vector<uint32_t> info;  // 4 words per instruction
+  std::vector<uint16_t> eta1, eta2;
+};
+
+// Validation + preprocessing of one region.  Readings R31-R38.
+aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P) {
+  const uint32_t n = d.n_insts, E = d.n_edges, G = d.n_regs;
+  if (n > ACO_MAX_INSTS || G > 16777215u) return ACO_E_TOO_LARGE;
+  if (n > kMaxKernelInsts) return ACO_E_TOO_LARGE;
+  if ((E && (!d.edge_src || !d.edge_dst || !d.edge_lat)) || (G && (!d.reg_class || !d.reg_flags)) ||
+      !d.def_ptr || !d.use_ptr)
+    return ACO_E_ARG;
+  if (d.def_ptr[0] != 0 || d.use_ptr[0] != 0) return ACO_E_ARG;
+  for (uint32_t j = 0; j < n; ++j)
+    if (d.def_ptr[j + 1] < d.def_ptr[j] || d.use_ptr[j + 1] < d.use_ptr[j]) return ACO_E_ARG;
+  if ((d.def_ptr[n] && !d.def_reg) || (d.use_ptr[n] && !d.use_reg)) return ACO_E_ARG;
+  for (uint32_t g = 0; g < G; ++g)
+    if (d.reg_class[g] >= n_classes || (d.reg_flags[g] & ~3u)) return ACO_E_ARG;
+  uint32_t max_lat = 0;
+  for (uint32_t e = 0; e < E; ++e) {
+    if (d.edge_src[e] >= n || d.edge_dst[e] >= n) return ACO_E_ARG;
+    if (d.edge_lat[e] > ACO_MAX_LATENCY) return ACO_E_TOO_LARGE;
+    if (d.edge_src[e] == d.edge_dst[e]) return ACO_E_DDG_CYCLE;
+    max_lat = std::max(max_lat, d.edge_lat[e]);
+  }
+  for (uint32_t k = 0; k < d.def_ptr[n]; ++k)
+    if (d.def_reg[k] >= G) return ACO_E_ARG;
+  for (uint32_t k = 0; k < d.use_ptr[n]; ++k)
+    if (d.use_reg[k] >= G) return ACO_E_ARG;
+  // successor CSR (stable by input order) + duplicate check
+  std::vector<uint32_t> sp(n + 1, 0), outs(E), lats(E), indeg(n, 0);
+  for (uint32_t e = 0; e < E; ++e) sp[d.edge_src[e] + 1]++;
+  for (uint32_t j = 0; j < n; ++j) sp[j + 1] += sp[j];
+  {
+    std::vector<uint32_t> fill(sp.begin(), sp.end() - 1);
+    for (uint32_t e = 0; e < E; ++e) {
+      const uint32_t s = d.edge_src[e];
+      outs[fill[s]] = d.edge_dst[e];
+      lats[fill[s]++] = d.edge_lat[e];
+      indeg[d.edge_dst[e]]++;
+    }
+  }
+  {
+    std::vector<uint32_t> mark(n, 0xFFFFFFFFu);
+    for (uint32_t j = 0; j < n; ++j)
+      for (uint32_t q = sp[j]; q < sp[j + 1]; ++q) {
+        if (mark[outs[q]] == j) return ACO_E_ARG;
+        mark[outs[q]] = j;
+      }
+  }
+  // topological order (Kahn), cycle detection
+  std::vector<uint32_t> topo;
+  topo.reserve(n);
+  {
+    std::vector<uint32_t> deg(indeg);
+    for (uint32_t j = 0; j < n; ++j)
+      if (!deg[j]) topo.push_back(j);
+    for (size_t h = 0; h < topo.size(); ++h) {
+      const uint32_t j = topo[h];
+      for (uint32_t q = sp[j]; q < sp[j + 1]; ++q)
+        if (--deg[outs[q]] == 0) topo.push_back(outs[q]);
+    }
+    if (topo.size() != n) return ACO_E_DDG_CYCLE;
+  }
+  // definitions
+  std::vector<uint32_t> def_by(G, 0xFFFFFFFFu);
+  for (uint32_t j = 0; j < n; ++j)
+    for (uint32_t k = d.def_ptr[j]; k < d.def_ptr[j + 1]; ++k) {
+      const uint32_t g = d.def_reg[k];
+      if (def_by[g] != 0xFFFFFFFFu || (d.reg_flags[g] & kFlagLiveIn)) return ACO_E_DDG_MULTIDEF;
+      def_by[g] = j;
+    }
+  // uses: de-duplicate per instruction (R33), check defining edges (R38)
+  std::vector<uint32_t> uptr(n + 1, 0), ureg;
+  std::vector<uint32_t> nuses(G, 0);
+  {
+    std::vector<uint32_t> seen(G, 0xFFFFFFFFu);
+    std::vector<uint32_t> has_edge(n, 0xFFFFFFFFu);
+    for (uint32_t j = 0; j < n; ++j) {
+      for (uint32_t k = d.use_ptr[j]; k < d.use_ptr[j + 1]; ++k) {
+        const uint32_t g = d.use_reg[k];
+        if (seen[g] == j) continue;
+        seen[g] = j;
+        if (!(d.reg_flags[g] & kFlagLiveIn)) {
+          const uint32_t p = def_by[g];
+          if (p == 0xFFFFFFFFu) return ACO_E_ARG;
+          bool found = false;
+          for (uint32_t q = sp[p]; q < sp[p + 1] && !found; ++q) found = outs[q] == j;
+          if (!found) return ACO_E_DDG_USE_NO_EDGE;
+        }
+        ureg.push_back(g);
+        nuses[g]++;
+      }
+      uptr[j + 1] = (uint32_t)ureg.size();
+    }
+  }
+  // device limits
+  for (uint32_t j = 0; j < n; ++j)
+    if (indeg[j] > ACO_MAX_INDEG || uptr[j + 1] - uptr[j] > 255u) return ACO_E_TOO_LARGE;
+  for (uint32_t g = 0; g < G; ++g)
+    if (nuses[g] > ACO_MAX_USES) return ACO_E_TOO_LARGE;
+  if ((uint64_t)n * ((uint64_t)max_lat + 1) >= (1ull << 24)) return ACO_E_TOO_LARGE;
+  // register categories: counters for multi-use, non-live-out registers
+  std::vector<uint32_t> ctr(G, 0xFFFFFFFFu);
+  uint32_t nmu = 0;
+  for (uint32_t g = 0; g < G; ++g)
+    if (nuses[g] >= 2 && !(d.reg_flags[g] & kFlagLiveOut)) ctr[g] = nmu++;
+  if (nmu > 65535u) return ACO_E_TOO_LARGE;
+  // critical path heights (reverse topological relaxation)
+  std::vector<uint32_t> cp(n, 0);
+  for (size_t h = n; h-- > 0;) {
+    const uint32_t j = topo[h];
+    uint32_t v = 0;
+    for (uint32_t q = sp[j]; q < sp[j + 1]; ++q) v = std::max(v, lats[q] + cp[outs[q]]);
+    cp[j] = v;
+  }
+  uint32_t cp_max = 0;
+  for (uint32_t j = 0; j < n; ++j) cp_max = std::max(cp_max, cp[j]);
+  // per-instruction info
+  P.info.assign((size_t)n * 4, 0);
+  uint32_t L = 0;
+  uint32_t lbvec[4] = {0, 0, 0, 0}, livein[4] = {0, 0, 0, 0}, liveout[4] = {0, 0, 0, 0};
+  for (uint32_t g = 0; g < G; ++g) {
+    if (d.reg_flags[g] & kFlagLiveIn) livein[d.reg_class[g]]++;
+    if (d.reg_flags[g] & kFlagLiveOut) liveout[d.reg_class[g]]++;
+  }
+  for (uint32_t c = 0; c < 4; ++c) lbvec[c] = std::max(livein[c], n ? liveout[c] : 0u);
+  for (uint32_t j = 0; j < n; ++j) {
+    uint32_t defs[4] = {0, 0, 0, 0}, dead[4] = {0, 0, 0, 0}, sk[4] = {0, 0, 0, 0}, usec[4] = {0, 0, 0, 0};
+    for (uint32_t k = d.def_ptr[j]; k < d.def_ptr[j + 1]; ++k) {
+      const uint32_t g = d.def_reg[k], c = d.reg_class[g];
+      defs[c]++;
+      if (nuses[g] == 0 && !(d.reg_flags[g] & kFlagLiveOut)) dead[c]++;
+    }
+    const uint32_t mstart = (uint32_t)P.muse.size();
+    uint32_t nonlo = 0;
+    for (uint32_t k = uptr[j]; k < uptr[j + 1]; ++k) {
+      const uint32_t g = ureg[k], c = d.reg_class[g];
+      usec[c]++;
+      if (d.reg_flags[g] & kFlagLiveOut) continue;
+      nonlo++;
+      if (nuses[g] == 1) sk[c]++;
+      else P.muse.push_back(ctr[g] | (c << 16));
+    }
+    L = std::max(L, nonlo);
+    const uint32_t mcnt = (uint32_t)P.muse.size() - mstart;
+    for (uint32_t c = 0; c < 4; ++c) {
+      if (defs[c] > 255u || dead[c] > 255u || sk[c] > 255u) return ACO_E_TOO_LARGE;
+      P.info[(size_t)j * 4 + 0] |= defs[c] << (8 * c);
+      P.info[(size_t)j * 4 + 1] |= dead[c] << (8 * c);
+      P.info[(size_t)j * 4 + 2] |= sk[c] << (8 * c);
+      lbvec[c] = std::max(lbvec[c], std::max(defs[c], usec[c]));
+    }
+    if (mstart >= (1u << 24)) return ACO_E_TOO_LARGE;
+    P.info[(size_t)j * 4 + 3] = (mstart << 8) | mcnt;
+  }
+  // heuristic tables (R4)
+  const uint64_t km1 = (uint64_t)L * (cp_max + 1ull) + cp_max;
+  const uint64_t d1 = km1 ? km1 : 1;
+  P.eta1.resize((size_t)n * (L + 1));
+  for (uint32_t j = 0; j < n; ++j)
+    for (uint32_t l = 0; l <= L; ++l) {
+      const uint64_t key = (uint64_t)l * (cp_max + 1ull) + cp[j];
+      P.eta1[(size_t)j * (L + 1) + l] = (uint16_t)(1 + key * 65534ull / d1);
+    }
+  P.eta2.resize(n);
+  for (uint32_t j = 0; j < n; ++j)
+    P.eta2[j] = (uint16_t)(1 + (uint64_t)cp[j] * 65534ull / (cp_max ? cp_max : 1));
+  // successor list packed v | lat << 16
+  P.succ_ptr = sp;
+  P.succ.resize(E);
+  for (uint32_t q = 0; q < E; ++q) P.succ[q] = outs[q] | (lats[q] << 16);
+  // initial per-ant state
+  const uint32_t nwr = (n + 31) / 32;
+  P.rb0.assign(nwr, 0);
+  for (uint32_t j = 0; j < n; ++j)
+    if (!indeg[j]) P.rb0[j >> 5] |= 1u << (j & 31);
+  P.cnt0.assign((n + 3) / 4, 0);
+  for (uint32_t j = 0; j < n; ++j) P.cnt0[j >> 2] |= indeg[j] << (8 * (j & 3));
+  P.rem0.assign((nmu + 1) / 2, 0);
+  for (uint32_t g = 0; g < G; ++g)
+    if (ctr[g] != 0xFFFFFFFFu) P.rem0[ctr[g] >> 1] |= nuses[g] << (16 * (ctr[g] & 1));
+  RegionDev &R = P.rd;
+  std::memset(&R, 0, sizeof(R));
+  R.n = n;
+  R.nwr = nwr;
+  R.nmu = nmu;
+  R.L = L;
+  R.region_id = d.region_id;
+  R.cp_max = cp_max;
+  R.lb_len = std::max(n, n ? cp_max + 1 : 0u);
+  R.ub_ready = 0;
+  for (uint32_t c = 0; c < 4; ++c) {
+    R.livein[c] = livein[c];
+    R.lbvec[c] = lbvec[c];
+  }
+  return ACO_OK;
+}
+
+template <typename T>
+uint64_t put(std::vector<unsigned char> &blob, const std::vector<T> &v) {
+  uint64_t off = align16(blob.size());
+  blob.resize(off + v.size() * sizeof(T) + 16, 0);
+  if (!v.empty()) std::memcpy(blob.data() + off, v.data(), v.size() * sizeof(T));
+  return off;
+}
+
+aco_status cuda_status(cudaError_t e) { return e == cudaSuccess ? ACO_OK : ACO_E_CUDA; }
+
+}  // namespace
+
+extern "C" {
+
+const char *aco_status_string(aco_status st) {
+  switch (st) {
+    case ACO_OK: return "ok";
+    case ACO_E_ARG: return "invalid argument";
+    case ACO_E_DDG_CYCLE: return "DDG has a cycle";
+    case ACO_E_DDG_MULTIDEF: return "register defined more than once (or live-in defined)";
+    case ACO_E_DDG_USE_NO_EDGE: return "use without a def->use edge";
+    case ACO_E_TOO_LARGE: return "over a compiled limit";
+    case ACO_E_WORKSPACE: return "buffer missing or too small";
+    case ACO_E_CUDA: return "CUDA error";
+    case ACO_E_STATE: return "call out of order";
+    default: return "unknown status";
+  }
+}
+
+aco_status aco_create(int device, const aco_machine *m, aco_ctx *out) {
+  if (!m || !out || m->n_classes < 1 || m->n_classes > 4) return ACO_E_ARG;
+  for (uint32_t c = 0; c < m->n_classes; ++c)
+    if (m->step_count[c] < 1 || m->step_count[c] > 16 || m->occ_max < m->step_count[c]) return ACO_E_ARG;
+  aco_ctx ctx = new (std::nothrow) aco_ctx_s();
+  if (!ctx) return ACO_E_ARG;
+  ctx->device = device;
+  ctx->mach.n_classes = m->n_classes;
+  ctx->mach.occ_max = m->occ_max;
+  for (int c = 0; c < 4; ++c) {
+    ctx->mach.step_count[c] = m->step_count[c];
+    for (int i = 0; i < 16; ++i) ctx->mach.step_max[c][i] = m->step_max[c][i];
+    ctx->mach.perp_limit[c] = m->perp_limit[c];
+  }
+  *out = ctx;  // no CUDA call here: the device is touched on first use
+  return ACO_OK;
+}
+
+void aco_destroy(aco_ctx ctx) { delete ctx; }
+
+aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_t count, void *d_arena,
+                            size_t arena_bytes, size_t *arena_needed, void *cuda_stream) {
+  if (!ctx || (count && !regions)) return ACO_E_ARG;
+  {  // unique region ids
+    std::vector<uint32_t> ids(count);
+    for (uint32_t i = 0; i < count; ++i) ids[i] = regions[i].region_id;
+    std::sort(ids.begin(), ids.end());
+    for (uint32_t i = 1; i < count; ++i)
+      if (ids[i] == ids[i - 1]) return ACO_E_ARG;
+  }
+  std::vector<Prepped> P(count);
+  for (uint32_t i = 0; i < count; ++i) {
+    aco_status st = prep_region(regions[i], ctx->mach.n_classes, P[i]);
+    if (st != ACO_OK) return st;
+  }
+  std::vector<unsigned char> blob(align16(sizeof(RegionDev) * (size_t)count + 16), 0);
+  for (uint32_t i = 0; i < count; ++i) {
+    RegionDev &R = P[i].rd;
+    R.o_succ_ptr = put(blob, P[i].succ_ptr);
+    R.o_succ = put(blob, P[i].succ);
+    R.o_info = put(blob, P[i].info);
+    R.o_muse = put(blob, P[i].muse);
+    R.o_rb0 = put(blob, P[i].rb0);
+    R.o_cnt0 = put(blob, P[i].cnt0);
+    R.o_rem0 = put(blob, P[i].rem0);
+    R.o_eta1 = put(blob, P[i].eta1);
+    R.o_eta2 = put(blob, P[i].eta2);
+    std::memcpy(blob.data() + sizeof(RegionDev) * (size_t)i, &R, sizeof(RegionDev));
+  }
+  const size_t need = align256(blob.size());
+  if (arena_needed) *arena_needed = need;
+  if (!d_arena) return ACO_OK;
+  if (arena_bytes < need) return ACO_E_WORKSPACE;
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
+  cudaError_t e = cudaMemcpyAsync(d_arena, blob.data(), blob.size(), cudaMemcpyHostToDevice,
+                                  (cudaStream_t)cuda_stream);
+  if (e != cudaSuccess) return ACO_E_CUDA;
+  // pageable source: make sure the copy has consumed `blob` before it is freed
+  e = cudaStreamSynchronize((cudaStream_t)cuda_stream);
+  if (e != cudaSuccess) return ACO_E_CUDA;
+  ctx->count = count;
+  ctx->regions.resize(count);
+  ctx->inst_off.assign(count + 1, 0);
+  for (uint32_t i = 0; i < count; ++i) {
+    ctx->regions[i] = P[i].rd;
+    ctx->inst_off[i + 1] = ctx->inst_off[i] + P[i].rd.n;
+  }
+  ctx->arena = (unsigned char *)d_arena;
+  ctx->arena_bytes = arena_bytes;
+  ctx->have_run = false;
+  return ACO_OK;
+}
+
+aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint32_t *d_cycles) {
+  if (!ctx) return ACO_E_ARG;
+  ctx->dump_cost = d_costs;
+  ctx->dump_order = d_orders;
+  ctx->dump_cycle = d_cycles;
+  return ACO_OK;
+}
+
+namespace {
+
+// Ants per block and the smem word cap for a per-ant state of W words.
+void pick_class(uint32_t W, uint32_t &ants_pb, uint32_t &wcap) {
+  static const uint32_t caps[] = {16, 32, 48, 64, 96, 128, 192, 256, 384, 512, 768, 1024, 1536, 1775};
+  wcap = 1775;
+  for (uint32_t c : caps)
+    if (W <= c) {
+      wcap = c;
+      break;
+    }
+  ants_pb = wcap <= 96 ? 128 : (wcap <= 384 ? 64 : 32);
+}
+
+}  // namespace
+
+aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspace, size_t ws_bytes,
+                              size_t *ws_needed, void *cuda_stream) {
+  if (!ctx || !p) return ACO_E_ARG;
+  if (!ctx->arena && ctx->count) return ACO_E_STATE;
+  if (p->pass < 1 || p->pass > 3 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
+      p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->tau0 > 65535u ||
+      p->tau0 < p->tau_min || p->tau0 > p->tau_max || p->q0_t > (1ull << 32) || p->rho_q16 > 65536u ||
+      p->iterations > 0x7FFFFFFFu)
+    return ACO_E_ARG;
+  if ((p->flags & ACO_FLAG_DUMP) && !ctx->dump_cost) return ACO_E_ARG;
+  const uint32_t count = ctx->count, A = p->ants;
+  // ---- per-pass construct classes
+  struct Cls {
+    uint32_t ants_pb, wcap;
+    bool mask;
+    std::vector<std::pair<uint64_t, uint32_t>> regs;  // (-work, region)
+  };
+  std::map<std::tuple<uint32_t, uint32_t, uint32_t, bool>, Cls> classes;  // (pass, ants_pb, wcap, mask)
+  uint32_t fin_smem[3] = {0, 0, 0}, max_n = 0, init_smem = 0, p2_smem = 0;
+  for (uint32_t r = 0; r < count; ++r) {
+    const RegionDev &R = ctx->regions[r];
+    max_n = std::max(max_n, R.n);
+    for (uint32_t pass = 1; pass <= 2; ++pass) {
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nmu);
+      if (W > 1775) return ACO_E_TOO_LARGE;
+      const uint32_t fs = 4 * W + 4 * R.n + 2 * ((R.n + 2) & ~1u) + 2 * (R.n + 1) + 64;
+      fin_smem[pass] = std::max(fin_smem[pass], fs);
+      if (pass == 1) init_smem = std::max(init_smem, 4 * W + 16);
+      if (!(p->pass & pass)) continue;
+      uint32_t apb, wcap;
+      pick_class(W, apb, wcap);
+      const bool mask = R.n <= 1024;
+      Cls &c = classes[std::make_tuple(pass, apb, wcap, mask)];
+      c.ants_pb = apb;
+      c.wcap = wcap;
+      c.mask = mask;
+      c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
+    }
+    p2_smem = std::max(p2_smem, 4 * R.n + 16);
+  }
+  if (std::max(fin_smem[1], fin_smem[2]) > 227 * 1024) return ACO_E_TOO_LARGE;
+  // ---- workspace layout
+  uint64_t off = 0;
+  const uint64_t o_state = off;
+  off = align256(off + sizeof(RegionState) * (uint64_t)count);
+  const uint64_t o_rws = off;
+  off = align16(off + sizeof(RegionWs) * (uint64_t)count);
+  const uint64_t o_items = off;
+  uint64_t n_items = 0;
+  std::vector<std::pair<std::tuple<uint32_t, uint32_t, uint32_t, bool>, uint64_t>> class_item_off;
+  for (auto &kv : classes) {
+    class_item_off.push_back({kv.first, n_items});
+    n_items += (uint64_t)kv.second.regs.size() * ((A + kv.second.ants_pb - 1) / kv.second.ants_pb);
+  }
+  off = align256(off + sizeof(BlockItem) * n_items);
+  const uint64_t sum_n = ctx->inst_off.empty() ? 0 : ctx->inst_off[count];
+  const uint64_t o_gb1 = off;
+  off = align256(off + 2 * sum_n + 16);
+  const uint64_t o_gb2 = off;
+  off = align256(off + 2 * sum_n + 16);
+  const uint64_t o_gb2c = off;
+  off = align256(off + 4 * sum_n + 16);
+  const uint64_t o_cost = off;
+  off = align256(off + 4ull * A * count);
+  std::vector<RegionWs> rws(count);
+  for (uint32_t r = 0; r < count; ++r) {
+    const uint32_t n = ctx->regions[r].n;
+    RegionWs &w = rws[r];
+    std::memset(&w, 0, sizeof(w));
+    w.tau_len = (uint32_t)(((uint64_t)(n + 1) * n + 7) & ~7ull);
+    w.o_tau = off;
+    off = align16(off + 2ull * w.tau_len);
+    w.o_cost = o_cost + 4ull * A * r;
+    w.o_gb1 = o_gb1 + 2 * ctx->inst_off[r];
+    w.o_gb2 = o_gb2 + 2 * ctx->inst_off[r];
+    w.o_gb2c = o_gb2c + 4 * ctx->inst_off[r];
+    w.o_dump = (uint64_t)A * ctx->inst_off[r];
+  }
+  const size_t need = align256(off);
+  if (ws_needed) *ws_needed = need;
+  if (!d_workspace) return ACO_OK;
+  if (ws_bytes < need) return ACO_E_WORKSPACE;
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
+  if (!ctx->machine_uploaded) {
+    if (set_machine(ctx->mach) != 0) return ACO_E_CUDA;
+    ctx->machine_uploaded = true;
+  }
+  unsigned char *ws = (unsigned char *)d_workspace;
+  // ---- host plan: RegionWs table + block items, one H2D
+  std::vector<unsigned char> &blob = ctx->plan_blob;
+  blob.assign(o_items - o_rws + sizeof(BlockItem) * n_items, 0);
+  std::memcpy(blob.data(), rws.data(), sizeof(RegionWs) * count);
+  std::vector<ClassLaunch> launches[3];
+  {
+    size_t ci = 0;
+    for (auto &kv : classes) {
+      Cls &c = kv.second;
+      std::sort(c.regs.begin(), c.regs.end());
+      const uint64_t base = class_item_off[ci++].second;
+      BlockItem *items = (BlockItem *)(blob.data() + (o_items - o_rws)) + base;
+      uint64_t k = 0;
+      for (auto &pr : c.regs)
+        for (uint32_t a0 = 0; a0 < A; a0 += c.ants_pb) items[k++] = BlockItem{pr.second, a0};
+      ClassLaunch cl;
+      cl.items = (const BlockItem *)(ws + o_items) + base;
+      cl.n_blocks = (uint32_t)k;
+      cl.ants_pb = c.ants_pb;
+      cl.smem_bytes = c.ants_pb * c.wcap * 4;
+      cl.max_n = c.mask ? 1024 : 65535;
+      launches[std::get<0>(kv.first)].push_back(cl);
+    }
+  }
+  cudaStream_t s = (cudaStream_t)cuda_stream;
+  if (cudaMemcpyAsync(ws + o_rws, blob.data(), blob.size(), cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return ACO_E_CUDA;
+  LaunchCtx L;
+  L.arena = ctx->arena;
+  L.ws = ws;
+  L.regions = (const RegionDev *)ctx->arena;
+  L.state = (RegionState *)(ws + o_state);
+  L.rws = (const RegionWs *)(ws + o_rws);
+  L.dump_cost = ctx->dump_cost;
+  L.dump_order = ctx->dump_order;
+  L.dump_cycle = ctx->dump_cycle;
+  RunCfg &cfg = L.cfg;
+  std::memset(&cfg, 0, sizeof(cfg));
+  cfg.seed = p->seed;
+  cfg.q0_t = p->q0_t;
+  cfg.ants = A;
+  cfg.iterations = p->iterations;
+  cfg.pass_mask = p->pass;
+  cfg.cost_mode = p->cost_mode;
+  cfg.group_size = p->group_size;
+  cfg.stall_mod = p->stall_mod;
+  cfg.stall_rem = p->stall_rem;
+  cfg.flags = p->flags;
+  cfg.tau0 = p->tau0;
+  cfg.rho_q16 = p->rho_q16;
+  cfg.delta = p->delta;
+  cfg.tau_min = p->tau_min;
+  cfg.tau_max = p->tau_max;
+  cfg.stop_no_improve = p->stop_no_improve;
+  cfg.stop_at_lb = p->stop_at_lb;
+  cfg.n_classes = ctx->mach.n_classes;
+  cfg.count = count;
+  cfg.dump_slice = (uint64_t)A * sum_n;
+  L.stream = cuda_stream;
+  L.launches = 0;
+  const bool timing = (p->flags & ACO_FLAG_TIMING) != 0;
+  ctx->ev_used = 0;
+  for (int ph = 0; ph < 3; ++ph) {
+    ctx->ev_pairs[ph].clear();
+    ctx->phase_launches[ph] = 0;
+  }
+  // phase bracket: record an event pair around a group of launches
+  auto begin = [&](int ph) -> size_t {
+    if (!timing) return 0;
+    const size_t i = ctx->ev_used;
+    cudaEvent_t e = ctx->next_event();
+    if (e) cudaEventRecord(e, s);
+    (void)ph;
+    return i;
+  };
+  auto end = [&](int ph, size_t i0, uint64_t l0) {
+    ctx->phase_launches[ph] += L.launches - l0;
+    if (!timing) return;
+    const size_t i1 = ctx->ev_used;
+    cudaEvent_t e = ctx->next_event();
+    if (e) cudaEventRecord(e, s);
+    ctx->ev_pairs[ph].push_back({i0, i1});
+  };
+  int err = 0;
+  {
+    const size_t e0 = begin(2);
+    const uint64_t l0 = L.launches;
+    err |= launch_init(L, init_smem, max_n);
+    end(2, e0, l0);
+  }
+  for (uint32_t pass = 1; pass <= 2 && !err; ++pass) {
+    if (pass == 2) {
+      const size_t e0 = begin(2);
+      const uint64_t l0 = L.launches;
+      err |= launch_pass2_init(L, p2_smem, max_n);
+      end(2, e0, l0);
+    }
+    if (!(p->pass & pass)) continue;
+    for (uint32_t it = 0; it < p->iterations && !err; ++it) {
+      size_t e0 = begin(0);
+      uint64_t l0 = L.launches;
+      for (const ClassLaunch &cl : launches[pass]) err |= launch_construct(L, pass, it, cl);
+      end(0, e0, l0);
+      e0 = begin(1);
+      l0 = L.launches;
+      err |= launch_finalize(L, pass, it, fin_smem[pass], max_n);
+      end(1, e0, l0);
+    }
+  }
+  ctx->launches = L.launches;
+  if (err) return ACO_E_CUDA;
+  ctx->ws = ws;
+  ctx->ws_bytes = ws_bytes;
+  ctx->stream = cuda_stream;
+  ctx->cfg = cfg;
+  ctx->o_state = o_state;
+  ctx->o_rws = o_rws;
+  ctx->o_gb2 = o_gb2;
+  ctx->o_gb2c = o_gb2c;
+  ctx->have_run = true;
+  return ACO_OK;
+}
+
+aco_status aco_get_timing(aco_ctx ctx, double ms[3], uint64_t launches[3]) {
+  if (!ctx || !ms || !launches) return ACO_E_ARG;
+  if (!ctx->have_run) return ACO_E_STATE;
+  if (cudaStreamSynchronize((cudaStream_t)ctx->stream) != cudaSuccess) return ACO_E_CUDA;
+  for (int ph = 0; ph < 3; ++ph) {
+    double t = 0;
+    for (auto &pr : ctx->ev_pairs[ph]) {
+      float f = 0;
+      if (cudaEventElapsedTime(&f, ctx->ev_pool[pr.first], ctx->ev_pool[pr.second]) != cudaSuccess)
+        return ACO_E_CUDA;
+      t += f;
+    }
+    ms[ph] = t;
+    launches[ph] = ctx->phase_launches[ph];
+  }
+  return ACO_OK;
+}
+
+aco_status aco_last_launch_count(aco_ctx ctx, uint64_t *launches) {
+  if (!ctx || !launches) return ACO_E_ARG;
+  *launches = ctx->launches;
+  return ACO_OK;
+}
+
+aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_result *out, uint32_t *orders,
+                           uint32_t *cycles) {
+  if (!ctx || (count && !out)) return ACO_E_ARG;
+  if (!ctx->have_run) return ACO_E_STATE;
+  if ((uint64_t)first + count > ctx->count) return ACO_E_ARG;
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
+  cudaStream_t s = (cudaStream_t)ctx->stream;
+  if (cudaStreamSynchronize(s) != cudaSuccess) return ACO_E_CUDA;
+  if (!count) return ACO_OK;
+  std::vector<RegionState> st(count);
+  const uint64_t i0 = ctx->inst_off[first], i1 = ctx->inst_off[first + count];
+  std::vector<uint16_t> o16(i1 - i0 + 1);
+  std::vector<uint32_t> c32(i1 - i0 + 1);
+  aco_status e = cuda_status(cudaMemcpy(st.data(), ctx->ws + ctx->o_state + sizeof(RegionState) * first,
+                                        sizeof(RegionState) * count, cudaMemcpyDeviceToHost));
+  if (e == ACO_OK && i1 > i0) {
+    e = cuda_status(cudaMemcpy(o16.data(), ctx->ws + ctx->o_gb2 + 2 * i0, 2 * (i1 - i0), cudaMemcpyDeviceToHost));
+    if (e == ACO_OK)
+      e = cuda_status(cudaMemcpy(c32.data(), ctx->ws + ctx->o_gb2c + 4 * i0, 4 * (i1 - i0), cudaMemcpyDeviceToHost));
+  }
+  if (e != ACO_OK) return e;
+  // host-side cost of the final PRP (R16) -- the machine tables
+  auto aprp = [&](uint32_t c, uint32_t x) {
+    for (uint32_t i = 0; i < ctx->mach.step_count[c]; ++i)
+      if (x <= ctx->mach.step_max[c][i]) return ctx->mach.step_max[c][i];
+    return x;
+  };
+  auto occ = [&](uint32_t c, uint32_t x) {
+    for (uint32_t i = 0; i < ctx->mach.step_count[c]; ++i)
+      if (x <= ctx->mach.step_max[c][i]) return ctx->mach.occ_max - i;
+    return 0u;
+  };
+  for (uint32_t k = 0; k < count; ++k) {
+    const RegionState &S = st[k];
+    const RegionDev &R = ctx->regions[first + k];
+    aco_result &o = out[k];
+    std::memset(&o, 0, sizeof(o));
+    o.n_insts = R.n;
+    o.length = S.best[1];
+    uint32_t cost = 0;
+    const uint32_t nc = ctx->mach.n_classes, mode = ctx->cfg.cost_mode;
+    if (mode == ACO_COST_PRP_SUM) {
+      for (uint32_t c = 0; c < nc; ++c) cost += S.prp2[c];
+    } else if (mode == ACO_COST_APRP_SUM) {
+      for (uint32_t c = 0; c < nc; ++c) cost += aprp(c, S.prp2[c]);
+    } else if (mode == ACO_COST_OCC) {
+      uint32_t m = ctx->mach.occ_max;
+      for (uint32_t c = 0; c < nc; ++c) m = std::min(m, occ(c, S.prp2[c]));
+      cost = ctx->mach.occ_max - m;
+    } else {
+      for (uint32_t c = 0; c < nc; ++c)
+        cost += S.prp2[c] > ctx->mach.perp_limit[c] ? S.prp2[c] - ctx->mach.perp_limit[c] : 0;
+    }
+    o.cost_rp = cost;
+    for (int c = 0; c < 4; ++c) {
+      o.prp[c] = S.prp2[c];
+      o.target[c] = S.target[c];
+    }
+    o.iters_run[0] = S.iters[0];
+    o.iters_run[1] = S.iters[1];
+    o.best_cost[0] = S.best[0];
+    o.best_cost[1] = S.best[1];
+    o.init_cost[0] = S.init[0];
+    o.init_cost[1] = S.init[1];
+    o.lb_cost = S.lb_cost;
+    o.lb_len = R.lb_len;
+    o.trace_hash = S.hash;
+  }
+  for (uint64_t q = 0; q < i1 - i0; ++q) {
+    if (orders) orders[q] = o16[q];
+    if (cycles) cycles[q] = c32[q];
+  }
+  return ACO_OK;
+}
+
+}  // extern "C"

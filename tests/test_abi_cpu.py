@@ -1,0 +1,95 @@
+"""Host-side checks of the C-ABI library that need no GPU: it loads, exports
+every symbol declared in include/aco.h, and its validation (aco_create and
+the sizing call of aco_load_regions make no CUDA call) agrees with the
+oracle's error codes."""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+from oracle import pyoracle as O
+from paper_conf_cgo_shobakimhlmkrg24_b200 import _lib, build
+from paper_conf_cgo_shobakimhlmkrg24_b200 import inputs as I
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    build.build()
+    return _lib.load()
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "aco.h")).read()
+    return sorted(set(re.findall(r"\b(aco_[a-z_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol(lib):
+    syms = declared_symbols()
+    assert "aco_load_regions" in syms and "aco_schedule_batch" in syms
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert set(_lib.EXPORTS) == set(syms)
+
+
+def test_status_strings(lib):
+    for st in range(0, -9, -1):
+        assert lib.aco_status_string(st)
+
+
+def _ctx(lib):
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import machine_struct
+    m = machine_struct(I.GFX906)
+    ctx = C.c_void_p()
+    assert lib.aco_create(0, C.byref(m), C.byref(ctx)) == 0
+    return ctx, m
+
+
+def _size_status(lib, regions, ids=None):
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch
+    ctx, m = _ctx(lib)
+    b = HostBatch(regions, ids or list(range(len(regions))))
+    need = C.c_size_t(0)
+    st = lib.aco_load_regions(ctx, b.descs, len(regions), None, 0, C.byref(need), None)
+    lib.aco_destroy(ctx)
+    return st, need.value
+
+
+def _tiny(edges, defs, uses, flags=None, n=3):
+    R = 1 + max([g for d in defs for g in d] + [g for u in uses for g in u] + [-1])
+    return I.Region.from_lists(n, edges, [0] * R, flags or [0] * R, defs, uses)
+
+
+CASES = [
+    _tiny([(0, 1, 1), (1, 2, 1)], [[0], [1], []], [[], [0], [1]]),
+    _tiny([(0, 1, 1), (1, 0, 1)], [[], [], []], [[], [], []]),
+    _tiny([(0, 0, 1)], [[], [], []], [[], [], []]),
+    _tiny([(0, 1, 1)], [[0], [0], []], [[], [], []]),
+    _tiny([(0, 1, 1)], [[0], [], []], [[], [], [0]]),
+    _tiny([(0, 1, 1), (0, 1, 2)], [[], [], []], [[], [], []]),
+    _tiny([], [[], [], []], [[], [], [0]]),
+    _tiny([], [[0], [], []], [[], [], []], flags=[1]),
+]
+
+
+@pytest.mark.parametrize("k", range(len(CASES)))
+def test_validation_matches_oracle(lib, k):
+    st, _ = _size_status(lib, [CASES[k]])
+    assert st == O.validate(CASES[k])
+
+
+def test_sizing_call_on_synthetic_batch(lib):
+    regs = I.gen_batch(40, base_seed=9)
+    st, need = _size_status(lib, regs)
+    assert st == 0 and need > 0
+    st, _ = _size_status(lib, regs[:2], [4, 4])
+    assert st == -1  # duplicate region ids
+
+
+def test_too_large_region(lib):
+    n = 9000
+    big = I.Region.from_lists(n, [], [], [], [[] for _ in range(n)], [[] for _ in range(n)])
+    st, _ = _size_status(lib, [big])
+    assert st == -5

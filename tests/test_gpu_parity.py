@@ -1,0 +1,196 @@
+"""Parity of the CUDA path (through the C ABI) with the CPU oracle.
+
+Integer / index work, so the bar is BIT-EXACT: every ant's cost, order and
+cycles in dump mode; the final schedule, PRP, length, iteration counts and
+the per-iteration winner-trace hash in production mode.
+"""
+import numpy as np
+import pytest
+
+from oracle import pyoracle as O
+from paper_conf_cgo_shobakimhlmkrg24_b200 import inputs as I
+from tests import checker
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def _sched(machine=I.GFX906):
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import Scheduler
+    return Scheduler(machine, device=0)
+
+
+def compare_results(gpu, ora, ctx=""):
+    assert gpu["length"] == ora["length"], ctx
+    assert gpu["prp"] == ora["prp"], ctx
+    assert gpu["cost_rp"] == ora["cost_rp"], ctx
+    assert gpu["iters1"] == ora["iters1"] and gpu["iters2"] == ora["iters2"], ctx
+    assert gpu["best1"] == ora["best1"] and gpu["best2"] == ora["best2"], ctx
+    assert gpu["init1"] == ora["init1"] and gpu["init2"] == ora["init2"], ctx
+    assert gpu["lb1"] == ora["lb1"] and gpu["lblen"] == ora["lblen"], ctx
+    assert gpu["target"][:2] == [ora["target0"], ora["target1"]], ctx
+    assert gpu["trace_hash"] == ora["trace_hash"], ctx
+    assert list(gpu["order"]) == list(ora["order"]), ctx
+    assert list(gpu["cycle"]) == list(ora["cycle"]), ctx
+
+
+def dump_parity(s, regions, ids, p, machine=I.GFX906):
+    c, o, y = s.dump_arrays()
+    A, n_it = p.ants, p.iterations
+    for k, (reg, rid) in enumerate(zip(regions, ids)):
+        ora = O.schedule(reg, rid, machine, p, dump=True, dump_orders=True)
+        n = reg.n_insts
+        base0 = A * int(s.batch.offsets[k])
+        for ps in (0, 1):
+            if not (p.passes & (ps + 1)):
+                continue
+            iters = ora["iters1"] if ps == 0 else ora["iters2"]
+            for it in range(iters):
+                oc = ora["dump_cost"][ps, it]
+                gc = c[ps, it, k]
+                assert np.array_equal(gc, oc), f"region {k} pass {ps+1} iter {it}: costs differ"
+                for a in range(A):
+                    if oc[a] == O.INVALID:
+                        continue
+                    g_ord = o[ps, it, base0 + a * n: base0 + (a + 1) * n].astype(np.uint32)
+                    assert np.array_equal(g_ord, ora["dump_order"][ps, it, a]), (k, ps, it, a)
+                    if ps == 1:
+                        g_cyc = y[ps, it, base0 + a * n: base0 + (a + 1) * n]
+                        assert np.array_equal(g_cyc, ora["dump_cycle"][ps, it, a]), (k, ps, it, a)
+        compare_results(s.results(k, 1)[0], ora, f"region {k}")
+
+
+def test_fig1_two_ants(torch_cuda):
+    m = I.Machine(n_classes=1, steps=((24, 28, 32, 36, 40, 48, 64, 84, 128, 256),))
+    f = I.fig1r()
+    p = I.Params(ants=2, iterations=1, seed=0, cost_mode=0, stall_mod=1)
+    s = _sched(m)
+    s.load([f], [0]).run(p, no_prune=True, dump=True)
+    dump_parity(s, [f], [0], p, m)
+    g = s.results()[0]
+    assert g["length"] == 10 and list(g["cycle"]) == [0, 1, 2, 5, 6, 8, 9]
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_config1_fix10a_every_ant(torch_cuda, seed):
+    """Config 1: FIX10-A, 2 classes, 64 ants x 20 iterations, PRP_SUM."""
+    x = I.fix10a()
+    p = I.Params(ants=64, iterations=20, seed=seed, cost_mode=0)
+    s = _sched()
+    s.load([x], [7]).run(p, no_prune=True, dump=True)
+    dump_parity(s, [x], [7], p)
+    g = s.results()[0]
+    checker.check_schedule(x, g["order"], g["cycle"], g["length"])
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2, 3])
+def test_synthetic_batch_every_ant(torch_cuda, mode):
+    """A ragged batch (sizes span several bitset words, mixed latencies) with
+    an ant count that is not a multiple of the block or group size."""
+    sizes = [1, 5, 23, 40, 64, 97, 130]
+    regs = [I.gen_region(n, 500 + i + 10 * mode, "mixed" if i % 2 else "unit") for i, n in enumerate(sizes)]
+    ids = [1000 + 3 * i for i in range(len(regs))]
+    p = I.Params(ants=100, iterations=3, seed=11 + mode, cost_mode=mode, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_pruning_is_winner_invariant(torch_cuda):
+    regs = [I.gen_region(n, 900 + n) for n in (30, 80, 150)]
+    ids = [0, 1, 2]
+    p = I.Params(ants=256, iterations=4, seed=5)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True)
+    a = s.results()
+    s.run(p, no_prune=False)
+    b = s.results()
+    for x, y in zip(a, b):
+        for k in ("length", "prp", "trace_hash", "iters1", "iters2"):
+            assert x[k] == y[k]
+        assert list(x["order"]) == list(y["order"])
+
+
+def test_config2_full(torch_cuda):
+    """Config 2: one synthetic region n = 100, both passes, 1024 ants x 100
+    iterations, production mode (pruning on), vs the oracle."""
+    reg = I.gen_region(100, I.region_seed(2, 0))
+    p = I.Params(ants=1024, iterations=100, seed=2)
+    s = _sched()
+    s.load([reg], [0]).run(p)
+    g = s.results()[0]
+    ora = O.schedule(reg, 0, I.GFX906, p)
+    compare_results(g, ora)
+    checker.check_schedule(reg, g["order"], g["cycle"], g["length"])
+
+
+def test_paper_mode_stop_rules(torch_cuda):
+    regs = I.gen_batch(24, base_seed=17)
+    ids = list(range(24))
+    p = I.Params(ants=192, iterations=8, seed=3, stop_no_improve=I.STOP_PAPER_CLASSES, stop_at_lb=1)
+    s = _sched()
+    s.load(regs, ids).run(p)
+    g = s.results()
+    _, _, stats, off = O.schedule_many(regs, ids, I.GFX906, p)
+    for k in range(len(regs)):
+        ora = {n: int(stats[k, i]) for n, i in O.ORS.items()}
+        assert g[k]["iters1"] == ora["iters1"] and g[k]["iters2"] == ora["iters2"], k
+        assert g[k]["trace_hash"] == ora["trace_hash"], k
+        assert g[k]["length"] == ora["length"] and g[k]["cost_rp"] == ora["cost_rp"], k
+
+
+def test_edge_regions(torch_cuda):
+    empty = I.Region.from_lists(0, [], [1], [1], [], [])
+    one = I.Region.from_lists(1, [], [0, 1], [0, 1], [[0]], [[1]])
+    noregs = I.Region.from_lists(4, [(0, 2, 3), (1, 2, 1)], [], [], [[], [], [], []], [[], [], [], []])
+    chain = I.Region.from_lists(6, [(i, i + 1, 2) for i in range(5)], [0] * 5, [0] * 5,
+                                [[i] for i in range(5)] + [[]], [[]] + [[i - 1] for i in range(1, 6)])
+    regs = [empty, one, noregs, chain]
+    ids = [10, 11, 12, 13]
+    p = I.Params(ants=40, iterations=3, seed=1, stall_mod=1)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_error_codes_through_abi(torch_cuda):
+    from paper_conf_cgo_shobakimhlmkrg24_b200._lib import AcoError
+    s = _sched()
+    bad = I.Region.from_lists(3, [(0, 1, 1), (1, 0, 1)], [], [], [[], [], []], [[], [], []])
+    with pytest.raises(AcoError) as e:
+        s.load([bad], [0])
+    assert e.value.status == -2
+    dup = [I.gen_region(10, 1), I.gen_region(12, 2)]
+    with pytest.raises(AcoError) as e:
+        s.load(dup, [5, 5])
+    assert e.value.status == -1
+
+
+def test_config3_sampled(torch_cuda):
+    """Config 3 at full size (5,000 regions, 1024 ants x 10 iterations per pass)
+    in the bench's launch configuration; the oracle recomputes a sample of
+    regions (the largest, the smallest and a spread) one by one."""
+    regs = I.gen_batch(5000, base_seed=3)
+    ids = list(range(5000))
+    p = I.Params(ants=1024, iterations=10, seed=3)
+    s = _sched()
+    s.load(regs, ids).run(p)
+    g = s.results()
+    sizes = np.array([r.n_insts for r in regs])
+    sample = sorted(set([int(np.argmax(sizes)), int(np.argmin(sizes))] + list(range(0, 5000, 499))))
+    _, _, stats, off = O.schedule_many([regs[k] for k in sample], [ids[k] for k in sample], I.GFX906, p)
+    for q, k in enumerate(sample):
+        ora = {n: int(stats[q, i]) for n, i in O.ORS.items()}
+        assert g[k]["trace_hash"] == ora["trace_hash"], k
+        assert g[k]["length"] == ora["length"] and g[k]["cost_rp"] == ora["cost_rp"], k
+        assert g[k]["prp"] == [ora["prp0"], ora["prp1"], ora["prp2"], ora["prp3"]], k
+    # every region's final schedule is valid (independent checker)
+    for k in range(0, 5000, 97):
+        checker.check_schedule(regs[k], g[k]["order"], g[k]["cycle"], g[k]["length"])
