@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""Benchmark: region-batch ACO throughput (ant-schedules/s) on 1..N B200s.
+
+One STEP = one full two-pass ACO run (aco_schedule_batch: every pass and
+iteration of every region: construction, argmin + winner replay, pheromone
+update, epilogue) over one batch of synthetic regions.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c3|c2|c1]
+  python bench.py --impl reference ...     # the CPU oracle on a bounded sample
+
+Multi-GPU: launched by torchrun, one process per GPU.  Regions shard with no
+data-path collective (each rank schedules its own batch with globally unique
+region ids); NCCL is used only for the barrier and the max-over-ranks time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_cgo_shobakimhlmkrg24_b200 import inputs as I  # noqa: E402
+
+METRIC = "ant-schedules/s"
+C3_REGIONS = 5000
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c3", choices=["c3", "c2", "c1"])
+    ap.add_argument("--regions", type=int, default=C3_REGIONS, help="regions per rank (c3)")
+    ap.add_argument("--ants", type=int, default=None)
+    ap.add_argument("--iterations", type=int, default=None)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=48, help="regions in the oracle sample")
+    return ap.parse_args()
+
+
+def workload(args, rank: int):
+    """(regions, region_ids, params, config dict) for this rank."""
+    if args.workload == "c3":
+        n = args.regions
+        first = rank * n
+        regs = I.gen_batch(n, base_seed=3, first_id=first)
+        ids = list(range(first, first + n))
+        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 10, seed=3)
+        cfg = {"workload": "c3-rocprim-shaped-batch", "regions_per_gpu": n,
+               "sizes": "20-500 (Table 3.a buckets)", "latency": "mixed"}
+    elif args.workload == "c2":
+        regs = [I.gen_region(100, I.region_seed(2, rank))]
+        ids = [rank]
+        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 100, seed=2)
+        cfg = {"workload": "c2-single-region-n100", "regions_per_gpu": 1, "latency": "mixed"}
+    else:
+        regs = [I.fix10a()]
+        ids = [rank]
+        p = I.Params(ants=args.ants or 64, iterations=args.iterations or 20, seed=0, cost_mode=0)
+        cfg = {"workload": "c1-fix10a", "regions_per_gpu": 1}
+    cfg.update({"ants": p.ants, "iterations_per_pass": p.iterations, "passes": "RP+ILP",
+                "cost": ["PRP_SUM", "APRP_SUM", "OCC", "PERP"][p.cost_mode], "stop_rules": "off (fixed work)"})
+    return regs, ids, p, cfg
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                  "--format=csv,noheader,nounits", "-lms", "200"],
+                                 stdout=subprocess.PIPE, text=True)
+        except Exception:
+            return
+        while not self._stop.is_set():
+            line = p.stdout.readline()
+            if not line:
+                break
+            self.samples.append([x.strip() for x in line.split(",")])
+        p.terminate()
+
+    def start(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        time.sleep(0.3)
+
+    def stop(self):
+        time.sleep(0.25)
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=3)
+        sm = [float(s[0]) for s in self.samples if s and s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if len(s) > 1 and s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4)
+                          if len(s) > 3 + i and s[3 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except Exception:
+        return {}
+
+
+def bytes_per_ant_step(stats: np.ndarray) -> float:
+    """SURVEY 8(d) algorithmic bytes per ant-step from oracle instrumentation:
+    8.5|F| + 2|R| + 12 deg + 6 |Use| + 2 |Def| + 16 per placed instruction."""
+    from oracle.pyoracle import ORS
+    s = stats.sum(axis=0).astype(np.float64)
+    pl = s[ORS["placements"]]
+    b = (8.5 * s[ORS["sum_F"]] + 2.0 * s[ORS["sum_R"]] + 12.0 * s[ORS["sum_deg"]] + 6.0 * s[ORS["sum_use"]]
+         + 2.0 * s[ORS["sum_def"]] + 16.0 * pl)
+    return float(b / max(pl, 1.0))
+
+
+def cpu_baseline(regs, ids, p, sample: int):
+    """The oracle as it stands on a bounded, stratified sample of the same workload."""
+    from oracle import pyoracle as O
+    k = min(sample, len(regs))
+    order = np.argsort([r.n_insts for r in regs], kind="stable")
+    pick = sorted(set(int(order[int(i)]) for i in np.linspace(0, len(regs) - 1, k)))
+    sub = [regs[i] for i in pick]
+    sid = [ids[i] for i in pick]
+    threads = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    _, _, stats, _ = O.schedule_many(sub, sid, I.GFX906, p, n_threads=threads)
+    dt = time.perf_counter() - t0
+    scheds = float(stats[:, O.ORS["ant_scheds"]].sum())
+    return {"value": scheds / dt, "unit": METRIC, "cores": threads, "kind": "oracle",
+            "sample": f"{len(sub)} of {len(regs)} regions (stratified by size), full A x I x 2 passes, "
+                      f"{scheds:.0f} ant-schedules in {dt:.1f} s"}, stats
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        return reference_arm(args, world, rank)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch, Scheduler
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    regs, ids, p, cfg = workload(args, rank)
+    batch = HostBatch(regs, ids)
+    sched = Scheduler(I.GFX906, device=local)
+    stream = torch.cuda.current_stream()
+    sched.load(regs, ids, batch=batch)
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{local}")
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(max(3, args.warmup)):
+        sched.run(p)
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    phase_ms = np.zeros(3)
+    phase_launches = np.zeros(3)
+    launches = 0
+    clk = ClockSampler(local)
+    clk.start()
+    barrier()
+    torch.cuda.synchronize()
+    for k in range(args.steps):
+        flush.zero_()  # L2 flush between timed steps (outside the events)
+        ev[k][0].record(stream)
+        sched.run(p, timing=True)
+        ev[k][1].record(stream)
+        ms, ln = sched.timing()  # syncs; events inside the library, same stream
+        phase_ms += ms
+        phase_launches += ln
+        launches += sched.launch_count()
+    torch.cuda.synchronize()
+    barrier()
+    clocks = clk.stop()
+    step_ms = sum(a.elapsed_time(b) for a, b in ev)
+    t = torch.tensor([step_ms], dtype=torch.float64, device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    max_ms = float(t.item())
+    res = sched.results()
+    iters = sum(r["iters1"] + r["iters2"] for r in res)
+    scheds_rank = p.ants * iters * args.steps
+    tot = torch.tensor([float(scheds_rank)], dtype=torch.float64, device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+    value = float(tot.item()) / (max_ms / 1000.0)
+
+    # ---- end to end through the public API: host inputs -> H2D -> run -> D2H results
+    e2e_ms = []
+    h2d = d2h = 0
+    sum_n = int(batch.offsets[-1])
+    orders = np.zeros(max(1, sum_n), np.uint32)
+    cycles = np.zeros(max(1, sum_n), np.uint32)
+    for _ in range(max(1, args.e2e_steps)):
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        sched.load(regs, ids, batch=batch)
+        sched.run(p)
+        sched.results_raw(0, len(regs), orders, cycles)
+        e2e_ms.append((time.perf_counter() - t0) * 1000.0)
+    h2d = int(sched.arena.numel()) if sched.arena is not None else 0
+    d2h = int(len(regs) * 64 + 4 * 2 * sum_n)
+    e = torch.tensor([float(np.median(e2e_ms))], dtype=torch.float64, device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(e, op=dist.ReduceOp.MAX)
+    e2e_value = float(tot.item()) / args.steps / (float(e.item()) / 1000.0)
+
+    out = None
+    if rank == 0:
+        peaks = measured_peaks()
+        cpu = None
+        bpas = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu, stats = cpu_baseline(regs, ids, p, args.cpu_sample)
+            bpas = bytes_per_ant_step(stats)
+        # roofline of the dominant kernel (ant construction): algorithmic bytes
+        construct_ms = phase_ms[0] / max(1, args.steps)
+        ant_steps = p.ants * sum(r["n"] * (r["iters1"] + r["iters2"]) for r in res)
+        sm_mhz = peaks.get("sm_max_mhz", 1965.0)
+        smem_peak = 148 * 128 * sm_mhz * 1e6 / 1e9  # GB/s, nominal smem crossbar (guide)
+        roof = None
+        if bpas is not None and construct_ms > 0:
+            n_launch = phase_launches[0] / max(1, args.steps)
+            achieved = bpas * ant_steps / (construct_ms / 1000.0) / 1e9
+            roof = {"bound": "smem", "achieved": round(achieved, 1), "peak": round(smem_peak, 1),
+                    "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": None,
+                    "kernel": "k_construct", "bytes_per_ant_step": round(bpas, 2),
+                    "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,
+                    "peak_source": "148 SM x 128 B/clk x sm_max_mhz (guide nominal smem)"}
+        out = {
+            "metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world,
+            "steps": args.steps, "warmup": max(3, args.warmup),
+            "ms_per_step": round(max_ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)", "data": "synthetic",
+            "config": dict(cfg, l2="flushed between timed steps (256 MB write)", parallelism=f"regions x{world}"),
+            "aco_ms_per_batch": round(max_ms / args.steps, 3),
+            "phase_ms_per_step": {"construct": round(phase_ms[0] / args.steps, 3),
+                                  "finalize": round(phase_ms[1] / args.steps, 3),
+                                  "init": round(phase_ms[2] / args.steps, 3)},
+            "gpu_launches": int(launches),
+            "e2e": {"value": round(e2e_value, 1), "unit": METRIC, "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "ms_per_step": round(float(e.item()), 3)},
+            "clocks": clocks, "roofline": roof, "cpu_baseline": cpu,
+        }
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return out
+
+
+def reference_arm(args, world, rank):
+    """--impl reference: the oracle (as it stands) on the host cores, on a
+    bounded sample of this arm's workload per step."""
+    if rank != 0:
+        return None
+    regs, ids, p, cfg = workload(args, 0)
+    cpu_times = []
+    scheds = 0.0
+    for _ in range(args.warmup):
+        pass  # the oracle has no warm-up state
+    for _ in range(args.steps):
+        cpu, stats = cpu_baseline(regs, ids, p, max(4, args.cpu_sample // max(1, args.steps)))
+        from oracle.pyoracle import ORS
+        s = float(stats[:, ORS["ant_scheds"]].sum())
+        scheds += s
+        cpu_times.append(s / cpu["value"])
+    tot_s = sum(cpu_times)
+    value = scheds / tot_s
+    out = {"metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(1000 * tot_s / args.steps, 3), "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
+           "data": "synthetic", "config": cfg, "impl": "reference",
+           "cpu_baseline": {"value": round(value, 1), "unit": METRIC, "cores": os.cpu_count(), "kind": "oracle",
+                            "sample": f"per step a stratified sample of {max(4, args.cpu_sample // max(1, args.steps))} "
+                                      f"regions of the {cfg['workload']} workload"},
+           "e2e": {"value": round(value, 1), "unit": METRIC, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return out
+
+
+if __name__ == "__main__":
+    main()

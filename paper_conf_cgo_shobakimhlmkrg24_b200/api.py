@@ -121,8 +121,10 @@ class Scheduler:
         sum_n = int(self.batch.offsets[-1])
         od = cy = None
         if orders:
-            od = torch.zeros((2, p.iterations, p.ants * sum_n + 1), dtype=torch.int16, device=dev)
-            cy = torch.zeros((2, p.iterations, p.ants * sum_n + 1), dtype=torch.int32, device=dev)
+            # flat [2][iterations][ants * sum_n] (+ padding so empty batches have storage)
+            size = 2 * p.iterations * p.ants * sum_n + 8
+            od = torch.zeros(size, dtype=torch.int16, device=dev)
+            cy = torch.zeros(size, dtype=torch.int32, device=dev)
         self.dump = (costs, od, cy)
         _lib.check(self.lib.aco_set_dump(self.ctx, C.c_void_p(costs.data_ptr()),
                                          C.c_void_p(od.data_ptr()) if od is not None else None,
@@ -133,7 +135,9 @@ class Scheduler:
             dump: bool = False, timing: bool = False):
         flags = ((_lib.ACO_FLAG_NO_PRUNE if no_prune else 0) | (_lib.ACO_FLAG_DUMP if dump else 0)
                  | (_lib.ACO_FLAG_TIMING if timing else 0))
-        if dump and self.dump is None:
+        if dump and (self.dump is None or self.params is None or
+                     (self.params.ants, self.params.iterations) != (p.ants, p.iterations) or
+                     self.dump[0].shape[2] != self.count):
             self.set_dump(p)
         need = self.workspace_bytes(p, flags)
         if self.ws is None or self.ws.numel() < need:
@@ -195,8 +199,10 @@ class Scheduler:
         torch.cuda.synchronize(self.device)
         costs, od, cy = self.dump
         c = costs.cpu().numpy().view(np.uint32)
-        o = od.cpu().numpy().view(np.uint16) if od is not None else None
-        y = cy.cpu().numpy().view(np.uint32) if cy is not None else None
+        sl = self.params.ants * int(self.batch.offsets[-1])
+        shape = (2, self.params.iterations, sl)
+        o = od.cpu().numpy().view(np.uint16)[:2 * shape[1] * sl].reshape(shape) if od is not None else None
+        y = cy.cpu().numpy().view(np.uint32)[:2 * shape[1] * sl].reshape(shape) if cy is not None else None
         return c, o, y
 
     def dump_ant(self, region: int, pass_: int, it: int, ant: int):

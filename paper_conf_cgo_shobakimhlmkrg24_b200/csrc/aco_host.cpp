@@ -43,8 +43,38 @@ struct aco_ctx_s {
   size_t ev_used = 0;
   std::vector<std::pair<size_t, size_t>> ev_pairs[3];
   uint64_t phase_launches[3] = {0, 0, 0};
+  // pinned staging buffers for the H2D copies (arena, plan); an event per
+  // buffer guards reuse while a previous async copy may still read it
+  void *pin[2] = {nullptr, nullptr};
+  size_t pin_bytes[2] = {0, 0};
+  cudaEvent_t pin_ev[2] = {nullptr, nullptr};
   ~aco_ctx_s() {
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+    for (int i = 0; i < 2; ++i) {
+      if (pin_ev[i]) cudaEventDestroy(pin_ev[i]);
+      if (pin[i]) cudaFreeHost(pin[i]);
+    }
+  }
+  // Copy `bytes` from host `src` to device `dst` through pinned staging slot k.
+  aco_status staged_h2d(int k, void *dst, const void *src, size_t bytes, cudaStream_t s) {
+    if (!bytes) return ACO_OK;
+    if (pin_ev[k]) {
+      if (cudaEventSynchronize(pin_ev[k]) != cudaSuccess) return ACO_E_CUDA;
+    } else if (cudaEventCreateWithFlags(&pin_ev[k], cudaEventDisableTiming) != cudaSuccess) {
+      return ACO_E_CUDA;
+    }
+    if (pin_bytes[k] < bytes) {
+      if (pin[k]) cudaFreeHost(pin[k]);
+      pin[k] = nullptr;
+      pin_bytes[k] = 0;
+      const size_t want = bytes + bytes / 4;
+      if (cudaMallocHost(&pin[k], want) != cudaSuccess) return ACO_E_CUDA;
+      pin_bytes[k] = want;
+    }
+    std::memcpy(pin[k], src, bytes);
+    if (cudaMemcpyAsync(dst, pin[k], bytes, cudaMemcpyHostToDevice, s) != cudaSuccess) return ACO_E_CUDA;
+    if (cudaEventRecord(pin_ev[k], s) != cudaSuccess) return ACO_E_CUDA;
+    return ACO_OK;
   }
   cudaEvent_t next_event() {
     if (ev_used == ev_pool.size()) {
@@ -343,12 +373,8 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   if (!d_arena) return ACO_OK;
   if (arena_bytes < need) return ACO_E_WORKSPACE;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
-  cudaError_t e = cudaMemcpyAsync(d_arena, blob.data(), blob.size(), cudaMemcpyHostToDevice,
-                                  (cudaStream_t)cuda_stream);
-  if (e != cudaSuccess) return ACO_E_CUDA;
-  // pageable source: make sure the copy has consumed `blob` before it is freed
-  e = cudaStreamSynchronize((cudaStream_t)cuda_stream);
-  if (e != cudaSuccess) return ACO_E_CUDA;
+  aco_status hs = ctx->staged_h2d(0, d_arena, blob.data(), blob.size(), (cudaStream_t)cuda_stream);
+  if (hs != ACO_OK) return hs;
   ctx->count = count;
   ctx->regions.resize(count);
   ctx->inst_off.assign(count + 1, 0);
@@ -499,8 +525,10 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     }
   }
   cudaStream_t s = (cudaStream_t)cuda_stream;
-  if (cudaMemcpyAsync(ws + o_rws, blob.data(), blob.size(), cudaMemcpyHostToDevice, s) != cudaSuccess)
-    return ACO_E_CUDA;
+  {
+    aco_status hs = ctx->staged_h2d(1, ws + o_rws, blob.data(), blob.size(), s);
+    if (hs != ACO_OK) return hs;
+  }
   LaunchCtx L;
   L.arena = ctx->arena;
   L.ws = ws;
