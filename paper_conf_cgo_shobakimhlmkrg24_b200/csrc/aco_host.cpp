@@ -6,6 +6,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <new>
@@ -48,7 +50,27 @@ struct aco_ctx_s {
   void *pin[2] = {nullptr, nullptr};
   size_t pin_bytes[2] = {0, 0};
   cudaEvent_t pin_ev[2] = {nullptr, nullptr};
+  // internal streams for concurrent construct classes (fork / join per iteration)
+  static constexpr int kStreams = 4;
+  cudaStream_t side[kStreams] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t fork_ev = nullptr, join_ev[kStreams] = {nullptr, nullptr, nullptr, nullptr};
+  bool side_ok = false;
+  bool make_side() {
+    if (side_ok) return true;
+    for (int i = 0; i < kStreams; ++i) {
+      if (cudaStreamCreateWithFlags(&side[i], cudaStreamNonBlocking) != cudaSuccess) return false;
+      if (cudaEventCreateWithFlags(&join_ev[i], cudaEventDisableTiming) != cudaSuccess) return false;
+    }
+    if (cudaEventCreateWithFlags(&fork_ev, cudaEventDisableTiming) != cudaSuccess) return false;
+    side_ok = true;
+    return true;
+  }
   ~aco_ctx_s() {
+    for (int i = 0; i < kStreams; ++i) {
+      if (side[i]) cudaStreamDestroy(side[i]);
+      if (join_ev[i]) cudaEventDestroy(join_ev[i]);
+    }
+    if (fork_ev) cudaEventDestroy(fork_ev);
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
     for (int i = 0; i < 2; ++i) {
       if (pin_ev[i]) cudaEventDestroy(pin_ev[i]);
@@ -90,10 +112,17 @@ namespace {
 
 struct Prepped {
   RegionDev rd{};
-  std::vector<uint32_t> succ_ptr, succ, muse, rb0, cnt0, rem0;
-  std::vector<uint32_t> info;  // 4 words per instruction
-  std::vector<uint16_t> eta1, eta2;
+  std::vector<unsigned char> image;  // the block image (ImageLayout)
 };
+
+// Append array v to the image at a 16-byte aligned offset; returns the offset.
+template <typename T>
+uint32_t img_put(std::vector<unsigned char> &img, const std::vector<T> &v) {
+  const uint64_t off = align16(img.size());
+  img.resize(off + v.size() * sizeof(T), 0);
+  if (!v.empty()) std::memcpy(img.data() + off, v.data(), v.size() * sizeof(T));
+  return (uint32_t)off;
+}
 
 // Validation + preprocessing of one region.  Readings R31-R38.
 aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P) {
@@ -193,12 +222,26 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   for (uint32_t g = 0; g < G; ++g)
     if (nuses[g] > ACO_MAX_USES) return ACO_E_TOO_LARGE;
   if ((uint64_t)n * ((uint64_t)max_lat + 1) >= (1ull << 24)) return ACO_E_TOO_LARGE;
-  // register categories: counters for multi-use, non-live-out registers
+  // register categories (R14, R15): single-use / 2-use (partner check) /
+  // >= 3 uses (u16 remaining-use counter); live-out registers never die
   std::vector<uint32_t> ctr(G, 0xFFFFFFFFu);
-  uint32_t nmu = 0;
+  uint32_t nctr = 0;
   for (uint32_t g = 0; g < G; ++g)
-    if (nuses[g] >= 2 && !(d.reg_flags[g] & kFlagLiveOut)) ctr[g] = nmu++;
-  if (nmu > 65535u) return ACO_E_TOO_LARGE;
+    if (nuses[g] >= 3 && !(d.reg_flags[g] & kFlagLiveOut)) ctr[g] = nctr++;
+  if (nctr > 65535u) return ACO_E_TOO_LARGE;
+  std::vector<uint32_t> user0(G, 0xFFFFFFFFu), user1(G, 0xFFFFFFFFu);
+  for (uint32_t j = 0; j < n; ++j)
+    for (uint32_t k = uptr[j]; k < uptr[j + 1]; ++k) {
+      const uint32_t g = ureg[k];
+      if (user0[g] == 0xFFFFFFFFu) user0[g] = j;
+      else if (user1[g] == 0xFFFFFFFFu) user1[g] = j;
+    }
+  {
+    uint32_t per_class[4] = {0, 0, 0, 0};
+    for (uint32_t g = 0; g < G; ++g) per_class[d.reg_class[g]]++;
+    for (uint32_t c = 0; c < 4; ++c)
+      if (per_class[c] > 65535u) return ACO_E_TOO_LARGE;  // u16 live counters
+  }
   // critical path heights (reverse topological relaxation)
   std::vector<uint32_t> cp(n, 0);
   for (size_t h = n; h-- > 0;) {
@@ -209,8 +252,8 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   }
   uint32_t cp_max = 0;
   for (uint32_t j = 0; j < n; ++j) cp_max = std::max(cp_max, cp[j]);
-  // per-instruction info
-  P.info.assign((size_t)n * 4, 0);
+  // per-instruction info + multi-use entries
+  std::vector<uint32_t> info((size_t)n * 4, 0), muse;
   uint32_t L = 0;
   uint32_t lbvec[4] = {0, 0, 0, 0}, livein[4] = {0, 0, 0, 0}, liveout[4] = {0, 0, 0, 0};
   for (uint32_t g = 0; g < G; ++g) {
@@ -225,77 +268,116 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
       defs[c]++;
       if (nuses[g] == 0 && !(d.reg_flags[g] & kFlagLiveOut)) dead[c]++;
     }
-    const uint32_t mstart = (uint32_t)P.muse.size();
+    const uint32_t mstart = (uint32_t)muse.size();
     uint32_t nonlo = 0;
     for (uint32_t k = uptr[j]; k < uptr[j + 1]; ++k) {
       const uint32_t g = ureg[k], c = d.reg_class[g];
       usec[c]++;
       if (d.reg_flags[g] & kFlagLiveOut) continue;
       nonlo++;
-      if (nuses[g] == 1) sk[c]++;
-      else P.muse.push_back(ctr[g] | (c << 16));
+      if (nuses[g] == 1) {
+        sk[c]++;
+      } else if (nuses[g] == 2) {
+        const uint32_t other = user0[g] == j ? user1[g] : user0[g];
+        muse.push_back(other | (c << 16));
+      } else {
+        muse.push_back(ctr[g] | (c << 16) | kMuseCounter);
+      }
     }
     L = std::max(L, nonlo);
-    const uint32_t mcnt = (uint32_t)P.muse.size() - mstart;
+    const uint32_t mcnt = (uint32_t)muse.size() - mstart;
+    if (mcnt > 15u) return ACO_E_TOO_LARGE;  // 4-bit last-use counters
     for (uint32_t c = 0; c < 4; ++c) {
       if (defs[c] > 255u || dead[c] > 255u || sk[c] > 255u) return ACO_E_TOO_LARGE;
-      P.info[(size_t)j * 4 + 0] |= defs[c] << (8 * c);
-      P.info[(size_t)j * 4 + 1] |= dead[c] << (8 * c);
-      P.info[(size_t)j * 4 + 2] |= sk[c] << (8 * c);
+      info[(size_t)j * 4 + 0] |= defs[c] << (8 * c);
+      info[(size_t)j * 4 + 1] |= sk[c] << (8 * c);
+      info[(size_t)j * 4 + 2] |= dead[c] << (8 * c);
       lbvec[c] = std::max(lbvec[c], std::max(defs[c], usec[c]));
     }
     if (mstart >= (1u << 24)) return ACO_E_TOO_LARGE;
-    P.info[(size_t)j * 4 + 3] = (mstart << 8) | mcnt;
+    info[(size_t)j * 4 + 3] = (mstart << 8) | mcnt;
   }
   // heuristic tables (R4)
   const uint64_t km1 = (uint64_t)L * (cp_max + 1ull) + cp_max;
   const uint64_t d1 = km1 ? km1 : 1;
-  P.eta1.resize((size_t)n * (L + 1));
+  std::vector<uint16_t> eta1((size_t)n * (L + 1)), eta2(n);
   for (uint32_t j = 0; j < n; ++j)
     for (uint32_t l = 0; l <= L; ++l) {
       const uint64_t key = (uint64_t)l * (cp_max + 1ull) + cp[j];
-      P.eta1[(size_t)j * (L + 1) + l] = (uint16_t)(1 + key * 65534ull / d1);
+      eta1[(size_t)j * (L + 1) + l] = (uint16_t)(1 + key * 65534ull / d1);
     }
-  P.eta2.resize(n);
-  for (uint32_t j = 0; j < n; ++j)
-    P.eta2[j] = (uint16_t)(1 + (uint64_t)cp[j] * 65534ull / (cp_max ? cp_max : 1));
-  // successor list packed v | lat << 16
-  P.succ_ptr = sp;
-  P.succ.resize(E);
-  for (uint32_t q = 0; q < E; ++q) P.succ[q] = outs[q] | (lats[q] << 16);
+  for (uint32_t j = 0; j < n; ++j) eta2[j] = (uint16_t)(1 + (uint64_t)cp[j] * 65534ull / (cp_max ? cp_max : 1));
+  // pass-specific compact per-instruction records
+  std::vector<uint32_t> ds((size_t)n * 2), e1b(n);
+  for (uint32_t j = 0; j < n; ++j) {
+    ds[2 * j] = info[(size_t)j * 4 + 0];
+    ds[2 * j + 1] = info[(size_t)j * 4 + 1];
+    const uint32_t skw = info[(size_t)j * 4 + 1];
+    e1b[j] = j * (L + 1) + (skw & 0xFF) + ((skw >> 8) & 0xFF) + ((skw >> 16) & 0xFF) + (skw >> 24);
+  }
+  // users of each counter register (to find the last remaining user)
+  std::vector<uint32_t> cu_ptr(nctr + 1, 0), cu;
+  for (uint32_t g = 0; g < G; ++g)
+    if (ctr[g] != 0xFFFFFFFFu) cu_ptr[ctr[g] + 1] = nuses[g];
+  for (uint32_t m = 0; m < nctr; ++m) cu_ptr[m + 1] += cu_ptr[m];
+  cu.resize(cu_ptr[nctr]);
+  {
+    std::vector<uint32_t> fill(cu_ptr.begin(), cu_ptr.end() - 1);
+    for (uint32_t j = 0; j < n; ++j)
+      for (uint32_t k = uptr[j]; k < uptr[j + 1]; ++k) {
+        const uint32_t g = ureg[k];
+        if (ctr[g] != 0xFFFFFFFFu) cu[fill[ctr[g]]++] = j;
+      }
+  }
+  // successor / predecessor lists
+  std::vector<uint32_t> succ(E), pp(n + 1, 0), pred(E);
+  for (uint32_t q = 0; q < E; ++q) succ[q] = outs[q] | (indeg[outs[q]] == 1 ? kSuccSingle : 0u) | (lats[q] << 16);
+  for (uint32_t j = 0; j < n; ++j) pp[j + 1] = pp[j] + indeg[j];
+  {
+    std::vector<uint32_t> fill(pp.begin(), pp.end() - 1);
+    for (uint32_t j = 0; j < n; ++j)
+      for (uint32_t q = sp[j]; q < sp[j + 1]; ++q) pred[fill[outs[q]]++] = j | (lats[q] << 16);
+  }
   // initial per-ant state
   const uint32_t nwr = (n + 31) / 32;
-  P.rb0.assign(nwr, 0);
+  std::vector<uint32_t> rb0(nwr, 0), rem0((nctr + 1) / 2, 0);
   for (uint32_t j = 0; j < n; ++j)
-    if (!indeg[j]) P.rb0[j >> 5] |= 1u << (j & 31);
-  P.cnt0.assign((n + 3) / 4, 0);
-  for (uint32_t j = 0; j < n; ++j) P.cnt0[j >> 2] |= indeg[j] << (8 * (j & 3));
-  P.rem0.assign((nmu + 1) / 2, 0);
+    if (!indeg[j]) rb0[j >> 5] |= 1u << (j & 31);
   for (uint32_t g = 0; g < G; ++g)
-    if (ctr[g] != 0xFFFFFFFFu) P.rem0[ctr[g] >> 1] |= nuses[g] << (16 * (ctr[g] & 1));
+    if (ctr[g] != 0xFFFFFFFFu) rem0[ctr[g] >> 1] |= nuses[g] << (16 * (ctr[g] & 1));
   RegionDev &R = P.rd;
   std::memset(&R, 0, sizeof(R));
+  std::vector<unsigned char> &img = P.image;
+  img.clear();
+  R.img.info = img_put(img, info);
+  R.img.ds = img_put(img, ds);
+  R.img.e1b = img_put(img, e1b);
+  R.img.muse = img_put(img, muse);
+  R.img.cu_ptr = img_put(img, cu_ptr);
+  R.img.cu = img_put(img, cu);
+  R.img.eta1 = img_put(img, eta1);
+  R.img.eta2 = img_put(img, eta2);
+  R.img.succ_ptr = img_put(img, sp);
+  R.img.succ = img_put(img, succ);
+  R.img.pred_ptr = img_put(img, pp);
+  R.img.pred = img_put(img, pred);
+  R.img.rb0 = img_put(img, rb0);
+  R.img.rem0 = img_put(img, rem0);
+  img.resize(align16(img.size()) + 16, 0);
+  R.img.bytes = (uint32_t)img.size();
   R.n = n;
   R.nwr = nwr;
-  R.nmu = nmu;
+  R.nremw = (nctr + 1) / 2;
   R.L = L;
   R.region_id = d.region_id;
   R.cp_max = cp_max;
   R.lb_len = std::max(n, n ? cp_max + 1 : 0u);
-  R.ub_ready = 0;
+  R.max_cycle_bound = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)n * (max_lat + 1ull) + 1);
   for (uint32_t c = 0; c < 4; ++c) {
     R.livein[c] = livein[c];
     R.lbvec[c] = lbvec[c];
   }
   return ACO_OK;
-}
-
-template <typename T>
-uint64_t put(std::vector<unsigned char> &blob, const std::vector<T> &v) {
-  uint64_t off = align16(blob.size());
-  blob.resize(off + v.size() * sizeof(T) + 16, 0);
-  if (!v.empty()) std::memcpy(blob.data() + off, v.data(), v.size() * sizeof(T));
-  return off;
 }
 
 aco_status cuda_status(cudaError_t e) { return e == cudaSuccess ? ACO_OK : ACO_E_CUDA; }
@@ -357,19 +439,23 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   std::vector<unsigned char> blob(align16(sizeof(RegionDev) * (size_t)count + 16), 0);
   for (uint32_t i = 0; i < count; ++i) {
     RegionDev &R = P[i].rd;
-    R.o_succ_ptr = put(blob, P[i].succ_ptr);
-    R.o_succ = put(blob, P[i].succ);
-    R.o_info = put(blob, P[i].info);
-    R.o_muse = put(blob, P[i].muse);
-    R.o_rb0 = put(blob, P[i].rb0);
-    R.o_cnt0 = put(blob, P[i].cnt0);
-    R.o_rem0 = put(blob, P[i].rem0);
-    R.o_eta1 = put(blob, P[i].eta1);
-    R.o_eta2 = put(blob, P[i].eta2);
+    R.o_image = align16(blob.size());
+    blob.resize(R.o_image + P[i].image.size(), 0);
+    std::memcpy(blob.data() + R.o_image, P[i].image.data(), P[i].image.size());
     std::memcpy(blob.data() + sizeof(RegionDev) * (size_t)i, &R, sizeof(RegionDev));
   }
   const size_t need = align256(blob.size());
   if (arena_needed) *arena_needed = need;
+  if (!d_arena && getenv("ACO_DEBUG_PLAN")) {  // debug: keep host metadata for a sizing-only plan
+    ctx->count = count;
+    ctx->regions.resize(count);
+    ctx->inst_off.assign(count + 1, 0);
+    for (uint32_t i = 0; i < count; ++i) {
+      ctx->regions[i] = P[i].rd;
+      ctx->inst_off[i + 1] = ctx->inst_off[i] + P[i].rd.n;
+    }
+    ctx->arena = nullptr;
+  }
   if (!d_arena) return ACO_OK;
   if (arena_bytes < need) return ACO_E_WORKSPACE;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
@@ -398,16 +484,46 @@ aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint
 
 namespace {
 
-// Ants per block and the smem word cap for a per-ant state of W words.
-void pick_class(uint32_t W, uint32_t &ants_pb, uint32_t &wcap) {
-  static const uint32_t caps[] = {16, 32, 48, 64, 96, 128, 192, 256, 384, 512, 768, 1024, 1536, 1775};
-  wcap = 1775;
-  for (uint32_t c : caps)
-    if (W <= c) {
-      wcap = c;
-      break;
-    }
-  ants_pb = wcap <= 96 ? 128 : (wcap <= 384 ? 64 : 32);
+// Launch shape of one region in one pass: ants per block and whether tau is
+// staged in shared memory, chosen to maximise resident ants per SM (tau in
+// smem is preferred unless it costs residency below 256 ants).
+struct Shape {
+  uint32_t apb, smem;
+  bool ts;
+};
+
+// Dynamic shared-memory buckets of a construct launch (all blocks of a
+// launch reserve the same amount).
+const uint32_t kBuckets[] = {12 * 1024, 24 * 1024, 36 * 1024, 56 * 1024, 76 * 1024,
+                             112 * 1024, 150 * 1024, kSmemPerSM - 1024};
+
+uint32_t bucket_of(uint32_t bytes) {
+  for (uint32_t b : kBuckets)
+    if (bytes <= b) return b;
+  return 0;
+}
+
+// max_threads: resident threads per SM allowed by the kernel's registers
+// (pass 1 ~48 regs -> 1280, pass 2 ~80 regs -> 768; see cuobjdump -res-usage).
+Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads) {
+  auto resident = [&](uint32_t apb, uint32_t bytes) -> uint32_t {
+    const uint32_t b = bucket_of(bytes);
+    if (!b) return 0;
+    uint32_t blocks = kSmemPerSM / (b + 1024);  // + per-block reserved smem
+    blocks = std::min(blocks, max_threads / apb);  // register budget
+    blocks = std::min(blocks, 32u);
+    return blocks * apb;
+  };
+  Shape best0{0, 0, false}, best1{0, 0, true};
+  uint32_t r0 = 0, r1 = 0;
+  for (uint32_t apb : {32u, 64u, 128u, 256u}) {
+    const uint32_t b0 = img + apb * W * 4, b1 = img + tb + apb * W * 4;
+    const uint32_t x0 = resident(apb, b0), x1 = resident(apb, b1);
+    if (x0 >= r0 && x0 > 0) { r0 = x0; best0 = Shape{apb, bucket_of(b0), false}; }
+    if (x1 >= r1 && x1 > 0) { r1 = x1; best1 = Shape{apb, bucket_of(b1), true}; }
+  }
+  if (r1 > 0 && r1 >= std::min(r0, 256u)) return best1;
+  return best0;
 }
 
 }  // namespace
@@ -415,7 +531,6 @@ void pick_class(uint32_t W, uint32_t &ants_pb, uint32_t &wcap) {
 aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspace, size_t ws_bytes,
                               size_t *ws_needed, void *cuda_stream) {
   if (!ctx || !p) return ACO_E_ARG;
-  if (!ctx->arena && ctx->count) return ACO_E_STATE;
   if (p->pass < 1 || p->pass > 3 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
       p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->tau0 > 65535u ||
       p->tau0 < p->tau_min || p->tau0 > p->tau_max || p->q0_t > (1ull << 32) || p->rho_q16 > 65536u ||
@@ -423,34 +538,47 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     return ACO_E_ARG;
   if ((p->flags & ACO_FLAG_DUMP) && !ctx->dump_cost) return ACO_E_ARG;
   const uint32_t count = ctx->count, A = p->ants;
-  // ---- per-pass construct classes
+  // ---- per-pass construct classes (pass, ants/block, tau in smem, u32 cycles, mask, smem bucket)
   struct Cls {
-    uint32_t ants_pb, wcap;
-    bool mask;
-    std::vector<std::pair<uint64_t, uint32_t>> regs;  // (-work, region)
+    Shape sh;
+    bool mask, t32;
+    uint32_t smem;
+    std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  std::map<std::tuple<uint32_t, uint32_t, uint32_t, bool>, Cls> classes;  // (pass, ants_pb, wcap, mask)
+  using Key = std::tuple<uint32_t, uint32_t, bool, bool, bool, uint32_t>;
+  std::map<Key, Cls> classes;
   uint32_t fin_smem[3] = {0, 0, 0}, max_n = 0, init_smem = 0, p2_smem = 0;
+  bool any_t32 = false;
+  const bool nc4 = ctx->mach.n_classes > 2;
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
     max_n = std::max(max_n, R.n);
+    const bool t32 = R.max_cycle_bound > 65535u;
+    any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
-      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nmu);
-      if (W > 1775) return ACO_E_TOO_LARGE;
-      const uint32_t fs = 4 * W + 4 * R.n + 2 * ((R.n + 2) & ~1u) + 2 * (R.n + 1) + 64;
-      fin_smem[pass] = std::max(fin_smem[pass], fs);
-      if (pass == 1) init_smem = std::max(init_smem, 4 * W + 16);
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, nc4);
+      if (pass == 1) init_smem = std::max(init_smem, R.img.bytes + 4 * W + 16);
       if (!(p->pass & pass)) continue;
-      uint32_t apb, wcap;
-      pick_class(W, apb, wcap);
+      const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u);
+      if (sh.apb == 0) return ACO_E_TOO_LARGE;
       const bool mask = R.n <= 1024;
-      Cls &c = classes[std::make_tuple(pass, apb, wcap, mask)];
-      c.ants_pb = apb;
-      c.wcap = wcap;
+      const Key key(pass, sh.apb, sh.ts, pass == 2 && t32, mask, sh.smem);
+      Cls &c = classes[key];
+      c.sh = sh;
       c.mask = mask;
+      c.t32 = pass == 2 && t32;
+      c.smem = std::max(c.smem, sh.smem);
       c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
     }
     p2_smem = std::max(p2_smem, 4 * R.n + 16);
+  }
+  for (uint32_t r = 0; r < count; ++r) {
+    const RegionDev &R = ctx->regions[r];
+    for (uint32_t pass = 1; pass <= 2; ++pass) {
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && any_t32, nc4);
+      const uint32_t fs = R.img.bytes + 4 * W + 4 * R.n + 2 * R.n + 64;
+      fin_smem[pass] = std::max(fin_smem[pass], fs);
+    }
   }
   if (std::max(fin_smem[1], fin_smem[2]) > 227 * 1024) return ACO_E_TOO_LARGE;
   // ---- workspace layout
@@ -461,12 +589,19 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   off = align16(off + sizeof(RegionWs) * (uint64_t)count);
   const uint64_t o_items = off;
   uint64_t n_items = 0;
-  std::vector<std::pair<std::tuple<uint32_t, uint32_t, uint32_t, bool>, uint64_t>> class_item_off;
+  std::vector<std::pair<Key, uint64_t>> class_item_off;
   for (auto &kv : classes) {
     class_item_off.push_back({kv.first, n_items});
-    n_items += (uint64_t)kv.second.regs.size() * ((A + kv.second.ants_pb - 1) / kv.second.ants_pb);
+    n_items += (uint64_t)kv.second.regs.size() * ((A + kv.second.sh.apb - 1) / kv.second.sh.apb);
   }
-  off = align256(off + sizeof(BlockItem) * n_items);
+  off = align16(off + sizeof(BlockItem) * n_items);
+  const uint64_t o_upd = off;
+  uint64_t n_upd_max = 0;
+  for (uint32_t r = 0; r < count; ++r) {
+    const uint64_t n = ctx->regions[r].n;
+    n_upd_max += ((((n + 1) * n + 7) / 8) + kUpdVec - 1) / kUpdVec;
+  }
+  off = align256(off + sizeof(UpdItem) * n_upd_max);
   const uint64_t sum_n = ctx->inst_off.empty() ? 0 : ctx->inst_off[count];
   const uint64_t o_gb1 = off;
   off = align256(off + 2 * sum_n + 16);
@@ -474,6 +609,8 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   off = align256(off + 2 * sum_n + 16);
   const uint64_t o_gb2c = off;
   off = align256(off + 4 * sum_n + 16);
+  const uint64_t o_next = off;
+  off = align256(off + 2 * (sum_n + count) + 16);
   const uint64_t o_cost = off;
   off = align256(off + 4ull * A * count);
   std::vector<RegionWs> rws(count);
@@ -489,22 +626,34 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     w.o_gb2 = o_gb2 + 2 * ctx->inst_off[r];
     w.o_gb2c = o_gb2c + 4 * ctx->inst_off[r];
     w.o_dump = (uint64_t)A * ctx->inst_off[r];
+    w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
   }
+  // pheromone-update items (after the construct items in the plan blob)
+  std::vector<UpdItem> upd;
+  for (uint32_t r = 0; r < count; ++r)
+    for (uint32_t v0 = 0; v0 < rws[r].tau_len / 8; v0 += kUpdVec) upd.push_back(UpdItem{r, v0});
   const size_t need = align256(off);
   if (ws_needed) *ws_needed = need;
-  if (!d_workspace) return ACO_OK;
-  if (ws_bytes < need) return ACO_E_WORKSPACE;
-  if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
-  if (!ctx->machine_uploaded) {
-    if (set_machine(ctx->mach) != 0) return ACO_E_CUDA;
-    ctx->machine_uploaded = true;
+  const bool plan_only = !d_workspace;  // (debug: ACO_DEBUG_PLAN prints the plan)
+  if (plan_only && !getenv("ACO_DEBUG_PLAN")) return ACO_OK;
+  if (!plan_only) {
+    if (!ctx->arena && ctx->count) return ACO_E_STATE;
+    if (ws_bytes < need) return ACO_E_WORKSPACE;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
+    if (!ctx->machine_uploaded) {
+      if (set_machine(ctx->mach) != 0) return ACO_E_CUDA;
+      ctx->machine_uploaded = true;
+    }
+    if (!ctx->make_side()) return ACO_E_CUDA;
   }
   unsigned char *ws = (unsigned char *)d_workspace;
   // ---- host plan: RegionWs table + block items, one H2D
   std::vector<unsigned char> &blob = ctx->plan_blob;
-  blob.assign(o_items - o_rws + sizeof(BlockItem) * n_items, 0);
+  blob.assign(o_upd - o_rws + sizeof(UpdItem) * upd.size(), 0);
+  if (!upd.empty()) std::memcpy(blob.data() + (o_upd - o_rws), upd.data(), sizeof(UpdItem) * upd.size());
   std::memcpy(blob.data(), rws.data(), sizeof(RegionWs) * count);
   std::vector<ClassLaunch> launches[3];
+  std::vector<uint64_t> class_work[3];
   {
     size_t ci = 0;
     for (auto &kv : classes) {
@@ -514,16 +663,35 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
       BlockItem *items = (BlockItem *)(blob.data() + (o_items - o_rws)) + base;
       uint64_t k = 0;
       for (auto &pr : c.regs)
-        for (uint32_t a0 = 0; a0 < A; a0 += c.ants_pb) items[k++] = BlockItem{pr.second, a0};
+        for (uint32_t a0 = 0; a0 < A; a0 += c.sh.apb) items[k++] = BlockItem{pr.second, a0};
       ClassLaunch cl;
       cl.items = (const BlockItem *)(ws + o_items) + base;
       cl.n_blocks = (uint32_t)k;
-      cl.ants_pb = c.ants_pb;
-      cl.smem_bytes = c.ants_pb * c.wcap * 4;
+      cl.ants_pb = c.sh.apb;
+      cl.smem_bytes = c.smem;
       cl.max_n = c.mask ? 1024 : 65535;
+      cl.tau_smem = c.sh.ts;
+      cl.t32 = c.t32;
+      cl.nc4 = nc4;
       launches[std::get<0>(kv.first)].push_back(cl);
+      class_work[std::get<0>(kv.first)].push_back(0);
+      for (auto &pr : c.regs) class_work[std::get<0>(kv.first)].back() += ~pr.first;
     }
   }
+  for (int pass = 1; pass <= 2; ++pass) {  // biggest classes first (fork round-robin)
+    std::vector<size_t> idx(launches[pass].size());
+    for (size_t i = 0; i < idx.size(); ++i) idx[i] = i;
+    std::sort(idx.begin(), idx.end(), [&](size_t a, size_t b) { return class_work[pass][a] > class_work[pass][b]; });
+    std::vector<ClassLaunch> sorted;
+    for (size_t i : idx) sorted.push_back(launches[pass][i]);
+    launches[pass] = sorted;
+    if (getenv("ACO_DEBUG_PLAN"))
+      for (size_t i = 0; i < idx.size(); ++i)
+        fprintf(stderr, "[aco plan] pass %d class %zu: blocks %u ants/blk %u smem %u tau_smem %d t32 %d work %.3g\n",
+                pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].smem_bytes, (int)sorted[i].tau_smem,
+                (int)sorted[i].t32, (double)class_work[pass][idx[i]]);
+  }
+  if (plan_only) return ACO_OK;
   cudaStream_t s = (cudaStream_t)cuda_stream;
   {
     aco_status hs = ctx->staged_h2d(1, ws + o_rws, blob.data(), blob.size(), s);
@@ -603,11 +771,29 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     for (uint32_t it = 0; it < p->iterations && !err; ++it) {
       size_t e0 = begin(0);
       uint64_t l0 = L.launches;
-      for (const ClassLaunch &cl : launches[pass]) err |= launch_construct(L, pass, it, cl);
+      const std::vector<ClassLaunch> &cls = launches[pass];
+      if (cls.size() <= 1) {
+        for (const ClassLaunch &cl : cls) err |= launch_construct(L, pass, it, cl);
+      } else {
+        // fork: classes round-robin over the internal streams, join on `s`
+        const int k = (int)std::min<size_t>(cls.size(), aco_ctx_s::kStreams);
+        err |= cudaEventRecord(ctx->fork_ev, s) != cudaSuccess;
+        for (int i = 0; i < k; ++i) err |= cudaStreamWaitEvent(ctx->side[i], ctx->fork_ev, 0) != cudaSuccess;
+        for (size_t c = 0; c < cls.size(); ++c) {
+          L.stream = ctx->side[c % k];
+          err |= launch_construct(L, pass, it, cls[c]);
+        }
+        L.stream = cuda_stream;
+        for (int i = 0; i < k; ++i) {
+          err |= cudaEventRecord(ctx->join_ev[i], ctx->side[i]) != cudaSuccess;
+          err |= cudaStreamWaitEvent(s, ctx->join_ev[i], 0) != cudaSuccess;
+        }
+      }
       end(0, e0, l0);
       e0 = begin(1);
       l0 = L.launches;
-      err |= launch_finalize(L, pass, it, fin_smem[pass], max_n);
+      err |= launch_finalize(L, pass, it, fin_smem[pass], max_n, pass == 2 && any_t32, nc4,
+                             (const UpdItem *)(ws + o_upd), (uint32_t)upd.size());
       end(1, e0, l0);
     }
   }

@@ -2,41 +2,70 @@
 // internal; shared by aco_host.cpp and aco_kernels.cu only).
 //
 // Region statics live in the caller's ARENA (written once by
-// aco_load_regions); run state lives in the caller's WORKSPACE (laid out by
-// aco_schedule_batch).  All offsets are in BYTES from the buffer base.
+// aco_load_regions) as one contiguous, 16-byte aligned BLOCK IMAGE per region
+// whose internal layout is exactly what the kernels keep in shared memory;
+// a block stages it with 16-byte copies.  Run state lives in the caller's
+// WORKSPACE (laid out by aco_schedule_batch).  Offsets are in bytes.
 #pragma once
 #include <stdint.h>
 
 #include "../../include/aco.h"
 
+#ifdef __CUDACC__
+#define ACO_HD __host__ __device__
+#else
+#define ACO_HD
+#endif
+
 namespace aco {
 
 constexpr uint32_t kInvalid = 0xFFFFFFFFu;  // R35
-constexpr uint32_t kMaxKernelInsts = 8192;  // compiled limit of this version
+constexpr uint32_t kMaxKernelInsts = 8191;  // ids use 13 bits in successor entries
 constexpr uint32_t kFlagLiveIn = 1, kFlagLiveOut = 2;
+constexpr uint32_t kSmemPerSM = 227 * 1024;
 
-// Per-region statics (arena).  Arrays are 16-byte aligned.
+// Successor entry: v (13 bits) | single-predecessor flag << 13 | latency << 16.
+constexpr uint32_t kSuccSingle = 1u << 13;
+// Multi-use register entry (uses of a register with >= 2 uses, not live-out):
+//   bit 31 = 0: the register has exactly 2 users; bits 0..12 = the OTHER user
+//   bit 31 = 1: >= 3 users; bits 0..15 = remaining-use counter index
+//   bits 16..17 = register class
+constexpr uint32_t kMuseCounter = 1u << 31;
+
+// Offsets (bytes, relative to the image start) of the arrays of the block image.
+struct ImageLayout {
+  uint32_t info;      // uint4 [n] {defs u8x4, static kills u8x4, dead defs u8x4, muse start << 8 | count}
+  uint32_t ds;        // uint2 [n] {defs u8x4, static kills u8x4} (pass-2 feasibility)
+  uint32_t e1b;       // u32 [n]: j*(L+1) + #static kills (row base into eta1 for pass 1)
+  uint32_t muse;      // u32 [nm]
+  uint32_t cu_ptr;    // u32 [nctr+1]: users of each counter register
+  uint32_t cu;        // u32 [..]
+  uint32_t eta1;      // u16 [n * (L+1)]: eta1(j, luc) at j*(L+1) + luc (R4)
+  uint32_t eta2;      // u16 [n]
+  uint32_t succ_ptr;  // u32 [n+1]
+  uint32_t succ;      // u32 [E]
+  uint32_t pred_ptr;  // u32 [n+1]
+  uint32_t pred;      // u32 [E]: p | latency << 16
+  uint32_t rb0;       // u32 [nwr]: roots bitset
+  uint32_t rem0;      // u32 [nremw]: u16 use counts of >= 3-use registers
+  uint32_t bytes;     // total, multiple of 16
+  uint32_t pad;
+};
+
+// Per-region statics (arena header array).
 struct RegionDev {
   uint32_t n;        // instructions
   uint32_t nwr;      // words of an instruction bitset = ceil(n/32)
-  uint32_t nmu;      // remaining-use counters (registers used >= 2 times, not live-out)
+  uint32_t nremw;    // words of packed u16 counters = ceil(#counters / 2)
   uint32_t L;        // max LUC over instructions (rows of eta1 minus one)
   uint32_t region_id;
   uint32_t cp_max;
   uint32_t lb_len;   // max(n, 1 + CPmax) (R30)
-  uint32_t ub_ready; // 1 + max #independent (L182), reporting only
+  uint32_t max_cycle_bound;  // n * (max latency + 1): pass-2 cycles are below it
   uint32_t livein[4];
   uint32_t lbvec[4]; // per-class PRP lower bound vector (R30)
-  uint64_t o_succ_ptr;  // u32 [n+1]
-  uint64_t o_succ;      // u32 [E]  v | lat << 16
-  uint64_t o_info;      // uint4 [n] {defs c0..3 u8, dead defs u8x4, static kills u8x4, muse start<<8 | count}
-  uint64_t o_muse;      // u32 [..] counter index | class << 16
-  uint64_t o_rb0;       // u32 [nwr] roots bitset
-  uint64_t o_cnt0;      // u32 [ceil(n/4)] packed u8 in-degrees
-  uint64_t o_rem0;      // u32 [ceil(nmu/2)] packed u16 use counts
-  uint64_t o_eta1;      // u16 [n * (L+1)] eta1(j, luc) at [j*(L+1) + luc]
-  uint64_t o_eta2;      // u16 [n]
-  uint64_t pad;
+  uint64_t o_image;  // byte offset of the block image in the arena
+  ImageLayout img;
 };
 
 // Mutable per-region state (workspace).
@@ -62,8 +91,16 @@ struct RegionWs {
   uint64_t o_gb2;    // u16 [n]  pass-2 global best order
   uint64_t o_gb2c;   // u32 [n]  pass-2 global best cycles (in order)
   uint64_t o_dump;   // element offset of this region in a dump (pass, iter) slice = ants * sum n_q
+  uint64_t o_next;   // u16 [n+1]: the iteration winner's successor of each row (0xFFFF: none)
   uint32_t tau_len;  // (n+1)*n rounded up to a multiple of 8
   uint32_t pad;
+};
+
+// Pheromone-update work item: vectors [v0, v0 + kUpdVec) of a region's table.
+constexpr uint32_t kUpdVec = 2048;  // 16-byte vectors per block
+struct UpdItem {
+  uint32_t region;
+  uint32_t v0;
 };
 
 // Constant run configuration.
@@ -95,16 +132,23 @@ struct BlockItem {
 inline uint64_t align16(uint64_t x) { return (x + 15) & ~uint64_t(15); }
 inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 
-// Per-ant state words (u32) of a region for a pass, in the [word][ant] layout.
-#ifdef __CUDACC__
-#define ACO_HD __host__ __device__
-#else
-#define ACO_HD
-#endif
-ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32_t nmu) {
-  uint32_t w = nwr + (nmu + 1) / 2;
-  return pass == 1 ? w + (n + 3) / 4 : w + n;
+// Per-ant state words (u32) of a region for a pass, [word][ant] interleave:
+//   RB [nwr] ready set, SCH [nwr] scheduled set, REM [nremw] u16 counters, then
+//   pass 1: DK [ceil(n/8)]  4-bit count of registers whose last remaining
+//                           user is the instruction (dynamic part of LUC)
+//   pass 2: T  [ceil(n/2)] u16 (or [n] u32 if t32): issue cycle (placed) or
+//                           ready time (ready instruction)
+//           DK [ceil(n/4)] u8 = 2 classes x 4 bits (or [ceil(n/2)] u16 = 4
+//                           classes x 4 bits if nc4): per-class last-use counts
+ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32_t nremw, bool t32,
+                                 bool nc4) {
+  const uint32_t w = 2 * nwr + nremw;
+  if (pass == 1) return w + (n + 7) / 8;
+  return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }
+
+// Bytes of the pheromone table as staged in shared memory.
+ACO_HD inline uint32_t tau_smem_bytes(uint32_t n) { return (((n + 1) * n * 2) + 15) & ~15u; }
 
 // ---- launch interface implemented in aco_kernels.cu ----
 struct LaunchCtx {
@@ -127,13 +171,17 @@ struct ClassLaunch {
   uint32_t ants_pb;
   uint32_t smem_bytes;
   uint32_t max_n;          // max n in the class (selects the mask variant)
+  bool tau_smem;           // stage tau in shared memory
+  bool t32;                // u32 pass-2 cycle array
+  bool nc4;                // 3-4 register classes (u16 last-use counts)
 };
 
 int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success
 int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);
-int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n);
+int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
+                    bool nc4, const UpdItem *upd, uint32_t n_upd);
 int last_cuda_error();
 
 }  // namespace aco

@@ -1,22 +1,28 @@
 // aco_kernels.cu -- sm_100a kernels of the ACO instruction scheduler.
 //
-// Mapping: ONE ANT PER THREAD, as in the paper (L126),
-// but with every per-ant mutable array in SHARED MEMORY in a [word][ant]
-// interleave (word w of ant a at smem[w * ants_per_block + a]) so that the
-// data-dependent gathers of 32 ants of a warp (each at its own instruction)
-// always hit 32 distinct banks: conflict-free regardless of which
-// instruction each ant touches.  Region statics are read-only and shared by
-// all ants of a block (L1/L2 via the read-only path).  Exploit/explore is a
-// coin per group of 64 ants (L198), so a warp (32 ants) takes one branch.
+// Mapping: ONE ANT PER THREAD (as the paper, L126), all
+// ants of a block belong to one region.  Everything an ant touches per step
+// is in SHARED MEMORY:
+//   * the region's block image (per-instruction info, multi-use register
+//     entries, eta tables, successor/predecessor lists) -- staged once per
+//     block with 16-byte copies;
+//   * the pheromone table when it fits (else read through L1 from the
+//     workspace);
+//   * the per-ant mutable state in a [word][ant] interleave (word w of ant a at
+//     st[w * ants_per_block + a]): bank = lane, so the 32 data-dependent
+//     accesses of a warp (each ant at its own instruction) never conflict.
+// Exploit/explore is a coin per group of 64 ants (L198): a warp takes one
+// branch in pass 1.  Candidates are scored four at a time so that their
+// shared-memory loads overlap (ILP).
 //
-// Kernels per pass and iteration (L135-L139):
-//   k_construct  : every ant builds a schedule, writes its cost (K1a)
-//   k_finalize   : per region: argmin over (cost, ant) (K1b), replay of the
-//                  winner to recover its order (no per-ant order is ever
-//                  stored), pheromone evaporate+deposit (K1c), global-best
-//                  epilogue and termination flags (K1d).
-// Plus k_init (tau0, the greedy heuristic schedule) and k_pass2_init
-// (target, ASAP of the pass-1 best, tau reset).
+// Per pass and iteration (L135-L139):
+//   k_construct : every ant builds a schedule and writes its cost (K1a)
+//   k_finalize  : per region: argmin over (cost, ant) (K1b), replay of the
+//                 winner to recover its order (no per-ant order is stored),
+//                 pheromone evaporate + deposit (K1c), global-best epilogue and
+//                 termination (K1d).
+// Plus k_init (tau0, greedy heuristic schedule) and k_pass2_init (target, ASAP
+// of the pass-1 best, tau reset).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -59,7 +65,8 @@ __device__ __forceinline__ uint32_t aprp_of(uint32_t c, uint32_t x) {
     if (x <= c_mach.step_max[c][i]) return c_mach.step_max[c][i];
   return x;
 }
-__device__ uint32_t cost_rp(uint32_t mode, const uint32_t prp[4]) {
+__device__ __noinline__ uint32_t cost_rp(uint32_t mode, uint32_t p0, uint32_t p1, uint32_t p2, uint32_t p3) {
+  const uint32_t prp[4] = {p0, p1, p2, p3};
   const uint32_t nc = c_mach.n_classes;
   uint32_t cost = 0;
   if (mode == ACO_COST_PRP_SUM) {
@@ -98,238 +105,349 @@ __device__ void target_of(uint32_t mode, const uint32_t best[4], uint32_t tgt[4]
   }
 }
 
-// ---------------------------------------------------------------- region view
-struct RV {
-  uint32_t n, nwr, nmu, Lp1, region_id;
-  const uint32_t *succ_ptr, *succ, *muse, *rb0, *cnt0, *rem0;
+// ---------------------------------------------------------------- statics view
+struct SV {
   const uint4 *info;
+  const uint2 *ds;
+  const uint32_t *e1b, *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0;
   const uint16_t *eta1, *eta2;
-  uint32_t livein[4];
+  uint32_t n, nwr, nremw, region_id;
+  uint32_t livein01, livein23;  // u16 x 2
 };
 
-__device__ __forceinline__ RV make_rv(const unsigned char *arena, const RegionDev *rd) {
-  RV R;
-  R.n = rd->n;
-  R.nwr = rd->nwr;
-  R.nmu = rd->nmu;
-  R.Lp1 = rd->L + 1;
-  R.region_id = rd->region_id;
-  R.succ_ptr = (const uint32_t *)(arena + rd->o_succ_ptr);
-  R.succ = (const uint32_t *)(arena + rd->o_succ);
-  R.info = (const uint4 *)(arena + rd->o_info);
-  R.muse = (const uint32_t *)(arena + rd->o_muse);
-  R.rb0 = (const uint32_t *)(arena + rd->o_rb0);
-  R.cnt0 = (const uint32_t *)(arena + rd->o_cnt0);
-  R.rem0 = (const uint32_t *)(arena + rd->o_rem0);
-  R.eta1 = (const uint16_t *)(arena + rd->o_eta1);
-  R.eta2 = (const uint16_t *)(arena + rd->o_eta2);
-  for (int c = 0; c < 4; ++c) R.livein[c] = rd->livein[c];
-  return R;
+__device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev *rd) {
+  SV V;
+  V.info = (const uint4 *)(img + rd->img.info);
+  V.ds = (const uint2 *)(img + rd->img.ds);
+  V.e1b = (const uint32_t *)(img + rd->img.e1b);
+  V.muse = (const uint32_t *)(img + rd->img.muse);
+  V.cu_ptr = (const uint32_t *)(img + rd->img.cu_ptr);
+  V.cu = (const uint32_t *)(img + rd->img.cu);
+  V.eta1 = (const uint16_t *)(img + rd->img.eta1);
+  V.eta2 = (const uint16_t *)(img + rd->img.eta2);
+  V.succ_ptr = (const uint32_t *)(img + rd->img.succ_ptr);
+  V.succ = (const uint32_t *)(img + rd->img.succ);
+  V.pred_ptr = (const uint32_t *)(img + rd->img.pred_ptr);
+  V.pred = (const uint32_t *)(img + rd->img.pred);
+  V.rb0 = (const uint32_t *)(img + rd->img.rb0);
+  V.rem0 = (const uint32_t *)(img + rd->img.rem0);
+  V.n = rd->n;
+  V.nwr = rd->nwr;
+  V.nremw = rd->nremw;
+  V.region_id = rd->region_id;
+  V.livein01 = (rd->livein[0] & 0xFFFFu) | (rd->livein[1] << 16);
+  V.livein23 = (rd->livein[2] & 0xFFFFu) | (rd->livein[3] << 16);
+  return V;
 }
 
-__device__ __forceinline__ uint32_t byte_of(uint32_t w, uint32_t c) { return (w >> (8 * c)) & 0xFFu; }
-__device__ __forceinline__ uint32_t byte_sum(uint32_t w) { return (w * 0x01010101u) >> 24; }
+__device__ __forceinline__ uint32_t lo_pair(uint32_t w) { return __byte_perm(w, 0, 0x4140); }  // u8 b0,b1 -> u16x2
+__device__ __forceinline__ uint32_t hi_pair(uint32_t w) { return __byte_perm(w, 0, 0x4342); }  // u8 b2,b3 -> u16x2
 
-// remaining-use counter m (u16 packed two per word)
-__device__ __forceinline__ uint32_t rem_get(const uint32_t *REM, uint32_t S, uint32_t m) {
-  return (REM[(m >> 1) * S] >> ((m & 1u) * 16)) & 0xFFFFu;
+// Per-ant state (stride S words between consecutive words of one ant).
+struct St {
+  uint32_t *RB, *SCH, *REM, *T, *DK;
+  uint32_t S;
+};
+
+template <int PASS, bool T32, bool NC4>
+__device__ __forceinline__ St make_st(uint32_t *st, uint32_t S, const SV &V) {
+  St A;
+  A.S = S;
+  A.RB = st;
+  A.SCH = st + V.nwr * S;
+  A.REM = A.SCH + V.nwr * S;
+  A.T = A.REM + V.nremw * S;
+  A.DK = PASS == 1 ? A.T : A.T + (T32 ? V.n : (V.n + 1) / 2) * S;
+  return A;
 }
 
-// Iterate set bits of the ant's instruction bitset in ascending order (R25).
-// MASK: a register holds one bit per non-empty bitset word (n <= 1024).
-#define ACO_FOR_EACH_BIT(MASK, wmask, RB, S, nwr, J, BODY)                  \
-  {                                                                         \
-    uint32_t _m = (wmask);                                                  \
-    uint32_t _w = 0;                                                        \
-    bool _stop = false;                                                     \
-    while (!_stop) {                                                        \
-      if (MASK) {                                                           \
-        if (!_m) break;                                                     \
-        _w = __ffs(_m) - 1;                                                 \
-        _m &= _m - 1;                                                       \
-      } else if (_w >= (nwr)) {                                             \
-        break;                                                              \
-      }                                                                     \
-      uint32_t _bits = (RB)[_w * (S)];                                      \
-      while (_bits) {                                                       \
-        const uint32_t J = _w * 32u + (__ffs(_bits) - 1);                   \
-        _bits &= _bits - 1;                                                 \
-        BODY                                                                \
-      }                                                                     \
-      if (!MASK) ++_w;                                                      \
-    }                                                                       \
+__device__ __forceinline__ uint32_t sch_bit(const St &A, uint32_t p) {
+  return (A.SCH[(p >> 5) * A.S] >> (p & 31u)) & 1u;
+}
+
+// ---- last-use counts (DK): how many registers read by instruction j have j
+// as their last unscheduled user (the dynamic part of kills_c(j), R14).
+// pass 1: one 4-bit total per instruction
+__device__ __forceinline__ uint32_t dk1_get(const St &A, uint32_t j) {
+  return (A.DK[(j >> 3) * A.S] >> ((j & 7u) * 4)) & 0xFu;
+}
+// pass 2: 4 bits per class; returned as packed u8 x 4 per class
+template <bool NC4>
+__device__ __forceinline__ uint32_t dk2_get(const St &A, uint32_t j) {
+  if (NC4) {
+    uint32_t x = (A.DK[(j >> 1) * A.S] >> ((j & 1u) * 16)) & 0xFFFFu;
+    x = (x | (x << 8)) & 0x00FF00FFu;
+    return (x | (x << 4)) & 0x0F0F0F0Fu;
   }
-#define ACO_BREAK_SCAN \
-  {                    \
-    _stop = true;      \
-    break;             \
+  const uint32_t x = (A.DK[(j >> 2) * A.S] >> ((j & 3u) * 8)) & 0xFFu;
+  return (x & 0xFu) | ((x & 0xF0u) << 4);
+}
+template <int PASS, bool NC4>
+__device__ __forceinline__ void dk_add(const St &A, uint32_t j, uint32_t c) {
+  if (PASS == 1) {
+    A.DK[(j >> 3) * A.S] += 1u << ((j & 7u) * 4);
+  } else if (NC4) {
+    A.DK[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 4 * c);
+  } else {
+    A.DK[(j >> 2) * A.S] += 1u << ((j & 3u) * 8 + 4 * c);
   }
+}
+
+template <bool T32>
+__device__ __forceinline__ uint32_t t_get(const St &A, uint32_t j) {
+  if (T32) return A.T[j * A.S];
+  return (A.T[(j >> 1) * A.S] >> ((j & 1u) * 16)) & 0xFFFFu;
+}
+template <bool T32>
+__device__ __forceinline__ void t_set(const St &A, uint32_t j, uint32_t v) {
+  if (T32) {
+    A.T[j * A.S] = v;
+  } else {
+    const uint32_t sh = (j & 1u) * 16;
+    uint32_t *p = A.T + (j >> 1) * A.S;
+    *p = (*p & ~(0xFFFFu << sh)) | (v << sh);
+  }
+}
+
+// Ascending iteration over the ready bitset (R25).  MASK: one register bit per
+// non-empty bitset word (n <= 1024).
+struct BitIt {
+  uint32_t m, w, bits;
+};
+template <bool MASK>
+__device__ __forceinline__ void it_init(BitIt &it, uint32_t wmask) {
+  it.m = wmask;
+  it.w = MASK ? 0u : 0xFFFFFFFFu;
+  it.bits = 0;
+}
+template <bool MASK>
+__device__ __forceinline__ bool it_next(BitIt &it, const St &A, uint32_t nwr, uint32_t &j) {
+  while (!it.bits) {
+    if (MASK) {
+      if (!it.m) return false;
+      it.w = __ffs(it.m) - 1;
+      it.m &= it.m - 1;
+    } else {
+      if (++it.w >= nwr) return false;
+    }
+    it.bits = A.RB[it.w * A.S];
+  }
+  j = it.w * 32u + (__ffs(it.bits) - 1);
+  it.bits &= it.bits - 1;
+  return true;
+}
+// Next up to four candidates (ascending); invalid slots repeat j[0].
+template <bool MASK>
+__device__ __forceinline__ uint32_t it_next4(BitIt &it, const St &A, uint32_t nwr, uint32_t j[4]) {
+  uint32_t cnt = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint32_t x = 0;
+    if (cnt == (uint32_t)q && it_next<MASK>(it, A, nwr, x)) {
+      j[q] = x;
+      ++cnt;
+    } else {
+      j[q] = j[0];
+    }
+  }
+  return cnt;
+}
 
 struct AntOut {
   uint32_t cost;
-  uint32_t prp[4];
+  uint32_t prp01, prp23;
 };
+
+__device__ __forceinline__ uint32_t cost_of(uint32_t mode, uint32_t prp01, uint32_t prp23) {
+  return cost_rp(mode, prp01 & 0xFFFFu, prp01 >> 16, prp23 & 0xFFFFu, prp23 >> 16);
+}
+
+// Commit of instruction j at cycle t (both passes): scheduled / ready sets,
+// the RP update (R14, R15), last-use bookkeeping of the registers j reads,
+// and the successors that become ready (pass 2: with their ready times).
+template <int PASS, bool MASK, bool T32, bool NC4>
+__device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uint32_t t, uint32_t &wmask,
+                                       uint32_t &live01, uint32_t &live23, uint32_t &prp01,
+                                       uint32_t &prp23) {
+  {
+    const uint32_t wi = j >> 5, bit = 1u << (j & 31u);
+    const uint32_t nw = A.RB[wi * A.S] & ~bit;
+    A.RB[wi * A.S] = nw;
+    if (MASK && !nw) wmask &= ~(1u << wi);
+    A.SCH[wi * A.S] |= bit;
+  }
+  if (PASS == 2) t_set<T32>(A, j, t);
+  const uint4 inf = V.info[j];
+  uint32_t K = inf.y;  // static kills (single-use registers)
+  {
+    const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;
+    for (uint32_t q = 0; q < mc; ++q) {
+      const uint32_t e = V.muse[m0 + q];
+      const uint32_t c = (e >> 16) & 3u;
+      if (e & kMuseCounter) {  // >= 3 users: remaining-use counter
+        const uint32_t m = e & 0xFFFFu, sh = (m & 1u) * 16;
+        uint32_t *p = A.REM + (m >> 1) * A.S;
+        const uint32_t w = *p;
+        *p = w - (1u << sh);
+        const uint32_t left = (w >> sh) & 0xFFFFu;  // users left including j
+        if (left == 1u) {
+          K += 1u << (8 * c);  // j is the last user: the register dies here
+        } else if (left == 2u) {  // one user remains: it becomes the last user
+          for (uint32_t k = V.cu_ptr[m]; k < V.cu_ptr[m + 1]; ++k) {
+            const uint32_t u = V.cu[k];
+            if (!sch_bit(A, u)) {
+              dk_add<PASS, NC4>(A, u, c);
+              break;
+            }
+          }
+        }
+      } else {  // 2 users: the partner
+        const uint32_t p = e & 0x1FFFu;
+        if (sch_bit(A, p)) K += 1u << (8 * c);
+        else dk_add<PASS, NC4>(A, p, c);
+      }
+    }
+  }
+  live01 = __vsub2(live01, lo_pair(K));
+  live23 = __vsub2(live23, hi_pair(K));
+  live01 = __vadd2(live01, lo_pair(inf.x));
+  live23 = __vadd2(live23, hi_pair(inf.x));
+  prp01 = __vmaxu2(prp01, live01);
+  prp23 = __vmaxu2(prp23, live23);
+  live01 = __vsub2(live01, lo_pair(inf.z));
+  live23 = __vsub2(live23, hi_pair(inf.z));
+  const uint32_t s0 = V.succ_ptr[j], s1 = V.succ_ptr[j + 1];
+  for (uint32_t q = s0; q < s1; ++q) {
+    const uint32_t e = V.succ[q];
+    const uint32_t v = e & 0x1FFFu;
+    bool ready = true;
+    uint32_t rdy = t + (e >> 16);
+    if (!(e & kSuccSingle)) {
+      const uint32_t p0 = V.pred_ptr[v], p1 = V.pred_ptr[v + 1];
+      if (PASS == 2) rdy = 0;
+      for (uint32_t k = p0; k < p1; ++k) {
+        const uint32_t pe = V.pred[k];
+        const uint32_t p = pe & 0xFFFFu;
+        if (!sch_bit(A, p)) {
+          ready = false;
+          break;
+        }
+        if (PASS == 2) rdy = max(rdy, t_get<T32>(A, p) + (pe >> 16));
+      }
+    }
+    if (ready) {
+      A.RB[(v >> 5) * A.S] |= 1u << (v & 31u);
+      if (MASK) wmask |= 1u << (v >> 5);
+      if (PASS == 2) t_set<T32>(A, v, rdy);
+    }
+  }
+}
+
+template <int PASS, bool MASK, bool T32, bool NC4>
+__device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
+  uint32_t wmask = 0;
+  for (uint32_t w = 0; w < V.nwr; ++w) {
+    const uint32_t x = V.rb0[w];
+    A.RB[w * A.S] = x;
+    A.SCH[w * A.S] = 0;
+    if (MASK && x) wmask |= 1u << w;
+  }
+  for (uint32_t w = 0; w < V.nremw; ++w) A.REM[w * A.S] = V.rem0[w];
+  const uint32_t n = V.n;
+  const uint32_t tw = PASS == 1 ? 0 : (T32 ? n : (n + 1) / 2);
+  const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (NC4 ? (n + 1) / 2 : (n + 3) / 4);
+  for (uint32_t w = 0; w < tw + dw; ++w) A.T[w * A.S] = 0;  // T and DK are contiguous
+  return wmask;
+}
 
 // ------------------------------------------------------------ pass-1 ant
 // RP pass (L108, L145; R19): latencies ignored, candidates = ready list,
-// eta1 = LUC-then-CP (R4), score tau[prev][j] * eta1 (R1).  One step per
-// instruction; the step index k is the Philox step (R26).
-template <bool MASK, bool REC>
-__device__ __forceinline__ AntOut ant_pass1(const RV &R, const uint16_t *__restrict__ tau,
-                                            uint32_t *st, const uint32_t S, const uint32_t ant,
-                                            const uint32_t iter, const RunCfg &cfg, const bool greedy,
-                                            uint16_t *rec) {
-  const uint32_t n = R.n, nwr = R.nwr;
-  uint32_t *RB = st;
-  uint32_t *CNT = st + nwr * S;
-  uint32_t *REM = CNT + ((n + 3) >> 2) * S;
-  uint32_t wmask = 0;
-  for (uint32_t w = 0; w < nwr; ++w) {
-    const uint32_t x = __ldg(R.rb0 + w);
-    RB[w * S] = x;
-    if (MASK && x) wmask |= 1u << w;
-  }
-  for (uint32_t w = 0; w < ((n + 3) >> 2); ++w) CNT[w * S] = __ldg(R.cnt0 + w);
-  for (uint32_t w = 0; w < ((R.nmu + 1) >> 1); ++w) REM[w * S] = __ldg(R.rem0 + w);
-  uint32_t live[4], prp[4];
-#pragma unroll
-  for (int c = 0; c < 4; ++c) live[c] = prp[c] = R.livein[c];
+// score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
+// Philox step (R26).  rec (may be NULL) receives the order.
+template <bool MASK>
+__device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
+                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
+                                            const bool greedy, uint16_t *rec) {
+  const uint32_t n = V.n, nwr = V.nwr;
+  uint32_t wmask = init_state<1, MASK, false, false>(V, A);
+  uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   uint32_t prev = n;
   for (uint32_t k = 0; k < n; ++k) {
     bool exploit = greedy;
     if (!greedy) {
-      const uint4 g = philox(k, 0x80000000u | group, iter, R.region_id, cfg.seed);
+      const uint4 g = philox(k, 0x80000000u | group, iter, V.region_id, cfg.seed);
       exploit = (uint64_t)g.x < cfg.q0_t;
     }
-    const uint16_t *trow = tau + (size_t)prev * n;
+    const uint16_t *trow = tau + prev * n;
     uint32_t best_s = 0, best_j = 0;
     uint64_t sum = 0;
-#define ACO_SCORE1(J, OUT)                                                   \
-  uint32_t OUT;                                                              \
-  {                                                                          \
-    const uint4 inf = __ldg(R.info + J);                                     \
-    uint32_t luc = byte_sum(inf.z);                                          \
-    const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;                      \
-    for (uint32_t q = 0; q < mc; ++q) {                                      \
-      const uint32_t mm = __ldg(R.muse + m0 + q) & 0xFFFFu;                  \
-      luc += rem_get(REM, S, mm) == 1u;                                      \
-    }                                                                        \
-    OUT = (uint32_t)__ldg(trow + J) * (uint32_t)__ldg(R.eta1 + J * R.Lp1 + luc); \
-  }
-    ACO_FOR_EACH_BIT(MASK, wmask, RB, S, nwr, j, {
-      ACO_SCORE1(j, s)
-      if (exploit) {
-        if (s > best_s) {
-          best_s = s;
-          best_j = j;
-        }
-      } else {
-        sum += s;
+    BitIt it;
+    it_init<MASK>(it, wmask);
+    for (;;) {
+      uint32_t j[4];
+      const uint32_t cnt = it_next4<MASK>(it, A, nwr, j);
+      if (!cnt) break;
+      uint32_t s[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {  // independent loads of four candidates
+        const uint32_t e1 = V.e1b[j[q]] + dk1_get(A, j[q]);
+        s[q] = (uint32_t)trow[j[q]] * (uint32_t)V.eta1[e1];
       }
-    })
-    if (!exploit) {
-      const uint4 x = philox(k, ant, iter, R.region_id, cfg.seed);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t sq = (uint32_t)q < cnt ? s[q] : 0u;
+        if (sq > best_s) {  // argmax, ties to the lowest index (ascending order)
+          best_s = sq;
+          best_j = j[q];
+        }
+        sum += sq;
+      }
+      if (cnt < 4) break;
+    }
+    if (!exploit) {  // roulette (R27)
+      const uint4 x = philox(k, ant, iter, V.region_id, cfg.seed);
       const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
       uint64_t pre = 0;
-      ACO_FOR_EACH_BIT(MASK, wmask, RB, S, nwr, j, {
-        ACO_SCORE1(j, s)
-        pre += s;
+      it_init<MASK>(it, wmask);
+      uint32_t j;
+      while (it_next<MASK>(it, A, nwr, j)) {
+        pre += (uint32_t)trow[j] * (uint32_t)V.eta1[V.e1b[j] + dk1_get(A, j)];
         if (pre > r) {
           best_j = j;
-          ACO_BREAK_SCAN
-        }
-      })
-    }
-#undef ACO_SCORE1
-    // ---- commit best_j: RP update (R14, R15), successors, order
-    const uint32_t j = best_j;
-    {
-      const uint32_t wi = j >> 5;
-      const uint32_t nw = RB[wi * S] & ~(1u << (j & 31u));
-      RB[wi * S] = nw;
-      if (MASK && !nw) wmask &= ~(1u << wi);
-    }
-    const uint4 inf = __ldg(R.info + j);
-#pragma unroll
-    for (int c = 0; c < 4; ++c) live[c] -= byte_of(inf.z, c);
-    {
-      const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;
-      for (uint32_t q = 0; q < mc; ++q) {
-        const uint32_t e = __ldg(R.muse + m0 + q);
-        const uint32_t mm = e & 0xFFFFu, cls = e >> 16;
-        const uint32_t sh = (mm & 1u) * 16;
-        const uint32_t word = REM[(mm >> 1) * S];
-        REM[(mm >> 1) * S] = word - (1u << sh);
-        if (((word >> sh) & 0xFFFFu) == 1u) {
-#pragma unroll
-          for (int c = 0; c < 4; ++c) live[c] -= (cls == (uint32_t)c);
+          break;
         }
       }
     }
-#pragma unroll
-    for (int c = 0; c < 4; ++c) {
-      live[c] += byte_of(inf.x, c);
-      prp[c] = max(prp[c], live[c]);
-      live[c] -= byte_of(inf.y, c);
-    }
-    {
-      const uint32_t s0 = __ldg(R.succ_ptr + j), s1 = __ldg(R.succ_ptr + j + 1);
-      for (uint32_t q = s0; q < s1; ++q) {
-        const uint32_t v = __ldg(R.succ + q) & 0xFFFFu;
-        const uint32_t sh = (v & 3u) * 8;
-        const uint32_t word = CNT[(v >> 2) * S] - (1u << sh);
-        CNT[(v >> 2) * S] = word;
-        if (((word >> sh) & 0xFFu) == 0u) {
-          RB[(v >> 5) * S] |= 1u << (v & 31u);
-          if (MASK) wmask |= 1u << (v >> 5);
-        }
-      }
-    }
-    if (REC) rec[k] = (uint16_t)j;
-    prev = j;
+    commit<1, MASK, false, false>(V, A, best_j, 0, wmask, live01, live23, prp01, prp23);
+    if (rec) rec[k] = (uint16_t)best_j;
+    prev = best_j;
   }
   AntOut o;
-#pragma unroll
-  for (int c = 0; c < 4; ++c) o.prp[c] = prp[c];
-  o.cost = cost_rp(cfg.cost_mode, prp);
+  o.prp01 = prp01;
+  o.prp23 = prp23;
+  o.cost = cost_of(cfg.cost_mode, prp01, prp23);
   return o;
 }
 
 // ------------------------------------------------------------ pass-2 ant
 // ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle and
-// the Philox step; stalls skip ahead without drawing.
-template <bool MASK, bool REC>
-__device__ __forceinline__ AntOut ant_pass2(const RV &R, const uint16_t *__restrict__ tau,
-                                            uint32_t *st, const uint32_t S, const uint32_t ant,
-                                            const uint32_t iter, const RunCfg &cfg,
+// the Philox step; stalls skip ahead without drawing.  rec_o / rec_c (may be
+// NULL) receive the order and the cycles.
+template <bool MASK, bool T32, bool NC4>
+__device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restrict__ tau, const St &A,
+                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
                                             const uint32_t tgt[4], uint32_t *prune_len, const bool prune,
                                             uint16_t *rec_o, uint32_t *rec_c) {
-  const uint32_t n = R.n, nwr = R.nwr;
-  uint32_t *RB = st;             // avail bitset: all preds placed, not placed
-  uint32_t *RC = st + nwr * S;   // per instruction: ready time << 8 | preds left
-  uint32_t *REM = RC + n * S;
-  uint32_t wmask = 0;
-  for (uint32_t w = 0; w < nwr; ++w) {
-    const uint32_t x = __ldg(R.rb0 + w);
-    RB[w * S] = x;
-    if (MASK && x) wmask |= 1u << w;
-  }
-  for (uint32_t w = 0; w < ((n + 3) >> 2); ++w) {
-    const uint32_t x = __ldg(R.cnt0 + w);
-#pragma unroll
-    for (uint32_t b = 0; b < 4; ++b)
-      if (w * 4 + b < n) RC[(w * 4 + b) * S] = byte_of(x, b);
-  }
-  for (uint32_t w = 0; w < ((R.nmu + 1) >> 1); ++w) REM[w * S] = __ldg(R.rem0 + w);
-  uint32_t live[4], prp[4];
-#pragma unroll
-  for (int c = 0; c < 4; ++c) live[c] = prp[c] = R.livein[c];
+  const uint32_t n = V.n, nwr = V.nwr;
+  uint32_t wmask = init_state<2, MASK, T32, NC4>(V, A);
+  uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const bool stall_en = (group % cfg.stall_mod) == cfg.stall_rem;  // R23
   const uint32_t c2 = 0x80000000u | iter;
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0;
   AntOut o;
+  o.prp01 = o.prp23 = 0;
   while (placed < n) {
     if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune
       const uint32_t bl = *(volatile uint32_t *)prune_len;
@@ -338,64 +456,57 @@ __device__ __forceinline__ AntOut ant_pass2(const RV &R, const uint16_t *__restr
         return o;
       }
     }
-    const uint16_t *trow = tau + (size_t)prev * n;
+    // slack_c = target_c - live_c, saturated to a byte (R21); live <= target always
+    uint32_t slack = 0;
+    {
+      const uint32_t lv[4] = {live01 & 0xFFFFu, live01 >> 16, live23 & 0xFFFFu, live23 >> 16};
+#pragma unroll
+      for (int c = 0; c < 4; ++c) slack |= min(tgt[c] - lv[c], 255u) << (8 * c);
+    }
+    const uint16_t *trow = tau + prev * n;
     uint32_t nr = 0, nf = 0, ns = 0, min_s = 0xFFFFFFFFu;
     bool all_f_inc = true, some_s_dec = false;
     uint32_t best_s = 0, best_j = 0;
     uint64_t sum = 0;
-    // Delta_c(j) = defs_c - kills_c at the current state; feasible iff
-    // live_c + Delta_c <= target_c for every class (R21).
-#define ACO_DELTA(J, D)                                                       \
-  int D[4];                                                                   \
-  {                                                                           \
-    const uint4 inf = __ldg(R.info + J);                                      \
-    _Pragma("unroll") for (int c = 0; c < 4; ++c) D[c] =                      \
-        (int)byte_of(inf.x, c) - (int)byte_of(inf.z, c);                      \
-    const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;                       \
-    for (uint32_t q = 0; q < mc; ++q) {                                       \
-      const uint32_t e = __ldg(R.muse + m0 + q);                              \
-      if (rem_get(REM, S, e & 0xFFFFu) == 1u) {                               \
-        const uint32_t cls = e >> 16;                                         \
-        _Pragma("unroll") for (int c = 0; c < 4; ++c) D[c] -= (cls == (uint32_t)c); \
-      }                                                                       \
-    }                                                                         \
-  }
-#define ACO_FEASIBLE(D, OK)                                                   \
-  bool OK = true;                                                             \
-  _Pragma("unroll") for (int c = 0; c < 4; ++c) OK =                          \
-      OK && ((uint32_t)((int)live[c] + D[c]) <= tgt[c]);
-    ACO_FOR_EACH_BIT(MASK, wmask, RB, S, nwr, j, {
-      const uint32_t rdy = RC[j * S] >> 8;
-      if (rdy <= t) {
-        ++nr;
-        ACO_DELTA(j, d)
-        ACO_FEASIBLE(d, ok)
-        if (ok) {
-          ++nf;
-          const uint32_t s = (uint32_t)__ldg(trow + j) * (uint32_t)__ldg(R.eta2 + j);
-          if (s > best_s) {
-            best_s = s;
-            best_j = j;
+    BitIt it;
+    it_init<MASK>(it, wmask);
+    for (;;) {
+      uint32_t j[4];
+      const uint32_t cnt = it_next4<MASK>(it, A, nwr, j);
+      if (!cnt) break;
+      uint32_t rdy[4], K[4], D[4], s[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {  // independent loads of four candidates
+        rdy[q] = t_get<T32>(A, j[q]);
+        const uint2 ds = V.ds[j[q]];
+        D[q] = ds.x;
+        K[q] = ds.y + dk2_get<NC4>(A, j[q]);  // kills per class (R14)
+        s[q] = (uint32_t)trow[j[q]] * (uint32_t)V.eta2[j[q]];
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if ((uint32_t)q >= cnt) break;
+        if (rdy[q] <= t) {
+          ++nr;
+          // feasible (R21): defs_c <= slack_c + kills_c for every class
+          if (__vcmpgtu4(D[q], __vaddus4(slack, K[q])) == 0u) {
+            ++nf;
+            if (__vcmpgtu4(D[q], K[q]) == 0u) all_f_inc = false;  // max_c Delta_c <= 0
+            if (s[q] > best_s) {
+              best_s = s[q];
+              best_j = j[q];
+            }
+            sum += s[q];
           }
-          sum += s;
-          if (stall_en) {
-            int mx = d[0];
-            _Pragma("unroll") for (int c = 1; c < 4; ++c) mx = max(mx, d[c]);
-            if (!(mx > 0)) all_f_inc = false;
-          }
-        }
-      } else {
-        ++ns;
-        min_s = min(min_s, rdy);
-        if (stall_en && !some_s_dec) {
-          ACO_DELTA(j, d)
-          int mn = d[0];
-          _Pragma("unroll") for (int c = 1; c < 4; ++c) mn = min(mn, d[c]);
-          if (mn < 0) some_s_dec = true;
+        } else {
+          ++ns;
+          min_s = min(min_s, rdy[q]);
+          if (__vcmpltu4(D[q], K[q]) != 0u) some_s_dec = true;  // min_c Delta_c < 0
         }
       }
-    })
-    if (nr == 0) {  // necessary stall (L153): skip ahead
+      if (cnt < 4) break;
+    }
+    if (nr == 0) {  // necessary stall (L153): skip ahead to the next ready time
       t = min_s;
       continue;
     }
@@ -411,7 +522,7 @@ __device__ __forceinline__ AntOut ant_pass2(const RV &R, const uint16_t *__restr
     uint4 x = make_uint4(0, 0, 0, 0);
     bool have_x = false;
     if (stall_en && ns > 0 && all_f_inc && some_s_dec) {  // discretionary stall (L157-L164)
-      x = philox(t, ant, c2, R.region_id, cfg.seed);
+      x = philox(t, ant, c2, V.region_id, cfg.seed);
       have_x = true;
       const uint32_t thr = (kopt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (kopt + 1));
       if (x.z < thr) {
@@ -420,84 +531,36 @@ __device__ __forceinline__ AntOut ant_pass2(const RV &R, const uint16_t *__restr
         continue;
       }
     }
-    const uint4 g = philox(t, 0x80000000u | group, c2, R.region_id, cfg.seed);
+    const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
     if (!((uint64_t)g.x < cfg.q0_t)) {  // explore: roulette over F (R27)
-      if (!have_x) x = philox(t, ant, c2, R.region_id, cfg.seed);
+      if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
       const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
       uint64_t pre = 0;
-      ACO_FOR_EACH_BIT(MASK, wmask, RB, S, nwr, j, {
-        if ((RC[j * S] >> 8) <= t) {
-          ACO_DELTA(j, d)
-          ACO_FEASIBLE(d, ok)
-          if (ok) {
-            pre += (uint32_t)__ldg(trow + j) * (uint32_t)__ldg(R.eta2 + j);
-            if (pre > r) {
-              best_j = j;
-              ACO_BREAK_SCAN
-            }
-          }
-        }
-      })
-    }
-#undef ACO_DELTA
-#undef ACO_FEASIBLE
-    // ---- commit best_j at cycle t
-    const uint32_t j = best_j;
-    {
-      const uint32_t wi = j >> 5;
-      const uint32_t nw = RB[wi * S] & ~(1u << (j & 31u));
-      RB[wi * S] = nw;
-      if (MASK && !nw) wmask &= ~(1u << wi);
-    }
-    const uint4 inf = __ldg(R.info + j);
-#pragma unroll
-    for (int c = 0; c < 4; ++c) live[c] -= byte_of(inf.z, c);
-    {
-      const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;
-      for (uint32_t q = 0; q < mc; ++q) {
-        const uint32_t e = __ldg(R.muse + m0 + q);
-        const uint32_t mm = e & 0xFFFFu, cls = e >> 16;
-        const uint32_t sh = (mm & 1u) * 16;
-        const uint32_t word = REM[(mm >> 1) * S];
-        REM[(mm >> 1) * S] = word - (1u << sh);
-        if (((word >> sh) & 0xFFFFu) == 1u) {
-#pragma unroll
-          for (int c = 0; c < 4; ++c) live[c] -= (cls == (uint32_t)c);
+      it_init<MASK>(it, wmask);
+      uint32_t j;
+      while (it_next<MASK>(it, A, nwr, j)) {
+        if (t_get<T32>(A, j) > t) continue;
+        const uint2 ds = V.ds[j];
+        if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk2_get<NC4>(A, j))) != 0u) continue;
+        pre += (uint32_t)trow[j] * (uint32_t)V.eta2[j];
+        if (pre > r) {
+          best_j = j;
+          break;
         }
       }
     }
-#pragma unroll
-    for (int c = 0; c < 4; ++c) {
-      live[c] += byte_of(inf.x, c);
-      prp[c] = max(prp[c], live[c]);
-      live[c] -= byte_of(inf.y, c);
-    }
-    {
-      const uint32_t s0 = __ldg(R.succ_ptr + j), s1 = __ldg(R.succ_ptr + j + 1);
-      for (uint32_t q = s0; q < s1; ++q) {
-        const uint32_t e = __ldg(R.succ + q);
-        const uint32_t v = e & 0xFFFFu, lat = e >> 16;
-        const uint32_t w = RC[v * S];
-        const uint32_t rdy = max(w >> 8, t + lat);
-        const uint32_t cnt = (w & 0xFFu) - 1u;
-        RC[v * S] = (rdy << 8) | cnt;
-        if (cnt == 0u) {
-          RB[(v >> 5) * S] |= 1u << (v & 31u);
-          if (MASK) wmask |= 1u << (v >> 5);
-        }
-      }
-    }
-    if (REC) {
-      rec_o[placed] = (uint16_t)j;
+    commit<2, MASK, T32, NC4>(V, A, best_j, t, wmask, live01, live23, prp01, prp23);
+    if (rec_o) {
+      rec_o[placed] = (uint16_t)best_j;
       rec_c[placed] = t;
     }
     ++placed;
-    prev = j;
+    prev = best_j;
     ++t;
   }
   if (prune) atomicMin(prune_len, t);
-#pragma unroll
-  for (int c = 0; c < 4; ++c) o.prp[c] = prp[c];
+  o.prp01 = prp01;
+  o.prp23 = prp23;
   o.cost = t;  // length = last issue cycle + 1 (R20)
   return o;
 }
@@ -515,51 +578,64 @@ struct KArgs {
   RunCfg cfg;
 };
 
-template <int PASS, bool MASK, bool DUMP>
+// Stage the region's block image (and tau) into shared memory.
+__device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t bytes) {
+  for (uint32_t i = threadIdx.x; i < bytes / 16; i += blockDim.x) dst[i] = src[i];
+}
+
+template <int PASS, bool MASK, bool TAU_SMEM, bool T32, bool NC4>
 __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__restrict__ items,
                                                    uint32_t iter) {
-  const BlockItem it = items[blockIdx.x];
-  RegionState &rs = A.state[it.region];
-  if (!rs.active) return;
-  const uint32_t ant = it.ant0 + threadIdx.x;
+  const BlockItem bi = items[blockIdx.x];
+  RegionState &rs = A.state[bi.region];
+  if (!rs.active) return;  // block-uniform
+  const RegionDev *rd = A.regions + bi.region;
+  const RegionWs &W = A.rws[bi.region];
+  extern __shared__ uint4 smem4[];
+  unsigned char *smem = (unsigned char *)smem4;
+  const uint32_t img_bytes = rd->img.bytes;
+  stage(smem4, (const uint4 *)(A.arena + rd->o_image), img_bytes);
+  const uint16_t *tau;
+  uint32_t state_off = img_bytes;
+  if (TAU_SMEM) {
+    const uint32_t tb = tau_smem_bytes(rd->n);
+    stage((uint4 *)(smem + img_bytes), (const uint4 *)(A.ws + W.o_tau), tb);
+    tau = (const uint16_t *)(smem + img_bytes);
+    state_off += tb;
+  } else {
+    tau = (const uint16_t *)(A.ws + W.o_tau);
+  }
+  __syncthreads();
+  const uint32_t ant = bi.ant0 + threadIdx.x;
   if (ant >= A.cfg.ants) return;
-  const RV R = make_rv(A.arena, A.regions + it.region);
-  const RegionWs &W = A.rws[it.region];
-  const uint16_t *tau = (const uint16_t *)(A.ws + W.o_tau);
-  extern __shared__ uint32_t smem[];
-  uint32_t *st = smem + threadIdx.x;
-  const uint32_t S = blockDim.x;
+  const SV V = make_sv(smem, rd);
+  const St S = make_st<PASS, T32, NC4>((uint32_t *)(smem + state_off) + threadIdx.x, blockDim.x, V);
+  const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
   if (PASS == 1) {
     uint16_t *rec = nullptr;
-    if (DUMP && A.dump_order)
-      rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ant * R.n;
-    o = ant_pass1<MASK, DUMP>(R, tau, st, S, ant, iter, A.cfg, false, rec);
+    if (dump && A.dump_order)
+      rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ant * V.n;
+    o = ant_pass1<MASK>(V, tau, S, ant, iter, A.cfg, false, rec);
   } else {
     uint32_t tgt[4];
 #pragma unroll
     for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
+    const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE);
     uint16_t *rec_o = nullptr;
     uint32_t *rec_c = nullptr;
-    uint16_t scratch_o[1];
-    uint32_t scratch_c[1];
-    if (DUMP) {
-      const size_t base = ((size_t)A.cfg.iterations + iter) * A.cfg.dump_slice + W.o_dump + (size_t)ant * R.n;
-      rec_o = A.dump_order ? A.dump_order + base : scratch_o;
-      rec_c = A.dump_cycle ? A.dump_cycle + base : scratch_c;
-      if (!A.dump_order || !A.dump_cycle) rec_o = nullptr;
+    if (dump && A.dump_order && A.dump_cycle) {
+      const size_t base =
+          ((size_t)A.cfg.iterations + iter) * A.cfg.dump_slice + W.o_dump + (size_t)ant * V.n;
+      rec_o = A.dump_order + base;
+      rec_c = A.dump_cycle + base;
     }
-    const bool prune = !DUMP && !(A.cfg.flags & ACO_FLAG_NO_PRUNE);
-    if (DUMP && rec_o)
-      o = ant_pass2<MASK, true>(R, tau, st, S, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c);
-    else
-      o = ant_pass2<MASK, false>(R, tau, st, S, ant, iter, A.cfg, tgt, &rs.prune_len, prune, nullptr,
-                                 nullptr);
+    o = ant_pass2<MASK, T32, NC4>(V, tau, S, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c);
   }
   uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
   costs[ant] = o.cost;
-  if (DUMP && A.dump_cost)
-    A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + it.region) * A.cfg.ants + ant] =
+  if (dump && A.dump_cost)
+    A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants + ant] =
         o.cost;
 }
 
@@ -585,27 +661,34 @@ __device__ void tau_fill(uint16_t *tau, uint32_t len, uint32_t tau0) {
   for (uint32_t i = threadIdx.x; i < len / 8; i += blockDim.x) t4[i] = q;
 }
 
-// Evaporate + deposit + clamp over the (n+1) x n table (R6-R9), 8 entries
-// per 16-byte access; next[i] = the winner's successor of i (0xFFFF: none).
-__device__ void tau_update(uint16_t *tau, uint32_t n, uint32_t len, const uint16_t *next,
-                           const RunCfg &cfg) {
+// Evaporate + deposit + clamp (R6-R9) over all active regions' tables, 8
+// entries per 16-byte access.  One block = kUpdVec vectors of one region;
+// next[i] = the winner's successor of row i (0xFFFF: no deposit).
+__global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restrict__ items) {
+  const UpdItem it = items[blockIdx.x];
+  if (!A.state[it.region].active) return;  // the pass ended: tau is not used again
+  const RegionDev *rd = A.regions + it.region;
+  const RegionWs &W = A.rws[it.region];
+  const uint32_t n = rd->n;
   const uint32_t total = (n + 1) * n;
-  uint4 *t4 = (uint4 *)tau;
-  for (uint32_t v = threadIdx.x; v < len / 8; v += blockDim.x) {
-    uint4 q = t4[v];
+  const uint16_t *next = (const uint16_t *)(A.ws + W.o_next);
+  uint4 *t4 = (uint4 *)(A.ws + W.o_tau);
+  const uint32_t vend = min(it.v0 + kUpdVec, W.tau_len / 8);
+  const uint32_t rho = A.cfg.rho_q16, dl = A.cfg.delta, lo = A.cfg.tau_min, hi = A.cfg.tau_max;
+  for (uint32_t v = it.v0 + threadIdx.x; v < vend; v += blockDim.x) {
+    const uint4 q = t4[v];
     uint32_t w[4] = {q.x, q.y, q.z, q.w};
     const uint32_t e0 = v * 8;
     uint32_t i = e0 / n, j = e0 - i * n;
     uint32_t nx = i <= n ? next[i] : 0xFFFFu;
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
-      const uint32_t e = e0 + u;
-      if (e < total) {
+      if (e0 + u < total) {
         const uint32_t sh = (u & 1) * 16;
         uint32_t x = (w[u >> 1] >> sh) & 0xFFFFu;
-        x = (x * cfg.rho_q16) >> 16;
-        if (nx == j) x += cfg.delta;
-        x = min(max(x, cfg.tau_min), cfg.tau_max);
+        x = (x * rho) >> 16;
+        if (nx == j) x += dl;
+        x = min(max(x, lo), hi);
         w[u >> 1] = (w[u >> 1] & ~(0xFFFFu << sh)) | (x << sh);
         if (++j == n) {
           j = 0;
@@ -623,28 +706,29 @@ __device__ void tau_update(uint16_t *tau, uint32_t n, uint32_t len, const uint16
 template <bool MASK>
 __global__ void __launch_bounds__(128) k_init(KArgs A) {
   const uint32_t r = blockIdx.x;
-  const RV R = make_rv(A.arena, A.regions + r);
+  const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
   RegionState &rs = A.state[r];
   uint16_t *tau = (uint16_t *)(A.ws + W.o_tau);
-  extern __shared__ uint32_t smem[];
+  extern __shared__ uint4 smem4[];
+  unsigned char *smem = (unsigned char *)smem4;
+  stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   __syncthreads();
   if (threadIdx.x == 0) {
+    const SV V = make_sv(smem, rd);
+    const St S = make_st<1, false, false>((uint32_t *)(smem + rd->img.bytes), 1, V);
     uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
-    AntOut o = ant_pass1<MASK, true>(R, tau, smem, 1, 0, 0, A.cfg, true, gb1);
-    const RegionDev *rd = A.regions + r;
-    uint32_t lbv[4];
-    for (int c = 0; c < 4; ++c) lbv[c] = rd->lbvec[c];
-    rs.lb_cost = cost_rp(A.cfg.cost_mode, lbv);
+    AntOut o = ant_pass1<MASK>(V, tau, S, 0, 0, A.cfg, true, gb1);
+    rs.lb_cost = cost_rp(A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
     rs.init[0] = rs.best[0] = o.cost;
-    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = o.prp[c];
+    const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
+    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = prp[c];
     rs.iters[0] = rs.iters[1] = 0;
     rs.no_imp = 0;
     rs.prune_len = kInvalid;
     rs.hash = 0xcbf29ce484222325ull;
-    rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 &&
-                !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
+    rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
   }
 }
 
@@ -652,34 +736,33 @@ __global__ void __launch_bounds__(128) k_init(KArgs A) {
 // initial pass-2 schedule = ASAP(pass-1 best order), tau reset.
 __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
   const uint32_t r = blockIdx.x;
-  const RV R = make_rv(A.arena, A.regions + r);
+  const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
   RegionState &rs = A.state[r];
   uint16_t *tau = (uint16_t *)(A.ws + W.o_tau);
-  extern __shared__ uint32_t smem[];  // rdy[n]
+  extern __shared__ uint32_t rdyv[];  // rdy[n]
+  const uint32_t n = rd->n;
   tau_fill(tau, W.tau_len, A.cfg.tau0);
-  for (uint32_t i = threadIdx.x; i < R.n; i += blockDim.x) smem[i] = 0;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) rdyv[i] = 0;
   __syncthreads();
   if (threadIdx.x == 0) {
+    const SV V = make_sv(A.arena + rd->o_image, rd);
     const uint16_t *gb1 = (const uint16_t *)(A.ws + W.o_gb1);
     uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
     uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
     uint32_t t = 0;
-    bool first = true;
-    for (uint32_t k = 0; k < R.n; ++k) {
+    for (uint32_t k = 0; k < n; ++k) {
       const uint32_t j = gb1[k];
-      t = first ? smem[j] : max(t + 1, smem[j]);
-      first = false;
+      t = k == 0 ? rdyv[j] : max(t + 1, rdyv[j]);
       gb2[k] = (uint16_t)j;
       gb2c[k] = t;
-      const uint32_t s0 = __ldg(R.succ_ptr + j), s1 = __ldg(R.succ_ptr + j + 1);
-      for (uint32_t q = s0; q < s1; ++q) {
-        const uint32_t e = __ldg(R.succ + q);
-        const uint32_t v = e & 0xFFFFu;
-        smem[v] = max(smem[v], t + (e >> 16));
+      for (uint32_t q = V.succ_ptr[j]; q < V.succ_ptr[j + 1]; ++q) {
+        const uint32_t e = V.succ[q];
+        const uint32_t v = e & 0x1FFFu;
+        rdyv[v] = max(rdyv[v], t + (e >> 16));
       }
     }
-    const uint32_t len = R.n ? t + 1 : 0;
+    const uint32_t len = n ? t + 1 : 0;
     rs.init[1] = rs.best[1] = len;
     for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.prp1[c];
     uint32_t tgt[4];
@@ -687,68 +770,61 @@ __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
     for (int c = 0; c < 4; ++c) rs.target[c] = tgt[c];
     rs.no_imp = 0;
     rs.prune_len = kInvalid;
-    const uint32_t lb_len = A.regions[r].lb_len;
-    rs.active = (A.cfg.pass_mask & 2u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && len == lb_len);
+    rs.active = (A.cfg.pass_mask & 2u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && len == rd->lb_len);
   }
 }
 
-// End of an iteration for one region (L137-L139).
-template <int PASS, bool MASK>
-__global__ void __launch_bounds__(256) k_finalize(KArgs A, uint32_t iter) {
+// End of an iteration for one region (L137-L139), one warp: argmin over
+// (cost, ant) (R10), replay of the winner (lane 0) to recover its order,
+// the winner's successor table for the pheromone update, and the epilogue.
+template <int PASS, bool MASK, bool T32, bool NC4>
+__global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   const uint32_t r = blockIdx.x;
   RegionState &rs = A.state[r];
   if (!rs.active) return;
-  const RV R = make_rv(A.arena, A.regions + r);
+  const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
-  const uint32_t n = R.n;
-  uint16_t *tau = (uint16_t *)(A.ws + W.o_tau);
+  const uint32_t n = rd->n;
+  const uint16_t *tau = (const uint16_t *)(A.ws + W.o_tau);
   const uint32_t *costs = (const uint32_t *)(A.ws + W.o_cost);
-  extern __shared__ uint32_t smem[];
-  __shared__ unsigned long long s_red[8];
-  __shared__ uint32_t s_flag;
-  // ---- argmin over (cost, ant) (R10): packed u64 keys, warp shuffles
+  extern __shared__ uint4 smem4[];
+  unsigned char *smem = (unsigned char *)smem4;
+  __shared__ uint32_t s_prp[2], s_flag;
+  stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
   unsigned long long best = ~0ull;
-  for (uint32_t a = threadIdx.x; a < A.cfg.ants; a += blockDim.x)
+  for (uint32_t a = threadIdx.x; a < A.cfg.ants; a += 32)
     best = min(best, ((unsigned long long)costs[a] << 32) | a);
 #pragma unroll
   for (int off = 16; off; off >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, off));
-  if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = best;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    for (uint32_t w = 1; w < blockDim.x / 32; ++w) best = min(best, s_red[w]);
-    s_red[0] = best;
-  }
-  __syncthreads();
-  best = s_red[0];
   const uint32_t wcost = (uint32_t)(best >> 32), want = (uint32_t)best;
   const bool have = wcost != kInvalid;
-  // smem: [ant state | order u16[n] | cycle u32[n] | next u16[n+1]]
-  const uint32_t words = ant_words(PASS, n, R.nwr, R.nmu);
-  uint32_t *cyc = smem + words;
+  // smem: [image | ant state | cycle u32[n] | order u16[n]]
+  const SV V = make_sv(smem, rd);
+  uint32_t *stw = (uint32_t *)(smem + rd->img.bytes);
+  uint32_t *cyc = stw + ant_words(PASS, n, rd->nwr, rd->nremw, T32, NC4);
   uint16_t *ord = (uint16_t *)(cyc + n);
-  uint16_t *next = ord + ((n + 1) & ~1u);
-  // ---- replay the winner (deterministic: same tau, same Philox counters)
+  __syncwarp();
   if (have && threadIdx.x == 0) {
+    const St S = make_st<PASS, T32, NC4>(stw, 1, V);
     AntOut o;
     if (PASS == 1) {
-      o = ant_pass1<MASK, true>(R, tau, smem, 1, want, iter, A.cfg, false, ord);
+      o = ant_pass1<MASK>(V, tau, S, want, iter, A.cfg, false, ord);
     } else {
       uint32_t tgt[4];
       for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
-      o = ant_pass2<MASK, true>(R, tau, smem, 1, want, iter, A.cfg, tgt, nullptr, false, ord, cyc);
+      o = ant_pass2<MASK, T32, NC4>(V, tau, S, want, iter, A.cfg, tgt, nullptr, false, ord, cyc);
     }
-    s_red[1] = o.prp[0] | ((unsigned long long)o.prp[1] << 32);
-    s_red[2] = o.prp[2] | ((unsigned long long)o.prp[3] << 32);
+    s_prp[0] = o.prp01;
+    s_prp[1] = o.prp23;
   }
-  __syncthreads();
-  for (uint32_t i = threadIdx.x; i <= n; i += blockDim.x) next[i] = 0xFFFFu;
-  __syncthreads();
+  __syncwarp();
+  uint16_t *next = (uint16_t *)(A.ws + W.o_next);
+  for (uint32_t i = threadIdx.x; i <= n; i += 32) next[i] = 0xFFFFu;
+  __syncwarp();
   if (have) {
-    for (uint32_t k = threadIdx.x; k + 1 < n; k += blockDim.x) next[ord[k]] = ord[k + 1];
+    for (uint32_t k = threadIdx.x; k + 1 < n; k += 32) next[ord[k]] = ord[k + 1];
     if (threadIdx.x == 0 && n) next[n] = ord[0];
   }
-  __syncthreads();
-  if (n) tau_update(tau, n, W.tau_len, next, A.cfg);
   // ---- epilogue (first thread, L139)
   if (threadIdx.x == 0) {
     rs.hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(rs.hash, PASS), iter), have ? wcost : kInvalid),
@@ -759,35 +835,44 @@ __global__ void __launch_bounds__(256) k_finalize(KArgs A, uint32_t iter) {
       rs.best[PASS - 1] = wcost;
       rs.no_imp = 0;
       uint32_t *prp = PASS == 1 ? rs.prp1 : rs.prp2;
-      prp[0] = (uint32_t)s_red[1];
-      prp[1] = (uint32_t)(s_red[1] >> 32);
-      prp[2] = (uint32_t)s_red[2];
-      prp[3] = (uint32_t)(s_red[2] >> 32);
+      prp[0] = s_prp[0] & 0xFFFFu;
+      prp[1] = s_prp[0] >> 16;
+      prp[2] = s_prp[1] & 0xFFFFu;
+      prp[3] = s_prp[1] >> 16;
     } else {
       rs.no_imp++;
     }
     rs.iters[PASS - 1] = iter + 1;
-    const uint32_t lim = no_improve_limit(A.cfg, n);
-    const uint32_t lb = PASS == 1 ? rs.lb_cost : A.regions[r].lb_len;
-    if ((A.cfg.stop_at_lb && rs.best[PASS - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
-        iter + 1 >= A.cfg.iterations)
-      rs.active = 0;
     rs.prune_len = kInvalid;
   }
-  __syncthreads();
+  __syncwarp();
   if (s_flag) {
     if (PASS == 1) {
       uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
-      for (uint32_t k = threadIdx.x; k < n; k += blockDim.x) gb1[k] = ord[k];
+      for (uint32_t k = threadIdx.x; k < n; k += 32) gb1[k] = ord[k];
     } else {
       uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
       uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
-      for (uint32_t k = threadIdx.x; k < n; k += blockDim.x) {
+      for (uint32_t k = threadIdx.x; k < n; k += 32) {
         gb2[k] = ord[k];
         gb2c[k] = cyc[k];
       }
     }
   }
+}
+
+// Termination (L110, L139, L226; R12), after the pheromone update.
+__global__ void k_stop(KArgs A, uint32_t pass) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.cfg.count) return;
+  RegionState &rs = A.state[r];
+  if (!rs.active) return;
+  const RegionDev *rd = A.regions + r;
+  const uint32_t lim = no_improve_limit(A.cfg, rd->n);
+  const uint32_t lb = pass == 1 ? rs.lb_cost : rd->lb_len;
+  if ((A.cfg.stop_at_lb && rs.best[pass - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
+      rs.iters[pass - 1] >= A.cfg.iterations)
+    rs.active = 0;
 }
 
 // ------------------------------------------------------------ launchers
@@ -812,22 +897,25 @@ static int check() {
 
 int last_cuda_error() { return check(); }
 
+template <typename K>
+static void big_smem(K kernel) {
+  cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemPerSM);
+}
+
 int set_machine(const MachineDev &m) {
   if (cudaMemcpyToSymbol(c_mach, &m, sizeof(m)) != cudaSuccess) return 1;
-  // allow large dynamic shared memory for every kernel variant
-  const int big = 227 * 1024;
-  cudaFuncSetAttribute(k_init<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_init<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_pass2_init, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_finalize<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_finalize<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_finalize<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  cudaFuncSetAttribute(k_finalize<2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-#define ACO_ATTR(P, M, D) \
-  cudaFuncSetAttribute(k_construct<P, M, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-  ACO_ATTR(1, true, false) ACO_ATTR(1, false, false) ACO_ATTR(1, true, true) ACO_ATTR(1, false, true)
-  ACO_ATTR(2, true, false) ACO_ATTR(2, false, false) ACO_ATTR(2, true, true) ACO_ATTR(2, false, true)
-#undef ACO_ATTR
+  big_smem(k_init<true>);
+  big_smem(k_init<false>);
+  big_smem(k_pass2_init);
+#define ACO_SEL(M) big_smem(k_select<1, M, false, false>); big_smem(k_select<2, M, false, false>); \
+  big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
+  ACO_SEL(true) ACO_SEL(false)
+#undef ACO_SEL
+#define ACO_CON(M, TS) big_smem(k_construct<1, M, TS, false, false>); big_smem(k_construct<2, M, TS, false, false>); \
+  big_smem(k_construct<2, M, TS, true, false>); big_smem(k_construct<2, M, TS, false, true>); \
+  big_smem(k_construct<2, M, TS, true, true>);
+  ACO_CON(true, true) ACO_CON(true, false) ACO_CON(false, true) ACO_CON(false, false)
+#undef ACO_CON
   return check();
 }
 
@@ -850,44 +938,56 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   return check();
 }
 
+template <int P, bool M, bool TS, bool T3, bool N4>
+static void go(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
+  k_construct<P, M, TS, T3, N4><<<c.n_blocks, c.ants_pb, c.smem_bytes, s>>>(a, c.items, iter);
+}
+
+template <bool M, bool TS>
+static void go_pass(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
+  if (pass == 1) go<1, M, TS, false, false>(c, s, a, iter);
+  else if (!c.t32 && !c.nc4) go<2, M, TS, false, false>(c, s, a, iter);
+  else if (c.t32 && !c.nc4) go<2, M, TS, true, false>(c, s, a, iter);
+  else if (!c.t32 && c.nc4) go<2, M, TS, false, true>(c, s, a, iter);
+  else go<2, M, TS, true, true>(c, s, a, iter);
+}
+
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c) {
   if (!c.n_blocks) return 0;
   cudaStream_t s = (cudaStream_t)L.stream;
   const bool mask = c.max_n <= 1024;
-  const bool dump = (L.cfg.flags & ACO_FLAG_DUMP) != 0;
   KArgs a = kargs(L);
-#define ACO_LAUNCH(P, M, D) k_construct<P, M, D><<<c.n_blocks, c.ants_pb, c.smem_bytes, s>>>(a, c.items, iter)
-  if (pass == 1) {
-    if (mask) {
-      if (dump) ACO_LAUNCH(1, true, true); else ACO_LAUNCH(1, true, false);
-    } else {
-      if (dump) ACO_LAUNCH(1, false, true); else ACO_LAUNCH(1, false, false);
-    }
+  if (mask) {
+    if (c.tau_smem) go_pass<true, true>(pass, c, s, a, iter);
+    else go_pass<true, false>(pass, c, s, a, iter);
   } else {
-    if (mask) {
-      if (dump) ACO_LAUNCH(2, true, true); else ACO_LAUNCH(2, true, false);
-    } else {
-      if (dump) ACO_LAUNCH(2, false, true); else ACO_LAUNCH(2, false, false);
-    }
+    if (c.tau_smem) go_pass<false, true>(pass, c, s, a, iter);
+    else go_pass<false, false>(pass, c, s, a, iter);
   }
-#undef ACO_LAUNCH
   L.launches++;
   return check();
 }
 
-int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n) {
+template <bool M>
+static void sel(uint32_t pass, bool t32, bool nc4, uint32_t grid, uint32_t smem, cudaStream_t s, const KArgs &a,
+                uint32_t iter) {
+  if (pass == 1) k_select<1, M, false, false><<<grid, 32, smem, s>>>(a, iter);
+  else if (!t32 && !nc4) k_select<2, M, false, false><<<grid, 32, smem, s>>>(a, iter);
+  else if (t32 && !nc4) k_select<2, M, true, false><<<grid, 32, smem, s>>>(a, iter);
+  else if (!t32 && nc4) k_select<2, M, false, true><<<grid, 32, smem, s>>>(a, iter);
+  else k_select<2, M, true, true><<<grid, 32, smem, s>>>(a, iter);
+}
+
+int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
+                    bool nc4, const UpdItem *upd, uint32_t n_upd) {
   if (!L.cfg.count) return 0;
   cudaStream_t s = (cudaStream_t)L.stream;
-  const bool mask = max_n <= 1024;
   KArgs a = kargs(L);
-  if (pass == 1) {
-    if (mask) k_finalize<1, true><<<L.cfg.count, 256, smem, s>>>(a, iter);
-    else k_finalize<1, false><<<L.cfg.count, 256, smem, s>>>(a, iter);
-  } else {
-    if (mask) k_finalize<2, true><<<L.cfg.count, 256, smem, s>>>(a, iter);
-    else k_finalize<2, false><<<L.cfg.count, 256, smem, s>>>(a, iter);
-  }
-  L.launches++;
+  if (max_n <= 1024) sel<true>(pass, t32, nc4, L.cfg.count, smem, s, a, iter);
+  else sel<false>(pass, t32, nc4, L.cfg.count, smem, s, a, iter);
+  if (n_upd) k_update<<<n_upd, 256, 0, s>>>(a, upd);
+  k_stop<<<(L.cfg.count + 255) / 256, 256, 0, s>>>(a, pass);
+  L.launches += 2 + (n_upd ? 1 : 0);
   return check();
 }
 

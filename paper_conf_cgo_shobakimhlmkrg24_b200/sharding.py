@@ -1,0 +1,55 @@
+"""Multi-GPU sharding of independent regions.
+
+Regions are independent (configs 3 and 5), so they shard across ranks with NO
+data-path collective: every rank runs aco_schedule_batch on its own regions.
+Region ids are global and key the Philox streams (R26), so a region produces
+the same schedule whichever rank runs it.  torch.distributed is used only to
+gather per-region results for reporting (gather_object) and, in bench.py,
+for the barrier and the max-over-ranks time.
+"""
+from __future__ import annotations
+
+from typing import Dict, List, Sequence
+
+
+def estimated_work(n: int, ants: int, iterations: int) -> int:
+    """Work estimate of one region: ants x iterations x n x (n + 16) (each ant
+    step scans a ready list that grows with n)."""
+    return ants * iterations * n * (n + 16)
+
+
+def lpt_partition(sizes: Sequence[int], world: int, ants: int = 1024, iterations: int = 10) -> List[List[int]]:
+    """Deterministic longest-processing-time assignment (strong scaling):
+    regions sorted by estimated work (descending, ties by index) go to the
+    least-loaded rank (ties to the lowest rank).  Returns per-rank index lists
+    in ascending index order."""
+    order = sorted(range(len(sizes)), key=lambda i: (-estimated_work(int(sizes[i]), ants, iterations), i))
+    load = [0] * world
+    parts: List[List[int]] = [[] for _ in range(world)]
+    for i in order:
+        r = min(range(world), key=lambda k: (load[k], k))
+        parts[r].append(i)
+        load[r] += estimated_work(int(sizes[i]), ants, iterations)
+    return [sorted(p) for p in parts]
+
+
+def weak_ids(per_rank: int, rank: int) -> List[int]:
+    """Weak scaling: rank r owns the global ids [r * per_rank, (r+1) * per_rank)."""
+    return list(range(rank * per_rank, (rank + 1) * per_rank))
+
+
+def gather_results(local: Dict[int, dict], world: int, rank: int, group=None) -> Dict[int, dict]:
+    """Gather {region_id: result} from every rank to rank 0 (reporting only)."""
+    import torch.distributed as dist
+    if world == 1:
+        return dict(local)
+    buf = [None] * world if rank == 0 else None
+    dist.gather_object(local, buf, dst=0, group=group)
+    if rank != 0:
+        return {}
+    out: Dict[int, dict] = {}
+    for part in buf:
+        for k, v in part.items():
+            assert k not in out, f"region {k} scheduled twice"
+            out[k] = v
+    return out
