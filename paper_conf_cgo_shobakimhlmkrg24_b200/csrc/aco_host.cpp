@@ -308,13 +308,14 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
     }
   for (uint32_t j = 0; j < n; ++j) eta2[j] = (uint16_t)(1 + (uint64_t)cp[j] * 65534ull / (cp_max ? cp_max : 1));
   // pass-specific compact per-instruction records
-  std::vector<uint32_t> ds((size_t)n * 2), e1b(n);
+  std::vector<uint32_t> ds((size_t)n * 4, 0), e1b(n);
   for (uint32_t j = 0; j < n; ++j) {
-    ds[2 * j] = info[(size_t)j * 4 + 0];
-    ds[2 * j + 1] = info[(size_t)j * 4 + 1];
+    ds[4 * j] = info[(size_t)j * 4 + 0];
+    ds[4 * j + 1] = info[(size_t)j * 4 + 1];
     const uint32_t skw = info[(size_t)j * 4 + 1];
     e1b[j] = j * (L + 1) + (skw & 0xFF) + ((skw >> 8) & 0xFF) + ((skw >> 16) & 0xFF) + (skw >> 24);
   }
+  for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j];
   // users of each counter register (to find the last remaining user)
   std::vector<uint32_t> cu_ptr(nctr + 1, 0), cu;
   for (uint32_t g = 0; g < G; ++g)
@@ -484,11 +485,14 @@ aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint
 
 namespace {
 
-// Launch shape of one region in one pass: ants per block and whether tau is
-// staged in shared memory, chosen to maximise resident ants per SM (tau in
-// smem is preferred unless it costs residency below 256 ants).
+// Launch shape of one region in one pass: ants per block, lanes per ant and
+// whether tau is staged in shared memory.  Ants per block maximise resident
+// ants per SM (shared memory is the usual limit); tau in smem is preferred
+// unless it costs residency below 256 ants; lanes per ant are the smallest
+// that give >= 16 resident warps per SM (latency hiding), within the
+// register budget.
 struct Shape {
-  uint32_t apb, smem;
+  uint32_t apb, lanes, smem;
   bool ts;
 };
 
@@ -503,27 +507,41 @@ uint32_t bucket_of(uint32_t bytes) {
   return 0;
 }
 
-// max_threads: resident threads per SM allowed by the kernel's registers
-// (pass 1 ~48 regs -> 1280, pass 2 ~80 regs -> 768; see cuobjdump -res-usage).
-Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads) {
-  auto resident = [&](uint32_t apb, uint32_t bytes) -> uint32_t {
-    const uint32_t b = bucket_of(bytes);
-    if (!b) return 0;
-    uint32_t blocks = kSmemPerSM / (b + 1024);  // + per-block reserved smem
-    blocks = std::min(blocks, max_threads / apb);  // register budget
-    blocks = std::min(blocks, 32u);
-    return blocks * apb;
-  };
-  Shape best0{0, 0, false}, best1{0, 0, true};
-  uint32_t r0 = 0, r1 = 0;
-  for (uint32_t apb : {32u, 64u, 128u, 256u}) {
-    const uint32_t b0 = img + apb * W * 4, b1 = img + tb + apb * W * 4;
-    const uint32_t x0 = resident(apb, b0), x1 = resident(apb, b1);
-    if (x0 >= r0 && x0 > 0) { r0 = x0; best0 = Shape{apb, bucket_of(b0), false}; }
-    if (x1 >= r1 && x1 > 0) { r1 = x1; best1 = Shape{apb, bucket_of(b1), true}; }
+// max_threads: resident threads per SM allowed by the kernel's registers.
+// Candidates (ants/block, lanes/ant, tau staging) are ranked by resident
+// threads per SM capped at 512 (16 warps hide the smem/ALU latency of the
+// per-ant step chain), then fewer lanes per ant (less reduction overhead),
+// then tau in shared memory, then more resident ants.
+Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
+                 uint32_t target_threads, uint32_t max_lanes) {
+  Shape best{0, 1, 0, false};
+  uint64_t best_score = 0;
+  for (int ts = 1; ts >= 0; --ts) {
+    if (ts && !allow_ts) continue;
+    for (uint32_t apb : {32u, 64u, 128u, 256u}) {
+      const uint32_t bytes = img + (ts ? tb : 0u) + apb * W * 4;
+      const uint32_t b = bucket_of(bytes);
+      if (!b) continue;
+      for (uint32_t L : {1u, 2u, 4u, 8u}) {
+        if (lanes14 && L != 1 && L != 4) continue;
+        if (L > max_lanes) continue;
+        const uint32_t threads = apb * L;
+        if (threads > 256) continue;
+        uint32_t blocks = kSmemPerSM / (b + 1024);  // + per-block reserved smem
+        blocks = std::min(blocks, max_threads / threads);
+        blocks = std::min(blocks, 32u);
+        if (!blocks) continue;
+        const uint64_t thr = std::min<uint64_t>((uint64_t)blocks * threads, target_threads);
+        const uint64_t ants = (uint64_t)blocks * apb;
+        const uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) | ants;
+        if (score > best_score) {
+          best_score = score;
+          best = Shape{apb, L, b, ts != 0};
+        }
+      }
+    }
   }
-  if (r1 > 0 && r1 >= std::min(r0, 256u)) return best1;
-  return best0;
+  return best;
 }
 
 }  // namespace
@@ -545,11 +563,15 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     uint32_t smem;
     std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  using Key = std::tuple<uint32_t, uint32_t, bool, bool, bool, uint32_t>;
+  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, uint32_t>;
   std::map<Key, Cls> classes;
   uint32_t fin_smem[3] = {0, 0, 0}, max_n = 0, init_smem = 0, p2_smem = 0;
   bool any_t32 = false;
   const bool nc4 = ctx->mach.n_classes > 2;
+  // launch-shape policy (tuning knobs; defaults measured on B200)
+  uint32_t tgt_threads[2] = {512, 256}, max_lanes[2] = {8, 1};
+  if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
+  if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
     max_n = std::max(max_n, R.n);
@@ -559,10 +581,12 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, nc4);
       if (pass == 1) init_smem = std::max(init_smem, R.img.bytes + 4 * W + 16);
       if (!(p->pass & pass)) continue;
-      const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u);
+      const bool rare = pass == 2 && (t32 || nc4);  // variants compiled without tau staging, 1|4 lanes
+      const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u, !rare, rare,
+                                  pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1]);
       if (sh.apb == 0) return ACO_E_TOO_LARGE;
       const bool mask = R.n <= 1024;
-      const Key key(pass, sh.apb, sh.ts, pass == 2 && t32, mask, sh.smem);
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, sh.smem);
       Cls &c = classes[key];
       c.sh = sh;
       c.mask = mask;
@@ -668,6 +692,7 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
       cl.items = (const BlockItem *)(ws + o_items) + base;
       cl.n_blocks = (uint32_t)k;
       cl.ants_pb = c.sh.apb;
+      cl.lanes = c.sh.lanes;
       cl.smem_bytes = c.smem;
       cl.max_n = c.mask ? 1024 : 65535;
       cl.tau_smem = c.sh.ts;
@@ -687,8 +712,8 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     launches[pass] = sorted;
     if (getenv("ACO_DEBUG_PLAN"))
       for (size_t i = 0; i < idx.size(); ++i)
-        fprintf(stderr, "[aco plan] pass %d class %zu: blocks %u ants/blk %u smem %u tau_smem %d t32 %d work %.3g\n",
-                pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].smem_bytes, (int)sorted[i].tau_smem,
+        fprintf(stderr, "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d work %.3g\n",
+                pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes, (int)sorted[i].tau_smem,
                 (int)sorted[i].t32, (double)class_work[pass][idx[i]]);
   }
   if (plan_only) return ACO_OK;

@@ -35,7 +35,7 @@ constexpr uint32_t kMuseCounter = 1u << 31;
 // Offsets (bytes, relative to the image start) of the arrays of the block image.
 struct ImageLayout {
   uint32_t info;      // uint4 [n] {defs u8x4, static kills u8x4, dead defs u8x4, muse start << 8 | count}
-  uint32_t ds;        // uint2 [n] {defs u8x4, static kills u8x4} (pass-2 feasibility)
+  uint32_t ds;        // uint4 [n] {defs u8x4, static kills u8x4, eta2, 0} (pass-2 candidates)
   uint32_t e1b;       // u32 [n]: j*(L+1) + #static kills (row base into eta1 for pass 1)
   uint32_t muse;      // u32 [nm]
   uint32_t cu_ptr;    // u32 [nctr+1]: users of each counter register
@@ -169,6 +169,7 @@ struct ClassLaunch {
   const BlockItem *items;  // device pointer (in ws)
   uint32_t n_blocks;
   uint32_t ants_pb;
+  uint32_t lanes;          // lanes per ant (1, 2, 4, 8): threads per block = ants_pb * lanes
   uint32_t smem_bytes;
   uint32_t max_n;          // max n in the class (selects the mask variant)
   bool tau_smem;           // stage tau in shared memory

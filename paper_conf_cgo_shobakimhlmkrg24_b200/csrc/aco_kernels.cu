@@ -108,7 +108,7 @@ __device__ void target_of(uint32_t mode, const uint32_t best[4], uint32_t tgt[4]
 // ---------------------------------------------------------------- statics view
 struct SV {
   const uint4 *info;
-  const uint2 *ds;
+  const uint4 *ds;
   const uint32_t *e1b, *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0;
   const uint16_t *eta1, *eta2;
   uint32_t n, nwr, nremw, region_id;
@@ -118,7 +118,7 @@ struct SV {
 __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev *rd) {
   SV V;
   V.info = (const uint4 *)(img + rd->img.info);
-  V.ds = (const uint2 *)(img + rd->img.ds);
+  V.ds = (const uint4 *)(img + rd->img.ds);
   V.e1b = (const uint32_t *)(img + rd->img.e1b);
   V.muse = (const uint32_t *)(img + rd->img.muse);
   V.cu_ptr = (const uint32_t *)(img + rd->img.cu_ptr);
@@ -209,48 +209,87 @@ __device__ __forceinline__ void t_set(const St &A, uint32_t j, uint32_t v) {
   }
 }
 
-// Ascending iteration over the ready bitset (R25).  MASK: one register bit per
-// non-empty bitset word (n <= 1024).
-struct BitIt {
-  uint32_t m, w, bits;
-};
-template <bool MASK>
-__device__ __forceinline__ void it_init(BitIt &it, uint32_t wmask) {
-  it.m = wmask;
-  it.w = MASK ? 0u : 0xFFFFFFFFu;
-  it.bits = 0;
-}
-template <bool MASK>
-__device__ __forceinline__ bool it_next(BitIt &it, const St &A, uint32_t nwr, uint32_t &j) {
-  while (!it.bits) {
-    if (MASK) {
-      if (!it.m) return false;
-      it.w = __ffs(it.m) - 1;
-      it.m &= it.m - 1;
-    } else {
-      if (++it.w >= nwr) return false;
-    }
-    it.bits = A.RB[it.w * A.S];
+// ---- lane groups: LG consecutive lanes of a warp build one ant together.
+// Lane l of a group scans the ready-bitset words w with w % LG == l; the group
+// reduces with shuffles; lane 0 (the leader) performs every state update.
+template <int LG>
+struct Grp {
+  uint32_t lane, mask;
+  __device__ __forceinline__ Grp(uint32_t tid) {
+    const uint32_t l = tid & 31u;
+    lane = l & (LG - 1);
+    mask = LG == 32 ? 0xFFFFFFFFu : (((1u << LG) - 1u) << (l - lane));
   }
-  j = it.w * 32u + (__ffs(it.bits) - 1);
-  it.bits &= it.bits - 1;
-  return true;
-}
-// Next up to four candidates (ascending); invalid slots repeat j[0].
-template <bool MASK>
-__device__ __forceinline__ uint32_t it_next4(BitIt &it, const St &A, uint32_t nwr, uint32_t j[4]) {
-  uint32_t cnt = 0;
+  __device__ __forceinline__ bool leader() const { return lane == 0; }
+  __device__ __forceinline__ uint32_t bcast(uint32_t v) const {
+    return LG == 1 ? v : __shfl_sync(mask, v, 0, LG);
+  }
+  __device__ __forceinline__ uint32_t sum(uint32_t v) const {
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    uint32_t x = 0;
-    if (cnt == (uint32_t)q && it_next<MASK>(it, A, nwr, x)) {
-      j[q] = x;
-      ++cnt;
-    } else {
-      j[q] = j[0];
+    for (int o = LG / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, LG);
+    return v;
+  }
+  __device__ __forceinline__ uint32_t min(uint32_t v) const {
+#pragma unroll
+    for (int o = LG / 2; o > 0; o >>= 1) v = ::min(v, __shfl_xor_sync(mask, v, o, LG));
+    return v;
+  }
+  __device__ __forceinline__ unsigned long long max64(unsigned long long v) const {
+#pragma unroll
+    for (int o = LG / 2; o > 0; o >>= 1) v = ::max(v, __shfl_xor_sync(mask, v, o, LG));
+    return v;
+  }
+  __device__ __forceinline__ unsigned long long sum64(unsigned long long v) const {
+#pragma unroll
+    for (int o = LG / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, LG);
+    return v;
+  }
+  __device__ __forceinline__ bool any(bool p) const {
+    return LG == 1 ? p : (__ballot_sync(mask, p) & mask) != 0u;
+  }
+  __device__ __forceinline__ void sync() const {
+    if (LG > 1) __syncwarp(mask);
+  }
+};
+
+// Bits of a word-subset mask: words w with w % LG == lane (n <= 1024).
+template <int LG>
+__device__ __forceinline__ uint32_t lane_words(uint32_t lane) {
+  return LG == 1 ? 0xFFFFFFFFu
+                 : (LG == 2 ? 0x55555555u
+                            : (LG == 4 ? 0x11111111u
+                                       : (LG == 8 ? 0x01010101u : (LG == 16 ? 0x00010001u : 1u))))
+                       << lane;
+}
+
+// Visit the set bits of the ready bitset in ascending order: all words
+// (stride 1) or this lane's words (stride LG).  MASK: wmask has one bit per
+// non-empty word (n <= 1024).
+template <bool MASK, typename F>
+__device__ __forceinline__ void scan_bits(const St &A, uint32_t nwr, uint32_t wmask, uint32_t first,
+                                          uint32_t stride, uint32_t sub, F &&visit) {
+  if (MASK) {
+    uint32_t m = wmask & sub;
+    while (m) {
+      const uint32_t w = __ffs(m) - 1;
+      m &= m - 1;
+      uint32_t bits = A.RB[w * A.S];
+      while (bits) {
+        const uint32_t j = w * 32u + (__ffs(bits) - 1);
+        bits &= bits - 1;
+        if (visit(j)) return;
+      }
+    }
+  } else {
+    for (uint32_t w = first; w < nwr; w += stride) {
+      uint32_t bits = A.RB[w * A.S];
+      while (bits) {
+        const uint32_t j = w * 32u + (__ffs(bits) - 1);
+        bits &= bits - 1;
+        if (visit(j)) return;
+      }
     }
   }
-  return cnt;
 }
 
 struct AntOut {
@@ -360,18 +399,28 @@ __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
   return wmask;
 }
 
+// Argmax key: highest score, ties to the lowest index (R1, R25).
+__device__ __forceinline__ unsigned long long akey(uint32_t s, uint32_t j) {
+  return ((unsigned long long)s << 32) | (0xFFFFFFFFu - j);
+}
+
 // ------------------------------------------------------------ pass-1 ant
 // RP pass (L108, L145; R19): latencies ignored, candidates = ready list,
 // score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
-// Philox step (R26).  rec (may be NULL) receives the order.
-template <bool MASK>
+// Philox step (R26).  rec (leader, may be NULL) receives the order.  The
+// result is valid in the leader lane.
+template <int LG, bool MASK>
 __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
-                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
-                                            const bool greedy, uint16_t *rec) {
+                                            const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
+                                            const RunCfg &cfg, const bool greedy, uint16_t *rec) {
   const uint32_t n = V.n, nwr = V.nwr;
-  uint32_t wmask = init_state<1, MASK, false, false>(V, A);
+  uint32_t wmask = 0;
+  if (G.leader()) wmask = init_state<1, MASK, false, false>(V, A);
+  wmask = G.bcast(wmask);
+  G.sync();
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
+  const uint32_t sub = lane_words<LG>(G.lane);
   uint32_t prev = n;
   for (uint32_t k = 0; k < n; ++k) {
     bool exploit = greedy;
@@ -380,77 +429,78 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       exploit = (uint64_t)g.x < cfg.q0_t;
     }
     const uint16_t *trow = tau + prev * n;
-    uint32_t best_s = 0, best_j = 0;
-    uint64_t sum = 0;
-    BitIt it;
-    it_init<MASK>(it, wmask);
-    for (;;) {
-      uint32_t j[4];
-      const uint32_t cnt = it_next4<MASK>(it, A, nwr, j);
-      if (!cnt) break;
-      uint32_t s[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {  // independent loads of four candidates
-        const uint32_t e1 = V.e1b[j[q]] + dk1_get(A, j[q]);
-        s[q] = (uint32_t)trow[j[q]] * (uint32_t)V.eta1[e1];
+    auto score = [&](uint32_t j) -> uint32_t {
+      return (uint32_t)trow[j] * (uint32_t)V.eta1[V.e1b[j] + dk1_get(A, j)];
+    };
+    unsigned long long best = 0;
+    unsigned long long sum = 0;
+    scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
+      const uint32_t s = score(j);
+      best = ::max(best, akey(s, j));
+      sum += s;
+      return false;
+    });
+    best = G.max64(best);
+    uint32_t jstar = 0xFFFFFFFFu - (uint32_t)best;
+    if (!exploit) {  // roulette (R27): the leader scans every candidate in ascending order
+      sum = G.sum64(sum);
+      if (G.leader()) {
+        const uint4 x = philox(k, ant, iter, V.region_id, cfg.seed);
+        const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
+        uint64_t pre = 0;
+        scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
+          pre += score(j);
+          if (pre > r) {
+            jstar = j;
+            return true;
+          }
+          return false;
+        });
       }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint32_t sq = (uint32_t)q < cnt ? s[q] : 0u;
-        if (sq > best_s) {  // argmax, ties to the lowest index (ascending order)
-          best_s = sq;
-          best_j = j[q];
-        }
-        sum += sq;
-      }
-      if (cnt < 4) break;
+      jstar = G.bcast(jstar);
     }
-    if (!exploit) {  // roulette (R27)
-      const uint4 x = philox(k, ant, iter, V.region_id, cfg.seed);
-      const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
-      uint64_t pre = 0;
-      it_init<MASK>(it, wmask);
-      uint32_t j;
-      while (it_next<MASK>(it, A, nwr, j)) {
-        pre += (uint32_t)trow[j] * (uint32_t)V.eta1[V.e1b[j] + dk1_get(A, j)];
-        if (pre > r) {
-          best_j = j;
-          break;
-        }
-      }
+    if (G.leader()) {
+      commit<1, MASK, false, false>(V, A, jstar, 0, wmask, live01, live23, prp01, prp23);
+      if (rec) rec[k] = (uint16_t)jstar;
     }
-    commit<1, MASK, false, false>(V, A, best_j, 0, wmask, live01, live23, prp01, prp23);
-    if (rec) rec[k] = (uint16_t)best_j;
-    prev = best_j;
+    wmask = G.bcast(wmask);
+    G.sync();
+    prev = jstar;
   }
   AntOut o;
   o.prp01 = prp01;
   o.prp23 = prp23;
-  o.cost = cost_of(cfg.cost_mode, prp01, prp23);
+  o.cost = G.leader() ? cost_of(cfg.cost_mode, prp01, prp23) : 0u;
   return o;
 }
 
 // ------------------------------------------------------------ pass-2 ant
 // ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle and
-// the Philox step; stalls skip ahead without drawing.  rec_o / rec_c (may be
-// NULL) receive the order and the cycles.
-template <bool MASK, bool T32, bool NC4>
+// the Philox step; stalls skip ahead without drawing.  rec_o / rec_c (leader,
+// may be NULL) receive the order and the cycles.  Valid in the leader lane.
+template <int LG, bool MASK, bool T32, bool NC4>
 __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restrict__ tau, const St &A,
-                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
-                                            const uint32_t tgt[4], uint32_t *prune_len, const bool prune,
-                                            uint16_t *rec_o, uint32_t *rec_c) {
+                                            const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
+                                            const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
+                                            const bool prune, uint16_t *rec_o, uint32_t *rec_c) {
   const uint32_t n = V.n, nwr = V.nwr;
-  uint32_t wmask = init_state<2, MASK, T32, NC4>(V, A);
+  uint32_t wmask = 0;
+  if (G.leader()) wmask = init_state<2, MASK, T32, NC4>(V, A);
+  wmask = G.bcast(wmask);
+  G.sync();
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const bool stall_en = (group % cfg.stall_mod) == cfg.stall_rem;  // R23
   const uint32_t c2 = 0x80000000u | iter;
+  const uint32_t sub = lane_words<LG>(G.lane);
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0;
   AntOut o;
   o.prp01 = o.prp23 = 0;
   while (placed < n) {
     if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune
-      const uint32_t bl = *(volatile uint32_t *)prune_len;
+      uint32_t bl = 0;
+      if (G.leader()) bl = *(volatile uint32_t *)prune_len;
+      bl = G.bcast(bl);
       if (t + (n - placed) > bl) {
         o.cost = kInvalid;
         return o;
@@ -461,57 +511,46 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     {
       const uint32_t lv[4] = {live01 & 0xFFFFu, live01 >> 16, live23 & 0xFFFFu, live23 >> 16};
 #pragma unroll
-      for (int c = 0; c < 4; ++c) slack |= min(tgt[c] - lv[c], 255u) << (8 * c);
+      for (int c = 0; c < 4; ++c) slack |= ::min(tgt[c] - lv[c], 255u) << (8 * c);
     }
     const uint16_t *trow = tau + prev * n;
-    uint32_t nr = 0, nf = 0, ns = 0, min_s = 0xFFFFFFFFu;
-    bool all_f_inc = true, some_s_dec = false;
-    uint32_t best_s = 0, best_j = 0;
-    uint64_t sum = 0;
-    BitIt it;
-    it_init<MASK>(it, wmask);
-    for (;;) {
-      uint32_t j[4];
-      const uint32_t cnt = it_next4<MASK>(it, A, nwr, j);
-      if (!cnt) break;
-      uint32_t rdy[4], K[4], D[4], s[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {  // independent loads of four candidates
-        rdy[q] = t_get<T32>(A, j[q]);
-        const uint2 ds = V.ds[j[q]];
-        D[q] = ds.x;
-        K[q] = ds.y + dk2_get<NC4>(A, j[q]);  // kills per class (R14)
-        s[q] = (uint32_t)trow[j[q]] * (uint32_t)V.eta2[j[q]];
-      }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        if ((uint32_t)q >= cnt) break;
-        if (rdy[q] <= t) {
-          ++nr;
-          // feasible (R21): defs_c <= slack_c + kills_c for every class
-          if (__vcmpgtu4(D[q], __vaddus4(slack, K[q])) == 0u) {
-            ++nf;
-            if (__vcmpgtu4(D[q], K[q]) == 0u) all_f_inc = false;  // max_c Delta_c <= 0
-            if (s[q] > best_s) {
-              best_s = s[q];
-              best_j = j[q];
-            }
-            sum += s[q];
-          }
-        } else {
-          ++ns;
-          min_s = min(min_s, rdy[q]);
-          if (__vcmpltu4(D[q], K[q]) != 0u) some_s_dec = true;  // min_c Delta_c < 0
+    uint32_t counts = 0, min_s = 0xFFFFFFFFu;  // counts = |R| | |F| << 16
+    bool f_not_inc = false, s_dec = false, any_s = false;
+    unsigned long long best = 0, sum = 0;
+    scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
+      const uint32_t rdy = t_get<T32>(A, j);
+      const uint4 ds = V.ds[j];                       // defs, static kills, eta2
+      const uint32_t K = ds.y + dk2_get<NC4>(A, j);   // kills per class (R14)
+      const uint32_t s = (uint32_t)trow[j] * ds.z;
+      if (rdy <= t) {
+        counts += 1u;
+        if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
+          counts += 1u << 16;
+          f_not_inc |= __vcmpgtu4(ds.x, K) == 0u;           // max_c Delta_c <= 0
+          best = ::max(best, akey(s, j));
+          sum += s;
         }
+      } else {
+        any_s = true;
+        min_s = ::min(min_s, rdy);
+        s_dec |= __vcmpltu4(ds.x, K) != 0u;                 // min_c Delta_c < 0
       }
-      if (cnt < 4) break;
-    }
+      return false;
+    });
+    counts = G.sum(counts);
+    min_s = G.min(min_s);
+    best = G.max64(best);
+    sum = G.sum64(sum);
+    any_s = G.any(any_s);
+    const bool all_f_inc = !G.any(f_not_inc);
+    const bool some_s_dec = G.any(s_dec);
+    const uint32_t nr = counts & 0xFFFFu, nf = counts >> 16;
     if (nr == 0) {  // necessary stall (L153): skip ahead to the next ready time
       t = min_s;
       continue;
     }
     if (nf == 0) {
-      if (stall_en && ns > 0) {  // forced optional stall (L155, R22)
+      if (stall_en && any_s) {  // forced optional stall (L155, R22)
         kopt += min_s - t;
         t = min_s;
         continue;
@@ -521,7 +560,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     }
     uint4 x = make_uint4(0, 0, 0, 0);
     bool have_x = false;
-    if (stall_en && ns > 0 && all_f_inc && some_s_dec) {  // discretionary stall (L157-L164)
+    if (stall_en && any_s && all_f_inc && some_s_dec) {  // discretionary stall (L157-L164)
       x = philox(t, ant, c2, V.region_id, cfg.seed);
       have_x = true;
       const uint32_t thr = (kopt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (kopt + 1));
@@ -532,33 +571,42 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       }
     }
     const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
-    if (!((uint64_t)g.x < cfg.q0_t)) {  // explore: roulette over F (R27)
-      if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
-      const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
-      uint64_t pre = 0;
-      it_init<MASK>(it, wmask);
-      uint32_t j;
-      while (it_next<MASK>(it, A, nwr, j)) {
-        if (t_get<T32>(A, j) > t) continue;
-        const uint2 ds = V.ds[j];
-        if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk2_get<NC4>(A, j))) != 0u) continue;
-        pre += (uint32_t)trow[j] * (uint32_t)V.eta2[j];
-        if (pre > r) {
-          best_j = j;
-          break;
-        }
+    uint32_t jstar = 0xFFFFFFFFu - (uint32_t)best;
+    if (!((uint64_t)g.x < cfg.q0_t)) {  // explore: roulette over F (R27), leader in ascending order
+      if (G.leader()) {
+        if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
+        const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
+        uint64_t pre = 0;
+        scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
+          if (t_get<T32>(A, j) > t) return false;
+          const uint4 ds = V.ds[j];
+          if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk2_get<NC4>(A, j))) != 0u) return false;
+          pre += (uint32_t)trow[j] * ds.z;
+          if (pre > r) {
+            jstar = j;
+            return true;
+          }
+          return false;
+        });
+      }
+      jstar = G.bcast(jstar);
+    }
+    if (G.leader()) {
+      commit<2, MASK, T32, NC4>(V, A, jstar, t, wmask, live01, live23, prp01, prp23);
+      if (rec_o) {
+        rec_o[placed] = (uint16_t)jstar;
+        rec_c[placed] = t;
       }
     }
-    commit<2, MASK, T32, NC4>(V, A, best_j, t, wmask, live01, live23, prp01, prp23);
-    if (rec_o) {
-      rec_o[placed] = (uint16_t)best_j;
-      rec_c[placed] = t;
-    }
+    wmask = G.bcast(wmask);
+    live01 = G.bcast(live01);
+    live23 = G.bcast(live23);
+    G.sync();
     ++placed;
-    prev = best_j;
+    prev = jstar;
     ++t;
   }
-  if (prune) atomicMin(prune_len, t);
+  if (prune && G.leader()) atomicMin(prune_len, t);
   o.prp01 = prp01;
   o.prp23 = prp23;
   o.cost = t;  // length = last issue cycle + 1 (R20)
@@ -583,7 +631,7 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
   for (uint32_t i = threadIdx.x; i < bytes / 16; i += blockDim.x) dst[i] = src[i];
 }
 
-template <int PASS, bool MASK, bool TAU_SMEM, bool T32, bool NC4>
+template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4>
 __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__restrict__ items,
                                                    uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
@@ -606,17 +654,19 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
     tau = (const uint16_t *)(A.ws + W.o_tau);
   }
   __syncthreads();
-  const uint32_t ant = bi.ant0 + threadIdx.x;
-  if (ant >= A.cfg.ants) return;
+  const uint32_t local = threadIdx.x / LG;  // ant within the block
+  const uint32_t ant = bi.ant0 + local;
+  if (ant >= A.cfg.ants) return;  // whole lane group
+  const Grp<LG> G(threadIdx.x);
   const SV V = make_sv(smem, rd);
-  const St S = make_st<PASS, T32, NC4>((uint32_t *)(smem + state_off) + threadIdx.x, blockDim.x, V);
+  const St S = make_st<PASS, T32, NC4>((uint32_t *)(smem + state_off) + local, blockDim.x / LG, V);
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
   if (PASS == 1) {
     uint16_t *rec = nullptr;
     if (dump && A.dump_order)
       rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ant * V.n;
-    o = ant_pass1<MASK>(V, tau, S, ant, iter, A.cfg, false, rec);
+    o = ant_pass1<LG, MASK>(V, tau, S, G, ant, iter, A.cfg, false, rec);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -630,13 +680,16 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
       rec_o = A.dump_order + base;
       rec_c = A.dump_cycle + base;
     }
-    o = ant_pass2<MASK, T32, NC4>(V, tau, S, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c);
+    o = ant_pass2<LG, MASK, T32, NC4>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
+                                      rec_c);
   }
-  uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
-  costs[ant] = o.cost;
-  if (dump && A.dump_cost)
-    A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants + ant] =
-        o.cost;
+  if (G.leader()) {
+    uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
+    costs[ant] = o.cost;
+    if (dump && A.dump_cost)
+      A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants +
+                  ant] = o.cost;
+  }
 }
 
 __device__ __forceinline__ uint64_t fnv_u32(uint64_t h, uint32_t v) {
@@ -715,11 +768,13 @@ __global__ void __launch_bounds__(128) k_init(KArgs A) {
   stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   __syncthreads();
-  if (threadIdx.x == 0) {
+  if (threadIdx.x < 32) {  // warp 0 builds the greedy schedule as one 32-lane group
     const SV V = make_sv(smem, rd);
     const St S = make_st<1, false, false>((uint32_t *)(smem + rd->img.bytes), 1, V);
     uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
-    AntOut o = ant_pass1<MASK>(V, tau, S, 0, 0, A.cfg, true, gb1);
+    const Grp<32> G32(threadIdx.x);
+    AntOut o = ant_pass1<32, MASK>(V, tau, S, G32, 0, 0, A.cfg, true, gb1);
+    if (threadIdx.x != 0) return;
     rs.lb_cost = cost_rp(A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
     rs.init[0] = rs.best[0] = o.cost;
     const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
@@ -804,18 +859,21 @@ __global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   uint32_t *cyc = stw + ant_words(PASS, n, rd->nwr, rd->nremw, T32, NC4);
   uint16_t *ord = (uint16_t *)(cyc + n);
   __syncwarp();
-  if (have && threadIdx.x == 0) {
+  if (have) {  // the whole warp replays the winner as one 32-lane group
     const St S = make_st<PASS, T32, NC4>(stw, 1, V);
+    const Grp<32> G32(threadIdx.x);
     AntOut o;
     if (PASS == 1) {
-      o = ant_pass1<MASK>(V, tau, S, want, iter, A.cfg, false, ord);
+      o = ant_pass1<32, MASK>(V, tau, S, G32, want, iter, A.cfg, false, ord);
     } else {
       uint32_t tgt[4];
       for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
-      o = ant_pass2<MASK, T32, NC4>(V, tau, S, want, iter, A.cfg, tgt, nullptr, false, ord, cyc);
+      o = ant_pass2<32, MASK, T32, NC4>(V, tau, S, G32, want, iter, A.cfg, tgt, nullptr, false, ord, cyc);
     }
-    s_prp[0] = o.prp01;
-    s_prp[1] = o.prp23;
+    if (threadIdx.x == 0) {
+      s_prp[0] = o.prp01;
+      s_prp[1] = o.prp23;
+    }
   }
   __syncwarp();
   uint16_t *next = (uint16_t *)(A.ws + W.o_next);
@@ -911,11 +969,16 @@ int set_machine(const MachineDev &m) {
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
 #undef ACO_SEL
-#define ACO_CON(M, TS) big_smem(k_construct<1, M, TS, false, false>); big_smem(k_construct<2, M, TS, false, false>); \
-  big_smem(k_construct<2, M, TS, true, false>); big_smem(k_construct<2, M, TS, false, true>); \
-  big_smem(k_construct<2, M, TS, true, true>);
-  ACO_CON(true, true) ACO_CON(true, false) ACO_CON(false, true) ACO_CON(false, false)
+#define ACO_CON(LG, M, TS) big_smem(k_construct<1, LG, M, TS, false, false>); \
+  big_smem(k_construct<2, LG, M, TS, false, false>);
+#define ACO_CON_M(LG) ACO_CON(LG, true, true) ACO_CON(LG, true, false) ACO_CON(LG, false, true) ACO_CON(LG, false, false)
+  ACO_CON_M(1) ACO_CON_M(2) ACO_CON_M(4) ACO_CON_M(8)
 #undef ACO_CON
+#undef ACO_CON_M
+#define ACO_CON_X(LG, M) big_smem(k_construct<2, LG, M, false, true, false>); \
+  big_smem(k_construct<2, LG, M, false, false, true>); big_smem(k_construct<2, LG, M, false, true, true>);
+  ACO_CON_X(1, true) ACO_CON_X(1, false) ACO_CON_X(4, true) ACO_CON_X(4, false)
+#undef ACO_CON_X
   return check();
 }
 
@@ -938,18 +1001,37 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   return check();
 }
 
-template <int P, bool M, bool TS, bool T3, bool N4>
+template <int P, int LG, bool M, bool TS, bool T3, bool N4>
 static void go(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  k_construct<P, M, TS, T3, N4><<<c.n_blocks, c.ants_pb, c.smem_bytes, s>>>(a, c.items, iter);
+  k_construct<P, LG, M, TS, T3, N4><<<c.n_blocks, c.ants_pb * LG, c.smem_bytes, s>>>(a, c.items, iter);
+}
+
+template <int LG, bool M, bool TS>
+static void go_lg(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
+  if (pass == 1) go<1, LG, M, TS, false, false>(c, s, a, iter);
+  else go<2, LG, M, TS, false, false>(c, s, a, iter);
+}
+
+template <int LG, bool M>
+static void go_x(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
+  if (c.t32 && !c.nc4) go<2, LG, M, false, true, false>(c, s, a, iter);
+  else if (!c.t32 && c.nc4) go<2, LG, M, false, false, true>(c, s, a, iter);
+  else go<2, LG, M, false, true, true>(c, s, a, iter);
 }
 
 template <bool M, bool TS>
 static void go_pass(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  if (pass == 1) go<1, M, TS, false, false>(c, s, a, iter);
-  else if (!c.t32 && !c.nc4) go<2, M, TS, false, false>(c, s, a, iter);
-  else if (c.t32 && !c.nc4) go<2, M, TS, true, false>(c, s, a, iter);
-  else if (!c.t32 && c.nc4) go<2, M, TS, false, true>(c, s, a, iter);
-  else go<2, M, TS, true, true>(c, s, a, iter);
+  if (pass == 2 && (c.t32 || c.nc4)) {  // rare variants: tau in global memory, 1 or 4 lanes per ant
+    if (c.lanes >= 4) go_x<4, M>(c, s, a, iter);
+    else go_x<1, M>(c, s, a, iter);
+    return;
+  }
+  switch (c.lanes) {
+    case 8: go_lg<8, M, TS>(pass, c, s, a, iter); break;
+    case 4: go_lg<4, M, TS>(pass, c, s, a, iter); break;
+    case 2: go_lg<2, M, TS>(pass, c, s, a, iter); break;
+    default: go_lg<1, M, TS>(pass, c, s, a, iter); break;
+  }
 }
 
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c) {
