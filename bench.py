@@ -45,7 +45,7 @@ def parse():
     ap.add_argument("--iterations", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-sample", type=int, default=48, help="regions in the oracle sample")
+    ap.add_argument("--cpu-sample", type=int, default=160, help="regions in the oracle sample")
     return ap.parse_args()
 
 
@@ -249,20 +249,26 @@ def main():
         if world == 1 and not args.no_cpu_baseline:
             cpu, stats = cpu_baseline(regs, ids, p, args.cpu_sample)
             bpas = bytes_per_ant_step(stats)
-        # roofline of the dominant kernel (ant construction): algorithmic bytes
+        # roofline of the dominant kernel (ant construction):
+        # algorithmic shared-memory bytes (SURVEY 8(d) per ant-step figure from
+        # the oracle's instrumentation of the sample) x ant-steps per launch,
+        # over the construct launches' CUDA-event time; peak = the SM shared
+        # memory crossbar, 148 SMs x 128 B/clk x the SM clock seen under load.
         construct_ms = phase_ms[0] / max(1, args.steps)
         ant_steps = p.ants * sum(r["n"] * (r["iters1"] + r["iters2"]) for r in res)
-        sm_mhz = peaks.get("sm_max_mhz", 1965.0)
-        smem_peak = 148 * 128 * sm_mhz * 1e6 / 1e9  # GB/s, nominal smem crossbar (guide)
+        sm_mhz = clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
+        smem_peak = 148 * 128 * sm_mhz * 1e6 / 1e9  # GB/s
         roof = None
         if bpas is not None and construct_ms > 0:
             n_launch = phase_launches[0] / max(1, args.steps)
             achieved = bpas * ant_steps / (construct_ms / 1000.0) / 1e9
             roof = {"bound": "smem", "achieved": round(achieved, 1), "peak": round(smem_peak, 1),
                     "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": None,
-                    "kernel": "k_construct", "bytes_per_ant_step": round(bpas, 2),
+                    "kernel": "k_construct (all classes)", "bytes_per_ant_step": round(bpas, 2),
                     "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,
-                    "peak_source": "148 SM x 128 B/clk x sm_max_mhz (guide nominal smem)"}
+                    "construct_ms_per_step": round(construct_ms, 3),
+                    "ant_steps_per_s": round(ant_steps / (construct_ms / 1000.0), 1),
+                    "peak_source": f"guide: 148 SM x 128 B/clk x {sm_mhz:.0f} MHz (smem crossbar, no measured peak)"}
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup),

@@ -150,6 +150,27 @@ aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_resu
  * Region r's block in a (pass, iteration) slice starts at ants * sum_{q<r} n_q. */
 aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint32_t *d_cycles);
 
+/* ---- Shared colony (config 4): the ants of the loaded regions are split
+ * across ranks (one context per GPU).  Ant ids are global: this context runs
+ * ants [ant_base, ant_base + p->ants) of p->ants * world ants.  Per pass and
+ * iteration the caller runs
+ *     aco_colony_construct(ctx, pass, iter, keys, stream)   (local ants; keys[r] = local best)
+ *     allreduce(keys, MIN) over ranks, on `stream`           (int64, one per region)
+ *     aco_colony_finalize(ctx, pass, iter, keys, stream)     (replay of the global winner,
+ *                                                             identical pheromone update)
+ * for pass in the requested passes and iter < p->iterations (stop rules are
+ * evaluated identically on every rank; finished regions idle), then
+ * aco_colony_end.  keys is a caller-owned device buffer of count int64:
+ * key = ((cost << 32) | global ant) XOR 2^63, so a signed MIN selects the
+ * lexicographically smallest (cost, ant) (R10).  The winner's order is never
+ * sent: every rank replays it from its identical pheromone table.  Results
+ * are bit-identical to one context running all ants (tested). */
+aco_status aco_colony_begin(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *d_workspace,
+                            size_t ws_bytes, size_t *ws_needed, void *cuda_stream);
+aco_status aco_colony_construct(aco_ctx ctx, uint32_t pass, uint32_t iter, int64_t *d_keys, void *cuda_stream);
+aco_status aco_colony_finalize(aco_ctx ctx, uint32_t pass, uint32_t iter, int64_t *d_keys, void *cuda_stream);
+aco_status aco_colony_end(aco_ctx ctx, void *cuda_stream);
+
 /* Device time of the phases of the last aco_schedule_batch run with
  * ACO_FLAG_TIMING (synchronises).  ms[0] = ant construction (all
  * k_construct launches), ms[1] = finalize (argmin + replay + pheromone +

@@ -20,6 +20,7 @@ INVALID = 0xFFFFFFFF
 EXPORTS = [
     "aco_create", "aco_load_regions", "aco_schedule_batch", "aco_get_results", "aco_set_dump",
     "aco_last_launch_count", "aco_get_timing", "aco_status_string", "aco_destroy",
+    "aco_colony_begin", "aco_colony_construct", "aco_colony_finalize", "aco_colony_end",
 ]
 
 
@@ -83,12 +84,17 @@ def load(path: str = LIB_PATH):
     L.aco_set_dump.argtypes = [vp, vp, vp, vp]
     L.aco_last_launch_count.argtypes = [vp, C.POINTER(C.c_uint64)]
     L.aco_get_timing.argtypes = [vp, vp, vp]
+    L.aco_colony_begin.argtypes = [vp, vp, u32, vp, sz, C.POINTER(sz), vp]
+    L.aco_colony_construct.argtypes = [vp, u32, u32, vp, vp]
+    L.aco_colony_finalize.argtypes = [vp, u32, u32, vp, vp]
+    L.aco_colony_end.argtypes = [vp, vp]
     L.aco_status_string.argtypes = [C.c_int32]
     L.aco_status_string.restype = C.c_char_p
     L.aco_destroy.argtypes = [vp]
     L.aco_destroy.restype = None
     for f in ("aco_create", "aco_load_regions", "aco_schedule_batch", "aco_get_results",
-              "aco_set_dump", "aco_last_launch_count", "aco_get_timing"):
+              "aco_set_dump", "aco_last_launch_count", "aco_get_timing", "aco_colony_begin",
+              "aco_colony_construct", "aco_colony_finalize", "aco_colony_end"):
         getattr(L, f).restype = C.c_int32
     _lib = L
     return L

@@ -150,6 +150,49 @@ class Scheduler:
         self.params = p
         return self
 
+    # ---------------------------------------------------------------- shared colony
+    def colony_begin(self, p: Params, ant_base: int, stream: Optional[torch.cuda.Stream] = None):
+        """Plan a shared-colony run: this context builds ants [ant_base, ant_base + p.ants)."""
+        need = C.c_size_t(0)
+        ps = params_struct(p, 0)
+        _lib.check(self.lib.aco_colony_begin(self.ctx, C.byref(ps), ant_base, None, 0, C.byref(need), None),
+                   "aco_colony_begin(size)")
+        if self.ws is None or self.ws.numel() < need.value:
+            self.ws = torch.empty(max(256, need.value), dtype=torch.uint8, device=f"cuda:{self.device}")
+        _lib.check(self.lib.aco_colony_begin(self.ctx, C.byref(ps), ant_base, C.c_void_p(self.ws.data_ptr()),
+                                             self.ws.numel(), C.byref(need), _stream_handle(stream)),
+                   "aco_colony_begin")
+        self.params = p
+        self.keys = torch.empty(max(1, self.count), dtype=torch.int64, device=f"cuda:{self.device}")
+        return self.keys
+
+    def colony_construct(self, pass_: int, it: int, stream: Optional[torch.cuda.Stream] = None):
+        _lib.check(self.lib.aco_colony_construct(self.ctx, pass_, it, C.c_void_p(self.keys.data_ptr()),
+                                                 _stream_handle(stream)), "aco_colony_construct")
+
+    def colony_finalize(self, pass_: int, it: int, stream: Optional[torch.cuda.Stream] = None):
+        _lib.check(self.lib.aco_colony_finalize(self.ctx, pass_, it, C.c_void_p(self.keys.data_ptr()),
+                                                _stream_handle(stream)), "aco_colony_finalize")
+
+    def colony_end(self, stream: Optional[torch.cuda.Stream] = None):
+        _lib.check(self.lib.aco_colony_end(self.ctx, _stream_handle(stream)), "aco_colony_end")
+
+    def run_colony(self, p: Params, rank: int, world: int, group=None):
+        """Shared colony over torch.distributed (NCCL): p.ants per rank, global
+        ants = p.ants * world; one int64 MIN allreduce per region per iteration."""
+        import torch.distributed as dist
+        keys = self.colony_begin(p, rank * p.ants)
+        for pass_ in (1, 2):
+            if not (p.passes & pass_):
+                continue
+            for it in range(p.iterations):
+                self.colony_construct(pass_, it)
+                if world > 1:
+                    dist.all_reduce(keys, op=dist.ReduceOp.MIN, group=group)
+                self.colony_finalize(pass_, it)
+        self.colony_end()
+        return self
+
     def timing(self):
         """(ms[construct, finalize, init], launches[...]) of the last timed run."""
         ms = (C.c_double * 3)()

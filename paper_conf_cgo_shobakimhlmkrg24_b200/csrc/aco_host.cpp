@@ -18,8 +18,21 @@
 
 using namespace aco;
 
+// A planned run: launch classes, workspace offsets and the launch context.
+struct Plan {
+  std::vector<ClassLaunch> launches[3];
+  uint32_t fin_smem[3] = {0, 0, 0};
+  uint32_t init_smem = 0, p2_smem = 0, max_n = 0, n_upd = 0;
+  uint32_t pass_mask = 0, iterations = 0;
+  bool any_t32 = false, nc4 = false, timing = false, p2_done = false;
+  uint64_t o_state = 0, o_rws = 0, o_upd = 0, o_gb2 = 0, o_gb2c = 0, o_keys = 0;
+  LaunchCtx L{};
+};
+
 struct aco_ctx_s {
   int device = 0;
+  Plan plan;
+  bool planned = false;
   MachineDev mach{};
   bool machine_uploaded = false;
   // loaded batch
@@ -546,70 +559,92 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
 
 }  // namespace
 
-aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspace, size_t ws_bytes,
-                              size_t *ws_needed, void *cuda_stream) {
-  if (!ctx || !p) return ACO_E_ARG;
+namespace {
+
+aco_status check_params(const aco_params *p) {
   if (p->pass < 1 || p->pass > 3 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
       p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->tau0 > 65535u ||
       p->tau0 < p->tau_min || p->tau0 > p->tau_max || p->q0_t > (1ull << 32) || p->rho_q16 > 65536u ||
       p->iterations > 0x7FFFFFFFu)
     return ACO_E_ARG;
-  if ((p->flags & ACO_FLAG_DUMP) && !ctx->dump_cost) return ACO_E_ARG;
+  return ACO_OK;
+}
+
+// Plan a run (launch classes, workspace layout), upload the plan blob and
+// fill ctx->plan.  ants = this context's ants (ant ids ant_base ..).
+aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *d_workspace, size_t ws_bytes,
+                     size_t *ws_needed, void *cuda_stream, bool colony) {
+  if (aco_status st = check_params(p)) return st;
+  if ((p->flags & ACO_FLAG_DUMP) && (!ctx->dump_cost || colony)) return ACO_E_ARG;
   const uint32_t count = ctx->count, A = p->ants;
-  // ---- per-pass construct classes (pass, ants/block, tau in smem, u32 cycles, mask, smem bucket)
+  Plan saved = ctx->plan;  // a sizing call must not disturb a planned run
+  Plan &P = ctx->plan;
+  P = Plan();
+  // ---- per-pass construct classes
   struct Cls {
     Shape sh;
-    bool mask, t32;
+    bool mask, t32, gs;
     uint32_t smem;
     std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, uint32_t>;
+  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t>;
   std::map<Key, Cls> classes;
-  uint32_t fin_smem[3] = {0, 0, 0}, max_n = 0, init_smem = 0, p2_smem = 0;
-  bool any_t32 = false;
-  const bool nc4 = ctx->mach.n_classes > 2;
+  P.nc4 = ctx->mach.n_classes > 2;
   // launch-shape policy (tuning knobs; defaults measured on B200)
   uint32_t tgt_threads[2] = {512, 256}, max_lanes[2] = {8, 1};
   if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
+  std::vector<uint8_t> gs(count, 0);
+  std::vector<uint32_t> gs_words(count, 0), scratch_words(count, 0);
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
-    max_n = std::max(max_n, R.n);
+    P.max_n = std::max(P.max_n, R.n);
     const bool t32 = R.max_cycle_bound > 65535u;
-    any_t32 |= t32;
+    P.any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
-      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, nc4);
-      if (pass == 1) init_smem = std::max(init_smem, R.img.bytes + 4 * W + 16);
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
       if (!(p->pass & pass)) continue;
-      const bool rare = pass == 2 && (t32 || nc4);  // variants compiled without tau staging, 1|4 lanes
-      const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u, !rare, rare,
-                                  pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1]);
-      if (sh.apb == 0) return ACO_E_TOO_LARGE;
-      const bool mask = R.n <= 1024;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, sh.smem);
+      const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
+      Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u, !rare, rare,
+                            pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1]);
+      bool g = false;
+      if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
+        sh = Shape{64, 4, 0, false};
+        g = true;
+        gs[r] = 1;
+        gs_words[r] = std::max(gs_words[r], W);
+      }
+      const bool mask = R.n <= 1024 && !g;
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem);
       Cls &c = classes[key];
       c.sh = sh;
       c.mask = mask;
       c.t32 = pass == 2 && t32;
+      c.gs = g;
       c.smem = std::max(c.smem, sh.smem);
       c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
     }
-    p2_smem = std::max(p2_smem, 4 * R.n + 16);
+    P.p2_smem = std::max(P.p2_smem, 4 * R.n + 16);
   }
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
     for (uint32_t pass = 1; pass <= 2; ++pass) {
-      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && any_t32, nc4);
-      const uint32_t fs = R.img.bytes + 4 * W + 4 * R.n + 2 * R.n + 64;
-      fin_smem[pass] = std::max(fin_smem[pass], fs);
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && P.any_t32, P.nc4);
+      const uint32_t need_words = W + R.n + (R.n + 1) / 2 + 4;  // state + cycles + order
+      const uint32_t fs = R.img.bytes + 4 * need_words + 64;
+      if (fs > kSmemPerSM - 2048) gs[r] = 1;  // replay scratch in the workspace too
+      scratch_words[r] = std::max(scratch_words[r], need_words);
+      if (!gs[r]) {
+        P.fin_smem[pass] = std::max(P.fin_smem[pass], fs);
+        if (pass == 1) P.init_smem = std::max(P.init_smem, fs);
+      }
     }
   }
-  if (std::max(fin_smem[1], fin_smem[2]) > 227 * 1024) return ACO_E_TOO_LARGE;
   // ---- workspace layout
   uint64_t off = 0;
-  const uint64_t o_state = off;
+  P.o_state = off;
   off = align256(off + sizeof(RegionState) * (uint64_t)count);
-  const uint64_t o_rws = off;
+  P.o_rws = off;
   off = align16(off + sizeof(RegionWs) * (uint64_t)count);
   const uint64_t o_items = off;
   uint64_t n_items = 0;
@@ -619,7 +654,7 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     n_items += (uint64_t)kv.second.regs.size() * ((A + kv.second.sh.apb - 1) / kv.second.sh.apb);
   }
   off = align16(off + sizeof(BlockItem) * n_items);
-  const uint64_t o_upd = off;
+  P.o_upd = off;
   uint64_t n_upd_max = 0;
   for (uint32_t r = 0; r < count; ++r) {
     const uint64_t n = ctx->regions[r].n;
@@ -629,14 +664,16 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   const uint64_t sum_n = ctx->inst_off.empty() ? 0 : ctx->inst_off[count];
   const uint64_t o_gb1 = off;
   off = align256(off + 2 * sum_n + 16);
-  const uint64_t o_gb2 = off;
+  P.o_gb2 = off;
   off = align256(off + 2 * sum_n + 16);
-  const uint64_t o_gb2c = off;
+  P.o_gb2c = off;
   off = align256(off + 4 * sum_n + 16);
   const uint64_t o_next = off;
   off = align256(off + 2 * (sum_n + count) + 16);
   const uint64_t o_cost = off;
   off = align256(off + 4ull * A * count);
+  P.o_keys = off;
+  off = align256(off + 8ull * count);
   std::vector<RegionWs> rws(count);
   for (uint32_t r = 0; r < count; ++r) {
     const uint32_t n = ctx->regions[r].n;
@@ -647,22 +684,37 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     off = align16(off + 2ull * w.tau_len);
     w.o_cost = o_cost + 4ull * A * r;
     w.o_gb1 = o_gb1 + 2 * ctx->inst_off[r];
-    w.o_gb2 = o_gb2 + 2 * ctx->inst_off[r];
-    w.o_gb2c = o_gb2c + 4 * ctx->inst_off[r];
+    w.o_gb2 = P.o_gb2 + 2 * ctx->inst_off[r];
+    w.o_gb2c = P.o_gb2c + 4 * ctx->inst_off[r];
     w.o_dump = (uint64_t)A * ctx->inst_off[r];
     w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
+    w.gs = gs[r];
+    if (gs[r]) {
+      off = align256(off);
+      w.o_gstate = off;
+      off += 4ull * A * gs_words[r];
+      off = align256(off);
+      w.o_scratch = off;
+      off = align256(off + 4ull * scratch_words[r]);
+    }
   }
-  // pheromone-update items (after the construct items in the plan blob)
   std::vector<UpdItem> upd;
   for (uint32_t r = 0; r < count; ++r)
     for (uint32_t v0 = 0; v0 < rws[r].tau_len / 8; v0 += kUpdVec) upd.push_back(UpdItem{r, v0});
+  P.n_upd = (uint32_t)upd.size();
   const size_t need = align256(off);
   if (ws_needed) *ws_needed = need;
   const bool plan_only = !d_workspace;  // (debug: ACO_DEBUG_PLAN prints the plan)
-  if (plan_only && !getenv("ACO_DEBUG_PLAN")) return ACO_OK;
+  if (plan_only && !getenv("ACO_DEBUG_PLAN")) {
+    ctx->plan = saved;
+    return ACO_OK;
+  }
   if (!plan_only) {
     if (!ctx->arena && ctx->count) return ACO_E_STATE;
-    if (ws_bytes < need) return ACO_E_WORKSPACE;
+    if (ws_bytes < need) {
+      ctx->plan = saved;
+      return ACO_E_WORKSPACE;
+    }
     if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
     if (!ctx->machine_uploaded) {
       if (set_machine(ctx->mach) != 0) return ACO_E_CUDA;
@@ -671,12 +723,11 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
     if (!ctx->make_side()) return ACO_E_CUDA;
   }
   unsigned char *ws = (unsigned char *)d_workspace;
-  // ---- host plan: RegionWs table + block items, one H2D
+  // ---- host plan: RegionWs table + block items + update items, one H2D
   std::vector<unsigned char> &blob = ctx->plan_blob;
-  blob.assign(o_upd - o_rws + sizeof(UpdItem) * upd.size(), 0);
-  if (!upd.empty()) std::memcpy(blob.data() + (o_upd - o_rws), upd.data(), sizeof(UpdItem) * upd.size());
+  blob.assign(P.o_upd - P.o_rws + sizeof(UpdItem) * upd.size(), 0);
+  if (!upd.empty()) std::memcpy(blob.data() + (P.o_upd - P.o_rws), upd.data(), sizeof(UpdItem) * upd.size());
   std::memcpy(blob.data(), rws.data(), sizeof(RegionWs) * count);
-  std::vector<ClassLaunch> launches[3];
   std::vector<uint64_t> class_work[3];
   {
     size_t ci = 0;
@@ -684,7 +735,7 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
       Cls &c = kv.second;
       std::sort(c.regs.begin(), c.regs.end());
       const uint64_t base = class_item_off[ci++].second;
-      BlockItem *items = (BlockItem *)(blob.data() + (o_items - o_rws)) + base;
+      BlockItem *items = (BlockItem *)(blob.data() + (o_items - P.o_rws)) + base;
       uint64_t k = 0;
       for (auto &pr : c.regs)
         for (uint32_t a0 = 0; a0 < A; a0 += c.sh.apb) items[k++] = BlockItem{pr.second, a0};
@@ -697,37 +748,40 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
       cl.max_n = c.mask ? 1024 : 65535;
       cl.tau_smem = c.sh.ts;
       cl.t32 = c.t32;
-      cl.nc4 = nc4;
-      launches[std::get<0>(kv.first)].push_back(cl);
+      cl.nc4 = P.nc4;
+      cl.gs = c.gs;
+      P.launches[std::get<0>(kv.first)].push_back(cl);
       class_work[std::get<0>(kv.first)].push_back(0);
       for (auto &pr : c.regs) class_work[std::get<0>(kv.first)].back() += ~pr.first;
     }
   }
   for (int pass = 1; pass <= 2; ++pass) {  // biggest classes first (fork round-robin)
-    std::vector<size_t> idx(launches[pass].size());
+    std::vector<size_t> idx(P.launches[pass].size());
     for (size_t i = 0; i < idx.size(); ++i) idx[i] = i;
     std::sort(idx.begin(), idx.end(), [&](size_t a, size_t b) { return class_work[pass][a] > class_work[pass][b]; });
     std::vector<ClassLaunch> sorted;
-    for (size_t i : idx) sorted.push_back(launches[pass][i]);
-    launches[pass] = sorted;
+    for (size_t i : idx) sorted.push_back(P.launches[pass][i]);
+    P.launches[pass] = sorted;
     if (getenv("ACO_DEBUG_PLAN"))
       for (size_t i = 0; i < idx.size(); ++i)
-        fprintf(stderr, "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d work %.3g\n",
-                pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes, (int)sorted[i].tau_smem,
-                (int)sorted[i].t32, (double)class_work[pass][idx[i]]);
+        fprintf(stderr,
+                "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d gs %d "
+                "work %.3g\n",
+                pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes,
+                (int)sorted[i].tau_smem, (int)sorted[i].t32, (int)sorted[i].gs, (double)class_work[pass][idx[i]]);
   }
-  if (plan_only) return ACO_OK;
+  if (plan_only) {
+    ctx->plan = saved;
+    return ACO_OK;
+  }
   cudaStream_t s = (cudaStream_t)cuda_stream;
-  {
-    aco_status hs = ctx->staged_h2d(1, ws + o_rws, blob.data(), blob.size(), s);
-    if (hs != ACO_OK) return hs;
-  }
-  LaunchCtx L;
+  if (aco_status hs = ctx->staged_h2d(1, ws + P.o_rws, blob.data(), blob.size(), s)) return hs;
+  LaunchCtx &L = P.L;
   L.arena = ctx->arena;
   L.ws = ws;
   L.regions = (const RegionDev *)ctx->arena;
-  L.state = (RegionState *)(ws + o_state);
-  L.rws = (const RegionWs *)(ws + o_rws);
+  L.state = (RegionState *)(ws + P.o_state);
+  L.rws = (const RegionWs *)(ws + P.o_rws);
   L.dump_cost = ctx->dump_cost;
   L.dump_order = ctx->dump_order;
   L.dump_cycle = ctx->dump_cycle;
@@ -752,88 +806,166 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   cfg.stop_at_lb = p->stop_at_lb;
   cfg.n_classes = ctx->mach.n_classes;
   cfg.count = count;
+  cfg.ant_base = ant_base;
   cfg.dump_slice = (uint64_t)A * sum_n;
+  cfg.keys = nullptr;
   L.stream = cuda_stream;
   L.launches = 0;
-  const bool timing = (p->flags & ACO_FLAG_TIMING) != 0;
+  P.timing = (p->flags & ACO_FLAG_TIMING) != 0;
+  P.pass_mask = p->pass;
+  P.iterations = p->iterations;
   ctx->ev_used = 0;
   for (int ph = 0; ph < 3; ++ph) {
     ctx->ev_pairs[ph].clear();
     ctx->phase_launches[ph] = 0;
   }
-  // phase bracket: record an event pair around a group of launches
-  auto begin = [&](int ph) -> size_t {
-    if (!timing) return 0;
-    const size_t i = ctx->ev_used;
-    cudaEvent_t e = ctx->next_event();
-    if (e) cudaEventRecord(e, s);
-    (void)ph;
-    return i;
-  };
-  auto end = [&](int ph, size_t i0, uint64_t l0) {
-    ctx->phase_launches[ph] += L.launches - l0;
-    if (!timing) return;
-    const size_t i1 = ctx->ev_used;
-    cudaEvent_t e = ctx->next_event();
-    if (e) cudaEventRecord(e, s);
-    ctx->ev_pairs[ph].push_back({i0, i1});
-  };
-  int err = 0;
-  {
-    const size_t e0 = begin(2);
-    const uint64_t l0 = L.launches;
-    err |= launch_init(L, init_smem, max_n);
-    end(2, e0, l0);
-  }
-  for (uint32_t pass = 1; pass <= 2 && !err; ++pass) {
-    if (pass == 2) {
-      const size_t e0 = begin(2);
-      const uint64_t l0 = L.launches;
-      err |= launch_pass2_init(L, p2_smem, max_n);
-      end(2, e0, l0);
-    }
-    if (!(p->pass & pass)) continue;
-    for (uint32_t it = 0; it < p->iterations && !err; ++it) {
-      size_t e0 = begin(0);
-      uint64_t l0 = L.launches;
-      const std::vector<ClassLaunch> &cls = launches[pass];
-      if (cls.size() <= 1) {
-        for (const ClassLaunch &cl : cls) err |= launch_construct(L, pass, it, cl);
-      } else {
-        // fork: classes round-robin over the internal streams, join on `s`
-        const int k = (int)std::min<size_t>(cls.size(), aco_ctx_s::kStreams);
-        err |= cudaEventRecord(ctx->fork_ev, s) != cudaSuccess;
-        for (int i = 0; i < k; ++i) err |= cudaStreamWaitEvent(ctx->side[i], ctx->fork_ev, 0) != cudaSuccess;
-        for (size_t c = 0; c < cls.size(); ++c) {
-          L.stream = ctx->side[c % k];
-          err |= launch_construct(L, pass, it, cls[c]);
-        }
-        L.stream = cuda_stream;
-        for (int i = 0; i < k; ++i) {
-          err |= cudaEventRecord(ctx->join_ev[i], ctx->side[i]) != cudaSuccess;
-          err |= cudaStreamWaitEvent(s, ctx->join_ev[i], 0) != cudaSuccess;
-        }
-      }
-      end(0, e0, l0);
-      e0 = begin(1);
-      l0 = L.launches;
-      err |= launch_finalize(L, pass, it, fin_smem[pass], max_n, pass == 2 && any_t32, nc4,
-                             (const UpdItem *)(ws + o_upd), (uint32_t)upd.size());
-      end(1, e0, l0);
-    }
-  }
-  ctx->launches = L.launches;
-  if (err) return ACO_E_CUDA;
   ctx->ws = ws;
   ctx->ws_bytes = ws_bytes;
   ctx->stream = cuda_stream;
   ctx->cfg = cfg;
-  ctx->o_state = o_state;
-  ctx->o_rws = o_rws;
-  ctx->o_gb2 = o_gb2;
-  ctx->o_gb2c = o_gb2c;
+  ctx->o_state = P.o_state;
+  ctx->o_rws = P.o_rws;
+  ctx->o_gb2 = P.o_gb2;
+  ctx->o_gb2c = P.o_gb2c;
   ctx->have_run = true;
+  ctx->planned = true;
   return ACO_OK;
+}
+
+// ---- phase runners (stream-ordered on the plan's stream)
+struct Bracket {  // ACO_FLAG_TIMING: an event pair around a group of launches
+  aco_ctx ctx;
+  int ph;
+  size_t e0;
+  uint64_t l0;
+  Bracket(aco_ctx c, int phase) : ctx(c), ph(phase), e0(0), l0(c->plan.L.launches) {
+    if (!ctx->plan.timing) return;
+    e0 = ctx->ev_used;
+    if (cudaEvent_t e = ctx->next_event()) cudaEventRecord(e, (cudaStream_t)ctx->plan.L.stream);
+  }
+  ~Bracket() {
+    ctx->phase_launches[ph] += ctx->plan.L.launches - l0;
+    if (!ctx->plan.timing) return;
+    const size_t e1 = ctx->ev_used;
+    if (cudaEvent_t e = ctx->next_event()) cudaEventRecord(e, (cudaStream_t)ctx->plan.L.stream);
+    ctx->ev_pairs[ph].push_back({e0, e1});
+  }
+};
+
+int run_init(aco_ctx ctx) {
+  Bracket b(ctx, 2);
+  return launch_init(ctx->plan.L, ctx->plan.init_smem, ctx->plan.max_n);
+}
+
+int run_pass2_init(aco_ctx ctx) {
+  Bracket b(ctx, 2);
+  ctx->plan.p2_done = true;
+  return launch_pass2_init(ctx->plan.L, ctx->plan.p2_smem, ctx->plan.max_n);
+}
+
+int run_construct(aco_ctx ctx, uint32_t pass, uint32_t it) {
+  Plan &P = ctx->plan;
+  LaunchCtx &L = P.L;
+  Bracket b(ctx, 0);
+  int err = 0;
+  const std::vector<ClassLaunch> &cls = P.launches[pass];
+  void *main = L.stream;
+  cudaStream_t s = (cudaStream_t)main;
+  if (cls.size() <= 1) {
+    for (const ClassLaunch &cl : cls) err |= launch_construct(L, pass, it, cl);
+  } else {  // fork: classes round-robin over the internal streams, join on the main stream
+    const int k = (int)std::min<size_t>(cls.size(), aco_ctx_s::kStreams);
+    err |= cudaEventRecord(ctx->fork_ev, s) != cudaSuccess;
+    for (int i = 0; i < k; ++i) err |= cudaStreamWaitEvent(ctx->side[i], ctx->fork_ev, 0) != cudaSuccess;
+    for (size_t c = 0; c < cls.size(); ++c) {
+      L.stream = ctx->side[c % k];
+      err |= launch_construct(L, pass, it, cls[c]);
+    }
+    L.stream = main;
+    for (int i = 0; i < k; ++i) {
+      err |= cudaEventRecord(ctx->join_ev[i], ctx->side[i]) != cudaSuccess;
+      err |= cudaStreamWaitEvent(s, ctx->join_ev[i], 0) != cudaSuccess;
+    }
+  }
+  return err;
+}
+
+int run_finalize(aco_ctx ctx, uint32_t pass, uint32_t it, int64_t *keys) {
+  Plan &P = ctx->plan;
+  Bracket b(ctx, 1);
+  P.L.cfg.keys = keys;
+  const int err = launch_finalize(P.L, pass, it, P.fin_smem[pass], P.max_n, pass == 2 && P.any_t32, P.nc4,
+                                  (const UpdItem *)(P.L.ws + P.o_upd), P.n_upd);
+  P.L.cfg.keys = nullptr;
+  return err;
+}
+
+}  // namespace
+
+aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspace, size_t ws_bytes,
+                              size_t *ws_needed, void *cuda_stream) {
+  if (!ctx || !p) return ACO_E_ARG;
+  aco_status st = make_plan(ctx, p, 0, d_workspace, ws_bytes, ws_needed, cuda_stream, false);
+  if (st != ACO_OK || !d_workspace) return st;
+  int err = run_init(ctx);
+  for (uint32_t pass = 1; pass <= 2 && !err; ++pass) {
+    if (pass == 2) err |= run_pass2_init(ctx);
+    if (!(p->pass & pass)) continue;
+    for (uint32_t it = 0; it < p->iterations && !err; ++it) {
+      err |= run_construct(ctx, pass, it);
+      err |= run_finalize(ctx, pass, it, nullptr);
+    }
+  }
+  ctx->launches = ctx->plan.L.launches;
+  return err ? ACO_E_CUDA : ACO_OK;
+}
+
+aco_status aco_colony_begin(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *d_workspace, size_t ws_bytes,
+                            size_t *ws_needed, void *cuda_stream) {
+  if (!ctx || !p) return ACO_E_ARG;
+  if (p->flags & ACO_FLAG_DUMP) return ACO_E_ARG;
+  aco_status st = make_plan(ctx, p, ant_base, d_workspace, ws_bytes, ws_needed, cuda_stream, true);
+  if (st != ACO_OK || !d_workspace) return st;
+  const int err = run_init(ctx);
+  ctx->launches = ctx->plan.L.launches;
+  return err ? ACO_E_CUDA : ACO_OK;
+}
+
+aco_status aco_colony_construct(aco_ctx ctx, uint32_t pass, uint32_t iter, int64_t *d_keys, void *cuda_stream) {
+  if (!ctx || !d_keys || pass < 1 || pass > 2) return ACO_E_ARG;
+  if (!ctx->planned) return ACO_E_STATE;
+  Plan &P = ctx->plan;
+  if (!(P.pass_mask & pass) || iter >= P.iterations) return ACO_E_ARG;
+  P.L.stream = cuda_stream;
+  int err = 0;
+  if (pass == 2 && iter == 0) err |= run_pass2_init(ctx);
+  err |= run_construct(ctx, pass, iter);
+  err |= launch_local_keys(P.L, d_keys);
+  ctx->launches = P.L.launches;
+  return err ? ACO_E_CUDA : ACO_OK;
+}
+
+aco_status aco_colony_finalize(aco_ctx ctx, uint32_t pass, uint32_t iter, int64_t *d_keys, void *cuda_stream) {
+  if (!ctx || !d_keys || pass < 1 || pass > 2) return ACO_E_ARG;
+  if (!ctx->planned) return ACO_E_STATE;
+  Plan &P = ctx->plan;
+  if (!(P.pass_mask & pass) || iter >= P.iterations) return ACO_E_ARG;
+  P.L.stream = cuda_stream;
+  const int err = run_finalize(ctx, pass, iter, d_keys);
+  ctx->launches = P.L.launches;
+  return err ? ACO_E_CUDA : ACO_OK;
+}
+
+aco_status aco_colony_end(aco_ctx ctx, void *cuda_stream) {
+  if (!ctx) return ACO_E_ARG;
+  if (!ctx->planned) return ACO_E_STATE;
+  Plan &P = ctx->plan;
+  P.L.stream = cuda_stream;
+  int err = 0;
+  if (!P.p2_done) err |= run_pass2_init(ctx);  // ASAP timing of the pass-1 result
+  ctx->stream = cuda_stream;
+  ctx->launches = P.L.launches;
+  return err ? ACO_E_CUDA : ACO_OK;
 }
 
 aco_status aco_get_timing(aco_ctx ctx, double ms[3], uint64_t launches[3]) {

@@ -92,8 +92,10 @@ struct RegionWs {
   uint64_t o_gb2c;   // u32 [n]  pass-2 global best cycles (in order)
   uint64_t o_dump;   // element offset of this region in a dump (pass, iter) slice = ants * sum n_q
   uint64_t o_next;   // u16 [n+1]: the iteration winner's successor of each row (0xFFFF: none)
+  uint64_t o_gstate; // global-state regions: per-ant state [word][ant] (ants x words u32)
+  uint64_t o_scratch;// global-state regions: replay scratch (words + cycles + order)
   uint32_t tau_len;  // (n+1)*n rounded up to a multiple of 8
-  uint32_t pad;
+  uint32_t gs;       // 1: the region's state does not fit shared memory (global-state kernels)
 };
 
 // Pheromone-update work item: vectors [v0, v0 + kUpdVec) of a region's table.
@@ -112,8 +114,9 @@ struct RunCfg {
   uint32_t tau0, rho_q16, delta, tau_min, tau_max;
   uint32_t stop_no_improve, stop_at_lb, n_classes;
   uint32_t count;       // regions
-  uint32_t pad;
+  uint32_t ant_base;    // global id of this context's first ant (shared colony), else 0
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
+  int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };
 
 struct MachineDev {
@@ -175,6 +178,7 @@ struct ClassLaunch {
   bool tau_smem;           // stage tau in shared memory
   bool t32;                // u32 pass-2 cycle array
   bool nc4;                // 3-4 register classes (u16 last-use counts)
+  bool gs;                 // per-ant state in global memory (huge regions)
 };
 
 int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success
@@ -183,6 +187,11 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);
 int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
                     bool nc4, const UpdItem *upd, uint32_t n_upd);
+int launch_local_keys(LaunchCtx &L, int64_t *keys);  // shared colony: per-region local argmin keys
+
+// Biased winner key: (cost << 32 | global ant) XOR 2^63, so that a signed
+// int64 MIN (NCCL / torch) orders keys like the unsigned (cost, ant) pair.
+constexpr uint64_t kKeyBias = 1ull << 63;
 int last_cuda_error();
 
 }  // namespace aco

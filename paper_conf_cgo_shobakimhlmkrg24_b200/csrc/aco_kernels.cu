@@ -631,7 +631,7 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
   for (uint32_t i = threadIdx.x; i < bytes / 16; i += blockDim.x) dst[i] = src[i];
 }
 
-template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4>
+template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, bool GS>
 __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__restrict__ items,
                                                    uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
@@ -641,42 +641,53 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
   const RegionWs &W = A.rws[bi.region];
   extern __shared__ uint4 smem4[];
   unsigned char *smem = (unsigned char *)smem4;
-  const uint32_t img_bytes = rd->img.bytes;
-  stage(smem4, (const uint4 *)(A.arena + rd->o_image), img_bytes);
-  const uint16_t *tau;
-  uint32_t state_off = img_bytes;
-  if (TAU_SMEM) {
-    const uint32_t tb = tau_smem_bytes(rd->n);
-    stage((uint4 *)(smem + img_bytes), (const uint4 *)(A.ws + W.o_tau), tb);
-    tau = (const uint16_t *)(smem + img_bytes);
-    state_off += tb;
-  } else {
-    tau = (const uint16_t *)(A.ws + W.o_tau);
-  }
-  __syncthreads();
   const uint32_t local = threadIdx.x / LG;  // ant within the block
-  const uint32_t ant = bi.ant0 + local;
-  if (ant >= A.cfg.ants) return;  // whole lane group
+  const uint32_t ai = bi.ant0 + local;      // ant within this context's share of the region
+  const uint32_t ant = A.cfg.ant_base + ai; // global ant id (Philox key, groups, winner key)
+  const uint16_t *tau = (const uint16_t *)(A.ws + W.o_tau);
+  const unsigned char *img = A.arena + rd->o_image;
+  uint32_t *stbase;
+  uint32_t stride;
+  if (GS) {  // huge region: statics through L1/L2, per-ant state in the workspace
+    if (ai >= A.cfg.ants) return;
+    stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
+    stride = A.cfg.ants;
+  } else {
+    const uint32_t img_bytes = rd->img.bytes;
+    stage(smem4, (const uint4 *)img, img_bytes);
+    uint32_t state_off = img_bytes;
+    if (TAU_SMEM) {
+      const uint32_t tb = tau_smem_bytes(rd->n);
+      stage((uint4 *)(smem + img_bytes), (const uint4 *)(A.ws + W.o_tau), tb);
+      tau = (const uint16_t *)(smem + img_bytes);
+      state_off += tb;
+    }
+    __syncthreads();
+    if (ai >= A.cfg.ants) return;  // whole lane group
+    img = smem;
+    stbase = (uint32_t *)(smem + state_off) + local;
+    stride = blockDim.x / LG;
+  }
   const Grp<LG> G(threadIdx.x);
-  const SV V = make_sv(smem, rd);
-  const St S = make_st<PASS, T32, NC4>((uint32_t *)(smem + state_off) + local, blockDim.x / LG, V);
+  const SV V = make_sv(img, rd);
+  const St S = make_st<PASS, T32, NC4>(stbase, stride, V);
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
   if (PASS == 1) {
     uint16_t *rec = nullptr;
     if (dump && A.dump_order)
-      rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ant * V.n;
+      rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
     o = ant_pass1<LG, MASK>(V, tau, S, G, ant, iter, A.cfg, false, rec);
   } else {
     uint32_t tgt[4];
 #pragma unroll
     for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
-    const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE);
+    const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys;
     uint16_t *rec_o = nullptr;
     uint32_t *rec_c = nullptr;
     if (dump && A.dump_order && A.dump_cycle) {
       const size_t base =
-          ((size_t)A.cfg.iterations + iter) * A.cfg.dump_slice + W.o_dump + (size_t)ant * V.n;
+          ((size_t)A.cfg.iterations + iter) * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
       rec_o = A.dump_order + base;
       rec_c = A.dump_cycle + base;
     }
@@ -685,10 +696,10 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
   }
   if (G.leader()) {
     uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
-    costs[ant] = o.cost;
+    costs[ai] = o.cost;
     if (dump && A.dump_cost)
-      A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants +
-                  ant] = o.cost;
+      A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants + ai] =
+          o.cost;
   }
 }
 
@@ -756,21 +767,25 @@ __global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restri
 
 // Per-region initialisation: tau0, the greedy pass-1 heuristic schedule
 // (R28: the q0 = 1 ant on a uniform tau), LB check (L251).
-template <bool MASK>
-__global__ void __launch_bounds__(128) k_init(KArgs A) {
+template <bool MASK, bool GS>
+__device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
   RegionState &rs = A.state[r];
   uint16_t *tau = (uint16_t *)(A.ws + W.o_tau);
-  extern __shared__ uint4 smem4[];
-  unsigned char *smem = (unsigned char *)smem4;
-  stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
+  const unsigned char *img = A.arena + rd->o_image;
+  uint32_t *stw = (uint32_t *)(A.ws + W.o_scratch);
+  if (!GS) {
+    stage((uint4 *)smem, (const uint4 *)img, rd->img.bytes);
+    img = smem;
+    stw = (uint32_t *)(smem + rd->img.bytes);
+  }
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   __syncthreads();
   if (threadIdx.x < 32) {  // warp 0 builds the greedy schedule as one 32-lane group
-    const SV V = make_sv(smem, rd);
-    const St S = make_st<1, false, false>((uint32_t *)(smem + rd->img.bytes), 1, V);
+    const SV V = make_sv(img, rd);
+    const St S = make_st<1, false, false>(stw, 1, V);
     uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
     const Grp<32> G32(threadIdx.x);
     AntOut o = ant_pass1<32, MASK>(V, tau, S, G32, 0, 0, A.cfg, true, gb1);
@@ -785,6 +800,13 @@ __global__ void __launch_bounds__(128) k_init(KArgs A) {
     rs.hash = 0xcbf29ce484222325ull;
     rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
   }
+}
+
+template <bool MASK>
+__global__ void __launch_bounds__(128) k_init(KArgs A) {
+  extern __shared__ uint4 smem4[];
+  if (A.rws[blockIdx.x].gs) init_body<false, true>(A, (unsigned char *)smem4);
+  else init_body<MASK, false>(A, (unsigned char *)smem4);
 }
 
 // Pass transition (L147; R13, R18, R29): target from the pass-1 best, the
@@ -830,32 +852,39 @@ __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
 }
 
 // End of an iteration for one region (L137-L139), one warp: argmin over
-// (cost, ant) (R10), replay of the winner (lane 0) to recover its order,
-// the winner's successor table for the pheromone update, and the epilogue.
-template <int PASS, bool MASK, bool T32, bool NC4>
-__global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
+// (cost, ant) (R10) -- or the shared colony's allreduced key -- replay of the
+// winner by the whole warp to recover its order, the winner's successor
+// table for the pheromone update, and the epilogue.
+template <int PASS, bool MASK, bool T32, bool NC4, bool GS>
+__device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsigned char *smem,
+                                            uint32_t *s_prp, uint32_t &s_flag) {
   const uint32_t r = blockIdx.x;
   RegionState &rs = A.state[r];
-  if (!rs.active) return;
   const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
   const uint32_t n = rd->n;
   const uint16_t *tau = (const uint16_t *)(A.ws + W.o_tau);
   const uint32_t *costs = (const uint32_t *)(A.ws + W.o_cost);
-  extern __shared__ uint4 smem4[];
-  unsigned char *smem = (unsigned char *)smem4;
-  __shared__ uint32_t s_prp[2], s_flag;
-  stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
+  const unsigned char *img = A.arena + rd->o_image;
+  uint32_t *stw = (uint32_t *)(A.ws + W.o_scratch);
+  if (!GS) {
+    stage((uint4 *)smem, (const uint4 *)img, rd->img.bytes);
+    img = smem;
+    stw = (uint32_t *)(smem + rd->img.bytes);
+  }
   unsigned long long best = ~0ull;
-  for (uint32_t a = threadIdx.x; a < A.cfg.ants; a += 32)
-    best = min(best, ((unsigned long long)costs[a] << 32) | a);
+  if (A.cfg.keys) {
+    best = (unsigned long long)A.cfg.keys[r] ^ kKeyBias;
+  } else {
+    for (uint32_t a = threadIdx.x; a < A.cfg.ants; a += 32)
+      best = min(best, ((unsigned long long)costs[a] << 32) | (A.cfg.ant_base + a));
 #pragma unroll
-  for (int off = 16; off; off >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, off));
+    for (int off = 16; off; off >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, off));
+  }
   const uint32_t wcost = (uint32_t)(best >> 32), want = (uint32_t)best;
   const bool have = wcost != kInvalid;
-  // smem: [image | ant state | cycle u32[n] | order u16[n]]
-  const SV V = make_sv(smem, rd);
-  uint32_t *stw = (uint32_t *)(smem + rd->img.bytes);
+  // state: [ant state | cycle u32[n] | order u16[n]]
+  const SV V = make_sv(img, rd);
   uint32_t *cyc = stw + ant_words(PASS, n, rd->nwr, rd->nremw, T32, NC4);
   uint16_t *ord = (uint16_t *)(cyc + n);
   __syncwarp();
@@ -919,6 +948,30 @@ __global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   }
 }
 
+template <int PASS, bool MASK, bool T32, bool NC4>
+__global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
+  if (!A.state[blockIdx.x].active) return;
+  extern __shared__ uint4 smem4[];
+  __shared__ uint32_t s_prp[2], s_flag;
+  if (A.rws[blockIdx.x].gs)
+    select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+  else
+    select_body<PASS, MASK, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+}
+
+// Shared colony: per-region local argmin over this context's ants, written as
+// a biased key for a signed int64 MIN allreduce across ranks.
+__global__ void __launch_bounds__(32) k_local_keys(KArgs A, int64_t *keys) {
+  const uint32_t r = blockIdx.x;
+  const uint32_t *costs = (const uint32_t *)(A.ws + A.rws[r].o_cost);
+  unsigned long long best = ~0ull;
+  for (uint32_t a = threadIdx.x; a < A.cfg.ants; a += 32)
+    best = min(best, ((unsigned long long)costs[a] << 32) | (A.cfg.ant_base + a));
+#pragma unroll
+  for (int off = 16; off; off >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, off));
+  if (threadIdx.x == 0) keys[r] = (int64_t)(best ^ kKeyBias);
+}
+
 // Termination (L110, L139, L226; R12), after the pheromone update.
 __global__ void k_stop(KArgs A, uint32_t pass) {
   const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
@@ -969,14 +1022,14 @@ int set_machine(const MachineDev &m) {
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
 #undef ACO_SEL
-#define ACO_CON(LG, M, TS) big_smem(k_construct<1, LG, M, TS, false, false>); \
-  big_smem(k_construct<2, LG, M, TS, false, false>);
+#define ACO_CON(LG, M, TS) big_smem(k_construct<1, LG, M, TS, false, false, false>); \
+  big_smem(k_construct<2, LG, M, TS, false, false, false>);
 #define ACO_CON_M(LG) ACO_CON(LG, true, true) ACO_CON(LG, true, false) ACO_CON(LG, false, true) ACO_CON(LG, false, false)
   ACO_CON_M(1) ACO_CON_M(2) ACO_CON_M(4) ACO_CON_M(8)
 #undef ACO_CON
 #undef ACO_CON_M
-#define ACO_CON_X(LG, M) big_smem(k_construct<2, LG, M, false, true, false>); \
-  big_smem(k_construct<2, LG, M, false, false, true>); big_smem(k_construct<2, LG, M, false, true, true>);
+#define ACO_CON_X(LG, M) big_smem(k_construct<2, LG, M, false, true, false, false>); \
+  big_smem(k_construct<2, LG, M, false, false, true, false>); big_smem(k_construct<2, LG, M, false, true, true, false>);
   ACO_CON_X(1, true) ACO_CON_X(1, false) ACO_CON_X(4, true) ACO_CON_X(4, false)
 #undef ACO_CON_X
   return check();
@@ -1001,9 +1054,18 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   return check();
 }
 
-template <int P, int LG, bool M, bool TS, bool T3, bool N4>
+template <int P, int LG, bool M, bool TS, bool T3, bool N4, bool GS = false>
 static void go(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  k_construct<P, LG, M, TS, T3, N4><<<c.n_blocks, c.ants_pb * LG, c.smem_bytes, s>>>(a, c.items, iter);
+  k_construct<P, LG, M, TS, T3, N4, GS><<<c.n_blocks, c.ants_pb * LG, c.smem_bytes, s>>>(a, c.items, iter);
+}
+
+// Huge regions: per-ant state in the workspace, 4 lanes per ant.
+static void go_gs(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
+  if (pass == 1) go<1, 4, false, false, false, false, true>(c, s, a, iter);
+  else if (!c.t32 && !c.nc4) go<2, 4, false, false, false, false, true>(c, s, a, iter);
+  else if (c.t32 && !c.nc4) go<2, 4, false, false, true, false, true>(c, s, a, iter);
+  else if (!c.t32 && c.nc4) go<2, 4, false, false, false, true, true>(c, s, a, iter);
+  else go<2, 4, false, false, true, true, true>(c, s, a, iter);
 }
 
 template <int LG, bool M, bool TS>
@@ -1039,7 +1101,9 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
   cudaStream_t s = (cudaStream_t)L.stream;
   const bool mask = c.max_n <= 1024;
   KArgs a = kargs(L);
-  if (mask) {
+  if (c.gs) {
+    go_gs(pass, c, s, a, iter);
+  } else if (mask) {
     if (c.tau_smem) go_pass<true, true>(pass, c, s, a, iter);
     else go_pass<true, false>(pass, c, s, a, iter);
   } else {
@@ -1070,6 +1134,13 @@ int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, u
   if (n_upd) k_update<<<n_upd, 256, 0, s>>>(a, upd);
   k_stop<<<(L.cfg.count + 255) / 256, 256, 0, s>>>(a, pass);
   L.launches += 2 + (n_upd ? 1 : 0);
+  return check();
+}
+
+int launch_local_keys(LaunchCtx &L, int64_t *keys) {
+  if (!L.cfg.count) return 0;
+  k_local_keys<<<L.cfg.count, 32, 0, (cudaStream_t)L.stream>>>(kargs(L), keys);
+  L.launches++;
   return check();
 }
 

@@ -194,3 +194,96 @@ def test_config3_sampled(torch_cuda):
     # every region's final schedule is valid (independent checker)
     for k in range(0, 5000, 97):
         checker.check_schedule(regs[k], g[k]["order"], g[k]["cycle"], g[k]["length"])
+
+
+def _three_class(reg):
+    """Move every third VGPR to a third class (exercises the 3-4 class path)."""
+    cls = reg.reg_class.copy()
+    v = [g for g in range(reg.n_regs) if cls[g] == 0]
+    for g in v[::3]:
+        cls[g] = 2
+    return I.Region(reg.n_insts, reg.edge_src, reg.edge_dst, reg.edge_lat, cls, reg.reg_flags,
+                    reg.def_ptr, reg.def_reg, reg.use_ptr, reg.use_reg, name=reg.name + "-3c")
+
+
+M3 = I.Machine(n_classes=3, steps=((24, 28, 32, 36, 40, 48, 64, 84, 128, 256), (80, 88, 100, 102),
+                                   (24, 28, 32, 36, 40, 48, 64, 84, 128, 256)),
+               perp_limit=(24, 80, 24, 0))
+
+
+def test_three_register_classes_every_ant(torch_cuda):
+    regs = [_three_class(I.gen_region(n, 700 + n)) for n in (18, 60, 140)]
+    ids = [5, 6, 7]
+    for mode in (1, 3):
+        p = I.Params(ants=72, iterations=2, seed=3 + mode, cost_mode=mode, stall_mod=2)
+        s = _sched(M3)
+        s.load(regs, ids).run(p, no_prune=True, dump=True)
+        dump_parity(s, regs, ids, p, M3)
+
+
+def test_large_regions_global_state_every_ant(torch_cuda):
+    """Regions whose per-ant state does not fit shared memory (global-state
+    kernels) and whose cycles need 32 bits, every ant vs the oracle."""
+    regs = [I.gen_region(n, 9000 + n) for n in (900, 1500, 2100)]
+    ids = [21, 22, 23]
+    p = I.Params(ants=40, iterations=2, seed=12, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_largest_region_sampled(torch_cuda):
+    """Config-5-sized region (n = 4000), production mode, vs the oracle."""
+    reg = I.gen_region(4000, 4242)
+    p = I.Params(ants=24, iterations=1, seed=1)
+    s = _sched()
+    s.load([reg], [3]).run(p)
+    g = s.results()[0]
+    ora = O.schedule(reg, 3, I.GFX906, p)
+    compare_results(g, ora)
+
+
+def _colony_ranks(regs, ids, p_rank, world):
+    """Emulate `world` ranks of the shared colony on one GPU: one context per
+    rank, keys combined with an elementwise MIN (what the NCCL allreduce does)."""
+    import torch
+    scheds = [_sched() for _ in range(world)]
+    keys = []
+    for r, s in enumerate(scheds):
+        s.load(regs, ids)
+        keys.append(s.colony_begin(p_rank, r * p_rank.ants))
+    for pass_ in (1, 2):
+        if not (p_rank.passes & pass_):
+            continue
+        for it in range(p_rank.iterations):
+            for s in scheds:
+                s.colony_construct(pass_, it)
+            m = keys[0].clone()
+            for k in keys[1:]:
+                m = torch.minimum(m, k)
+            for k in keys:
+                k.copy_(m)
+            for s in scheds:
+                s.colony_finalize(pass_, it)
+    for s in scheds:
+        s.colony_end()
+    return [s.results() for s in scheds]
+
+
+def test_shared_colony_equals_single_context(torch_cuda):
+    """Config 4's scheme: 4 ranks x 64 ants == one context with 256 ants ==
+    the oracle with 256 ants, bit for bit (final schedule + winner trace)."""
+    import dataclasses
+    regs = [I.gen_region(n, 300 + n) for n in (45, 120)]
+    ids = [0, 1]
+    p_all = I.Params(ants=256, iterations=4, seed=8)
+    p_rank = dataclasses.replace(p_all, ants=64)
+    ranks = _colony_ranks(regs, ids, p_rank, 4)
+    s = _sched()
+    s.load(regs, ids).run(p_all, no_prune=True)
+    single = s.results()
+    for k, (reg, rid) in enumerate(zip(regs, ids)):
+        ora = O.schedule(reg, rid, I.GFX906, p_all)
+        compare_results(single[k], ora, f"single {k}")
+        for r in range(4):
+            compare_results(ranks[r][k], ora, f"rank {r} region {k}")
