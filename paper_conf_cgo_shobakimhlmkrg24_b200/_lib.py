@@ -10,6 +10,8 @@ import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libaco_b200.so")
+if os.environ.get("ACO_LIB_VARIANT"):  # A/B builds of the same sources (tools/, never the default)
+    LIB_PATH = os.path.join(HERE, f"libaco_b200_{os.environ['ACO_LIB_VARIANT']}.so")
 
 ACO_OK = 0
 ACO_FLAG_NO_PRUNE = 1

@@ -23,18 +23,22 @@ def stale() -> bool:
     return any(os.path.getmtime(f) > t for f in SOURCES + HEADERS)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if force or stale():
-        cmd = [NVCC] + FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", LIB] + SOURCES
+def build(force: bool = False, verbose: bool = False, variant: str = "", defines=()) -> str:
+    """variant/defines: an A/B build (libaco_b200_<variant>.so) for tools/ only."""
+    lib = LIB if not variant else os.path.join(HERE, f"libaco_b200_{variant}.so")
+    if force or variant or stale():
+        cmd = ([NVCC] + FLAGS + (["-Xptxas", "-v"] if verbose else []) + [f"-D{d}" for d in defines]
+               + ["-o", lib] + SOURCES)
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
             raise RuntimeError("nvcc failed building libaco_b200.so")
         if verbose:
             sys.stderr.write(r.stderr)
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
-    build(force=True, verbose="-v" in sys.argv)
-    print(LIB)
+    # build.py [-v] [variant DEF1 DEF2 ...]
+    args = [a for a in sys.argv[1:] if a != "-v"]
+    print(build(force=True, verbose="-v" in sys.argv, variant=args[0] if args else "", defines=args[1:]))

@@ -320,13 +320,24 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
       eta1[(size_t)j * (L + 1) + l] = (uint16_t)(1 + key * 65534ull / d1);
     }
   for (uint32_t j = 0; j < n; ++j) eta2[j] = (uint16_t)(1 + (uint64_t)cp[j] * 65534ull / (cp_max ? cp_max : 1));
+  // Row j of the device eta1 table is shifted by j's static kills (single-use
+  // registers, always last uses): entry j*(L+1) + d = eta1(j, LUC = sk(j) + d),
+  // so a candidate's score needs only its dynamic last-use count d.
+  {
+    std::vector<uint16_t> sh(eta1.size());
+    for (uint32_t j = 0; j < n; ++j) {
+      const uint32_t skw = info[(size_t)j * 4 + 1];
+      const uint32_t skj = (skw & 0xFF) + ((skw >> 8) & 0xFF) + ((skw >> 16) & 0xFF) + (skw >> 24);
+      for (uint32_t d = 0; d <= L; ++d)
+        sh[(size_t)j * (L + 1) + d] = eta1[(size_t)j * (L + 1) + std::min(L, skj + d)];
+    }
+    eta1.swap(sh);
+  }
   // pass-specific compact per-instruction records
-  std::vector<uint32_t> ds((size_t)n * 4, 0), e1b(n);
+  std::vector<uint32_t> ds((size_t)n * 4, 0);
   for (uint32_t j = 0; j < n; ++j) {
     ds[4 * j] = info[(size_t)j * 4 + 0];
     ds[4 * j + 1] = info[(size_t)j * 4 + 1];
-    const uint32_t skw = info[(size_t)j * 4 + 1];
-    e1b[j] = j * (L + 1) + (skw & 0xFF) + ((skw >> 8) & 0xFF) + ((skw >> 16) & 0xFF) + (skw >> 24);
   }
   for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j];
   // users of each counter register (to find the last remaining user)
@@ -365,7 +376,6 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   img.clear();
   R.img.info = img_put(img, info);
   R.img.ds = img_put(img, ds);
-  R.img.e1b = img_put(img, e1b);
   R.img.muse = img_put(img, muse);
   R.img.cu_ptr = img_put(img, cu_ptr);
   R.img.cu = img_put(img, cu);
@@ -509,47 +519,49 @@ struct Shape {
   bool ts;
 };
 
-// Dynamic shared-memory buckets of a construct launch (all blocks of a
-// launch reserve the same amount).
-const uint32_t kBuckets[] = {12 * 1024, 24 * 1024, 36 * 1024, 56 * 1024, 76 * 1024,
-                             112 * 1024, 150 * 1024, kSmemPerSM - 1024};
+// Shared memory per SM and per-block reservation (sm_100: 228 KB per SM,
+// at most 227 KB per block, 1 KB reserved by the system per resident block).
+constexpr uint32_t kSmemSM = 228 * 1024, kBlockReserve = 1024;
 
-uint32_t bucket_of(uint32_t bytes) {
-  for (uint32_t b : kBuckets)
-    if (bytes <= b) return b;
-  return 0;
-}
+// Dynamic shared memory of a launch whose blocks must fit k per SM: every
+// class is keyed by k, so all its blocks reserve exactly this much.
+uint32_t smem_for_k(uint32_t k) { return std::min(kSmemPerSM, (kSmemSM / k - kBlockReserve) & ~127u); }
 
-// max_threads: resident threads per SM allowed by the kernel's registers.
-// Candidates (ants/block, lanes/ant, tau staging) are ranked by resident
-// threads per SM capped at 512 (16 warps hide the smem/ALU latency of the
-// per-ant step chain), then fewer lanes per ant (less reduction overhead),
-// then tau in shared memory, then more resident ants.
+// Launch shape of one region and pass.  Candidates: block = any multiple of
+// 32 threads up to 512, lanes per ant L, tau staged or not; k = resident
+// blocks per SM allowed by shared memory (smem_for_k), the register budget
+// (max_threads) and the hardware (32).  Ranked by resident threads per SM
+// capped at target_threads (latency hiding of the per-ant step chain), then
+// fewer lanes per ant (less reduction overhead), then tau in shared memory,
+// then more resident USEFUL ants (A ants of a region fill ceil(A/apb) blocks),
+// then fewer blocks (one image copy per block).
 Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
-                 uint32_t target_threads, uint32_t max_lanes) {
+                 uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w) {
   Shape best{0, 1, 0, false};
   uint64_t best_score = 0;
   for (int ts = 1; ts >= 0; --ts) {
     if (ts && !allow_ts) continue;
-    for (uint32_t apb : {32u, 64u, 128u, 256u}) {
-      const uint32_t bytes = img + (ts ? tb : 0u) + apb * W * 4;
-      const uint32_t b = bucket_of(bytes);
-      if (!b) continue;
-      for (uint32_t L : {1u, 2u, 4u, 8u}) {
-        if (lanes14 && L != 1 && L != 4) continue;
-        if (L > max_lanes) continue;
-        const uint32_t threads = apb * L;
-        if (threads > 256) continue;
-        uint32_t blocks = kSmemPerSM / (b + 1024);  // + per-block reserved smem
-        blocks = std::min(blocks, max_threads / threads);
-        blocks = std::min(blocks, 32u);
-        if (!blocks) continue;
-        const uint64_t thr = std::min<uint64_t>((uint64_t)blocks * threads, target_threads);
-        const uint64_t ants = (uint64_t)blocks * apb;
-        const uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) | ants;
+    for (uint32_t L : {1u, 2u, 4u, 8u}) {
+      if (lanes14 && L != 1 && L != 4) continue;
+      if (L > max_lanes) continue;
+      for (uint32_t threads : {32u, 64u, 96u, 128u, 192u, 256u, 384u, 512u}) {
+        if (threads > kMaxBlockThreads) break;
+        const uint32_t apb = threads / L;
+        const uint64_t bytes = (uint64_t)img + (ts ? tb : 0u) + (uint64_t)ant_stride(apb, L) * W * 4 +
+                               (uint64_t)coin_groups(apb, gsz) * coin_w * 4;
+        if (bytes > kSmemPerSM) break;
+        uint32_t k = kSmemSM / ((uint32_t)bytes + kBlockReserve);
+        k = std::min(k, max_threads / threads);
+        k = std::min(k, 32u);
+        while (k && smem_for_k(k) < bytes) --k;
+        if (!k) continue;
+        const uint64_t thr = std::min<uint64_t>((uint64_t)k * threads, target_threads);
+        const uint64_t ants = std::min<uint64_t>((uint64_t)k * std::max(1u, A) / ((std::max(1u, A) + apb - 1) / apb), 4095);
+        const uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) |
+                               (ants << 12) | (uint64_t)(4095 - k);
         if (score > best_score) {
           best_score = score;
-          best = Shape{apb, L, b, ts != 0};
+          best = Shape{apb, L, smem_for_k(k), ts != 0};
         }
       }
     }
@@ -583,17 +595,27 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // ---- per-pass construct classes
   struct Cls {
     Shape sh;
-    bool mask, t32, gs;
+    bool mask, t32, gs, wide = false;
     uint32_t smem;
     std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t>;
+  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t, bool>;
   std::map<Key, Cls> classes;
   P.nc4 = ctx->mach.n_classes > 2;
   // launch-shape policy (tuning knobs; defaults measured on B200)
-  uint32_t tgt_threads[2] = {512, 256}, max_lanes[2] = {8, 1};
+  uint32_t tgt_threads[2] = {512, 768}, max_lanes[2] = {8, 1};
   if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
+  // registers of the construct kernels bound the resident threads per SM
+  static uint32_t s_mt[16][2][2];
+  static bool s_mt_ok[16];
+  uint32_t mt[2][2];
+  {
+    const int dv = ctx->device >= 0 && ctx->device < 16 ? ctx->device : 0;
+    if (!s_mt_ok[dv]) s_mt_ok[dv] = construct_max_threads(ctx->device, s_mt[dv]) == 0;
+    if (s_mt_ok[dv]) std::memcpy(mt, s_mt[dv], sizeof(mt));
+    else construct_max_threads(-2, mt);  // conservative defaults (no device: sizing only)
+  }
   std::vector<uint8_t> gs(count, 0);
   std::vector<uint32_t> gs_words(count, 0), scratch_words(count, 0);
   for (uint32_t r = 0; r < count; ++r) {
@@ -604,9 +626,14 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     for (uint32_t pass = 1; pass <= 2; ++pass) {
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
       if (!(p->pass & pass)) continue;
+      if (getenv("ACO_DEBUG_REGIONS"))
+        fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
+                R.nremw, R.L);
       const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
-      Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, pass == 1 ? 1280u : 768u, !rare, rare,
-                            pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1]);
+      const bool wide = R.n >= kWideN && R.n <= 1024;
+      Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
+                            pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1], A,
+                            p->group_size, coin_words(pass, R.n));
       bool g = false;
       if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
         sh = Shape{64, 4, 0, false};
@@ -615,8 +642,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         gs_words[r] = std::max(gs_words[r], W);
       }
       const bool mask = R.n <= 1024 && !g;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem);
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask);
       Cls &c = classes[key];
+      c.wide = wide && mask;
       c.sh = sh;
       c.mask = mask;
       c.t32 = pass == 2 && t32;
@@ -750,6 +778,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       cl.t32 = c.t32;
       cl.nc4 = P.nc4;
       cl.gs = c.gs;
+      cl.wide = c.wide;
       P.launches[std::get<0>(kv.first)].push_back(cl);
       class_work[std::get<0>(kv.first)].push_back(0);
       for (auto &pr : c.regs) class_work[std::get<0>(kv.first)].back() += ~pr.first;
@@ -766,9 +795,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       for (size_t i = 0; i < idx.size(); ++i)
         fprintf(stderr,
                 "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d gs %d "
-                "work %.3g\n",
+                "wide %d work %.3g\n",
                 pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes,
-                (int)sorted[i].tau_smem, (int)sorted[i].t32, (int)sorted[i].gs, (double)class_work[pass][idx[i]]);
+                (int)sorted[i].tau_smem, (int)sorted[i].t32, (int)sorted[i].gs, (int)sorted[i].wide,
+                (double)class_work[pass][idx[i]]);
   }
   if (plan_only) {
     ctx->plan = saved;

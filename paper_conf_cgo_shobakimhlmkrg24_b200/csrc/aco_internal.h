@@ -22,7 +22,11 @@ namespace aco {
 constexpr uint32_t kInvalid = 0xFFFFFFFFu;  // R35
 constexpr uint32_t kMaxKernelInsts = 8191;  // ids use 13 bits in successor entries
 constexpr uint32_t kFlagLiveIn = 1, kFlagLiveOut = 2;
-constexpr uint32_t kSmemPerSM = 227 * 1024;
+constexpr uint32_t kSmemPerSM = 227 * 1024;  // max dynamic shared memory per block
+constexpr uint32_t kMaxBlockThreads = 512;   // construct blocks (launch bounds)
+// Regions with at least this many instructions use the 4-wide candidate scan
+// (latency-bound: few ants fit an SM); smaller ones the 1-wide scan (issue-bound).
+constexpr uint32_t kWideN = 160;
 
 // Successor entry: v (13 bits) | single-predecessor flag << 13 | latency << 16.
 constexpr uint32_t kSuccSingle = 1u << 13;
@@ -36,11 +40,10 @@ constexpr uint32_t kMuseCounter = 1u << 31;
 struct ImageLayout {
   uint32_t info;      // uint4 [n] {defs u8x4, static kills u8x4, dead defs u8x4, muse start << 8 | count}
   uint32_t ds;        // uint4 [n] {defs u8x4, static kills u8x4, eta2, 0} (pass-2 candidates)
-  uint32_t e1b;       // u32 [n]: j*(L+1) + #static kills (row base into eta1 for pass 1)
   uint32_t muse;      // u32 [nm]
   uint32_t cu_ptr;    // u32 [nctr+1]: users of each counter register
   uint32_t cu;        // u32 [..]
-  uint32_t eta1;      // u16 [n * (L+1)]: eta1(j, luc) at j*(L+1) + luc (R4)
+  uint32_t eta1;      // u16 [n * (L+1)]: eta1(j, sk(j) + d) at j*(L+1) + d, d = dynamic last uses (R4)
   uint32_t eta2;      // u16 [n]
   uint32_t succ_ptr;  // u32 [n+1]
   uint32_t succ;      // u32 [E]
@@ -49,7 +52,7 @@ struct ImageLayout {
   uint32_t rb0;       // u32 [nwr]: roots bitset
   uint32_t rem0;      // u32 [nremw]: u16 use counts of >= 3-use registers
   uint32_t bytes;     // total, multiple of 16
-  uint32_t pad;
+  uint32_t pad[2];
 };
 
 // Per-region statics (arena header array).
@@ -150,6 +153,26 @@ ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }
 
+// Stride (in words) between consecutive state words of one ant in a block of
+// apb ants x lg lanes.  stride = 32/lg (mod 32) makes the 32 lanes of a warp
+// hit 32 distinct banks when lane l of every ant touches a word w = l (mod lg)
+// (the split ready-bitset scan) and when only the group leaders touch
+// arbitrary words (commit): bank = ant + (w mod lg) * 32/lg.
+ACO_HD inline uint32_t ant_stride(uint32_t apb, uint32_t lg) {
+  if (lg <= 1) return apb;
+  const uint32_t m = 32 / lg;
+  return ((apb + 31 - m) / 32) * 32 + m;
+}
+
+// Group-coin table of a construct block (R3): one bit per (step, group) for
+// every exploit/explore group its apb consecutive ants span (group size g),
+// pass 1 for the steps k < n, pass 2 for the cycles t < 32 * coin_words
+// (later cycles draw their coin inline).
+ACO_HD inline uint32_t coin_groups(uint32_t apb, uint32_t g) { return g >= apb ? 2u : (apb - 1) / g + 2u; }
+ACO_HD inline uint32_t coin_words(uint32_t pass, uint32_t n) {
+  return pass == 1 ? (n + 31) / 32 : (2 * n + 63) / 32;
+}
+
 // Bytes of the pheromone table as staged in shared memory.
 ACO_HD inline uint32_t tau_smem_bytes(uint32_t n) { return (((n + 1) * n * 2) + 15) & ~15u; }
 
@@ -179,9 +202,13 @@ struct ClassLaunch {
   bool t32;                // u32 pass-2 cycle array
   bool nc4;                // 3-4 register classes (u16 last-use counts)
   bool gs;                 // per-ant state in global memory (huge regions)
+  bool wide;               // 4-wide candidate scan (n >= kWideN, word-mask variant)
 };
 
 int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success
+// Resident threads per SM that the construct kernels' registers allow, per
+// [pass-1][wide]; returns nonzero (and conservative defaults) without a device.
+int construct_max_threads(int device, uint32_t out[2][2]);
 int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);

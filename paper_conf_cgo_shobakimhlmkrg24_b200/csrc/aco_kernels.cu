@@ -24,9 +24,12 @@
 // Plus k_init (tau0, greedy heuristic schedule) and k_pass2_init (target, ASAP
 // of the pass-1 best, tau reset).
 #include <cuda_runtime.h>
+
+#include <algorithm>
 #include <stdint.h>
 
 #include "aco_internal.h"
+
 
 namespace aco {
 
@@ -109,9 +112,9 @@ __device__ void target_of(uint32_t mode, const uint32_t best[4], uint32_t tgt[4]
 struct SV {
   const uint4 *info;
   const uint4 *ds;
-  const uint32_t *e1b, *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0;
+  const uint32_t *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0;
   const uint16_t *eta1, *eta2;
-  uint32_t n, nwr, nremw, region_id;
+  uint32_t n, nwr, nremw, region_id, L1;
   uint32_t livein01, livein23;  // u16 x 2
 };
 
@@ -119,7 +122,6 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   SV V;
   V.info = (const uint4 *)(img + rd->img.info);
   V.ds = (const uint4 *)(img + rd->img.ds);
-  V.e1b = (const uint32_t *)(img + rd->img.e1b);
   V.muse = (const uint32_t *)(img + rd->img.muse);
   V.cu_ptr = (const uint32_t *)(img + rd->img.cu_ptr);
   V.cu = (const uint32_t *)(img + rd->img.cu);
@@ -135,6 +137,7 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   V.nwr = rd->nwr;
   V.nremw = rd->nremw;
   V.region_id = rd->region_id;
+  V.L1 = rd->L + 1;
   V.livein01 = (rd->livein[0] & 0xFFFFu) | (rd->livein[1] << 16);
   V.livein23 = (rd->livein[2] & 0xFFFFu) | (rd->livein[3] << 16);
   return V;
@@ -292,6 +295,37 @@ __device__ __forceinline__ void scan_bits(const St &A, uint32_t nwr, uint32_t wm
   }
 }
 
+// Batched scan (MASK variant, n <= 1024): visit(j[4], v[4]) receives the
+// next four set bits of this lane's words in ascending order (v[u] = valid;
+// an invalid slot repeats j[0], so its loads stay in bounds).  Extracting
+// four candidates before touching their data lets a thread issue the four
+// candidates' shared-memory / L2 loads back to back instead of one dependent
+// chain per candidate (the step is latency-bound for large regions, where
+// few ants fit on an SM).  wmask has exactly the non-empty words' bits, so
+// one word fetch always refills an exhausted bits register.
+template <typename F>
+__device__ __forceinline__ void scan4(const St &A, uint32_t m, F &&visit) {
+  uint32_t w = 0, bits = 0;
+  while (true) {
+    uint32_t j[4];
+    bool v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      if (!bits && m) {
+        w = __ffs(m) - 1;
+        m &= m - 1;
+        bits = A.RB[w * A.S];
+      }
+      v[u] = bits != 0u;
+      j[u] = v[u] ? w * 32u + (__ffs(bits) - 1) : j[0];
+      bits &= bits - 1;
+    }
+    if (!v[0]) return;
+    visit(j, v);
+    if (!v[3] || (!bits && !m)) return;
+  }
+}
+
 struct AntOut {
   uint32_t cost;
   uint32_t prp01, prp23;
@@ -409,11 +443,12 @@ __device__ __forceinline__ unsigned long long akey(uint32_t s, uint32_t j) {
 // score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
 // Philox step (R26).  rec (leader, may be NULL) receives the order.  The
 // result is valid in the leader lane.
-template <int LG, bool MASK>
+template <int LG, bool MASK, bool WIDE = false>
 __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
-                                            const RunCfg &cfg, const bool greedy, uint16_t *rec) {
-  const uint32_t n = V.n, nwr = V.nwr;
+                                            const RunCfg &cfg, const bool greedy, uint16_t *rec,
+                                            const uint32_t *coins = nullptr) {
+  const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<1, MASK, false, false>(V, A);
   wmask = G.bcast(wmask);
@@ -421,27 +456,68 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const uint32_t sub = lane_words<LG>(G.lane);
+  constexpr bool wide = MASK && WIDE;
   uint32_t prev = n;
   for (uint32_t k = 0; k < n; ++k) {
     bool exploit = greedy;
     if (!greedy) {
-      const uint4 g = philox(k, 0x80000000u | group, iter, V.region_id, cfg.seed);
-      exploit = (uint64_t)g.x < cfg.q0_t;
+      if (coins) {  // the block's precomputed group coins (R3)
+        exploit = (coins[k >> 5] >> (k & 31u)) & 1u;
+      } else {
+        const uint4 g = philox(k, 0x80000000u | group, iter, V.region_id, cfg.seed);
+        exploit = (uint64_t)g.x < cfg.q0_t;
+      }
     }
     const uint16_t *trow = tau + prev * n;
+    // score(j) = tau[prev][j] * eta1(j, sk(j) + d(j)) (R1, R4)
     auto score = [&](uint32_t j) -> uint32_t {
-      return (uint32_t)trow[j] * (uint32_t)V.eta1[V.e1b[j] + dk1_get(A, j)];
+      return (uint32_t)trow[j] * (uint32_t)V.eta1[j * L1 + dk1_get(A, j)];
     };
-    unsigned long long best = 0;
+    // Lane-local argmax in ascending order: strict '>' keeps the lowest
+    // index among equal scores; bs1 = best score + 1 (0 = no candidate; a
+    // score is < 2^32 - 1, so +1 cannot wrap).
+    uint32_t bs1 = 0, bj = 0;
     unsigned long long sum = 0;
-    scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
-      const uint32_t s = score(j);
-      best = ::max(best, akey(s, j));
-      sum += s;
-      return false;
-    });
-    best = G.max64(best);
-    uint32_t jstar = 0xFFFFFFFFu - (uint32_t)best;
+    if constexpr (wide) {
+      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v)[4]) {
+        uint32_t tv[4], dk[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          tv[u] = trow[j[u]];
+          dk[u] = A.DK[(j[u] >> 3) * A.S];
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) dk[u] = V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t sc = tv[u] * dk[u];
+          if (v[u]) {
+            if (sc + 1u > bs1) {
+              bs1 = sc + 1u;
+              bj = j[u];
+            }
+            if (!exploit) sum += sc;
+          }
+        }
+      });
+    } else {
+      scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
+        const uint32_t sc = score(j);
+        if (sc + 1u > bs1) {
+          bs1 = sc + 1u;
+          bj = j;
+        }
+        if (!exploit) sum += sc;
+        return false;
+      });
+    }
+    uint32_t jstar;
+    if (LG == 1) {
+      jstar = bj;
+    } else {
+      const unsigned long long best = G.max64(bs1 ? akey(bs1 - 1u, bj) : 0ull);
+      jstar = 0xFFFFFFFFu - (uint32_t)best;
+    }
     if (!exploit) {  // roulette (R27): the leader scans every candidate in ascending order
       sum = G.sum64(sum);
       if (G.leader()) {
@@ -478,11 +554,12 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
 // ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle and
 // the Philox step; stalls skip ahead without drawing.  rec_o / rec_c (leader,
 // may be NULL) receive the order and the cycles.  Valid in the leader lane.
-template <int LG, bool MASK, bool T32, bool NC4>
+template <int LG, bool MASK, bool T32, bool NC4, bool WIDE = false>
 __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
-                                            const bool prune, uint16_t *rec_o, uint32_t *rec_c) {
+                                            const bool prune, uint16_t *rec_o, uint32_t *rec_c,
+                                            const uint32_t *coins = nullptr, uint32_t coin_t = 0) {
   const uint32_t n = V.n, nwr = V.nwr;
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<2, MASK, T32, NC4>(V, A);
@@ -493,6 +570,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   const bool stall_en = (group % cfg.stall_mod) == cfg.stall_rem;  // R23
   const uint32_t c2 = 0x80000000u | iter;
   const uint32_t sub = lane_words<LG>(G.lane);
+  constexpr bool wide = MASK && WIDE;
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0;
   AntOut o;
   o.prp01 = o.prp23 = 0;
@@ -516,31 +594,54 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     const uint16_t *trow = tau + prev * n;
     uint32_t counts = 0, min_s = 0xFFFFFFFFu;  // counts = |R| | |F| << 16
     bool f_not_inc = false, s_dec = false, any_s = false;
-    unsigned long long best = 0, sum = 0;
-    scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
-      const uint32_t rdy = t_get<T32>(A, j);
-      const uint4 ds = V.ds[j];                       // defs, static kills, eta2
-      const uint32_t K = ds.y + dk2_get<NC4>(A, j);   // kills per class (R14)
-      const uint32_t s = (uint32_t)trow[j] * ds.z;
+    uint32_t bs1 = 0, bj = 0;  // lane-local best score + 1 (0 = none) and its index
+    unsigned long long sum = 0;
+    // the roulette sum is needed unless this cycle's group coin is a known exploit
+    const bool need_sum = !(t < coin_t && ((coins[t >> 5] >> (t & 31u)) & 1u));
+    auto eval = [&](uint32_t j, uint32_t rdy, const uint4 &ds, uint32_t dk, uint32_t tv) {
+      const uint32_t K = ds.y + dk;                   // kills per class (R14)
+      const uint32_t s = tv * ds.z;
       if (rdy <= t) {
         counts += 1u;
         if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
           counts += 1u << 16;
           f_not_inc |= __vcmpgtu4(ds.x, K) == 0u;           // max_c Delta_c <= 0
-          best = ::max(best, akey(s, j));
-          sum += s;
+          if (s + 1u > bs1) {  // ascending: strict keeps the lowest index (R1, R25)
+            bs1 = s + 1u;
+            bj = j;
+          }
+          if (need_sum) sum += s;
         }
       } else {
         any_s = true;
         min_s = ::min(min_s, rdy);
         s_dec |= __vcmpltu4(ds.x, K) != 0u;                 // min_c Delta_c < 0
       }
-      return false;
-    });
+    };
+    if constexpr (wide) {
+      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v)[4]) {
+        uint32_t rd[4], dk[4], tv[4];
+        uint4 ds[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          rd[u] = t_get<T32>(A, j[u]);
+          ds[u] = V.ds[j[u]];                         // defs, static kills, eta2
+          dk[u] = dk2_get<NC4>(A, j[u]);
+          tv[u] = trow[j[u]];
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (v[u]) eval(j[u], rd[u], ds[u], dk[u], tv[u]);
+      });
+    } else {
+      scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
+        eval(j, t_get<T32>(A, j), V.ds[j], dk2_get<NC4>(A, j), trow[j]);
+        return false;
+      });
+    }
     counts = G.sum(counts);
     min_s = G.min(min_s);
-    best = G.max64(best);
-    sum = G.sum64(sum);
+    if (need_sum) sum = G.sum64(sum);
     any_s = G.any(any_s);
     const bool all_f_inc = !G.any(f_not_inc);
     const bool some_s_dec = G.any(s_dec);
@@ -570,9 +671,16 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         continue;
       }
     }
-    const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
-    uint32_t jstar = 0xFFFFFFFFu - (uint32_t)best;
-    if (!((uint64_t)g.x < cfg.q0_t)) {  // explore: roulette over F (R27), leader in ascending order
+    bool exploit;
+    if (t < coin_t) {  // the block's precomputed group coins (R3)
+      exploit = (coins[t >> 5] >> (t & 31u)) & 1u;
+    } else {
+      const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
+      exploit = (uint64_t)g.x < cfg.q0_t;
+    }
+    uint32_t jstar = bj;
+    if (LG > 1) jstar = 0xFFFFFFFFu - (uint32_t)G.max64(bs1 ? akey(bs1 - 1u, bj) : 0ull);
+    if (!exploit) {  // explore: roulette over F (R27), leader in ascending order
       if (G.leader()) {
         if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
         const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
@@ -631,9 +739,12 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
   for (uint32_t i = threadIdx.x; i < bytes / 16; i += blockDim.x) dst[i] = src[i];
 }
 
-template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, bool GS>
-__global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__restrict__ items,
-                                                   uint32_t iter) {
+// Launch bounds: the 1-wide variants keep <= 64 registers (2 x 512 threads per
+// SM); the 4-wide ones (large regions, few ants per SM by shared memory) may
+// use up to 128.
+template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, bool GS, bool WIDE>
+__global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
+    k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
   if (!rs.active) return;  // block-uniform
@@ -648,6 +759,8 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
   const unsigned char *img = A.arena + rd->o_image;
   uint32_t *stbase;
   uint32_t stride;
+  const uint32_t *coins = nullptr;
+  uint32_t coin_t = 0;
   if (GS) {  // huge region: statics through L1/L2, per-ant state in the workspace
     if (ai >= A.cfg.ants) return;
     stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
@@ -662,11 +775,29 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
       tau = (const uint16_t *)(smem + img_bytes);
       state_off += tb;
     }
+    const uint32_t apb = blockDim.x / LG;
+    stride = ant_stride(apb, LG);
+    // Group coins (R3) of every (step, group) of this block, one warp per
+    // 32 steps of a group (ballot), instead of one Philox per ant-step.
+    {
+      const uint32_t gsz = A.cfg.group_size, abase = A.cfg.ant_base + bi.ant0, g0 = abase / gsz;
+      const uint32_t ng = (abase + apb - 1) / gsz - g0 + 1, cw = coin_words(PASS, rd->n);
+      uint32_t *cz = (uint32_t *)(smem + state_off) +
+                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4);
+      const uint32_t lane = threadIdx.x & 31u, c2 = PASS == 1 ? iter : (0x80000000u | iter);
+      for (uint32_t task = threadIdx.x >> 5; task < ng * cw; task += blockDim.x >> 5) {
+        const uint32_t gi = task / cw, k = (task - gi * cw) * 32 + lane;
+        const uint4 x = philox(k, 0x80000000u | (g0 + gi), c2, rd->region_id, A.cfg.seed);
+        const uint32_t word = __ballot_sync(0xFFFFFFFFu, (uint64_t)x.x < A.cfg.q0_t);
+        if (lane == 0) cz[task] = word;
+      }
+      coins = cz + (ant / gsz - g0) * cw;
+      coin_t = PASS == 1 ? 0xFFFFFFFFu : cw * 32;
+    }
     __syncthreads();
     if (ai >= A.cfg.ants) return;  // whole lane group
     img = smem;
     stbase = (uint32_t *)(smem + state_off) + local;
-    stride = blockDim.x / LG;
   }
   const Grp<LG> G(threadIdx.x);
   const SV V = make_sv(img, rd);
@@ -677,7 +808,7 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
     uint16_t *rec = nullptr;
     if (dump && A.dump_order)
       rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
-    o = ant_pass1<LG, MASK>(V, tau, S, G, ant, iter, A.cfg, false, rec);
+    o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -691,8 +822,8 @@ __global__ void __launch_bounds__(256) k_construct(KArgs A, const BlockItem *__r
       rec_o = A.dump_order + base;
       rec_c = A.dump_cycle + base;
     }
-    o = ant_pass2<LG, MASK, T32, NC4>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
-                                      rec_c);
+    o = ant_pass2<LG, MASK, T32, NC4, WIDE>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
+                                      rec_c, coins, coin_t);
   }
   if (G.leader()) {
     uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
@@ -1008,13 +1139,121 @@ static int check() {
 
 int last_cuda_error() { return check(); }
 
+// ---- construct-kernel variants: one table of every instantiation, used for
+// the shared-memory opt-in, the register limits the planner needs and the
+// launch dispatch (a class launch looks its kernel up by variant code).
+using ConstructFn = void (*)(KArgs, const BlockItem *, uint32_t);
+
+__host__ __device__ constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4,
+                                                     bool gs, bool wd) {
+  return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
+         ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((uint32_t)gs << 1) | (uint32_t)wd;
+}
+
+template <int P, int LG, bool M, bool TS, bool T3, bool N4, bool GS, bool WD, typename F>
+static void reg1(F &f) {
+  f(&k_construct<P, LG, M, TS, T3, N4, GS, WD>, variant_code(P, LG, M, TS, T3, N4, GS, WD));
+}
+template <int P, int LG, bool M, bool TS, bool T3, bool N4, typename F>
+static void reg_w(F &f) {  // the 4-wide scan exists only with the word mask (n <= 1024)
+  reg1<P, LG, M, TS, T3, N4, false, false>(f);
+  if constexpr (M) reg1<P, LG, M, TS, T3, N4, false, true>(f);
+}
+template <int LG, typename F>
+static void reg_lg(F &f) {
+  reg_w<1, LG, true, true, false, false>(f);
+  reg_w<1, LG, true, false, false, false>(f);
+  reg_w<1, LG, false, true, false, false>(f);
+  reg_w<1, LG, false, false, false, false>(f);
+  reg_w<2, LG, true, true, false, false>(f);
+  reg_w<2, LG, true, false, false, false>(f);
+  reg_w<2, LG, false, true, false, false>(f);
+  reg_w<2, LG, false, false, false, false>(f);
+}
+template <int LG, bool M, typename F>
+static void reg_rare(F &f) {  // pass 2 with u32 cycles and/or 3-4 classes: tau in global memory, 1 or 4 lanes
+  reg_w<2, LG, M, false, true, false>(f);
+  reg_w<2, LG, M, false, false, true>(f);
+  reg_w<2, LG, M, false, true, true>(f);
+}
+template <typename F>
+static void for_each_construct(F &&f) {
+  reg_lg<1>(f);
+  reg_lg<2>(f);
+  reg_lg<4>(f);
+  reg_lg<8>(f);
+  reg_rare<1, true>(f);
+  reg_rare<1, false>(f);
+  reg_rare<4, true>(f);
+  reg_rare<4, false>(f);
+  // huge regions: per-ant state in the workspace, 4 lanes per ant
+  reg1<1, 4, false, false, false, false, true, false>(f);
+  reg1<2, 4, false, false, false, false, true, false>(f);
+  reg1<2, 4, false, false, true, false, true, false>(f);
+  reg1<2, 4, false, false, false, true, true, false>(f);
+  reg1<2, 4, false, false, true, true, true, false>(f);
+}
+
+static ConstructFn g_construct[512];
+static bool g_table_ready = false;
+static void build_table() {
+  if (g_table_ready) return;
+  for_each_construct([](ConstructFn f, uint32_t code) { g_construct[code] = f; });
+  g_table_ready = true;
+}
+
+// Resident threads per SM the registers of the construct kernels allow, per
+// (pass, wide); conservative defaults when no device is visible.
+int construct_max_threads(int device, uint32_t out[2][2]) {
+  out[0][0] = out[1][0] = 1024;
+  out[0][1] = out[1][1] = 512;
+  int cur = -1;
+  if (cudaGetDevice(&cur) != cudaSuccess || (device >= 0 && cur != device && cudaSetDevice(device) != cudaSuccess)) {
+    cudaGetLastError();
+    return 1;
+  }
+  uint32_t regs[2][2] = {{0, 0}, {0, 0}};
+  bool ok = true;
+  for_each_construct([&](ConstructFn f, uint32_t code) {
+    cudaFuncAttributes fa;
+    if (cudaFuncGetAttributes(&fa, f) != cudaSuccess) {
+      ok = false;
+      return;
+    }
+    const uint32_t p = code >> 8, w = code & 1u;
+    regs[p][w] = std::max(regs[p][w], (uint32_t)fa.numRegs);
+  });
+  if (!ok) {
+    cudaGetLastError();
+    return 1;
+  }
+  for (int p = 0; p < 2; ++p)
+    for (int w = 0; w < 2; ++w) {
+      const uint32_t r8 = std::max(8u, (regs[p][w] + 7u) & ~7u);  // allocation unit: 8 registers per thread
+      const uint32_t warps = std::min(64u, 65536u / (32u * r8));
+      out[p][w] = warps * 32u;
+    }
+  return 0;
+}
+
+// Opt every kernel into the largest dynamic shared memory it can use (the
+// per-block maximum minus its static shared memory, rounded down to 1 KB).
+static int g_attr_err = 0;
 template <typename K>
 static void big_smem(K kernel) {
-  cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemPerSM);
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, kernel) != cudaSuccess) {
+    g_attr_err = 1;
+    return;
+  }
+  const int dyn = (int)((kSmemPerSM - (uint32_t)fa.sharedSizeBytes) & ~1023u);
+  if (cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn) != cudaSuccess)
+    g_attr_err = 1;
 }
 
 int set_machine(const MachineDev &m) {
   if (cudaMemcpyToSymbol(c_mach, &m, sizeof(m)) != cudaSuccess) return 1;
+  g_attr_err = 0;
   big_smem(k_init<true>);
   big_smem(k_init<false>);
   big_smem(k_pass2_init);
@@ -1022,17 +1261,9 @@ int set_machine(const MachineDev &m) {
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
 #undef ACO_SEL
-#define ACO_CON(LG, M, TS) big_smem(k_construct<1, LG, M, TS, false, false, false>); \
-  big_smem(k_construct<2, LG, M, TS, false, false, false>);
-#define ACO_CON_M(LG) ACO_CON(LG, true, true) ACO_CON(LG, true, false) ACO_CON(LG, false, true) ACO_CON(LG, false, false)
-  ACO_CON_M(1) ACO_CON_M(2) ACO_CON_M(4) ACO_CON_M(8)
-#undef ACO_CON
-#undef ACO_CON_M
-#define ACO_CON_X(LG, M) big_smem(k_construct<2, LG, M, false, true, false, false>); \
-  big_smem(k_construct<2, LG, M, false, false, true, false>); big_smem(k_construct<2, LG, M, false, true, true, false>);
-  ACO_CON_X(1, true) ACO_CON_X(1, false) ACO_CON_X(4, true) ACO_CON_X(4, false)
-#undef ACO_CON_X
-  return check();
+  for_each_construct([](ConstructFn f, uint32_t) { big_smem(f); });
+  const int e = check();
+  return e ? e : g_attr_err;
 }
 
 int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
@@ -1054,62 +1285,17 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   return check();
 }
 
-template <int P, int LG, bool M, bool TS, bool T3, bool N4, bool GS = false>
-static void go(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  k_construct<P, LG, M, TS, T3, N4, GS><<<c.n_blocks, c.ants_pb * LG, c.smem_bytes, s>>>(a, c.items, iter);
-}
-
-// Huge regions: per-ant state in the workspace, 4 lanes per ant.
-static void go_gs(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  if (pass == 1) go<1, 4, false, false, false, false, true>(c, s, a, iter);
-  else if (!c.t32 && !c.nc4) go<2, 4, false, false, false, false, true>(c, s, a, iter);
-  else if (c.t32 && !c.nc4) go<2, 4, false, false, true, false, true>(c, s, a, iter);
-  else if (!c.t32 && c.nc4) go<2, 4, false, false, false, true, true>(c, s, a, iter);
-  else go<2, 4, false, false, true, true, true>(c, s, a, iter);
-}
-
-template <int LG, bool M, bool TS>
-static void go_lg(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  if (pass == 1) go<1, LG, M, TS, false, false>(c, s, a, iter);
-  else go<2, LG, M, TS, false, false>(c, s, a, iter);
-}
-
-template <int LG, bool M>
-static void go_x(const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  if (c.t32 && !c.nc4) go<2, LG, M, false, true, false>(c, s, a, iter);
-  else if (!c.t32 && c.nc4) go<2, LG, M, false, false, true>(c, s, a, iter);
-  else go<2, LG, M, false, true, true>(c, s, a, iter);
-}
-
-template <bool M, bool TS>
-static void go_pass(uint32_t pass, const ClassLaunch &c, cudaStream_t s, const KArgs &a, uint32_t iter) {
-  if (pass == 2 && (c.t32 || c.nc4)) {  // rare variants: tau in global memory, 1 or 4 lanes per ant
-    if (c.lanes >= 4) go_x<4, M>(c, s, a, iter);
-    else go_x<1, M>(c, s, a, iter);
-    return;
-  }
-  switch (c.lanes) {
-    case 8: go_lg<8, M, TS>(pass, c, s, a, iter); break;
-    case 4: go_lg<4, M, TS>(pass, c, s, a, iter); break;
-    case 2: go_lg<2, M, TS>(pass, c, s, a, iter); break;
-    default: go_lg<1, M, TS>(pass, c, s, a, iter); break;
-  }
-}
-
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c) {
   if (!c.n_blocks) return 0;
-  cudaStream_t s = (cudaStream_t)L.stream;
-  const bool mask = c.max_n <= 1024;
-  KArgs a = kargs(L);
-  if (c.gs) {
-    go_gs(pass, c, s, a, iter);
-  } else if (mask) {
-    if (c.tau_smem) go_pass<true, true>(pass, c, s, a, iter);
-    else go_pass<true, false>(pass, c, s, a, iter);
-  } else {
-    if (c.tau_smem) go_pass<false, true>(pass, c, s, a, iter);
-    else go_pass<false, false>(pass, c, s, a, iter);
-  }
+  build_table();
+  const bool mask = c.max_n <= 1024 && !c.gs;
+  const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
+  const uint32_t lg = c.gs ? 4u : c.lanes;
+  const uint32_t code = variant_code(pass, lg, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32,
+                                     pass == 2 && c.nc4, c.gs, c.wide && mask);
+  const ConstructFn f = g_construct[code];
+  if (!f) return (int)cudaErrorInvalidDeviceFunction;
+  f<<<c.n_blocks, c.ants_pb * lg, c.smem_bytes, (cudaStream_t)L.stream>>>(kargs(L), c.items, iter);
   L.launches++;
   return check();
 }
