@@ -606,6 +606,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t tgt_threads[2] = {512, 768}, max_lanes[2] = {8, 1};
   if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
+  uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
+  if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
   // registers of the construct kernels bound the resident threads per SM
   static uint32_t s_mt[16][2][2];
   static bool s_mt_ok[16];
@@ -632,7 +634,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
       const bool wide = R.n >= kWideN && R.n <= 1024;
       Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
-                            pass == 1 ? tgt_threads[0] : tgt_threads[1], pass == 1 ? max_lanes[0] : max_lanes[1], A,
+                            pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
                             p->group_size, coin_words(pass, R.n));
       bool g = false;
       if (sh.apb == 0) {  // does not fit shared memory: global-state kernels

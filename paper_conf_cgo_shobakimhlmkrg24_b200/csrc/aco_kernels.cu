@@ -31,6 +31,18 @@
 #include "aco_internal.h"
 
 
+// Compile-time switches for A/B measurement (tools/ab_run.sh); the defaults
+// are the product configuration.
+#ifndef ACO_PREFETCH
+#define ACO_PREFETCH 0
+#endif
+#ifndef ACO_BRANCHLESS1  // pass-1 4-wide evaluation without branches (measured faster)
+#define ACO_BRANCHLESS1 1
+#endif
+#ifndef ACO_BRANCHLESS2  // pass-2 likewise (measured slower: keep the branches)
+#define ACO_BRANCHLESS2 0
+#endif
+
 namespace aco {
 
 __constant__ MachineDev c_mach;
@@ -305,6 +317,40 @@ __device__ __forceinline__ void scan_bits(const St &A, uint32_t nwr, uint32_t wm
 // one word fetch always refills an exhausted bits register.
 template <typename F>
 __device__ __forceinline__ void scan4(const St &A, uint32_t m, F &&visit) {
+#if ACO_PREFETCH
+  // the next non-empty word is fetched one word ahead (its load overlaps the
+  // current word's candidates)
+  uint32_t w = 0, bits = 0, nw = 0, nbits = 0;
+  bool pend = m != 0u;
+  if (pend) {
+    nw = __ffs(m) - 1;
+    m &= m - 1;
+    nbits = A.RB[nw * A.S];
+  }
+  while (true) {
+    uint32_t j[4];
+    bool v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      if (!bits && pend) {
+        w = nw;
+        bits = nbits;
+        pend = m != 0u;
+        if (pend) {
+          nw = __ffs(m) - 1;
+          m &= m - 1;
+          nbits = A.RB[nw * A.S];
+        }
+      }
+      v[u] = bits != 0u;
+      j[u] = v[u] ? w * 32u + (__ffs(bits) - 1) : j[0];
+      bits &= bits - 1;
+    }
+    if (!v[0]) return;
+    visit(j, v);
+    if (!v[3] || (!bits && !pend)) return;
+  }
+#else
   uint32_t w = 0, bits = 0;
   while (true) {
     uint32_t j[4];
@@ -324,6 +370,7 @@ __device__ __forceinline__ void scan4(const St &A, uint32_t m, F &&visit) {
     visit(j, v);
     if (!v[3] || (!bits && !m)) return;
   }
+#endif
 }
 
 struct AntOut {
@@ -488,6 +535,24 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) dk[u] = V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+#if ACO_BRANCHLESS1
+        // branch-free: the four candidates' chains interleave (ILP)
+        uint32_t sc[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) sc[u] = v[u] ? tv[u] * dk[u] + 1u : 0u;  // score + 1, 0 = none
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {  // ascending: strict keeps the lowest index
+          const bool b = sc[u] > bs1;
+          bs1 = b ? sc[u] : bs1;
+          bj = b ? j[u] : bj;
+        }
+        if (!exploit) {
+          uint32_t s01 = (sc[0] ? sc[0] - 1u : 0u), s23 = (sc[2] ? sc[2] - 1u : 0u);
+          const uint64_t a = (uint64_t)s01 + (sc[1] ? sc[1] - 1u : 0u);
+          const uint64_t b = (uint64_t)s23 + (sc[3] ? sc[3] - 1u : 0u);
+          sum += a + b;
+        }
+#else
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const uint32_t sc = tv[u] * dk[u];
@@ -499,6 +564,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
             if (!exploit) sum += sc;
           }
         }
+#endif
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
@@ -629,9 +695,40 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
           dk[u] = dk2_get<NC4>(A, j[u]);
           tv[u] = trow[j[u]];
         }
+#if ACO_BRANCHLESS2
+        // branch-free evaluation of the four candidates (ILP); same
+        // semantics as eval() (R21, R22)
+        uint32_t sc[4];
+        bool fe[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t K = ds[u].y + dk[u];
+          const bool ready = v[u] && rd[u] <= t;
+          const bool semi = v[u] && rd[u] > t;
+          fe[u] = ready && __vcmpgtu4(ds[u].x, __vaddus4(slack, K)) == 0u;
+          counts += (ready ? 1u : 0u) + (fe[u] ? 0x10000u : 0u);
+          f_not_inc |= fe[u] && __vcmpgtu4(ds[u].x, K) == 0u;
+          any_s |= semi;
+          min_s = ::min(min_s, semi ? rd[u] : 0xFFFFFFFFu);
+          s_dec |= semi && __vcmpltu4(ds[u].x, K) != 0u;
+          sc[u] = fe[u] ? tv[u] * ds[u].z + 1u : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const bool b = sc[u] > bs1;
+          bs1 = b ? sc[u] : bs1;
+          bj = b ? j[u] : bj;
+        }
+        if (need_sum) {
+          const uint64_t a = (uint64_t)(sc[0] ? sc[0] - 1u : 0u) + (sc[1] ? sc[1] - 1u : 0u);
+          const uint64_t b = (uint64_t)(sc[2] ? sc[2] - 1u : 0u) + (sc[3] ? sc[3] - 1u : 0u);
+          sum += a + b;
+        }
+#else
 #pragma unroll
         for (int u = 0; u < 4; ++u)
           if (v[u]) eval(j[u], rd[u], ds[u], dk[u], tv[u]);
+#endif
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {

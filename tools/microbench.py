@@ -16,7 +16,7 @@ ants = int(os.environ.get("MB_ANTS", "1024"))
 iters = int(os.environ.get("MB_ITERS", "4"))
 tot = {}
 for n in sizes:
-    count = max(8, int(6e6 / (n * n)))
+    count = max(int(os.environ.get("MB_MIN_REGIONS", "160")), int(6e6 / (n * n)))
     regs = [I.gen_region(n, I.region_seed(77, i)) for i in range(count)]
     out = []
     for passes in (1, 3):

@@ -1,4 +1,5 @@
-"""One C3 aco_schedule_batch for profiling under ncu (no timing is reported)."""
+"""One aco_schedule_batch for profiling under ncu (no timing is reported).
+PROF_N=<n>: PROF_REGIONS regions all of n instructions; else the C3 batch."""
 import os
 import sys
 
@@ -10,7 +11,11 @@ from paper_conf_cgo_shobakimhlmkrg24_b200.api import Scheduler  # noqa: E402
 
 n = int(os.environ.get("PROF_REGIONS", "5000"))
 iters = int(os.environ.get("PROF_ITERS", "10"))
-regs = I.gen_batch(n, base_seed=3)
+size = int(os.environ.get("PROF_N", "0"))
+if size:
+    regs = [I.gen_region(size, I.region_seed(77, i)) for i in range(n)]
+else:
+    regs = I.gen_batch(n, base_seed=3)
 s = Scheduler(I.GFX906, device=0)
 s.load(regs, list(range(n)))
 s.run(I.Params(ants=1024, iterations=iters, seed=3))
