@@ -397,6 +397,7 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   R.cp_max = cp_max;
   R.lb_len = std::max(n, n ? cp_max + 1 : 0u);
   R.max_cycle_bound = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)n * (max_lat + 1ull) + 1);
+  R.max_lat = max_lat;
   for (uint32_t c = 0; c < 4; ++c) {
     R.livein[c] = livein[c];
     R.lbvec[c] = lbvec[c];
@@ -623,7 +624,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
     P.max_n = std::max(P.max_n, R.n);
-    const bool t32 = R.max_cycle_bound > 65535u;
+    // pass-2 state variant: the compact layout (windowed u8 ready times) needs
+    // latencies <= 127 and 2 classes; otherwise u16 cycles, or u32 when a
+    // schedule may exceed 65535 cycles (or a latency exceeds 127)
+    const bool t32 = P.nc4 ? R.max_cycle_bound > 65535u : R.max_lat > 127u;
     P.any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);

@@ -67,6 +67,8 @@ struct RegionDev {
   uint32_t max_cycle_bound;  // n * (max latency + 1): pass-2 cycles are below it
   uint32_t livein[4];
   uint32_t lbvec[4]; // per-class PRP lower bound vector (R30)
+  uint32_t max_lat;  // largest edge latency
+  uint32_t pad0;
   uint64_t o_image;  // byte offset of the block image in the arena
   ImageLayout img;
 };
@@ -142,7 +144,11 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 //   RB [nwr] ready set, SCH [nwr] scheduled set, REM [nremw] u16 counters, then
 //   pass 1: DK [ceil(n/8)]  4-bit count of registers whose last remaining
 //                           user is the instruction (dynamic part of LUC)
-//   pass 2: T  [ceil(n/2)] u16 (or [n] u32 if t32): issue cycle (placed) or
+//   pass 2, compact (2 classes, latencies <= 127):
+//           X  [ceil(n/2)] u16: windowed ready time (u8) | last-use counts
+//                           (2 classes x 4 bits) << 8
+//   pass 2, otherwise:
+//           T  [ceil(n/2)] u16 (or [n] u32 if t32): issue cycle (placed) or
 //                           ready time (ready instruction)
 //           DK [ceil(n/4)] u8 = 2 classes x 4 bits (or [ceil(n/2)] u16 = 4
 //                           classes x 4 bits if nc4): per-class last-use counts
@@ -150,6 +156,7 @@ ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32
                                  bool nc4) {
   const uint32_t w = 2 * nwr + nremw;
   if (pass == 1) return w + (n + 7) / 8;
+  if (!t32 && !nc4) return w + (n + 1) / 2;  // compact: u16 (windowed ready time | last uses)
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }
 

@@ -172,7 +172,9 @@ __device__ __forceinline__ St make_st(uint32_t *st, uint32_t S, const SV &V) {
   A.SCH = st + V.nwr * S;
   A.REM = A.SCH + V.nwr * S;
   A.T = A.REM + V.nremw * S;
-  A.DK = PASS == 1 ? A.T : A.T + (T32 ? V.n : (V.n + 1) / 2) * S;
+  // pass 2, compact layout (!T32 && !NC4): one u16 per instruction in T,
+  // ready time (windowed u8) | last-use counts << 8; DK aliases T
+  A.DK = (PASS == 1 || (!T32 && !NC4)) ? A.T : A.T + (T32 ? V.n : (V.n + 1) / 2) * S;
   return A;
 }
 
@@ -197,10 +199,12 @@ __device__ __forceinline__ uint32_t dk2_get(const St &A, uint32_t j) {
   const uint32_t x = (A.DK[(j >> 2) * A.S] >> ((j & 3u) * 8)) & 0xFFu;
   return (x & 0xFu) | ((x & 0xF0u) << 4);
 }
-template <int PASS, bool NC4>
+template <int PASS, bool T32, bool NC4>
 __device__ __forceinline__ void dk_add(const St &A, uint32_t j, uint32_t c) {
   if (PASS == 1) {
     A.DK[(j >> 3) * A.S] += 1u << ((j & 7u) * 4);
+  } else if (!T32 && !NC4) {  // compact: the high byte of j's u16
+    A.T[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 8 + 4 * c);
   } else if (NC4) {
     A.DK[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 4 * c);
   } else {
@@ -222,6 +226,25 @@ __device__ __forceinline__ void t_set(const St &A, uint32_t j, uint32_t v) {
     uint32_t *p = A.T + (j >> 1) * A.S;
     *p = (*p & ~(0xFFFFu << sh)) | (v << sh);
   }
+}
+
+// ---- pass-2 compact layout: x = u16 of instruction j = rt | dk << 8, where
+// rt = (ready time - B) for an unplaced instruction whose predecessors were
+// placed (a push-style maximum of t_p + lat over placed predecessors; 0 for
+// none) and B is the ant's window base.  Invariant: t - B < 128 at every
+// turn and latencies <= 127 (host), so every stored rt <= 254; when t - B
+// reaches 128 the window slides by 128 (saturating: a clamped rt still reads
+// as "ready now", which is all that matters for a value below t).
+__device__ __forceinline__ uint32_t x_get(const St &A, uint32_t j) {
+  return (A.T[(j >> 1) * A.S] >> ((j & 1u) * 16)) & 0xFFFFu;
+}
+__device__ __forceinline__ uint32_t x_dk(uint32_t x) {  // packed u8 x 4 per class
+  return ((x >> 8) & 0xFu) | ((x & 0xF000u) >> 4);
+}
+__device__ __forceinline__ void x_push_rt(const St &A, uint32_t v, uint32_t rt) {
+  uint32_t *p = A.T + (v >> 1) * A.S;
+  const uint32_t sh = (v & 1u) * 16, w = *p, cur = (w >> sh) & 0xFFu;
+  if (rt > cur) *p = w + ((rt - cur) << sh);
 }
 
 // ---- lane groups: LG consecutive lanes of a warp build one ant together.
@@ -388,7 +411,8 @@ __device__ __forceinline__ uint32_t cost_of(uint32_t mode, uint32_t prp01, uint3
 template <int PASS, bool MASK, bool T32, bool NC4>
 __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uint32_t t, uint32_t &wmask,
                                        uint32_t &live01, uint32_t &live23, uint32_t &prp01,
-                                       uint32_t &prp23) {
+                                       uint32_t &prp23, uint32_t B = 0) {
+  constexpr bool CT = PASS == 2 && !T32 && !NC4;
   {
     const uint32_t wi = j >> 5, bit = 1u << (j & 31u);
     const uint32_t nw = A.RB[wi * A.S] & ~bit;
@@ -396,7 +420,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
     if (MASK && !nw) wmask &= ~(1u << wi);
     A.SCH[wi * A.S] |= bit;
   }
-  if (PASS == 2) t_set<T32>(A, j, t);
+  if (PASS == 2 && !CT) t_set<T32>(A, j, t);
   const uint4 inf = V.info[j];
   uint32_t K = inf.y;  // static kills (single-use registers)
   {
@@ -416,7 +440,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
           for (uint32_t k = V.cu_ptr[m]; k < V.cu_ptr[m + 1]; ++k) {
             const uint32_t u = V.cu[k];
             if (!sch_bit(A, u)) {
-              dk_add<PASS, NC4>(A, u, c);
+              dk_add<PASS, T32, NC4>(A, u, c);
               break;
             }
           }
@@ -424,7 +448,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
       } else {  // 2 users: the partner
         const uint32_t p = e & 0x1FFFu;
         if (sch_bit(A, p)) K += 1u << (8 * c);
-        else dk_add<PASS, NC4>(A, p, c);
+        else dk_add<PASS, T32, NC4>(A, p, c);
       }
     }
   }
@@ -442,9 +466,10 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
     const uint32_t v = e & 0x1FFFu;
     bool ready = true;
     uint32_t rdy = t + (e >> 16);
+    if (CT) x_push_rt(A, v, rdy - B);  // ready time = max over placed predecessors
     if (!(e & kSuccSingle)) {
       const uint32_t p0 = V.pred_ptr[v], p1 = V.pred_ptr[v + 1];
-      if (PASS == 2) rdy = 0;
+      if (PASS == 2 && !CT) rdy = 0;
       for (uint32_t k = p0; k < p1; ++k) {
         const uint32_t pe = V.pred[k];
         const uint32_t p = pe & 0xFFFFu;
@@ -452,13 +477,13 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
           ready = false;
           break;
         }
-        if (PASS == 2) rdy = max(rdy, t_get<T32>(A, p) + (pe >> 16));
+        if (PASS == 2 && !CT) rdy = max(rdy, t_get<T32>(A, p) + (pe >> 16));
       }
     }
     if (ready) {
       A.RB[(v >> 5) * A.S] |= 1u << (v & 31u);
       if (MASK) wmask |= 1u << (v >> 5);
-      if (PASS == 2) t_set<T32>(A, v, rdy);
+      if (PASS == 2 && !CT) t_set<T32>(A, v, rdy);
     }
   }
 }
@@ -474,8 +499,9 @@ __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
   }
   for (uint32_t w = 0; w < V.nremw; ++w) A.REM[w * A.S] = V.rem0[w];
   const uint32_t n = V.n;
+  const bool ct = PASS == 2 && !T32 && !NC4;
   const uint32_t tw = PASS == 1 ? 0 : (T32 ? n : (n + 1) / 2);
-  const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (NC4 ? (n + 1) / 2 : (n + 3) / 4);
+  const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
   for (uint32_t w = 0; w < tw + dw; ++w) A.T[w * A.S] = 0;  // T and DK are contiguous
   return wmask;
 }
@@ -637,10 +663,27 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   const uint32_t c2 = 0x80000000u | iter;
   const uint32_t sub = lane_words<LG>(G.lane);
   constexpr bool wide = MASK && WIDE;
-  uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0;
+  constexpr bool CT = !T32 && !NC4;  // compact layout (x_get)
+  uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0, B = 0;
+  // ready time and per-class last-use counts of instruction j
+  auto rd_dk = [&](uint32_t j, uint32_t &rd, uint32_t &dk) {
+    if constexpr (CT) {
+      const uint32_t x = x_get(A, j);
+      rd = B + (x & 0xFFu);
+      dk = x_dk(x);
+    } else {
+      rd = t_get<T32>(A, j);
+      dk = dk2_get<NC4>(A, j);
+    }
+  };
   AntOut o;
   o.prp01 = o.prp23 = 0;
   while (placed < n) {
+    if (CT && t - B >= 128u) {  // slide the ready-time window (t - B <= 254 here)
+      for (uint32_t w = G.lane; w < (n + 1) / 2; w += LG) A.T[w * A.S] = __vsubus4(A.T[w * A.S], 0x00800080u);
+      B += 128u;
+      G.sync();
+    }
     if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune
       uint32_t bl = 0;
       if (G.leader()) bl = *(volatile uint32_t *)prune_len;
@@ -690,9 +733,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         uint4 ds[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          rd[u] = t_get<T32>(A, j[u]);
+          rd_dk(j[u], rd[u], dk[u]);
           ds[u] = V.ds[j[u]];                         // defs, static kills, eta2
-          dk[u] = dk2_get<NC4>(A, j[u]);
           tv[u] = trow[j[u]];
         }
 #if ACO_BRANCHLESS2
@@ -732,7 +774,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
-        eval(j, t_get<T32>(A, j), V.ds[j], dk2_get<NC4>(A, j), trow[j]);
+        uint32_t rd, dk;
+        rd_dk(j, rd, dk);
+        eval(j, rd, V.ds[j], dk, trow[j]);
         return false;
       });
     }
@@ -783,9 +827,11 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
         uint64_t pre = 0;
         scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
-          if (t_get<T32>(A, j) > t) return false;
+          uint32_t rd, dk;
+          rd_dk(j, rd, dk);
+          if (rd > t) return false;
           const uint4 ds = V.ds[j];
-          if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk2_get<NC4>(A, j))) != 0u) return false;
+          if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u) return false;
           pre += (uint32_t)trow[j] * ds.z;
           if (pre > r) {
             jstar = j;
@@ -797,7 +843,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       jstar = G.bcast(jstar);
     }
     if (G.leader()) {
-      commit<2, MASK, T32, NC4>(V, A, jstar, t, wmask, live01, live23, prp01, prp23);
+      commit<2, MASK, T32, NC4>(V, A, jstar, t, wmask, live01, live23, prp01, prp23, B);
       if (rec_o) {
         rec_o[placed] = (uint16_t)jstar;
         rec_c[placed] = t;

@@ -287,3 +287,32 @@ def test_shared_colony_equals_single_context(torch_cuda):
         compare_results(single[k], ora, f"single {k}")
         for r in range(4):
             compare_results(ranks[r][k], ora, f"rank {r} region {k}")
+
+
+def _relat(reg, f, tag):
+    """The same DDG with every edge latency mapped by f (exercises the
+    pass-2 ready-time layouts: windowed u8 for latencies <= 127, u32 beyond)."""
+    lat = np.asarray([f(int(x)) for x in reg.edge_lat], np.uint32)
+    return I.Region(reg.n_insts, reg.edge_src, reg.edge_dst, lat, reg.reg_class, reg.reg_flags,
+                    reg.def_ptr, reg.def_reg, reg.use_ptr, reg.use_reg, name=reg.name + tag)
+
+
+def test_latency_window_boundary_every_ant(torch_cuda):
+    """Latencies up to exactly 127 (the compact layout's bound) and schedules
+    of several hundred cycles (the ready-time window slides many times)."""
+    regs = [_relat(I.gen_region(n, 800 + n), lambda x: 127 if x >= 20 else x, "-l127") for n in (25, 70, 180)]
+    ids = [31, 32, 33]
+    p = I.Params(ants=72, iterations=2, seed=21, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_long_latencies_every_ant(torch_cuda):
+    """Latencies above 127 force the u32 ready-time layout."""
+    regs = [_relat(I.gen_region(n, 900 + n), lambda x: x * 3 + (150 if x >= 20 else 0), "-long") for n in (25, 70, 180)]
+    ids = [41, 42, 43]
+    p = I.Params(ants=72, iterations=2, seed=22, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
