@@ -190,6 +190,30 @@ static int first_occurrence(const orc_region *r, uint32_t j, uint32_t k) {
   return 1;
 }
 
+/* General machine model (L64; R42).  issue_width <= 1: single issue, any
+ * type (R32).  Otherwise at most issue_width instructions per cycle and at
+ * most type_slots[y] of type y. */
+static uint32_t m_width(const orc_machine *m) { return m->issue_width > 1 ? m->issue_width : 1u; }
+static uint32_t m_slots(const orc_machine *m, uint32_t y) {
+  if (m->issue_width <= 1) return 1u;
+  return m->type_slots[y];
+}
+static uint32_t itype(const orc_region *r, uint32_t j) { return r->inst_type ? r->inst_type[j] : 0u; }
+
+/* The machine model and instruction types are consistent (R42). */
+static int machine_check(const orc_region *r, const orc_machine *m) {
+  if (m->issue_width > 1) {
+    if (m->n_types < 1 || m->n_types > 4) return ORC_E_ARG;
+    for (uint32_t y = 0; y < m->n_types; ++y)
+      if (m->type_slots[y] < 1) return ORC_E_ARG;
+  }
+  uint32_t nt = m->issue_width > 1 ? m->n_types : 4u;
+  if (r->inst_type)
+    for (uint32_t j = 0; j < r->n_insts; ++j)
+      if (r->inst_type[j] >= nt) return ORC_E_ARG;
+  return ORC_OK;
+}
+
 static int model_build(model *m, const orc_region *r, uint32_t n_classes) {
   memset(m, 0, sizeof(*m));
   int st = orc_validate(r, n_classes);
@@ -391,6 +415,40 @@ int64_t orc_asap(const orc_region *r, const uint32_t *order, uint32_t *cycle) {
   return prev + 1;
 }
 
+/* ASAP timing of an order on the general machine model (R42, R29): in-order
+ * issue; c_k = max(c_{k-1}, ready time of o_k), moved to c_{k-1} + 1 when
+ * that cycle has no free slot for o_k (issue width or o_k's type); a later
+ * cycle is empty.  For issue_width 1 this is orc_asap. */
+int64_t orc_asap_m(const orc_region *r, const orc_machine *m, const uint32_t *order, uint32_t *cycle) {
+  uint32_t n = r->n_insts;
+  if (n == 0) return 0;
+  uint32_t *c_of = malloc(sizeof(uint32_t) * n);
+  char *placed = calloc(n, 1);
+  int64_t prev = -1;
+  uint32_t used = 0, used_t[4] = {0, 0, 0, 0};
+  for (uint32_t k = 0; k < n; ++k) {
+    uint32_t j = order[k], y = itype(r, j);
+    int64_t t = prev < 0 ? 0 : prev;
+    for (uint32_t e = 0; e < r->n_edges; ++e)
+      if (r->edge_dst[e] == j) {
+        uint32_t p = r->edge_src[e];
+        if (!placed[p]) { free(c_of); free(placed); return -1; }
+        int64_t need = (int64_t)c_of[p] + r->edge_lat[e];
+        if (need > t) t = need;
+      }
+    if (t == prev && (used >= m_width(m) || used_t[y] >= m_slots(m, y))) t = prev + 1;
+    if (t != prev) { used = 0; used_t[0] = used_t[1] = used_t[2] = used_t[3] = 0; }
+    used++;
+    used_t[y]++;
+    c_of[j] = (uint32_t)t;
+    placed[j] = 1;
+    cycle[k] = (uint32_t)t;
+    prev = t;
+  }
+  free(c_of); free(placed);
+  return prev + 1;
+}
+
 /* ------------------------------------------------------------------------ */
 /* Costs (L68-L74; R16-R18).                                                 */
 /* ------------------------------------------------------------------------ */
@@ -475,8 +533,17 @@ int orc_lower_bounds(const orc_region *r, const orc_machine *mach, uint32_t mode
       if (u > lbv[c]) lbv[c] = u;
     }
   *lb_cost = orc_cost_rp(mach, mode, lbv);
-  uint32_t l = n;
+  /* LB_len = max(1 + CPmax, ceil(n / w), max_y ceil(n_y / min(slots_y, w)))
+   * (R30, R42); for the single-issue machine max(n, 1 + CPmax). */
+  uint32_t w = m_width(mach);
+  uint32_t l = (n + w - 1) / w;
   if (n > 0 && m.cp_max + 1 > l) l = m.cp_max + 1;
+  if (w > 1)
+    for (uint32_t y = 0; y < mach->n_types; ++y) {
+      uint32_t ny = 0, s = m_slots(mach, y) < w ? m_slots(mach, y) : w;
+      for (uint32_t j = 0; j < n; ++j) if (itype(r, j) == y) ny++;
+      if ((ny + s - 1) / s > l) l = (ny + s - 1) / s;
+    }
   *lb_len = l;
   /* transitive closure by DFS from each node; UB = 1 + max #independent */
   uint32_t best = 0;
@@ -604,7 +671,11 @@ static void ant_pass1(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
     for (uint32_t j = 0; j < n; ++j) /* ascending index order (R25) */
       if (!a->scheduled[j] && a->pred_left[j] == 0) {
         a->cand[cnt] = j;
-        a->score[cnt] = (uint32_t)tau[(size_t)prev * n + j] * eta1(m, &a->rp, j);
+        /* R43: with heur_mix, odd ant groups are guided by the ILP heuristic
+         * (CP, eta2) instead of LUC-then-CP; the greedy schedule never is */
+        uint32_t e = (!greedy && a->p->heur_mix && ((ant / a->p->group_size) & 1u)) ? eta2(m, j)
+                                                                                    : eta1(m, &a->rp, j);
+        a->score[cnt] = (uint32_t)tau[(size_t)prev * n + j] * e;
         cnt++;
       }
     int exploit;
@@ -640,30 +711,55 @@ static void ant_pass1(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
   out->length = 0;
 }
 
-/* Pass-2 ant (L108, L118, L147-L164, L200-L206; R19-R24).  Each loop turn
- * either stalls (necessary, forced optional, or discretionary) or places one
- * instruction.  Pruning (R24) is a GPU-only, winner-invariant shortcut; the
- * oracle never prunes. */
+/* Is ant group g allowed optional stalls?  (L202-L204; R23, R44) */
+static int stall_enabled_group(const orc_params *p, uint32_t g) {
+  uint32_t mod = p->stall_mod, rem = p->stall_rem % mod;
+  return ((g % mod) + mod - rem) % mod < p->stall_num;
+}
+
+/* Pass-2 ant (L108, L118, L147-L164, L200-L206; R19-R24), on the general
+ * machine model (L64; R42).  Each loop turn either stalls (necessary, forced
+ * optional, or discretionary), or places one instruction in the current
+ * cycle t; the cycle is complete when issue_width instructions were placed
+ * in it.  An instruction whose latency is met but whose issue slot (width or
+ * type) is full this cycle counts as semi-ready with ready time t + 1.
+ * The Philox step is t * issue_width + (instructions already placed in t),
+ * which is t on the single-issue machine.
+ * weighted (pass 4, R41): no RP target, cost = length + W * cost_rp(PRP).
+ * Pruning (R24) is a GPU-only, winner-invariant shortcut; the oracle never
+ * prunes. */
 static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *tau,
                       uint32_t *order, uint32_t *cycle_of, ant_out *out) {
   const model *m = a->m;
   const orc_params *p = a->p;
-  uint32_t n = m->n, nc = m->n_classes;
+  const orc_machine *mach = a->mach;
+  const orc_region *src = m->src;
+  uint32_t n = m->n, nc = m->n_classes, w = m_width(mach);
   for (uint32_t j = 0; j < n; ++j) { a->pred_left[j] = m->indeg[j]; a->rdy[j] = 0; a->scheduled[j] = 0; }
   rp_init(m, &a->rp);
   uint32_t prev = ROOT_ROW(n), placed = 0;
-  uint64_t t = 0, k_opt = 0;
-  int stall_enabled = ((ant / p->group_size) % p->stall_mod) == p->stall_rem; /* R23 */
+  uint64_t t = 0, k_opt = 0, last = 0;
+  uint32_t used = 0, used_t[4] = {0, 0, 0, 0};
+  uint32_t group = ant / p->group_size;
+  int stall_enabled = stall_enabled_group(p, group); /* R23, R44 */
+  int use_eta1 = p->heur_mix && (group & 1u);        /* R43 */
   uint32_t *rlist = a->cand;   /* R in ascending order */
   uint32_t *flist = a->flist;
   uint32_t *fscore = a->score;
   while (placed < n) {
+    uint32_t step = (uint32_t)(t * w + used);
     uint32_t nr = 0, nf = 0, ns = 0;
     uint64_t min_s = UINT64_MAX;
     for (uint32_t j = 0; j < n; ++j) {
       if (a->scheduled[j] || a->pred_left[j]) continue;
-      if (a->rdy[j] <= t) rlist[nr++] = j;
-      else { ns++; if (a->rdy[j] < min_s) min_s = a->rdy[j]; }
+      uint32_t y = itype(src, j);
+      int slot = used < w && used_t[y] < m_slots(mach, y);
+      if (a->rdy[j] <= t && slot) rlist[nr++] = j;
+      else {
+        uint64_t eff = a->rdy[j] <= t ? t + 1 : a->rdy[j]; /* slot-blocked: next cycle */
+        ns++;
+        if (eff < min_s) min_s = eff;
+      }
     }
     for (uint32_t q = 0; q < nr; ++q) { /* F = RP-feasible part of R (R21) */
       uint32_t j = rlist[q];
@@ -675,6 +771,7 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
     if (a->stats) { a->stats[ORS_SUM_R] += nr; a->stats[ORS_SUM_S] += ns; }
     if (nr == 0) { /* necessary stall (L153): skip ahead to the next ready time */
       t = min_s;
+      used = 0; used_t[0] = used_t[1] = used_t[2] = used_t[3] = 0;
       if (a->stats) a->stats[ORS_STALL_EVENTS]++;
       continue;
     }
@@ -682,6 +779,7 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
       if (stall_enabled && ns > 0) { /* forced optional stall (L155, R22) */
         k_opt += min_s - t;
         t = min_s;
+        used = 0; used_t[0] = used_t[1] = used_t[2] = used_t[3] = 0;
         if (a->stats) a->stats[ORS_STALL_EVENTS]++;
         continue;
       }
@@ -704,7 +802,9 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
         if (!(mx > 0)) all_f_increase = 0;
       }
       for (uint32_t j = 0; j < n; ++j) {
-        if (a->scheduled[j] || a->pred_left[j] || a->rdy[j] <= t) continue;
+        if (a->scheduled[j] || a->pred_left[j]) continue;
+        uint32_t y = itype(src, j);
+        if (a->rdy[j] <= t && used < w && used_t[y] < m_slots(mach, y)) continue; /* in R */
         int64_t mn = INT64_MAX;
         for (uint32_t c = 0; c < nc; ++c) {
           int64_t d = rp_delta(m, &a->rp, j, c);
@@ -713,24 +813,26 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
         if (mn < 0) some_s_decrease = 1;
       }
       if (all_f_increase && some_s_decrease) {
-        draw_ant(p->seed, a->region_id, 2, iter, ant, (uint32_t)t, x);
+        draw_ant(p->seed, a->region_id, 2, iter, ant, step, x);
         have_x = 1;
         uint32_t thr = (k_opt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (k_opt + 1));
         if (x[2] < thr) { /* probability 2^-(k_opt+1) */
           k_opt++;
           t++;
+          used = 0; used_t[0] = used_t[1] = used_t[2] = used_t[3] = 0;
           if (a->stats) a->stats[ORS_STALL_EVENTS]++;
           continue;
         }
       }
     }
     for (uint32_t q = 0; q < nf; ++q)
-      fscore[q] = (uint32_t)tau[(size_t)prev * n + flist[q]] * eta2(m, flist[q]);
-    uint32_t coin = draw_group_coin(p->seed, a->region_id, 2, iter, ant / p->group_size, (uint32_t)t);
+      fscore[q] = (uint32_t)tau[(size_t)prev * n + flist[q]] *
+                  (use_eta1 ? eta1(m, &a->rp, flist[q]) : eta2(m, flist[q]));
+    uint32_t coin = draw_group_coin(p->seed, a->region_id, 2, iter, group, step);
     int exploit = (uint64_t)coin < p->q0_t;
     uint64_t r64 = 0;
     if (!exploit) {
-      if (!have_x) draw_ant(p->seed, a->region_id, 2, iter, ant, (uint32_t)t, x);
+      if (!have_x) draw_ant(p->seed, a->region_id, 2, iter, ant, step, x);
       r64 = ((uint64_t)x[1] << 32) | x[0];
     }
     uint32_t j = flist[orc_select(fscore, nf, exploit, r64)];
@@ -744,6 +846,7 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
     rp_issue(m, &a->rp, j);
     a->scheduled[j] = 1;
     cycle_of[j] = (uint32_t)t;
+    last = t;
     order[placed++] = j;
     for (uint32_t q = m->succ_ptr[j]; q < m->succ_ptr[j + 1]; ++q) {
       uint32_t v = m->succ[q];
@@ -752,11 +855,18 @@ static void ant_pass2(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *t
       if (need > a->rdy[v]) a->rdy[v] = (uint32_t)need;
     }
     prev = j;
-    t++;
+    used++;
+    used_t[itype(src, j)]++;
+    if (used == w) { /* the cycle is full */
+      t++;
+      used = 0; used_t[0] = used_t[1] = used_t[2] = used_t[3] = 0;
+    }
   }
   for (uint32_t c = 0; c < 4; ++c) out->prp[c] = a->rp.prp[c];
-  out->length = (uint32_t)t; /* last issue cycle + 1 (R20) */
+  out->length = n ? (uint32_t)last + 1 : 0; /* last issue cycle + 1 (R20) */
   out->cost = out->length;
+  if (p->pass == 4) /* weighted single pass (L74; R41) */
+    out->cost = out->length + p->ws_weight * orc_cost_rp(a->mach, p->cost_mode, a->rp.prp);
 }
 
 /* FNV-1a (64-bit) over (pass, iter, winner cost, winner ant), little endian. */
@@ -774,17 +884,88 @@ static uint32_t no_improve_limit(const orc_params *p, uint32_t n) {
 }
 
 /* ------------------------------------------------------------------------ */
+/* The single weighted-sum pass (L74; R41): the ILP-pass construction with  */
+/* no RP target, cost = length + W * cost_rp(PRP), from the heuristic order  */
+/* timed ASAP.  Same iteration loop as the two passes (R5-R12).              */
+/* ------------------------------------------------------------------------ */
+static int weighted_pass(ant_ctx *a, const orc_region *r, const orc_machine *mach, const orc_params *p,
+                         const model *m, uint16_t *tau, const uint32_t *heur_order, uint32_t lb_cost,
+                         uint32_t lb_len, uint32_t *ant_order, uint32_t *ant_cycle_of, uint32_t *win_order,
+                         uint32_t *win_cycle_of, uint32_t *best_order, uint32_t *best_cycle_of,
+                         uint32_t *tmp_cycle, uint64_t *hash, uint64_t *stats, uint32_t *dump_cost,
+                         uint32_t *dump_order, uint32_t *dump_cycle) {
+  uint32_t n = m->n;
+  for (uint32_t c = 0; c < 4; ++c) a->target[c] = 0xFFFFFFFFu; /* no target */
+  for (uint32_t c = 0; c < 4; ++c) stats[ORS_TARGET0 + c] = a->target[c];
+  int64_t init_len = orc_asap_m(r, mach, heur_order, tmp_cycle);
+  uint32_t prp[4];
+  orc_prp_of_order(r, mach->n_classes, heur_order, prp);
+  uint32_t best = (uint32_t)init_len + p->ws_weight * orc_cost_rp(mach, p->cost_mode, prp);
+  uint32_t best_len = (uint32_t)init_len;
+  uint32_t lb = lb_len + p->ws_weight * lb_cost;
+  for (uint32_t k = 0; k < n; ++k) {
+    best_order[k] = heur_order[k];
+    best_cycle_of[heur_order[k]] = tmp_cycle[k];
+  }
+  stats[ORS_INIT2] = best;
+  for (size_t q = 0; q < (size_t)(n + 1) * n; ++q) tau[q] = (uint16_t)p->tau0;
+  uint32_t nimp = 0, lim = no_improve_limit(p, n);
+  int skip = p->stop_at_lb && best == lb;
+  for (uint32_t it = 0; it < p->iterations && !skip; ++it) {
+    uint64_t wkey = UINT64_MAX;
+    uint32_t wcost = INVALID_COST, wlen = 0;
+    for (uint32_t ant = 0; ant < p->ants; ++ant) {
+      ant_out o;
+      ant_pass2(a, it, ant, tau, ant_order, ant_cycle_of, &o);
+      stats[ORS_ANT_SCHEDS]++;
+      if (dump_cost) dump_cost[((size_t)1 * p->iterations + it) * p->ants + ant] = o.cost;
+      if (dump_order || dump_cycle) {
+        size_t base = (((size_t)1 * p->iterations + it) * p->ants + ant) * n;
+        if (dump_order) memcpy(dump_order + base, ant_order, sizeof(uint32_t) * n);
+        if (dump_cycle)
+          for (uint32_t k = 0; k < n; ++k) dump_cycle[base + k] = ant_cycle_of[ant_order[k]];
+      }
+      uint64_t key = ((uint64_t)o.cost << 32) | ant; /* R10 */
+      if (key < wkey) {
+        wkey = key; wcost = o.cost; wlen = o.length;
+        memcpy(win_order, ant_order, sizeof(uint32_t) * n);
+        memcpy(win_cycle_of, ant_cycle_of, sizeof(uint32_t) * n);
+      }
+    }
+    orc_pheromone_update(tau, n, win_order, p);
+    *hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(*hash, 4), it), wcost), (uint32_t)wkey);
+    if (wcost < best) { /* R11 */
+      best = wcost; best_len = wlen;
+      memcpy(best_order, win_order, sizeof(uint32_t) * n);
+      memcpy(best_cycle_of, win_cycle_of, sizeof(uint32_t) * n);
+      nimp = 0;
+    } else {
+      nimp++;
+    }
+    stats[ORS_ITERS2] = it + 1;
+    if ((p->stop_at_lb && best == lb) || (lim > 0 && nimp >= lim)) break;
+  }
+  stats[ORS_BEST2] = best;
+  stats[ORS_WS_COST] = best;
+  stats[ORS_LENGTH] = best_len;
+  return ORC_OK;
+}
+
+/* ------------------------------------------------------------------------ */
 /* The two-pass ACO (L106-L139; R5-R13).                                     */
 /* ------------------------------------------------------------------------ */
 int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mach,
                  const orc_params *p, uint32_t *order_out, uint32_t *cycle_out,
                  uint64_t *stats, uint32_t *dump_cost, uint32_t *dump_order,
                  uint32_t *dump_cycle, uint16_t *tau_out) {
-  if (p->pass < 1 || p->pass > 3 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
-      p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u)
+  if (p->pass < 1 || p->pass > 4 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
+      p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->ws_weight > 1024u ||
+      p->heur_mix > 1u)
     return ORC_E_ARG;
+  int st = machine_check(r, mach);
+  if (st != ORC_OK) return st;
   model m;
-  int st = model_build(&m, r, mach->n_classes);
+  st = model_build(&m, r, mach->n_classes);
   if (st != ORC_OK) return st;
   uint32_t n = m.n;
   uint64_t local_stats[ORS_COUNT];
@@ -810,7 +991,7 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
   uint32_t *win_cycle_of = malloc(sizeof(uint32_t) * (n + 1));
   uint32_t *tmp_cycle = malloc(sizeof(uint32_t) * (n + 1));
 
-  uint32_t lb_cost, lb_len, ub;
+  uint32_t lb_cost, lb_len, ub, final_len = 0;
   orc_lower_bounds(r, mach, p->cost_mode, &lb_cost, &lb_len, &ub);
   stats[ORS_LB1] = lb_cost; stats[ORS_LBLEN] = lb_len; stats[ORS_UB_READY] = ub;
   uint64_t hash = 0xcbf29ce484222325ull;
@@ -821,6 +1002,20 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
   ant_out best1;
   ant_pass1(&a, 0, 0, tau, 1, best_order, &best1);
   stats[ORS_INIT1] = best1.cost;
+  /* the heuristic schedule H (R40): the greedy order timed ASAP */
+  uint32_t *heur_order = malloc(sizeof(uint32_t) * (n + 1));
+  memcpy(heur_order, best_order, sizeof(uint32_t) * n);
+  ant_out heur = best1;
+  stats[ORS_HEUR_LEN] = (uint64_t)orc_asap_m(r, mach, heur_order, tmp_cycle);
+  stats[ORS_POLICY] = 0;
+  if (p->pass == 4) { /* the single weighted-sum pass (L74; R41) */
+    stats[ORS_BEST1] = best1.cost;
+    st = weighted_pass(&a, r, mach, p, &m, tau, heur_order, lb_cost, lb_len, ant_order, ant_cycle_of,
+                       win_order, win_cycle_of, best_order, best_cycle_of, tmp_cycle, &hash, stats,
+                       dump_cost, dump_order, dump_cycle);
+    final_len = (uint32_t)stats[ORS_LENGTH];
+    goto report;
+  }
 
   /* ---- pass 1 (the RP pass) ---- */
   if (p->pass & 1u) {
@@ -857,14 +1052,17 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
   stats[ORS_BEST1] = best1.cost;
 
   /* ---- pass 2 (the ILP pass) ---- */
-  uint32_t final_len;
-  int64_t init_len = orc_asap(r, best_order, tmp_cycle); /* R29 */
+  int64_t init_len = orc_asap_m(r, mach, best_order, tmp_cycle); /* R29, R42 */
   for (uint32_t k = 0; k < n; ++k) best_cycle_of[best_order[k]] = tmp_cycle[k];
   final_len = (uint32_t)init_len;
   stats[ORS_INIT2] = (uint32_t)init_len;
   orc_target(mach, p->cost_mode, best1.prp, a.target); /* R18 */
   for (uint32_t c = 0; c < 4; ++c) stats[ORS_TARGET0 + c] = a.target[c];
-  if (p->pass & 2u) {
+  /* cycle-gap filter (L362, L393-L417; R39): pass 2 only if the input
+   * schedule is at least pass2_gap cycles above LB_len */
+  int gap_skip = (p->pass & 2u) && p->pass2_gap > 0 && init_len - (int64_t)lb_len < (int64_t)p->pass2_gap;
+  if (gap_skip) stats[ORS_POLICY] |= 1u;
+  if ((p->pass & 2u) && !gap_skip) {
     for (size_t q = 0; q < (size_t)(n + 1) * n; ++q) tau[q] = (uint16_t)p->tau0; /* R13 */
     uint32_t best_len = (uint32_t)init_len;
     uint32_t nimp = 0, lim = no_improve_limit(p, n);
@@ -911,11 +1109,33 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
   } else {
     stats[ORS_BEST2] = (uint32_t)init_len;
   }
+report:
   if (tau_out) memcpy(tau_out, tau, sizeof(uint16_t) * (size_t)(n + 1) * n);
 
   /* report: final order, its cycles, its PRP recomputed, cost_rp, length */
   uint32_t prp[4];
   orc_prp_of_order(r, mach->n_classes, best_order, prp);
+  /* post-scheduling revert filter (L366; R40): when ACO raised the
+   * occupancy by at least revert_occ but lengthened the schedule by more
+   * than revert_len cycles, the heuristic schedule H is reported instead */
+  if (p->revert_occ > 0) {
+    uint32_t occ_f = mach->occ_max, occ_h = mach->occ_max;
+    for (uint32_t c = 0; c < mach->n_classes; ++c) {
+      uint32_t of = orc_occupancy(mach, c, prp[c]), oh = orc_occupancy(mach, c, heur.prp[c]);
+      if (of < occ_f) occ_f = of;
+      if (oh < occ_h) occ_h = oh;
+    }
+    if (occ_f >= occ_h + p->revert_occ && (uint64_t)final_len > stats[ORS_HEUR_LEN] + p->revert_len) {
+      stats[ORS_POLICY] |= 2u;
+      orc_asap_m(r, mach, heur_order, tmp_cycle);
+      for (uint32_t k = 0; k < n; ++k) {
+        best_order[k] = heur_order[k];
+        best_cycle_of[heur_order[k]] = tmp_cycle[k];
+      }
+      final_len = (uint32_t)stats[ORS_HEUR_LEN];
+      for (uint32_t c = 0; c < 4; ++c) prp[c] = heur.prp[c];
+    }
+  }
   for (uint32_t k = 0; k < n; ++k) {
     order_out[k] = best_order[k];
     cycle_out[k] = best_cycle_of[best_order[k]];
@@ -927,9 +1147,9 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
 
   free(a.pred_left); free(a.rdy); free(a.cand); free(a.score); free(a.flist); free(a.scheduled); free(a.rp.rem);
   free(tau); free(ant_order); free(ant_cycle_of); free(best_order); free(win_order);
-  free(best_cycle_of); free(win_cycle_of); free(tmp_cycle);
+  free(best_cycle_of); free(win_cycle_of); free(tmp_cycle); free(heur_order);
   model_free(&m);
-  return ORC_OK;
+  return st;
 }
 
 /* ------------------------------------------------------------------------ */

@@ -38,6 +38,7 @@ typedef struct {
   const uint8_t *reg_flags; /* bit0 LIVE_IN, bit1 LIVE_OUT */
   const uint32_t *def_ptr, *def_reg; /* CSR over instructions */
   const uint32_t *use_ptr, *use_reg; /* CSR over instructions */
+  const uint8_t *inst_type; /* issue type of each instruction (R42); NULL = all type 0 */
 } orc_region;
 
 /* Occupancy model per register class (R16). */
@@ -46,18 +47,30 @@ typedef struct {
   uint32_t step_count[4];
   uint32_t step_max[4][16]; /* max PRP giving occupancy occ_max, occ_max-1, ... */
   uint32_t perp_limit[4];
+  /* general machine model (L64; R42): up to issue_width instructions per
+   * cycle, at most type_slots[y] of issue type y.  issue_width <= 1 is the
+   * single-issue machine of the paper's experiments (R32). */
+  uint32_t issue_width, n_types;
+  uint32_t type_slots[4];
 } orc_machine;
 
 typedef struct {
   uint32_t ants, iterations;
   uint64_t seed;
-  uint32_t pass;      /* 1 = RP pass only, 2 = ILP pass only (pass-1 best = heuristic), 3 = both */
+  uint32_t pass;      /* 1 = RP pass only, 2 = ILP pass only (pass-1 best = heuristic), 3 = both,
+                         4 = single weighted-sum pass (L74; R41) */
   uint32_t cost_mode; /* 0 PRP_SUM, 1 APRP_SUM, 2 OCC, 3 PERP */
   uint64_t q0_t;      /* exploit iff group coin (u32) < q0_t; 2^32 = always */
   uint32_t group_size, stall_mod, stall_rem;
   uint32_t tau0, rho_q16, delta, tau_min, tau_max;
   uint32_t stop_no_improve; /* 0 off; 0xFFFFFFFF = paper size classes */
   uint32_t stop_at_lb;
+  /* region-level compile policy (L362, L366, L393-L417; R39, R40) */
+  uint32_t pass2_gap;              /* run pass 2 iff initial length - LB_len >= pass2_gap (0 = off) */
+  uint32_t revert_occ, revert_len; /* revert to the heuristic schedule (revert_occ 0 = off) */
+  uint32_t ws_weight;              /* pass 4: cost = length + ws_weight * cost_rp (R41) */
+  uint32_t heur_mix;               /* 1: odd ant groups use the other pass's heuristic (L216-L218; R43) */
+  uint32_t stall_num;              /* group g may stall iff (g - stall_rem) mod stall_mod < stall_num (R44) */
 } orc_params;
 
 /* Indices into the u64 result vector filled by orc_schedule. */
@@ -70,6 +83,10 @@ enum {
   ORS_ANT_SCHEDS, ORS_PLACEMENTS, ORS_STALL_EVENTS, ORS_SUM_R, ORS_SUM_F,
   ORS_SUM_S, ORS_SUM_DEG, ORS_SUM_USE, ORS_SUM_DEF, ORS_SUM_MUSE_CHECKS,
   ORS_DEAD_ANTS, ORS_UB_READY,
+  /* compile policy / weighted pass (R39-R41) */
+  ORS_POLICY,   /* bit0: pass 2 filtered by the cycle gap; bit1: reverted to the heuristic */
+  ORS_HEUR_LEN, /* length of the heuristic schedule (greedy order, ASAP) */
+  ORS_WS_COST,  /* pass 4: final weighted cost */
   ORS_COUNT
 };
 
@@ -84,6 +101,9 @@ int orc_prp_of_order(const orc_region *r, uint32_t n_classes, const uint32_t *or
 
 /* ASAP cycles of an order (R29); returns the length. */
 int64_t orc_asap(const orc_region *r, const uint32_t *order, uint32_t *cycle);
+/* Same on the general machine model (R42): in-order issue, <= issue_width per
+ * cycle and <= type_slots[y] of type y per cycle. */
+int64_t orc_asap_m(const orc_region *r, const orc_machine *m, const uint32_t *order, uint32_t *cycle);
 
 /* Critical path heights (R4). */
 int orc_critical_path(const orc_region *r, uint32_t *cp);

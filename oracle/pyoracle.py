@@ -23,6 +23,7 @@ ORS_NAMES = [
     "best1", "best2", "lb1", "lblen", "init1", "init2", "target0", "target1", "target2",
     "target3", "ant_scheds", "placements", "stall_events", "sum_R", "sum_F", "sum_S",
     "sum_deg", "sum_use", "sum_def", "sum_muse_checks", "dead_ants", "ub_ready",
+    "policy", "heur_len", "ws_cost",
 ]
 ORS = {name: i for i, name in enumerate(ORS_NAMES)}
 ORS_COUNT = len(ORS_NAMES)
@@ -45,7 +46,7 @@ class _Region(C.Structure):
         ("edge_src", C.c_void_p), ("edge_dst", C.c_void_p), ("edge_lat", C.c_void_p),
         ("reg_class", C.c_void_p), ("reg_flags", C.c_void_p),
         ("def_ptr", C.c_void_p), ("def_reg", C.c_void_p),
-        ("use_ptr", C.c_void_p), ("use_reg", C.c_void_p),
+        ("use_ptr", C.c_void_p), ("use_reg", C.c_void_p), ("inst_type", C.c_void_p),
     ]
 
 
@@ -54,6 +55,7 @@ class _Machine(C.Structure):
         ("n_classes", C.c_uint32), ("occ_max", C.c_uint32),
         ("step_count", C.c_uint32 * 4), ("step_max", (C.c_uint32 * 16) * 4),
         ("perp_limit", C.c_uint32 * 4),
+        ("issue_width", C.c_uint32), ("n_types", C.c_uint32), ("type_slots", C.c_uint32 * 4),
     ]
 
 
@@ -65,6 +67,8 @@ class _Params(C.Structure):
         ("tau0", C.c_uint32), ("rho_q16", C.c_uint32), ("delta", C.c_uint32),
         ("tau_min", C.c_uint32), ("tau_max", C.c_uint32),
         ("stop_no_improve", C.c_uint32), ("stop_at_lb", C.c_uint32),
+        ("pass2_gap", C.c_uint32), ("revert_occ", C.c_uint32), ("revert_len", C.c_uint32),
+        ("ws_weight", C.c_uint32), ("heur_mix", C.c_uint32), ("stall_num", C.c_uint32),
     ]
 
 
@@ -82,6 +86,8 @@ def lib():
         L.orc_prp_of_order.argtypes = [vp, u32, vp, vp]
         L.orc_asap.argtypes = [vp, vp, vp]
         L.orc_asap.restype = C.c_int64
+        L.orc_asap_m.argtypes = [vp, vp, vp, vp]
+        L.orc_asap_m.restype = C.c_int64
         L.orc_critical_path.argtypes = [vp, vp]
         L.orc_occupancy.argtypes = [vp, u32, u32]
         L.orc_occupancy.restype = u32
@@ -119,7 +125,10 @@ class RegionRef:
         self.arrays = [a if a.size else np.zeros(1, a.dtype) for a in self.arrays]
         a = self.arrays
         self.n = int(r.n_insts)
-        self.s = _Region(self.n, int(r.n_edges), int(r.n_regs), *[x.ctypes.data for x in a])
+        it = getattr(r, "inst_type", None)
+        self.types = None if it is None else np.ascontiguousarray(it, np.uint8)
+        tp = None if self.types is None or not self.types.size else self.types.ctypes.data
+        self.s = _Region(self.n, int(r.n_edges), int(r.n_regs), *[x.ctypes.data for x in a], tp)
 
     @property
     def ref(self):
@@ -136,13 +145,18 @@ def machine_struct(m) -> _Machine:
             s.step_max[c][i] = v
     for c in range(4):
         s.perp_limit[c] = m.perp_limit[c] if c < len(m.perp_limit) else 0
+    s.issue_width = getattr(m, "issue_width", 1)
+    s.n_types = getattr(m, "n_types", 1)
+    for y, v in enumerate(getattr(m, "type_slots", (1, 1, 1, 1))):
+        s.type_slots[y] = v
     return s
 
 
 def params_struct(p) -> _Params:
     return _Params(p.ants, p.iterations, p.seed, p.passes, p.cost_mode, p.q0_t, p.group_size,
                    p.stall_mod, p.stall_rem, p.tau0, p.rho_q16, p.delta, p.tau_min, p.tau_max,
-                   p.stop_no_improve, p.stop_at_lb)
+                   p.stop_no_improve, p.stop_at_lb, p.pass2_gap, p.revert_occ, p.revert_len,
+                   p.ws_weight, p.heur_mix, p.stall_num)
 
 
 def philox(ctr: Sequence[int], key: Sequence[int]):
@@ -172,6 +186,16 @@ def asap(region, order):
     o = np.ascontiguousarray(order, np.uint32)
     cyc = np.zeros(max(1, len(o)), np.uint32)
     length = lib().orc_asap(rr.ref, _ptr(o) if o.size else None, cyc.ctypes.data)
+    return int(length), [int(x) for x in cyc[:len(o)]]
+
+
+def asap_m(region, machine, order):
+    """ASAP timing on the general machine model (R42)."""
+    rr = RegionRef(region)
+    m = machine_struct(machine)
+    o = np.ascontiguousarray(order, np.uint32)
+    cyc = np.zeros(max(1, len(o)), np.uint32)
+    length = lib().orc_asap_m(rr.ref, C.byref(m), _ptr(o) if o.size else None, cyc.ctypes.data)
     return int(length), [int(x) for x in cyc[:len(o)]]
 
 

@@ -46,6 +46,7 @@ class Region:
     use_ptr: np.ndarray  # uint32 [n+1]
     use_reg: np.ndarray  # uint32
     name: str = ""
+    inst_type: Optional[np.ndarray] = None  # uint8 [n] issue type (R42); None = all type 0
 
     @property
     def n_edges(self) -> int:
@@ -56,7 +57,7 @@ class Region:
         return int(self.reg_class.shape[0])
 
     @staticmethod
-    def from_lists(n, edges, reg_class, reg_flags, defs, uses, name=""):
+    def from_lists(n, edges, reg_class, reg_flags, defs, uses, name="", inst_type=None):
         """edges: [(src, dst, lat)], defs/uses: per-instruction lists of reg ids."""
         e = np.asarray(edges, dtype=np.uint32).reshape(-1, 3)
         dptr = np.zeros(n + 1, np.uint32)
@@ -78,6 +79,7 @@ class Region:
             use_ptr=uptr,
             use_reg=ureg,
             name=name,
+            inst_type=None if inst_type is None else np.asarray(inst_type, np.uint8),
         )
 
     def defs(self, j: int) -> List[int]:
@@ -103,9 +105,18 @@ class Machine:
         (80, 88, 100, 102),  # SGPR: occupancy 10..7
     )
     perp_limit: Sequence[int] = (24, 80, 0, 0)
+    # general machine model (L64; R42): issue_width <= 1 = single issue, any type
+    issue_width: int = 1
+    n_types: int = 1
+    type_slots: Sequence[int] = (1, 1, 1, 1)
 
 
 GFX906 = Machine()
+# Issue types of the synthetic generator (R42): VALU, SALU, memory (VMEM/SMEM/LDS/store).
+TYPE_VALU, TYPE_SALU, TYPE_MEM = 0, 1, 2
+# A dual-issue machine for the general-model rows: two instructions per cycle,
+# at most one of each type (a VLIW-like pairing; not a GCN fact).
+DUAL_ISSUE = Machine(issue_width=2, n_types=3, type_slots=(1, 1, 1, 1))
 
 # --------------------------------------------------------------------------
 # Parameters (defaults: DESIGN.md section 3).  Integers only.
@@ -132,6 +143,21 @@ class Params:
     tau_max: int = 32768
     stop_no_improve: int = 0
     stop_at_lb: int = 0
+    # region-level compile policy (L362, L366; R39, R40): 0 = off
+    pass2_gap: int = 0
+    revert_occ: int = 0
+    revert_len: int = 0
+    ws_weight: int = 0  # passes == 4: cost = length + ws_weight * cost_rp (L74; R41)
+    heur_mix: int = 0  # 1: odd ant groups use the other pass's heuristic (L216-L218; R43)
+    stall_num: int = 1  # group g may stall iff (g - stall_rem) % stall_mod < stall_num (R44)
+
+
+def paper_policy(p: "Params") -> "Params":
+    """The paper's compile-time filters on top of p: stop at the LB (L251),
+    size-class termination (L226), pass-2 cycle gap 21 (L362, Table 7) and
+    the 3-occupancy / 63-cycle revert filter (L366)."""
+    return dataclasses.replace(p, stop_at_lb=1, stop_no_improve=STOP_PAPER_CLASSES, pass2_gap=21,
+                               revert_occ=3, revert_len=63)
 
 
 # --------------------------------------------------------------------------
@@ -248,7 +274,10 @@ def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "") -> Reg
         elif rng.random() < 0.03:
             reg_flags[g] |= LIVE_OUT
     edges = sorted((s, d, l) for (s, d), l in edge_lat.items())
-    return Region.from_lists(n, edges, reg_class, reg_flags, defs, uses, name=name or f"synth-n{n}-s{seed}")
+    itype = [TYPE_VALU if _KINDS[int(k)] == "valu" else TYPE_SALU if _KINDS[int(k)] == "salu" else TYPE_MEM
+             for k in kinds]
+    return Region.from_lists(n, edges, reg_class, reg_flags, defs, uses, name=name or f"synth-n{n}-s{seed}",
+                             inst_type=itype)
 
 
 def region_seed(base: int, region_id: int) -> int:

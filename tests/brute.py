@@ -187,3 +187,62 @@ def no_optional_stall_schedules(region, target, n_classes=2):
 
     rec(0)
     return found
+
+
+# ---------------------------------------------------------------------------
+# General machine model (R42), written as a
+# cycle-stepped simulation (the oracle uses a closed max() recurrence).
+def asap_machine(region, order: Sequence[int], width: int, slots: Sequence[int],
+                 types: Sequence[int]) -> Tuple[int, List[int]]:
+    """In-order issue of `order`: at cycle t issue the next instruction if its
+    operands are ready and the cycle has a free slot (width and its type),
+    else move to cycle t + 1."""
+    P = preds_of(region)
+    cyc: Dict[int, int] = {}
+    out: List[int] = []
+    t, used, used_t = 0, 0, [0, 0, 0, 0]
+    k = 0
+    while k < len(order):
+        j = order[k]
+        y = int(types[j]) if types is not None else 0
+        ready = max([cyc[p] + l for p, l in P[j]] + [0])
+        free = used < width and (width <= 1 or used_t[y] < slots[y])
+        if ready <= t and free:
+            cyc[j] = t
+            out.append(t)
+            used += 1
+            used_t[y] += 1
+            k += 1
+        else:
+            t += 1
+            used, used_t = 0, [0, 0, 0, 0]
+    return (out[-1] + 1 if out else 0), out
+
+
+def optimum_machine(region, machine, mode: int, target=None, weight=None):
+    """Best length under target (and/or best length + weight * cost) over all
+    topological orders, each timed by asap_machine."""
+    w = max(1, machine.issue_width)
+    best_t = math.inf
+    best_w = math.inf
+    for o in topo_orders(region):
+        prp = prp_interval(region, o, machine.n_classes)
+        L, _ = asap_machine(region, o, w, machine.type_slots, region.inst_type)
+        if target is None or all(prp[c] <= target[c] for c in range(machine.n_classes)):
+            best_t = min(best_t, L)
+        if weight is not None:
+            best_w = min(best_w, L + weight * cost(machine, mode, prp))
+    return best_t, best_w
+
+
+def occupancy(machine, prp: Sequence[int]) -> int:
+    """min over classes of the occupancy table lookup (L68-L72)."""
+    occ = machine.occ_max
+    for c in range(machine.n_classes):
+        o = 0
+        for i, s in enumerate(machine.steps[c]):
+            if prp[c] <= s:
+                o = machine.occ_max - i
+                break
+        occ = min(occ, o)
+    return occ

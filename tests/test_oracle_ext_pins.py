@@ -1,0 +1,356 @@
+"""Pins for the oracle's SURVEY 8(f) rows: the general machine model (f1),
+mixed heuristics and the optional-stall fraction (f2), the region-level
+compile policy (f3) and the weighted-sum single pass (f4).
+
+Each check pins the oracle to something other than itself: textbook list
+scheduling written here from its definition, exhaustive enumeration with the
+cycle-stepped machine simulation of tests/brute.py, closed forms, and the
+independent schedule checker.  DESIGN.md R39-R44 state the readings.
+"""
+import dataclasses
+
+import numpy as np
+import pytest
+
+from oracle import pyoracle as O
+from paper_conf_cgo_shobakimhlmkrg24_b200 import inputs as I
+from tests import brute, checker
+from tests.test_oracle_pins import independent_greedy
+
+
+def fix10a_typed():
+    """FIX10-A with issue types: loads/stores = memory, s_add = SALU, rest VALU."""
+    x = I.fix10a()
+    x.inst_type = np.array([2, 2, 2, 2, 1, 0, 0, 0, 0, 2], np.uint8)
+    return x
+
+
+def cp_heights(region):
+    n = region.n_insts
+    cp = [0] * n
+    for j in reversed(range(n)):  # program order is topological
+        for s, d, l in region.edges():
+            if s == j:
+                cp[j] = max(cp[j], l + cp[d])
+    return cp
+
+
+def textbook_cp_list_schedule(region, machine):
+    """Cycle-driven list scheduling [1] on the machine model (L64): at each
+    cycle, repeatedly issue the data-ready instruction with the largest
+    critical path (ties to the lowest index) that still has a free slot;
+    when none remains, go to the next cycle.  Written from the definition."""
+    n = region.n_insts
+    P = brute.preds_of(region)
+    cp = cp_heights(region)
+    w = max(1, machine.issue_width)
+    types = region.inst_type
+    cyc, order, cycles = {}, [], []
+    t = 0
+    while len(order) < n:
+        used, used_t = 0, [0, 0, 0, 0]
+        while True:
+            def ok(j):
+                if j in cyc or not all(p in cyc for p, _ in P[j]):
+                    return False
+                if max([cyc[p] + l for p, l in P[j]] + [0]) > t:
+                    return False
+                y = int(types[j]) if types is not None else 0
+                return used < w and (w <= 1 or used_t[y] < machine.type_slots[y])
+            R = [j for j in range(n) if ok(j)]
+            if not R:
+                break
+            j = max(R, key=lambda j: (cp[j], -j))
+            cyc[j] = t
+            order.append(j)
+            cycles.append(t)
+            used += 1
+            y = int(types[j]) if types is not None else 0
+            used_t[y] += 1
+        t += 1
+    return order, cycles
+
+
+def textbook_cp_order(region):
+    """Latency-free list scheduling by critical path (ties lowest index)."""
+    n = region.n_insts
+    P = brute.preds_of(region)
+    cp = cp_heights(region)
+    done, order = set(), []
+    for _ in range(n):
+        R = [j for j in range(n) if j not in done and all(p in done for p, _ in P[j])]
+        j = max(R, key=lambda j: (cp[j], -j))
+        order.append(j)
+        done.add(j)
+    return order
+
+
+# ------------------------------------------------ f1: general machine (R42)
+def test_asap_machine_closed_forms():
+    n = 9
+    anti = I.Region.from_lists(n, [], [], [], [[]] * n, [[]] * n)
+    # all of one type with one slot: one per cycle; alternating types: two per cycle
+    anti.inst_type = np.zeros(n, np.uint8)
+    assert O.asap_m(anti, I.DUAL_ISSUE, list(range(n)))[0] == n
+    anti.inst_type = np.array([j % 2 for j in range(n)], np.uint8)
+    assert O.asap_m(anti, I.DUAL_ISSUE, list(range(n)))[0] == (n + 1) // 2
+    wide = dataclasses.replace(I.DUAL_ISSUE, issue_width=4, n_types=1, type_slots=(4, 1, 1, 1))
+    anti.inst_type = np.zeros(n, np.uint8)
+    assert O.asap_m(anti, wide, list(range(n)))[0] == (n + 3) // 4
+    chain = I.Region.from_lists(4, [(0, 1, 3), (1, 2, 5), (2, 3, 2)], [], [], [[]] * 4, [[]] * 4)
+    chain.inst_type = np.zeros(4, np.uint8)
+    assert O.asap_m(chain, wide, [0, 1, 2, 3])[0] == 3 + 5 + 2 + 1
+    # zero latency: a dependent pair may share a cycle on a wide machine
+    z = I.Region.from_lists(2, [(0, 1, 0)], [], [], [[]] * 2, [[]] * 2)
+    z.inst_type = np.array([0, 1], np.uint8)
+    assert O.asap_m(z, I.DUAL_ISSUE, [0, 1]) == (1, [0, 0])
+    assert O.asap_m(z, I.GFX906, [0, 1]) == (2, [0, 1])
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_asap_machine_against_cycle_stepped_simulation(seed):
+    reg = I.gen_region(40, 500 + seed)
+    order = independent_greedy(reg)
+    for m in (I.GFX906, I.DUAL_ISSUE,
+              dataclasses.replace(I.DUAL_ISSUE, issue_width=3, type_slots=(2, 1, 1, 1))):
+        L, cyc = O.asap_m(reg, m, order)
+        Lb, cb = brute.asap_machine(reg, order, max(1, m.issue_width), m.type_slots, reg.inst_type)
+        assert (L, cyc) == (Lb, cb)
+    assert O.asap_m(reg, I.GFX906, order) == O.asap(reg, order)
+
+
+def test_lower_bound_length_on_machine():
+    x = fix10a_typed()
+    _, lblen, _ = O.lower_bounds(x, I.DUAL_ISSUE, 0)
+    opt, _ = brute.optimum_machine(x, I.DUAL_ISSUE, 0)
+    assert lblen <= opt
+    # 5 memory instructions with one memory slot: at least 5 cycles; CP 13 -> 14
+    assert lblen == 14
+    n = 10
+    anti = I.Region.from_lists(n, [], [], [], [[]] * n, [[]] * n)
+    anti.inst_type = np.zeros(n, np.uint8)
+    assert O.lower_bounds(anti, I.DUAL_ISSUE, 0)[1] == n
+    anti.inst_type = np.array([j % 3 for j in range(n)], np.uint8)
+    assert O.lower_bounds(anti, I.DUAL_ISSUE, 0)[1] == 5
+    assert O.lower_bounds(anti, I.GFX906, 0)[1] == n
+
+
+@pytest.mark.parametrize("machine", ["dual", "triple"])
+@pytest.mark.parametrize("seed", range(3))
+def test_q0_one_ilp_ants_are_the_cp_list_schedule(machine, seed):
+    """With q0 = 1, uniform tau, no optional stalls and no RP target (the
+    weighted pass), every ant of the first iteration is the textbook
+    cycle-driven critical-path list schedule on the machine (L64, L122)."""
+    m = I.DUAL_ISSUE if machine == "dual" else dataclasses.replace(
+        I.DUAL_ISSUE, issue_width=3, type_slots=(2, 1, 1, 1))
+    reg = I.gen_region(30, 700 + seed)
+    p = I.Params(ants=6, iterations=1, seed=seed, q0_t=1 << 32, passes=4, ws_weight=1, stall_num=0)
+    r = O.schedule(reg, 3, m, p, dump=True, dump_orders=True)
+    order, cycles = textbook_cp_list_schedule(reg, m)
+    for a in range(6):
+        assert list(r["dump_order"][1, 0, a]) == order
+        assert list(r["dump_cycle"][1, 0, a]) == cycles
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_machine_two_pass_against_enumeration(seed):
+    reg = I.gen_region(8, 1000 + seed, profile="mixed" if seed % 2 else "unit")
+    for m in (I.DUAL_ISSUE, dataclasses.replace(I.DUAL_ISSUE, issue_width=3, type_slots=(2, 1, 1, 1))):
+        p = I.Params(ants=32, iterations=4, seed=seed, cost_mode=1, stall_mod=1)
+        r = O.schedule(reg, seed, m, p, dump=True, dump_orders=True)
+        tgt = [r["target0"], r["target1"]]
+        opt, _ = brute.optimum_machine(reg, m, 1, target=tgt)
+        assert r["lblen"] <= opt <= r["length"]
+        checker.check_machine_schedule(reg, m, r["order"], r["cycle"], r["length"])
+        prp = checker.prp(reg, r["order"])
+        assert prp == r["prp"] and prp[0] <= tgt[0] and prp[1] <= tgt[1]
+        for it in range(p.iterations):
+            for a in range(p.ants):
+                c2 = r["dump_cost"][1, it, a]
+                if c2 != O.INVALID:
+                    checker.check_machine_schedule(reg, m, r["dump_order"][1, it, a],
+                                                   r["dump_cycle"][1, it, a], int(c2))
+
+
+def test_dual_issue_fix10a_reaches_enumerated_optimum():
+    x = fix10a_typed()
+    for seed in range(5):
+        r = O.schedule(x, 0, I.DUAL_ISSUE, I.Params(ants=64, iterations=20, seed=seed, cost_mode=0))
+        tgt = [r["target0"], r["target1"]]
+        opt, _ = brute.optimum_machine(x, I.DUAL_ISSUE, 0, target=tgt)
+        assert r["length"] == opt  # 22 under (2, 2), 15 under (3, 2)
+
+
+def test_single_issue_ignores_types_and_slots():
+    reg = I.gen_region(50, 4242)
+    p = I.Params(ants=64, iterations=3, seed=5)
+    a = O.schedule(reg, 1, I.GFX906, p)
+    b = O.schedule(reg, 1, dataclasses.replace(I.GFX906, n_types=3, type_slots=(1, 1, 1, 1)), p)
+    untyped = dataclasses.replace(reg, inst_type=None)
+    c = O.schedule(untyped, 1, I.GFX906, p)
+    for k in ("length", "cost_rp", "trace_hash", "iters1", "iters2"):
+        assert a[k] == b[k] == c[k]
+    assert np.array_equal(a["order"], c["order"])
+
+
+# ------------------------------------------ f2: mixed heuristics (R43, R44)
+@pytest.mark.parametrize("seed", range(4))
+def test_heur_mix_odd_groups_pass1_is_cp_list_schedule(seed):
+    reg = I.gen_region(24, 300 + seed)
+    p = I.Params(ants=8, iterations=1, seed=seed, q0_t=1 << 32, passes=1, group_size=2, heur_mix=1)
+    r = O.schedule(reg, 5, I.GFX906, p, dump=True, dump_orders=True)
+    luc, cp = independent_greedy(reg), textbook_cp_order(reg)
+    for a in range(8):
+        assert list(r["dump_order"][0, 0, a]) == (cp if (a // 2) % 2 else luc)
+    assert list(O.greedy_pass1(reg, I.GFX906, p)[0]) == luc  # the heuristic schedule is not mixed
+
+
+def test_heur_mix_off_is_unchanged_and_on_changes_only_odd_groups():
+    reg = I.gen_region(60, 99)
+    p = I.Params(ants=128, iterations=1, seed=2, group_size=16)
+    a = O.schedule(reg, 0, I.GFX906, p, dump=True, dump_orders=True)
+    b = O.schedule(reg, 0, I.GFX906, dataclasses.replace(p, heur_mix=0), dump=True, dump_orders=True)
+    c = O.schedule(reg, 0, I.GFX906, dataclasses.replace(p, heur_mix=1), dump=True, dump_orders=True)
+    assert a["trace_hash"] == b["trace_hash"]
+    for ps in (0, 1):  # iteration 0: same tau, same draws; only the odd groups' heuristic differs
+        same = [np.array_equal(a["dump_order"][ps, 0, k], c["dump_order"][ps, 0, k]) for k in range(128)]
+        assert all(same[k] for k in range(128) if (k // 16) % 2 == 0)
+        assert not all(same[k] for k in range(128) if (k // 16) % 2 == 1)
+
+
+def test_stall_fraction_groups():
+    """Table 6 percentages (L387-L402): stall_num of stall_mod groups may take
+    optional stalls.  FIX10-A under target (2,2) has no schedule without an
+    optional stall, so exactly the other groups' ants die."""
+    x = I.fix10a()
+    assert brute.no_optional_stall_schedules(x, [2, 2]) == 0
+    for num, rem in ((0, 0), (1, 0), (2, 1), (3, 3), (4, 0)):
+        bit = False
+        for seed in range(10):  # pass 1 must reach (2,2) for the target to bite
+            p = I.Params(ants=512, iterations=6, seed=seed, cost_mode=0, group_size=64,
+                         stall_mod=4, stall_rem=rem, stall_num=num)
+            r = O.schedule(x, 0, I.GFX906, p, dump=True)
+            if [r["target0"], r["target1"]] != [2, 2]:
+                continue
+            bit = True
+            enabled = {g for g in range(8) if (g - rem) % 4 < num}
+            assert len(enabled) == 2 * num
+            for it in range(r["iters2"]):
+                costs = r["dump_cost"][1, it]
+                for a in range(512):
+                    if a // 64 not in enabled:
+                        assert costs[a] == O.INVALID
+                if num > 0 and it == 0:
+                    assert any(costs[a] != O.INVALID for a in range(512))
+            if num == 0:
+                assert r["length"] == r["init2"]
+            break
+        assert bit
+
+
+# ------------------------------------------------ f3: compile policy (R39, R40)
+@pytest.mark.parametrize("seed", range(6))
+def test_cycle_gap_filter_boundary(seed):
+    reg = I.gen_region(60 + 10 * seed, 800 + seed)
+    p = I.Params(ants=64, iterations=3, seed=seed)
+    base = O.schedule(reg, seed, I.GFX906, p)
+    gap = base["init2"] - base["lblen"]
+    if gap > 0:  # threshold equal to the gap: pass 2 runs, identical results
+        same = O.schedule(reg, seed, I.GFX906, dataclasses.replace(p, pass2_gap=gap))
+        assert same["trace_hash"] == base["trace_hash"] and same["policy"] == 0
+        assert np.array_equal(same["order"], base["order"])
+    cut = O.schedule(reg, seed, I.GFX906, dataclasses.replace(p, pass2_gap=gap + 1))
+    assert cut["policy"] == 1 and cut["iters2"] == 0
+    assert cut["length"] == cut["init2"] == base["init2"]
+    assert cut["iters1"] == base["iters1"] and cut["best1"] == base["best1"]
+    # the reported schedule is the pass-2 input: ASAP of the pass-1 best
+    L, cyc = brute.asap(reg, [int(j) for j in cut["order"]])
+    assert L == cut["length"] and cyc == [int(c) for c in cut["cycle"]]
+
+
+def test_heuristic_length_is_asap_of_greedy():
+    for seed in range(4):
+        reg = I.gen_region(50, 900 + seed)
+        r = O.schedule(reg, 0, I.GFX906, I.Params(ants=16, iterations=1, seed=seed))
+        g = independent_greedy(reg)
+        assert r["heur_len"] == brute.asap(reg, g)[0]
+        rm = O.schedule(reg, 0, I.DUAL_ISSUE, I.Params(ants=16, iterations=1, seed=seed))
+        assert rm["heur_len"] == brute.asap_machine(reg, g, 2, I.DUAL_ISSUE.type_slots, reg.inst_type)[0]
+
+
+def test_revert_filter_rule():
+    """Revert iff occupancy(final) - occupancy(heuristic) >= revert_occ and
+    length(final) - length(heuristic) > revert_len (L366), decided here from
+    the occupancy table and the independent greedy + ASAP."""
+    m = I.GFX906
+    fired = kept = 0
+    for seed in range(12, 18):  # seed 14 (n = 150): ACO gains an occupancy level and 3 cycles
+        reg = I.gen_region((60, 100, 150, 200, 250, 300)[seed % 6], 1300 + seed)
+        p = I.Params(ants=64, iterations=4, seed=seed, cost_mode=1)
+        base = O.schedule(reg, seed, m, p)
+        g = independent_greedy(reg)
+        h_len, h_cyc = brute.asap(reg, g)
+        h_occ = brute.occupancy(m, checker.prp(reg, g))
+        f_occ = brute.occupancy(m, checker.prp(reg, base["order"]))
+        for occ_thr, len_thr in ((1, 0), (1, 5), (2, 0), (3, 63)):
+            q = dataclasses.replace(p, revert_occ=occ_thr, revert_len=len_thr)
+            r = O.schedule(reg, seed, m, q)
+            expect = f_occ - h_occ >= occ_thr and base["length"] - h_len > len_thr
+            assert bool(r["policy"] & 2) == expect
+            if expect:
+                fired += 1
+                assert [int(j) for j in r["order"]] == g
+                assert r["length"] == h_len and [int(c) for c in r["cycle"]] == h_cyc
+                assert r["prp"] == checker.prp(reg, g)
+            else:
+                kept += 1
+                assert np.array_equal(r["order"], base["order"]) and r["length"] == base["length"]
+    assert fired > 0 and kept > 0
+
+
+def test_paper_policy_preset():
+    p = I.paper_policy(I.Params())
+    assert (p.pass2_gap, p.revert_occ, p.revert_len, p.stop_at_lb) == (21, 3, 63, 1)
+    assert p.stop_no_improve == I.STOP_PAPER_CLASSES
+
+
+# ------------------------------------------------ f4: weighted sum (R41)
+@pytest.mark.parametrize("seed", range(8))
+def test_weighted_pass_against_enumeration(seed):
+    reg = I.gen_region(8, 1000 + seed, profile="mixed")
+    for W, m in ((0, I.GFX906), (1, I.GFX906), (3, I.GFX906), (2, I.DUAL_ISSUE)):
+        p = I.Params(ants=32, iterations=5, seed=seed, cost_mode=0, passes=4, ws_weight=W, stall_mod=1)
+        r = O.schedule(reg, seed, m, p, dump=True, dump_orders=True)
+        _, opt = brute.optimum_machine(reg, m, 0, weight=W)
+        assert r["ws_cost"] >= opt
+        assert r["ws_cost"] <= r["init2"]
+        assert r["iters1"] == 0
+        checker.check_machine_schedule(reg, m, r["order"], r["cycle"], r["length"])
+        prp = checker.prp(reg, r["order"])
+        assert r["prp"] == prp
+        assert r["ws_cost"] == r["length"] + W * brute.cost(m, 0, prp)
+        # the initial schedule: the greedy order timed ASAP, with its weighted cost
+        g = independent_greedy(reg)
+        gl = brute.asap_machine(reg, g, max(1, m.issue_width), m.type_slots, reg.inst_type)[0]
+        assert r["init2"] == gl + W * brute.cost(m, 0, checker.prp(reg, g))
+        # every ant: a valid schedule (never dies: no target) with its cost recomputed
+        for it in range(r["iters2"]):
+            for a in range(p.ants):
+                c = int(r["dump_cost"][1, it, a])
+                o, y = r["dump_order"][1, it, a], r["dump_cycle"][1, it, a]
+                L = int(y[-1]) + 1
+                checker.check_machine_schedule(reg, m, o, y, L)
+                assert c == L + W * brute.cost(m, 0, checker.prp(reg, o))
+
+
+def test_weighted_pass_fix10a():
+    """W <= 8: the heuristic (PRP (3,2), 15 cycles) is optimal, W = 10 prefers
+    (2,2) at 23 cycles (63 < 65); the single pass keeps the heuristic there
+    (reaching (2,2) needs 8 optional stall cycles), which is why the paper
+    uses two passes (L74, L108)."""
+    x = I.fix10a()
+    for W, opt in ((1, 20), (4, 35), (8, 55)):
+        r = O.schedule(x, 0, I.GFX906, I.Params(ants=64, iterations=20, seed=1, cost_mode=0, passes=4,
+                                                   ws_weight=W))
+        assert brute.optimum_machine(x, I.GFX906, 0, weight=W)[1] == opt == r["ws_cost"]
+    assert brute.optimum_machine(x, I.GFX906, 0, weight=10)[1] == 63
