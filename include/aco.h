@@ -65,6 +65,8 @@ typedef struct {
   const uint8_t *reg_flags;                       /* [n_regs] bit0 LIVE_IN, bit1 LIVE_OUT */
   const uint32_t *def_ptr, *def_reg;              /* CSR: defs of j = def_reg[def_ptr[j]..def_ptr[j+1]) */
   const uint32_t *use_ptr, *use_reg;              /* CSR: uses of j (duplicates count once, R33) */
+  const uint8_t *inst_type; /* [n_insts] issue type of each instruction for the general machine
+                               model (L64; R42), < aco_machine.n_types; NULL = all type 0 */
 } aco_region_desc;
 
 /* Occupancy model per register class (L68-L72; R16, R17).  step_max[c][i] is
@@ -75,6 +77,14 @@ typedef struct {
   uint32_t step_count[4];
   uint32_t step_max[4][16];
   uint32_t perp_limit[4];
+  /* General machine model (L64 "supports a general machine model"; R42).
+   * issue_width <= 1: single issue, any instruction type per cycle (the
+   * paper's experiments, R32; n_types / type_slots ignored).  Otherwise at
+   * most issue_width instructions per cycle, of which at most type_slots[y]
+   * of issue type y < n_types <= 4.  Affects the ILP pass (and pass 4), the
+   * ASAP timing of R29 and LB_len; the RP pass ignores latencies (R19). */
+  uint32_t issue_width, n_types;
+  uint32_t type_slots[4];
 } aco_machine;
 
 enum { ACO_COST_PRP_SUM = 0, ACO_COST_APRP_SUM = 1, ACO_COST_OCC = 2, ACO_COST_PERP = 3 };
@@ -90,7 +100,8 @@ typedef struct {
   uint32_t ants;       /* ants per region per iteration (A) */
   uint32_t iterations; /* iterations per pass (a hard cap, R12) */
   uint64_t seed;       /* Philox key (R26) */
-  uint32_t pass;       /* 1 RP pass, 2 ILP pass from the heuristic, 3 both (L108) */
+  uint32_t pass;       /* 1 RP pass, 2 ILP pass from the heuristic, 3 both (L108),
+                          4 single weighted-sum pass (L74; R41) */
   uint32_t cost_mode;  /* ACO_COST_* (R16) */
   uint64_t q0_t;       /* exploit iff group coin < q0_t; 2^32 = always (R1-R3) */
   uint32_t group_size; /* ants sharing the exploit/explore coin (L198), default 64 */
@@ -99,6 +110,13 @@ typedef struct {
   uint32_t stop_no_improve; /* 0 = off, 0xFFFFFFFF = paper size classes 1/2/3 (L226) */
   uint32_t stop_at_lb;      /* stop a pass when its best cost equals the LB (L110, L251) */
   uint32_t flags;           /* ACO_FLAG_* */
+  /* region-level compile policy (L362, L366, L393-L417; R39, R40) */
+  uint32_t pass2_gap;       /* run pass 2 only if initial length - LB_len >= pass2_gap (0 off; paper 21) */
+  uint32_t revert_occ;      /* report the heuristic schedule when ACO gains >= revert_occ occupancy */
+  uint32_t revert_len;      /*   but lengthens the schedule by > revert_len cycles (paper 3, 63; 0 off) */
+  uint32_t ws_weight;       /* pass 4: cost = length + ws_weight * cost_rp (<= 1024; R41) */
+  uint32_t heur_mix;        /* 1: odd ant groups use the other pass's heuristic (L216-L218; R43) */
+  uint32_t stall_num;       /* group g may stall iff (g - stall_rem) % stall_mod < stall_num (R44; paper 1) */
 } aco_params;
 
 /* Per-region result (sizes fixed; the schedule itself is returned through
@@ -114,6 +132,10 @@ typedef struct {
   uint32_t lb_cost, lb_len; /* lower bounds (R30) */
   uint32_t target[4];    /* pass-2 PRP target per class (R18) */
   uint64_t trace_hash;   /* FNV-1a over (pass, iter, winner cost, winner ant) */
+  uint32_t policy;       /* bit0: pass 2 filtered by the cycle gap (R39); bit1: reverted (R40) */
+  uint32_t heur_len;     /* length of the heuristic schedule (greedy order timed ASAP, R40) */
+  uint32_t ws_cost;      /* pass 4: final weighted cost (R41), else 0 */
+  uint32_t pad;
 } aco_result;
 
 /* Create a context on CUDA device `device` for machine model *m (copied). */

@@ -33,7 +33,7 @@ class RegionDesc(C.Structure):
         ("edge_src", C.c_void_p), ("edge_dst", C.c_void_p), ("edge_lat", C.c_void_p),
         ("reg_class", C.c_void_p), ("reg_flags", C.c_void_p),
         ("def_ptr", C.c_void_p), ("def_reg", C.c_void_p),
-        ("use_ptr", C.c_void_p), ("use_reg", C.c_void_p),
+        ("use_ptr", C.c_void_p), ("use_reg", C.c_void_p), ("inst_type", C.c_void_p),
     ]
 
 
@@ -42,6 +42,7 @@ class Machine(C.Structure):
         ("n_classes", C.c_uint32), ("occ_max", C.c_uint32),
         ("step_count", C.c_uint32 * 4), ("step_max", (C.c_uint32 * 16) * 4),
         ("perp_limit", C.c_uint32 * 4),
+        ("issue_width", C.c_uint32), ("n_types", C.c_uint32), ("type_slots", C.c_uint32 * 4),
     ]
 
 
@@ -53,6 +54,8 @@ class Params(C.Structure):
         ("tau0", C.c_uint32), ("rho_q16", C.c_uint32), ("delta", C.c_uint32),
         ("tau_min", C.c_uint32), ("tau_max", C.c_uint32),
         ("stop_no_improve", C.c_uint32), ("stop_at_lb", C.c_uint32), ("flags", C.c_uint32),
+        ("pass2_gap", C.c_uint32), ("revert_occ", C.c_uint32), ("revert_len", C.c_uint32),
+        ("ws_weight", C.c_uint32), ("heur_mix", C.c_uint32), ("stall_num", C.c_uint32),
     ]
 
 
@@ -62,6 +65,7 @@ class Result(C.Structure):
         ("prp", C.c_uint32 * 4), ("iters_run", C.c_uint32 * 2), ("best_cost", C.c_uint32 * 2),
         ("init_cost", C.c_uint32 * 2), ("lb_cost", C.c_uint32), ("lb_len", C.c_uint32),
         ("target", C.c_uint32 * 4), ("trace_hash", C.c_uint64),
+        ("policy", C.c_uint32), ("heur_len", C.c_uint32), ("ws_cost", C.c_uint32), ("pad", C.c_uint32),
     ]
 
 

@@ -33,13 +33,18 @@ def machine_struct(m: Machine) -> _lib.Machine:
             s.step_max[c][i] = v
     for c in range(4):
         s.perp_limit[c] = m.perp_limit[c] if c < len(m.perp_limit) else 0
+    s.issue_width = m.issue_width
+    s.n_types = m.n_types
+    for y, v in enumerate(m.type_slots):
+        s.type_slots[y] = v
     return s
 
 
 def params_struct(p: Params, flags: int = 0) -> _lib.Params:
     return _lib.Params(p.ants, p.iterations, p.seed, p.passes, p.cost_mode, p.q0_t, p.group_size,
                        p.stall_mod, p.stall_rem, p.tau0, p.rho_q16, p.delta, p.tau_min, p.tau_max,
-                       p.stop_no_improve, p.stop_at_lb, flags)
+                       p.stop_no_improve, p.stop_at_lb, flags, p.pass2_gap, p.revert_occ, p.revert_len,
+                       p.ws_weight, p.heur_mix, p.stall_num)
 
 
 class HostBatch:
@@ -57,9 +62,14 @@ class HostBatch:
                 if a.size == 0:
                     a = np.zeros(1, dt)
                 arrs.append(a)
+            it = None
+            if r.inst_type is not None and r.n_insts:
+                it = np.ascontiguousarray(r.inst_type, dtype=np.uint8)
+                arrs.append(it)
             self.keep.append(arrs)
             self.descs[i] = _lib.RegionDesc(int(rid), int(r.n_insts), int(r.n_edges), int(r.n_regs),
-                                            *[a.ctypes.data for a in arrs])
+                                            *[a.ctypes.data for a in arrs[:9]],
+                                            None if it is None else it.ctypes.data)
         self.sizes = np.array([r.n_insts for r in regions], np.int64)
         self.offsets = np.concatenate([[0], np.cumsum(self.sizes)]).astype(np.int64)
 
@@ -182,8 +192,9 @@ class Scheduler:
         ants = p.ants * world; one int64 MIN allreduce per region per iteration."""
         import torch.distributed as dist
         keys = self.colony_begin(p, rank * p.ants)
+        pmask = 2 if p.passes == 4 else p.passes  # pass 4 runs on the pass-2 machinery (R41)
         for pass_ in (1, 2):
-            if not (p.passes & pass_):
+            if not (pmask & pass_):
                 continue
             for it in range(p.iterations):
                 self.colony_construct(pass_, it)
@@ -234,6 +245,7 @@ class Scheduler:
                 iters1=r.iters_run[0], iters2=r.iters_run[1], best1=r.best_cost[0], best2=r.best_cost[1],
                 init1=r.init_cost[0], init2=r.init_cost[1], lb1=r.lb_cost, lblen=r.lb_len,
                 target=list(r.target), trace_hash=int(r.trace_hash),
+                policy=r.policy, heur_len=r.heur_len, ws_cost=r.ws_cost,
                 order=orders[a:b].copy(), cycle=cycles[a:b].copy()))
         return res
 

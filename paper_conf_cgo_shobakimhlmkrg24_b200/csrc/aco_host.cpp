@@ -138,7 +138,8 @@ uint32_t img_put(std::vector<unsigned char> &img, const std::vector<T> &v) {
 }
 
 // Validation + preprocessing of one region.  Readings R31-R38.
-aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P) {
+aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped &P) {
+  const uint32_t n_classes = mach.n_classes;
   const uint32_t n = d.n_insts, E = d.n_edges, G = d.n_regs;
   if (n > ACO_MAX_INSTS || G > 16777215u) return ACO_E_TOO_LARGE;
   if (n > kMaxKernelInsts) return ACO_E_TOO_LARGE;
@@ -151,6 +152,11 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   if ((d.def_ptr[n] && !d.def_reg) || (d.use_ptr[n] && !d.use_reg)) return ACO_E_ARG;
   for (uint32_t g = 0; g < G; ++g)
     if (d.reg_class[g] >= n_classes || (d.reg_flags[g] & ~3u)) return ACO_E_ARG;
+  // issue types (R42): < n_types on a multi-issue machine, else any type < 4
+  const uint32_t n_types = mach.issue_width > 1 ? mach.n_types : 4u;
+  if (d.inst_type)
+    for (uint32_t j = 0; j < n; ++j)
+      if (d.inst_type[j] >= n_types) return ACO_E_ARG;
   uint32_t max_lat = 0;
   for (uint32_t e = 0; e < E; ++e) {
     if (d.edge_src[e] >= n || d.edge_dst[e] >= n) return ACO_E_ARG;
@@ -340,6 +346,7 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
     ds[4 * j + 1] = info[(size_t)j * 4 + 1];
   }
   for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j];
+  for (uint32_t j = 0; j < n; ++j) ds[4 * j + 3] = d.inst_type ? d.inst_type[j] : 0u;  // issue type (R42)
   // users of each counter register (to find the last remaining user)
   std::vector<uint32_t> cu_ptr(nctr + 1, 0), cu;
   for (uint32_t g = 0; g < G; ++g)
@@ -395,7 +402,21 @@ aco_status prep_region(const aco_region_desc &d, uint32_t n_classes, Prepped &P)
   R.L = L;
   R.region_id = d.region_id;
   R.cp_max = cp_max;
-  R.lb_len = std::max(n, n ? cp_max + 1 : 0u);
+  // LB_len = max(1 + CPmax, ceil(n / w), max_y ceil(n_y / min(slots_y, w))) (R30, R42)
+  {
+    const uint32_t w = std::max(1u, mach.issue_width);
+    uint32_t l = (n + w - 1) / w;
+    if (n) l = std::max(l, cp_max + 1);
+    if (w > 1) {
+      uint32_t ny[4] = {0, 0, 0, 0};
+      for (uint32_t j = 0; j < n; ++j) ny[d.inst_type ? d.inst_type[j] : 0]++;
+      for (uint32_t y = 0; y < 4; ++y) {
+        const uint32_t s = std::min(w, (mach.type_slots >> (8 * y)) & 0xFFu);
+        if (ny[y]) l = std::max(l, (ny[y] + s - 1) / s);
+      }
+    }
+    R.lb_len = l;
+  }
   R.max_cycle_bound = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)n * (max_lat + 1ull) + 1);
   R.max_lat = max_lat;
   for (uint32_t c = 0; c < 4; ++c) {
@@ -428,6 +449,12 @@ const char *aco_status_string(aco_status st) {
 
 aco_status aco_create(int device, const aco_machine *m, aco_ctx *out) {
   if (!m || !out || m->n_classes < 1 || m->n_classes > 4) return ACO_E_ARG;
+  if (m->issue_width > 255u) return ACO_E_ARG;
+  if (m->issue_width > 1) {  // R42
+    if (m->n_types < 1 || m->n_types > 4) return ACO_E_ARG;
+    for (uint32_t y = 0; y < m->n_types; ++y)
+      if (m->type_slots[y] < 1 || m->type_slots[y] > 255u) return ACO_E_ARG;
+  }
   for (uint32_t c = 0; c < m->n_classes; ++c)
     if (m->step_count[c] < 1 || m->step_count[c] > 16 || m->occ_max < m->step_count[c]) return ACO_E_ARG;
   aco_ctx ctx = new (std::nothrow) aco_ctx_s();
@@ -440,6 +467,11 @@ aco_status aco_create(int device, const aco_machine *m, aco_ctx *out) {
     for (int i = 0; i < 16; ++i) ctx->mach.step_max[c][i] = m->step_max[c][i];
     ctx->mach.perp_limit[c] = m->perp_limit[c];
   }
+  ctx->mach.issue_width = std::max(1u, m->issue_width);
+  ctx->mach.n_types = m->issue_width > 1 ? m->n_types : 1u;
+  ctx->mach.type_slots = 0;
+  if (m->issue_width > 1)
+    for (uint32_t y = 0; y < m->n_types; ++y) ctx->mach.type_slots |= m->type_slots[y] << (8 * y);
   *out = ctx;  // no CUDA call here: the device is touched on first use
   return ACO_OK;
 }
@@ -458,7 +490,7 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   }
   std::vector<Prepped> P(count);
   for (uint32_t i = 0; i < count; ++i) {
-    aco_status st = prep_region(regions[i], ctx->mach.n_classes, P[i]);
+    aco_status st = prep_region(regions[i], ctx->mach, P[i]);
     if (st != ACO_OK) return st;
   }
   std::vector<unsigned char> blob(align16(sizeof(RegionDev) * (size_t)count + 16), 0);
@@ -575,7 +607,8 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
 namespace {
 
 aco_status check_params(const aco_params *p) {
-  if (p->pass < 1 || p->pass > 3 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
+  if (p->pass < 1 || p->pass > 4 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
+      p->ws_weight > 1024u || p->heur_mix > 1u ||
       p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->tau0 > 65535u ||
       p->tau0 < p->tau_min || p->tau0 > p->tau_max || p->q0_t > (1ull << 32) || p->rho_q16 > 65536u ||
       p->iterations > 0x7FFFFFFFu)
@@ -589,6 +622,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                      size_t *ws_needed, void *cuda_stream, bool colony) {
   if (aco_status st = check_params(p)) return st;
   if ((p->flags & ACO_FLAG_DUMP) && (!ctx->dump_cost || colony)) return ACO_E_ARG;
+  // passes that run construct/finalize launches: pass 4 (weighted, R41) uses the pass-2 machinery
+  const uint32_t pmask = p->pass == 4 ? 2u : p->pass;
   const uint32_t count = ctx->count, A = p->ants;
   Plan saved = ctx->plan;  // a sizing call must not disturb a planned run
   Plan &P = ctx->plan;
@@ -627,11 +662,12 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // pass-2 state variant: the compact layout (windowed u8 ready times) needs
     // latencies <= 127 and 2 classes; otherwise u16 cycles, or u32 when a
     // schedule may exceed 65535 cycles (or a latency exceeds 127)
-    const bool t32 = P.nc4 ? R.max_cycle_bound > 65535u : R.max_lat > 127u;
+    // the general machine model (R42) runs in the u32-cycle variants
+    const bool t32 = ctx->mach.issue_width > 1 || (P.nc4 ? R.max_cycle_bound > 65535u : R.max_lat > 127u);
     P.any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
-      if (!(p->pass & pass)) continue;
+      if (!(pmask & pass)) continue;
       if (getenv("ACO_DEBUG_REGIONS"))
         fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
                 R.nremw, R.L);
@@ -658,7 +694,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       c.smem = std::max(c.smem, sh.smem);
       c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
     }
-    P.p2_smem = std::max(P.p2_smem, 4 * R.n + 16);
+    P.p2_smem = std::max(P.p2_smem, 4 * R.n + 16);  // also k_post
   }
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
@@ -702,6 +738,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   off = align256(off + 2 * sum_n + 16);
   P.o_gb2c = off;
   off = align256(off + 4 * sum_n + 16);
+  const uint64_t o_heur = off;
+  off = align256(off + 2 * sum_n + 16);
   const uint64_t o_next = off;
   off = align256(off + 2 * (sum_n + count) + 16);
   const uint64_t o_cost = off;
@@ -722,6 +760,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     w.o_gb2c = P.o_gb2c + 4 * ctx->inst_off[r];
     w.o_dump = (uint64_t)A * ctx->inst_off[r];
     w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
+    w.o_heur = o_heur + 2 * ctx->inst_off[r];
     w.gs = gs[r];
     if (gs[r]) {
       off = align256(off);
@@ -827,7 +866,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.q0_t = p->q0_t;
   cfg.ants = A;
   cfg.iterations = p->iterations;
-  cfg.pass_mask = p->pass;
+  cfg.pass_mask = pmask;
   cfg.cost_mode = p->cost_mode;
   cfg.group_size = p->group_size;
   cfg.stall_mod = p->stall_mod;
@@ -843,12 +882,19 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.n_classes = ctx->mach.n_classes;
   cfg.count = count;
   cfg.ant_base = ant_base;
+  cfg.weighted = p->pass == 4;
+  cfg.ws_weight = p->ws_weight;
+  cfg.pass2_gap = p->pass2_gap;
+  cfg.revert_occ = p->revert_occ;
+  cfg.revert_len = p->revert_len;
+  cfg.heur_mix = p->heur_mix;
+  cfg.stall_num = p->stall_num;
   cfg.dump_slice = (uint64_t)A * sum_n;
   cfg.keys = nullptr;
   L.stream = cuda_stream;
   L.launches = 0;
   P.timing = (p->flags & ACO_FLAG_TIMING) != 0;
-  P.pass_mask = p->pass;
+  P.pass_mask = pmask;
   P.iterations = p->iterations;
   ctx->ev_used = 0;
   for (int ph = 0; ph < 3; ++ph) {
@@ -899,6 +945,11 @@ int run_pass2_init(aco_ctx ctx) {
   return launch_pass2_init(ctx->plan.L, ctx->plan.p2_smem, ctx->plan.max_n);
 }
 
+int run_post(aco_ctx ctx) {
+  Bracket b(ctx, 2);
+  return launch_post(ctx->plan.L, ctx->plan.p2_smem);
+}
+
 int run_construct(aco_ctx ctx, uint32_t pass, uint32_t it) {
   Plan &P = ctx->plan;
   LaunchCtx &L = P.L;
@@ -946,12 +997,13 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   int err = run_init(ctx);
   for (uint32_t pass = 1; pass <= 2 && !err; ++pass) {
     if (pass == 2) err |= run_pass2_init(ctx);
-    if (!(p->pass & pass)) continue;
+    if (!(ctx->plan.pass_mask & pass)) continue;
     for (uint32_t it = 0; it < p->iterations && !err; ++it) {
       err |= run_construct(ctx, pass, it);
       err |= run_finalize(ctx, pass, it, nullptr);
     }
   }
+  if (!err) err |= run_post(ctx);
   ctx->launches = ctx->plan.L.launches;
   return err ? ACO_E_CUDA : ACO_OK;
 }
@@ -999,6 +1051,7 @@ aco_status aco_colony_end(aco_ctx ctx, void *cuda_stream) {
   P.L.stream = cuda_stream;
   int err = 0;
   if (!P.p2_done) err |= run_pass2_init(ctx);  // ASAP timing of the pass-1 result
+  err |= run_post(ctx);
   ctx->stream = cuda_stream;
   ctx->launches = P.L.launches;
   return err ? ACO_E_CUDA : ACO_OK;
@@ -1066,7 +1119,7 @@ aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_resu
     aco_result &o = out[k];
     std::memset(&o, 0, sizeof(o));
     o.n_insts = R.n;
-    o.length = S.best[1];
+    o.length = S.len2;
     uint32_t cost = 0;
     const uint32_t nc = ctx->mach.n_classes, mode = ctx->cfg.cost_mode;
     if (mode == ACO_COST_PRP_SUM) {
@@ -1095,6 +1148,9 @@ aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_resu
     o.lb_cost = S.lb_cost;
     o.lb_len = R.lb_len;
     o.trace_hash = S.hash;
+    o.policy = S.policy;
+    o.heur_len = S.heur_len;
+    o.ws_cost = ctx->cfg.weighted ? S.best[1] : 0u;
   }
   for (uint64_t q = 0; q < i1 - i0; ++q) {
     if (orders) orders[q] = o16[q];

@@ -85,6 +85,11 @@ struct RegionState {
   uint32_t target[4];    // pass-2 target (R18)
   uint32_t prune_len;    // best completed length of the running iteration (R24)
   uint32_t lb_cost;
+  uint32_t len2;         // length of the pass-2 global best (pass 4: best[1] is the weighted cost)
+  uint32_t policy;       // bit0 gap-filtered (R39), bit1 reverted (R40)
+  uint32_t heur_len;     // the heuristic schedule's length (R40)
+  uint32_t heur_prp[4];  // the heuristic schedule's PRP
+  uint32_t pad;
   uint64_t hash;         // FNV-1a trace
 };
 
@@ -99,6 +104,7 @@ struct RegionWs {
   uint64_t o_next;   // u16 [n+1]: the iteration winner's successor of each row (0xFFFF: none)
   uint64_t o_gstate; // global-state regions: per-ant state [word][ant] (ants x words u32)
   uint64_t o_scratch;// global-state regions: replay scratch (words + cycles + order)
+  uint64_t o_heur;   // u16 [n]  the heuristic (greedy pass-1) order, R40
   uint32_t tau_len;  // (n+1)*n rounded up to a multiple of 8
   uint32_t gs;       // 1: the region's state does not fit shared memory (global-state kernels)
 };
@@ -120,6 +126,10 @@ struct RunCfg {
   uint32_t stop_no_improve, stop_at_lb, n_classes;
   uint32_t count;       // regions
   uint32_t ant_base;    // global id of this context's first ant (shared colony), else 0
+  uint32_t weighted;    // pass 4: single weighted-sum pass on the pass-2 machinery (R41)
+  uint32_t ws_weight;
+  uint32_t pass2_gap, revert_occ, revert_len;  // compile policy (R39, R40)
+  uint32_t heur_mix, stall_num;                // R43, R44
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
   int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };
@@ -129,6 +139,9 @@ struct MachineDev {
   uint32_t step_count[4];
   uint32_t step_max[4][16];
   uint32_t perp_limit[4];
+  uint32_t issue_width;  // >= 1 (R42)
+  uint32_t type_slots;   // u8 x 4: issue slots per type (issue_width > 1)
+  uint32_t n_types;
 };
 
 // Construct-kernel work item: one block = ants [ant0, ant0 + blockDim) of a region.
@@ -221,7 +234,8 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);
 int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
                     bool nc4, const UpdItem *upd, uint32_t n_upd);
-int launch_local_keys(LaunchCtx &L, int64_t *keys);  // shared colony: per-region local argmin keys
+int launch_local_keys(LaunchCtx &L, int64_t *keys);
+int launch_post(LaunchCtx &L, uint32_t smem);  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys
 
 // Biased winner key: (cost << 32 | global ant) XOR 2^63, so that a signed
 // int64 MIN (NCCL / torch) orders keys like the unsigned (cost, ant) pair.

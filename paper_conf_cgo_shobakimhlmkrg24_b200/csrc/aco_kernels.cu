@@ -39,9 +39,6 @@
 #ifndef ACO_BRANCHLESS1  // pass-1 4-wide evaluation without branches (measured faster)
 #define ACO_BRANCHLESS1 1
 #endif
-#ifndef ACO_BRANCHLESS2  // pass-2 likewise (measured slower: keep the branches)
-#define ACO_BRANCHLESS2 0
-#endif
 
 namespace aco {
 
@@ -399,7 +396,16 @@ __device__ __forceinline__ void scan4(const St &A, uint32_t m, F &&visit) {
 struct AntOut {
   uint32_t cost;
   uint32_t prp01, prp23;
+  uint32_t len;  // pass 2: schedule length (cost is the weighted cost in pass 4, R41)
 };
+
+// Optional stalls for ant group g (L202-L204; R23, R44).
+__device__ __forceinline__ bool stall_group(const RunCfg &cfg, uint32_t g) {
+  const uint32_t mod = cfg.stall_mod, rem = cfg.stall_rem % mod;
+  return ((g % mod) + mod - rem) % mod < cfg.stall_num;
+}
+// Sum of the four u8 lanes (per-class last-use counts -> LUC).
+__device__ __forceinline__ uint32_t sum_u8x4(uint32_t x) { return __dp4a(x, 0x01010101u, 0u); }
 
 __device__ __forceinline__ uint32_t cost_of(uint32_t mode, uint32_t prp01, uint32_t prp23) {
   return cost_rp(mode, prp01 & 0xFFFFu, prp01 >> 16, prp23 & 0xFFFFu, prp23 >> 16);
@@ -530,6 +536,8 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
   const uint32_t group = ant / cfg.group_size;
   const uint32_t sub = lane_words<LG>(G.lane);
   constexpr bool wide = MASK && WIDE;
+  // R43: odd groups are guided by the ILP heuristic (CP, eta2) instead
+  const bool mix = !greedy && cfg.heur_mix && (group & 1u);
   uint32_t prev = n;
   for (uint32_t k = 0; k < n; ++k) {
     bool exploit = greedy;
@@ -544,7 +552,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     const uint16_t *trow = tau + prev * n;
     // score(j) = tau[prev][j] * eta1(j, sk(j) + d(j)) (R1, R4)
     auto score = [&](uint32_t j) -> uint32_t {
-      return (uint32_t)trow[j] * (uint32_t)V.eta1[j * L1 + dk1_get(A, j)];
+      return (uint32_t)trow[j] * (mix ? V.ds[j].z : (uint32_t)V.eta1[j * L1 + dk1_get(A, j)]);
     };
     // Lane-local argmax in ascending order: strict '>' keeps the lowest
     // index among equal scores; bs1 = best score + 1 (0 = no candidate; a
@@ -560,7 +568,8 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
           dk[u] = A.DK[(j[u] >> 3) * A.S];
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) dk[u] = V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+        for (int u = 0; u < 4; ++u)
+          dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
 #if ACO_BRANCHLESS1
         // branch-free: the four candidates' chains interleave (ILP)
         uint32_t sc[4];
@@ -638,32 +647,44 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
   AntOut o;
   o.prp01 = prp01;
   o.prp23 = prp23;
+  o.len = 0;
   o.cost = G.leader() ? cost_of(cfg.cost_mode, prp01, prp23) : 0u;
   return o;
 }
 
 // ------------------------------------------------------------ pass-2 ant
-// ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle and
-// the Philox step; stalls skip ahead without drawing.  rec_o / rec_c (leader,
-// may be NULL) receive the order and the cycles.  Valid in the leader lane.
+// ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle;
+// stalls skip ahead without drawing.  rec_o / rec_c (leader, may be NULL)
+// receive the order and the cycles.  Valid in the leader lane.
+// General machine model (L64; R42, T32 variants only): the ant stays in
+// cycle t until issue_width instructions were placed; a latency-met
+// instruction whose slot (width / type) is full counts as semi-ready with
+// ready time t + 1; the Philox step is t * issue_width + used.
+// Weighted single pass (pass 4, R41): no target, cost = length + W * cost_rp.
 template <int LG, bool MASK, bool T32, bool NC4, bool WIDE = false>
 __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
                                             const bool prune, uint16_t *rec_o, uint32_t *rec_c,
                                             const uint32_t *coins = nullptr, uint32_t coin_t = 0) {
-  const uint32_t n = V.n, nwr = V.nwr;
+  const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<2, MASK, T32, NC4>(V, A);
   wmask = G.bcast(wmask);
   G.sync();
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
-  const bool stall_en = (group % cfg.stall_mod) == cfg.stall_rem;  // R23
+  const bool stall_en = stall_group(cfg, group);      // R23, R44
+  const bool mix = cfg.heur_mix && (group & 1u);      // R43: odd groups use eta1 (LUC, CP)
   const uint32_t c2 = 0x80000000u | iter;
   const uint32_t sub = lane_words<LG>(G.lane);
   constexpr bool wide = MASK && WIDE;
   constexpr bool CT = !T32 && !NC4;  // compact layout (x_get)
+  // general machine model (R42): runtime, only in the u32-cycle variants
+  const uint32_t w = T32 ? c_mach.issue_width : 1u;
+  const bool mi = T32 && w > 1u;
+  const uint32_t slots = c_mach.type_slots;  // u8 x 4
+  uint32_t used = 0, used_t = 0;              // placed in cycle t: total, per type (u8 x 4)
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0, B = 0;
   // ready time and per-class last-use counts of instruction j
   auto rd_dk = [&](uint32_t j, uint32_t &rd, uint32_t &dk) {
@@ -676,11 +697,16 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       dk = dk2_get<NC4>(A, j);
     }
   };
+  // heuristic of a feasible candidate: eta2 (CP), or eta1 (LUC, CP) for mixed odd groups
+  auto eta_of = [&](uint32_t j, uint32_t e2, uint32_t dk) -> uint32_t {
+    return mix ? (uint32_t)V.eta1[j * L1 + sum_u8x4(dk)] : e2;
+  };
   AntOut o;
   o.prp01 = o.prp23 = 0;
+  o.len = kInvalid;
   while (placed < n) {
     if (CT && t - B >= 128u) {  // slide the ready-time window (t - B <= 254 here)
-      for (uint32_t w = G.lane; w < (n + 1) / 2; w += LG) A.T[w * A.S] = __vsubus4(A.T[w * A.S], 0x00800080u);
+      for (uint32_t q = G.lane; q < (n + 1) / 2; q += LG) A.T[q * A.S] = __vsubus4(A.T[q * A.S], 0x00800080u);
       B += 128u;
       G.sync();
     }
@@ -688,11 +714,15 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       uint32_t bl = 0;
       if (G.leader()) bl = *(volatile uint32_t *)prune_len;
       bl = G.bcast(bl);
-      if (t + (n - placed) > bl) {
+      const uint32_t lbf = mi ? t + (n - placed + used + w - 1) / w : t + (n - placed);
+      if (lbf > bl) {
         o.cost = kInvalid;
         return o;
       }
     }
+    const uint32_t step = mi ? t * w + used : t;  // Philox step (R26, R42)
+    // free issue slots per type this cycle (0xFF per byte = free), R42
+    const uint32_t avail = mi ? (used < w ? __vcmpltu4(used_t, slots) : 0u) : 0xFFFFFFFFu;
     // slack_c = target_c - live_c, saturated to a byte (R21); live <= target always
     uint32_t slack = 0;
     {
@@ -705,14 +735,15 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     bool f_not_inc = false, s_dec = false, any_s = false;
     uint32_t bs1 = 0, bj = 0;  // lane-local best score + 1 (0 = none) and its index
     unsigned long long sum = 0;
-    // the roulette sum is needed unless this cycle's group coin is a known exploit
-    const bool need_sum = !(t < coin_t && ((coins[t >> 5] >> (t & 31u)) & 1u));
+    // the roulette sum is needed unless this step's group coin is a known exploit
+    const bool need_sum = !(step < coin_t && ((coins[step >> 5] >> (step & 31u)) & 1u));
     auto eval = [&](uint32_t j, uint32_t rdy, const uint4 &ds, uint32_t dk, uint32_t tv) {
       const uint32_t K = ds.y + dk;                   // kills per class (R14)
-      const uint32_t s = tv * ds.z;
-      if (rdy <= t) {
+      const bool lat_ok = rdy <= t;
+      if (lat_ok && (!mi || ((avail >> (8 * ds.w)) & 1u))) {
         counts += 1u;
         if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
+          const uint32_t s = tv * eta_of(j, ds.z, dk);
           counts += 1u << 16;
           f_not_inc |= __vcmpgtu4(ds.x, K) == 0u;           // max_c Delta_c <= 0
           if (s + 1u > bs1) {  // ascending: strict keeps the lowest index (R1, R25)
@@ -723,7 +754,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         }
       } else {
         any_s = true;
-        min_s = ::min(min_s, rdy);
+        min_s = ::min(min_s, lat_ok ? t + 1u : rdy);        // slot-blocked: next cycle (R42)
         s_dec |= __vcmpltu4(ds.x, K) != 0u;                 // min_c Delta_c < 0
       }
     };
@@ -734,43 +765,12 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           rd_dk(j[u], rd[u], dk[u]);
-          ds[u] = V.ds[j[u]];                         // defs, static kills, eta2
+          ds[u] = V.ds[j[u]];                         // defs, static kills, eta2, type
           tv[u] = trow[j[u]];
         }
-#if ACO_BRANCHLESS2
-        // branch-free evaluation of the four candidates (ILP); same
-        // semantics as eval() (R21, R22)
-        uint32_t sc[4];
-        bool fe[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const uint32_t K = ds[u].y + dk[u];
-          const bool ready = v[u] && rd[u] <= t;
-          const bool semi = v[u] && rd[u] > t;
-          fe[u] = ready && __vcmpgtu4(ds[u].x, __vaddus4(slack, K)) == 0u;
-          counts += (ready ? 1u : 0u) + (fe[u] ? 0x10000u : 0u);
-          f_not_inc |= fe[u] && __vcmpgtu4(ds[u].x, K) == 0u;
-          any_s |= semi;
-          min_s = ::min(min_s, semi ? rd[u] : 0xFFFFFFFFu);
-          s_dec |= semi && __vcmpltu4(ds[u].x, K) != 0u;
-          sc[u] = fe[u] ? tv[u] * ds[u].z + 1u : 0u;
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const bool b = sc[u] > bs1;
-          bs1 = b ? sc[u] : bs1;
-          bj = b ? j[u] : bj;
-        }
-        if (need_sum) {
-          const uint64_t a = (uint64_t)(sc[0] ? sc[0] - 1u : 0u) + (sc[1] ? sc[1] - 1u : 0u);
-          const uint64_t b = (uint64_t)(sc[2] ? sc[2] - 1u : 0u) + (sc[3] ? sc[3] - 1u : 0u);
-          sum += a + b;
-        }
-#else
 #pragma unroll
         for (int u = 0; u < 4; ++u)
           if (v[u]) eval(j[u], rd[u], ds[u], dk[u], tv[u]);
-#endif
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
@@ -789,12 +789,14 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     const uint32_t nr = counts & 0xFFFFu, nf = counts >> 16;
     if (nr == 0) {  // necessary stall (L153): skip ahead to the next ready time
       t = min_s;
+      used = used_t = 0;
       continue;
     }
     if (nf == 0) {
       if (stall_en && any_s) {  // forced optional stall (L155, R22)
         kopt += min_s - t;
         t = min_s;
+        used = used_t = 0;
         continue;
       }
       o.cost = kInvalid;  // the ant is terminated (L149)
@@ -803,27 +805,28 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     uint4 x = make_uint4(0, 0, 0, 0);
     bool have_x = false;
     if (stall_en && any_s && all_f_inc && some_s_dec) {  // discretionary stall (L157-L164)
-      x = philox(t, ant, c2, V.region_id, cfg.seed);
+      x = philox(step, ant, c2, V.region_id, cfg.seed);
       have_x = true;
       const uint32_t thr = (kopt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (kopt + 1));
       if (x.z < thr) {
         ++kopt;
         ++t;
+        used = used_t = 0;
         continue;
       }
     }
     bool exploit;
-    if (t < coin_t) {  // the block's precomputed group coins (R3)
-      exploit = (coins[t >> 5] >> (t & 31u)) & 1u;
+    if (step < coin_t) {  // the block's precomputed group coins (R3)
+      exploit = (coins[step >> 5] >> (step & 31u)) & 1u;
     } else {
-      const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
+      const uint4 g = philox(step, 0x80000000u | group, c2, V.region_id, cfg.seed);
       exploit = (uint64_t)g.x < cfg.q0_t;
     }
     uint32_t jstar = bj;
     if (LG > 1) jstar = 0xFFFFFFFFu - (uint32_t)G.max64(bs1 ? akey(bs1 - 1u, bj) : 0ull);
     if (!exploit) {  // explore: roulette over F (R27), leader in ascending order
       if (G.leader()) {
-        if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
+        if (!have_x) x = philox(step, ant, c2, V.region_id, cfg.seed);
         const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
         uint64_t pre = 0;
         scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
@@ -831,8 +834,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
           rd_dk(j, rd, dk);
           if (rd > t) return false;
           const uint4 ds = V.ds[j];
+          if (mi && !((avail >> (8 * ds.w)) & 1u)) return false;
           if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u) return false;
-          pre += (uint32_t)trow[j] * ds.z;
+          pre += (uint32_t)trow[j] * eta_of(j, ds.z, dk);
           if (pre > r) {
             jstar = j;
             return true;
@@ -855,12 +859,24 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     G.sync();
     ++placed;
     prev = jstar;
-    ++t;
+    if (mi) {  // R42: the cycle is complete after issue_width placements
+      ++used;
+      used_t += 1u << (8 * V.ds[jstar].w);
+      if (used == w) {
+        ++t;
+        used = used_t = 0;
+      }
+    } else {
+      ++t;
+    }
   }
-  if (prune && G.leader()) atomicMin(prune_len, t);
+  const uint32_t len = t + (used ? 1u : 0u);  // last issue cycle + 1 (R20)
+  if (prune && G.leader()) atomicMin(prune_len, len);
   o.prp01 = prp01;
   o.prp23 = prp23;
-  o.cost = t;  // length = last issue cycle + 1 (R20)
+  o.len = len;
+  o.cost = len;
+  if (cfg.weighted && G.leader()) o.cost = len + cfg.ws_weight * cost_of(cfg.cost_mode, prp01, prp23);  // R41
   return o;
 }
 
@@ -956,7 +972,7 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
     uint32_t tgt[4];
 #pragma unroll
     for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
-    const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys;
+    const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
     uint16_t *rec_o = nullptr;
     uint32_t *rec_c = nullptr;
     if (dump && A.dump_order && A.dump_cycle) {
@@ -1063,11 +1079,16 @@ __device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
     uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
     const Grp<32> G32(threadIdx.x);
     AntOut o = ant_pass1<32, MASK>(V, tau, S, G32, 0, 0, A.cfg, true, gb1);
+    __syncwarp();
+    uint16_t *heur = (uint16_t *)(A.ws + W.o_heur);  // the heuristic order, kept for R40
+    for (uint32_t k = threadIdx.x; k < rd->n; k += 32) heur[k] = gb1[k];
     if (threadIdx.x != 0) return;
     rs.lb_cost = cost_rp(A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
     rs.init[0] = rs.best[0] = o.cost;
     const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
-    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = prp[c];
+    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = rs.heur_prp[c] = prp[c];
+    rs.policy = 0;
+    rs.heur_len = 0;
     rs.iters[0] = rs.iters[1] = 0;
     rs.no_imp = 0;
     rs.prune_len = kInvalid;
@@ -1083,8 +1104,37 @@ __global__ void __launch_bounds__(128) k_init(KArgs A) {
   else init_body<MASK, false>(A, (unsigned char *)smem4);
 }
 
+// ASAP timing of an order (R29) on the general machine model (R42): in-order
+// issue, c_k = max(c_{k-1}, ready time), moved to c_{k-1} + 1 when cycle
+// c_{k-1} has no free slot (width or the instruction's type).  One thread;
+// rdyv[n] is zeroed scratch.  Returns the length.
+__device__ uint32_t asap_order(const SV &V, const uint16_t *order, uint16_t *out_o, uint32_t *out_c,
+                               uint32_t *rdyv) {
+  const uint32_t n = V.n, w = c_mach.issue_width;
+  uint32_t t = 0, used = 0, used_t = 0;
+  for (uint32_t k = 0; k < n; ++k) {
+    const uint32_t j = order[k], y = V.ds[j].w;
+    uint32_t c = k == 0 ? rdyv[j] : max(t, rdyv[j]);
+    if (k > 0 && c == t && (used >= w || ((used_t >> (8 * y)) & 0xFFu) >= ((c_mach.type_slots >> (8 * y)) & 0xFFu)))
+      c = t + 1;
+    if (k == 0 || c != t) used = used_t = 0;
+    t = c;
+    ++used;
+    used_t += 1u << (8 * y);
+    if (out_o) out_o[k] = (uint16_t)j;
+    if (out_c) out_c[k] = t;
+    for (uint32_t q = V.succ_ptr[j]; q < V.succ_ptr[j + 1]; ++q) {
+      const uint32_t e = V.succ[q];
+      const uint32_t v = e & 0x1FFFu;
+      rdyv[v] = max(rdyv[v], t + (e >> 16));
+    }
+  }
+  return n ? t + 1 : 0;
+}
+
 // Pass transition (L147; R13, R18, R29): target from the pass-1 best, the
-// initial pass-2 schedule = ASAP(pass-1 best order), tau reset.
+// initial pass-2 schedule = ASAP(pass-1 best order), tau reset, the cycle-gap
+// filter (R39).  Weighted pass (R41): no target, weighted initial cost.
 __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
@@ -1101,27 +1151,59 @@ __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
     const uint16_t *gb1 = (const uint16_t *)(A.ws + W.o_gb1);
     uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
     uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
-    uint32_t t = 0;
-    for (uint32_t k = 0; k < n; ++k) {
-      const uint32_t j = gb1[k];
-      t = k == 0 ? rdyv[j] : max(t + 1, rdyv[j]);
-      gb2[k] = (uint16_t)j;
-      gb2c[k] = t;
-      for (uint32_t q = V.succ_ptr[j]; q < V.succ_ptr[j + 1]; ++q) {
-        const uint32_t e = V.succ[q];
-        const uint32_t v = e & 0x1FFFu;
-        rdyv[v] = max(rdyv[v], t + (e >> 16));
-      }
-    }
-    const uint32_t len = n ? t + 1 : 0;
-    rs.init[1] = rs.best[1] = len;
+    const uint32_t len = asap_order(V, gb1, gb2, gb2c, rdyv);
     for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.prp1[c];
+    rs.len2 = len;
     uint32_t tgt[4];
-    target_of(A.cfg.cost_mode, rs.prp1, tgt);
+    uint32_t best = len, lb = rd->lb_len;
+    if (A.cfg.weighted) {  // R41: cost = length + W * cost_rp, no RP target
+      for (int c = 0; c < 4; ++c) tgt[c] = kInvalid;
+      best = len + A.cfg.ws_weight * cost_rp(A.cfg.cost_mode, rs.prp1[0], rs.prp1[1], rs.prp1[2], rs.prp1[3]);
+      lb = rd->lb_len + A.cfg.ws_weight * rs.lb_cost;
+    } else {
+      target_of(A.cfg.cost_mode, rs.prp1, tgt);
+    }
+    rs.init[1] = rs.best[1] = best;
     for (int c = 0; c < 4; ++c) rs.target[c] = tgt[c];
     rs.no_imp = 0;
     rs.prune_len = kInvalid;
-    rs.active = (A.cfg.pass_mask & 2u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && len == rd->lb_len);
+    // R39: pass 2 only if the input schedule is >= pass2_gap cycles above LB_len
+    const bool gap_cut = !A.cfg.weighted && (A.cfg.pass_mask & 2u) && A.cfg.pass2_gap > 0 &&
+                         len < rd->lb_len + A.cfg.pass2_gap;
+    if (gap_cut) rs.policy |= 1u;
+    rs.active = (A.cfg.pass_mask & 2u) && A.cfg.iterations > 0 && !gap_cut && !(A.cfg.stop_at_lb && best == lb);
+  }
+}
+
+// After the last pass (L366; R40): the heuristic schedule's length, and the
+// revert filter -- report the heuristic schedule when the result gained at
+// least revert_occ occupancy but is more than revert_len cycles longer.
+__global__ void __launch_bounds__(32) k_post(KArgs A) {
+  const uint32_t r = blockIdx.x;
+  const RegionDev *rd = A.regions + r;
+  const RegionWs &W = A.rws[r];
+  RegionState &rs = A.state[r];
+  extern __shared__ uint32_t rdyv[];  // rdy[n]
+  const uint32_t n = rd->n;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) rdyv[i] = 0;
+  __syncwarp();
+  if (threadIdx.x != 0) return;
+  const SV V = make_sv(A.arena + rd->o_image, rd);
+  const uint16_t *heur = (const uint16_t *)(A.ws + W.o_heur);
+  const uint32_t hlen = asap_order(V, heur, nullptr, nullptr, rdyv);
+  rs.heur_len = hlen;
+  if (A.cfg.revert_occ == 0) return;
+  uint32_t of = c_mach.occ_max, oh = c_mach.occ_max;
+  for (uint32_t c = 0; c < c_mach.n_classes; ++c) {
+    of = min(of, occ_of(c, rs.prp2[c]));
+    oh = min(oh, occ_of(c, rs.heur_prp[c]));
+  }
+  if (of >= oh + A.cfg.revert_occ && (uint64_t)rs.len2 > (uint64_t)hlen + A.cfg.revert_len) {
+    for (uint32_t i = 0; i < n; ++i) rdyv[i] = 0;
+    asap_order(V, heur, (uint16_t *)(A.ws + W.o_gb2), (uint32_t *)(A.ws + W.o_gb2c), rdyv);
+    for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.heur_prp[c];
+    rs.len2 = hlen;
+    rs.policy |= 2u;
   }
 }
 
@@ -1176,6 +1258,7 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
     if (threadIdx.x == 0) {
       s_prp[0] = o.prp01;
       s_prp[1] = o.prp23;
+      s_prp[2] = o.len;
     }
   }
   __syncwarp();
@@ -1188,7 +1271,8 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
   }
   // ---- epilogue (first thread, L139)
   if (threadIdx.x == 0) {
-    rs.hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(rs.hash, PASS), iter), have ? wcost : kInvalid),
+    rs.hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(rs.hash, PASS == 2 && A.cfg.weighted ? 4u : PASS), iter),
+                              have ? wcost : kInvalid),
                       have ? want : kInvalid);
     const bool improved = have && wcost < rs.best[PASS - 1];  // strict (R11)
     s_flag = improved;
@@ -1200,6 +1284,7 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
       prp[1] = s_prp[0] >> 16;
       prp[2] = s_prp[1] & 0xFFFFu;
       prp[3] = s_prp[1] >> 16;
+      if (PASS == 2) rs.len2 = s_prp[2];
     } else {
       rs.no_imp++;
     }
@@ -1226,7 +1311,7 @@ template <int PASS, bool MASK, bool T32, bool NC4>
 __global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   if (!A.state[blockIdx.x].active) return;
   extern __shared__ uint4 smem4[];
-  __shared__ uint32_t s_prp[2], s_flag;
+  __shared__ uint32_t s_prp[3], s_flag;
   if (A.rws[blockIdx.x].gs)
     select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
   else
@@ -1254,7 +1339,7 @@ __global__ void k_stop(KArgs A, uint32_t pass) {
   if (!rs.active) return;
   const RegionDev *rd = A.regions + r;
   const uint32_t lim = no_improve_limit(A.cfg, rd->n);
-  const uint32_t lb = pass == 1 ? rs.lb_cost : rd->lb_len;
+  const uint32_t lb = pass == 1 ? rs.lb_cost : rd->lb_len + (A.cfg.weighted ? A.cfg.ws_weight * rs.lb_cost : 0u);
   if ((A.cfg.stop_at_lb && rs.best[pass - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
       rs.iters[pass - 1] >= A.cfg.iterations)
     rs.active = 0;
@@ -1400,6 +1485,7 @@ int set_machine(const MachineDev &m) {
   big_smem(k_init<true>);
   big_smem(k_init<false>);
   big_smem(k_pass2_init);
+  big_smem(k_post);
 #define ACO_SEL(M) big_smem(k_select<1, M, false, false>); big_smem(k_select<2, M, false, false>); \
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
@@ -1463,6 +1549,13 @@ int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, u
   if (n_upd) k_update<<<n_upd, 256, 0, s>>>(a, upd);
   k_stop<<<(L.cfg.count + 255) / 256, 256, 0, s>>>(a, pass);
   L.launches += 2 + (n_upd ? 1 : 0);
+  return check();
+}
+
+int launch_post(LaunchCtx &L, uint32_t smem) {
+  if (!L.cfg.count) return 0;
+  k_post<<<L.cfg.count, 32, smem, (cudaStream_t)L.stream>>>(kargs(L));
+  L.launches++;
   return check();
 }
 

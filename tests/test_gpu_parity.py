@@ -39,6 +39,8 @@ def compare_results(gpu, ora, ctx=""):
     assert gpu["trace_hash"] == ora["trace_hash"], ctx
     assert list(gpu["order"]) == list(ora["order"]), ctx
     assert list(gpu["cycle"]) == list(ora["cycle"]), ctx
+    assert gpu["policy"] == ora["policy"] and gpu["heur_len"] == ora["heur_len"], ctx
+    assert gpu["ws_cost"] == ora["ws_cost"], ctx
 
 
 def dump_parity(s, regions, ids, p, machine=I.GFX906):
@@ -48,8 +50,9 @@ def dump_parity(s, regions, ids, p, machine=I.GFX906):
         ora = O.schedule(reg, rid, machine, p, dump=True, dump_orders=True)
         n = reg.n_insts
         base0 = A * int(s.batch.offsets[k])
+        pmask = 2 if p.passes == 4 else p.passes  # pass 4 (R41) fills the pass-2 slots
         for ps in (0, 1):
-            if not (p.passes & (ps + 1)):
+            if not (pmask & (ps + 1)):
                 continue
             iters = ora["iters1"] if ps == 0 else ora["iters2"]
             for it in range(iters):
