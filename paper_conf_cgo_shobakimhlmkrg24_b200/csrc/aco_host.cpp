@@ -273,7 +273,7 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   for (uint32_t j = 0; j < n; ++j) cp_max = std::max(cp_max, cp[j]);
   // per-instruction info + multi-use entries
   std::vector<uint32_t> info((size_t)n * 4, 0), muse;
-  uint32_t L = 0;
+  uint32_t L = 0, mc_max = 0;
   uint32_t lbvec[4] = {0, 0, 0, 0}, livein[4] = {0, 0, 0, 0}, liveout[4] = {0, 0, 0, 0};
   for (uint32_t g = 0; g < G; ++g) {
     if (d.reg_flags[g] & kFlagLiveIn) livein[d.reg_class[g]]++;
@@ -306,6 +306,11 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
     L = std::max(L, nonlo);
     const uint32_t mcnt = (uint32_t)muse.size() - mstart;
     if (mcnt > 15u) return ACO_E_TOO_LARGE;  // 4-bit last-use counters
+    {
+      uint32_t mc[4] = {0, 0, 0, 0};
+      for (uint32_t q = mstart; q < mstart + mcnt; ++q) mc[(muse[q] >> 16) & 3u]++;
+      for (uint32_t c = 0; c < 4; ++c) mc_max = std::max(mc_max, mc[c]);
+    }
     for (uint32_t c = 0; c < 4; ++c) {
       if (defs[c] > 255u || dead[c] > 255u || sk[c] > 255u) return ACO_E_TOO_LARGE;
       info[(size_t)j * 4 + 0] |= defs[c] << (8 * c);
@@ -419,6 +424,7 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   }
   R.max_cycle_bound = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)n * (max_lat + 1ull) + 1);
   R.max_lat = max_lat;
+  R.mc_max = mc_max;
   for (uint32_t c = 0; c < 4; ++c) {
     R.livein[c] = livein[c];
     R.lbvec[c] = lbvec[c];
@@ -660,10 +666,12 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     const RegionDev &R = ctx->regions[r];
     P.max_n = std::max(P.max_n, R.n);
     // pass-2 state variant: the compact layout (windowed u8 ready times) needs
-    // latencies <= 127 and 2 classes; otherwise u16 cycles, or u32 when a
-    // schedule may exceed 65535 cycles (or a latency exceeds 127)
+    // latencies < 512, 2 classes and <= 7 multi-use registers per class and
+    // instruction; otherwise u16 cycles (3-4 classes), or u32 when a
+    // schedule may exceed 65535 cycles (or the compact layout does not apply)
     // the general machine model (R42) runs in the u32-cycle variants
-    const bool t32 = ctx->mach.issue_width > 1 || (P.nc4 ? R.max_cycle_bound > 65535u : R.max_lat > 127u);
+    const bool t32 = ctx->mach.issue_width > 1 ||
+                     (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
     P.any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);

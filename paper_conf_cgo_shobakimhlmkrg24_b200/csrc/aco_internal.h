@@ -68,7 +68,7 @@ struct RegionDev {
   uint32_t livein[4];
   uint32_t lbvec[4]; // per-class PRP lower bound vector (R30)
   uint32_t max_lat;  // largest edge latency
-  uint32_t pad0;
+  uint32_t mc_max;   // max over instructions and classes of multi-use registers read
   uint64_t o_image;  // byte offset of the block image in the arena
   ImageLayout img;
 };
@@ -157,9 +157,10 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 //   RB [nwr] ready set, SCH [nwr] scheduled set, REM [nremw] u16 counters, then
 //   pass 1: DK [ceil(n/8)]  4-bit count of registers whose last remaining
 //                           user is the instruction (dynamic part of LUC)
-//   pass 2, compact (2 classes, latencies <= 127):
-//           X  [ceil(n/2)] u16: windowed ready time (u8) | last-use counts
-//                           (2 classes x 4 bits) << 8
+//   pass 2, compact (2 classes, latencies < 512, <= 7 multi-use registers
+//           per class and instruction):
+//           X  [ceil(n/2)] u16: windowed ready time (10 bits) | last-use
+//                           counts (2 classes x 3 bits) << 10
 //   pass 2, otherwise:
 //           T  [ceil(n/2)] u16 (or [n] u32 if t32): issue cycle (placed) or
 //                           ready time (ready instruction)

@@ -201,7 +201,7 @@ __device__ __forceinline__ void dk_add(const St &A, uint32_t j, uint32_t c) {
   if (PASS == 1) {
     A.DK[(j >> 3) * A.S] += 1u << ((j & 7u) * 4);
   } else if (!T32 && !NC4) {  // compact: the high byte of j's u16
-    A.T[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 8 + 4 * c);
+    A.T[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 10 + 3 * c);
   } else if (NC4) {
     A.DK[(j >> 1) * A.S] += 1u << ((j & 1u) * 16 + 4 * c);
   } else {
@@ -225,23 +225,33 @@ __device__ __forceinline__ void t_set(const St &A, uint32_t j, uint32_t v) {
   }
 }
 
-// ---- pass-2 compact layout: x = u16 of instruction j = rt | dk << 8, where
-// rt = (ready time - B) for an unplaced instruction whose predecessors were
-// placed (a push-style maximum of t_p + lat over placed predecessors; 0 for
-// none) and B is the ant's window base.  Invariant: t - B < 128 at every
-// turn and latencies <= 127 (host), so every stored rt <= 254; when t - B
-// reaches 128 the window slides by 128 (saturating: a clamped rt still reads
-// as "ready now", which is all that matters for a value below t).
+// ---- pass-2 compact layout: x = u16 of instruction j = rt | dk0 << 10 |
+// dk1 << 13, where rt (10 bits) = (ready time - B) for an unplaced
+// instruction whose predecessors were placed (a push-style maximum of
+// t_p + lat over placed predecessors; 0 for none), B is the ant's window base
+// and dk_c (3 bits) the class-c last-use counts.  Invariant: t - B < kWin at
+// every turn and latencies < kWin (host), so every stored rt <= 2 kWin - 2;
+// when t - B reaches kWin (one jump moves t at most to B + 2 kWin - 2) the
+// window slides by kWin (saturating: a clamped rt still reads as "ready now",
+// which is all that matters for a value below t).  Host: the compact layout
+// needs 2 classes, latencies < kWin and <= 7 multi-use registers per class
+// and instruction.
+constexpr uint32_t kWin = 512;
 __device__ __forceinline__ uint32_t x_get(const St &A, uint32_t j) {
   return (A.T[(j >> 1) * A.S] >> ((j & 1u) * 16)) & 0xFFFFu;
 }
 __device__ __forceinline__ uint32_t x_dk(uint32_t x) {  // packed u8 x 4 per class
-  return ((x >> 8) & 0xFu) | ((x & 0xF000u) >> 4);
+  return ((x >> 10) & 0x7u) | ((x & 0xE000u) >> 5);
 }
 __device__ __forceinline__ void x_push_rt(const St &A, uint32_t v, uint32_t rt) {
   uint32_t *p = A.T + (v >> 1) * A.S;
-  const uint32_t sh = (v & 1u) * 16, w = *p, cur = (w >> sh) & 0xFFu;
+  const uint32_t sh = (v & 1u) * 16, w = *p, cur = (w >> sh) & 0x3FFu;
   if (rt > cur) *p = w + ((rt - cur) << sh);
+}
+// Slide both halves' 10-bit rt by kWin = 512, saturating at 0:
+// rt >= 512 -> rt & 0x1FF, else 0 (rt < 1024).
+__device__ __forceinline__ uint32_t x_slide2(uint32_t w) {
+  return (w & 0xFC00FC00u) | (w & (((w >> 9) & 0x00010001u) * 0x1FFu));
 }
 
 // ---- lane groups: LG consecutive lanes of a warp build one ant together.
@@ -690,7 +700,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   auto rd_dk = [&](uint32_t j, uint32_t &rd, uint32_t &dk) {
     if constexpr (CT) {
       const uint32_t x = x_get(A, j);
-      rd = B + (x & 0xFFu);
+      rd = B + (x & 0x3FFu);
       dk = x_dk(x);
     } else {
       rd = t_get<T32>(A, j);
@@ -705,9 +715,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   o.prp01 = o.prp23 = 0;
   o.len = kInvalid;
   while (placed < n) {
-    if (CT && t - B >= 128u) {  // slide the ready-time window (t - B <= 254 here)
-      for (uint32_t q = G.lane; q < (n + 1) / 2; q += LG) A.T[q * A.S] = __vsubus4(A.T[q * A.S], 0x00800080u);
-      B += 128u;
+    if (CT && t - B >= kWin) {  // slide the ready-time window (t - B <= 2 kWin - 2 here)
+      for (uint32_t q = G.lane; q < (n + 1) / 2; q += LG) A.T[q * A.S] = x_slide2(A.T[q * A.S]);
+      B += kWin;
       G.sync();
     }
     if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune

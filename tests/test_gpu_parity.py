@@ -294,16 +294,17 @@ def test_shared_colony_equals_single_context(torch_cuda):
 
 def _relat(reg, f, tag):
     """The same DDG with every edge latency mapped by f (exercises the
-    pass-2 ready-time layouts: windowed u8 for latencies <= 127, u32 beyond)."""
+    pass-2 ready-time layouts: windowed 10-bit for latencies < 512, u32 beyond)."""
     lat = np.asarray([f(int(x)) for x in reg.edge_lat], np.uint32)
     return I.Region(reg.n_insts, reg.edge_src, reg.edge_dst, lat, reg.reg_class, reg.reg_flags,
                     reg.def_ptr, reg.def_reg, reg.use_ptr, reg.use_reg, name=reg.name + tag)
 
 
 def test_latency_window_boundary_every_ant(torch_cuda):
-    """Latencies up to exactly 127 (the compact layout's bound) and schedules
-    of several hundred cycles (the ready-time window slides many times)."""
-    regs = [_relat(I.gen_region(n, 800 + n), lambda x: 127 if x >= 20 else x, "-l127") for n in (25, 70, 180)]
+    """Latencies up to exactly 511 (the compact layout's bound) and schedules
+    of thousands of cycles (the ready-time window slides many times)."""
+    regs = [_relat(I.gen_region(n, 800 + n), lambda x: 511 if x >= 20 else (127 if x >= 8 else x), "-l511")
+            for n in (25, 70, 180)]
     ids = [31, 32, 33]
     p = I.Params(ants=72, iterations=2, seed=21, stall_mod=2)
     s = _sched()
@@ -312,10 +313,34 @@ def test_latency_window_boundary_every_ant(torch_cuda):
 
 
 def test_long_latencies_every_ant(torch_cuda):
-    """Latencies above 127 force the u32 ready-time layout."""
-    regs = [_relat(I.gen_region(n, 900 + n), lambda x: x * 3 + (150 if x >= 20 else 0), "-long") for n in (25, 70, 180)]
+    """Latencies of 512 and above force the u32 ready-time layout."""
+    regs = [_relat(I.gen_region(n, 900 + n), lambda x: x * 8 + (600 if x >= 20 else 0), "-long") for n in (25, 70, 180)]
     ids = [41, 42, 43]
     p = I.Params(ants=72, iterations=2, seed=22, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def many_multiuse_region():
+    """Instructions reading 9 VGPRs that each have several users: more than 7
+    multi-use registers of one class per instruction (3-bit last-use counts
+    do not fit -> the u32 layout)."""
+    n = 24
+    defs = [[g] for g in range(9)] + [[9 + k] for k in range(12)] + [[], [], []]
+    uses = [[] for _ in range(9)] + [list(range(9)) for _ in range(12)] + [[9, 10, 11], [12, 13, 14], list(range(15, 21))]
+    edges = set()
+    for j, u in enumerate(uses):
+        for g in u:
+            d = next(i for i, dd in enumerate(defs) if g in dd)
+            edges.add((d, j, 1 + (d % 5)))
+    return I.Region.from_lists(n, sorted(edges), [0] * 21, [0] * 21, defs, uses, name="multiuse9")
+
+
+def test_many_multiuse_registers_every_ant(torch_cuda):
+    regs = [many_multiuse_region(), I.gen_region(40, 4242)]
+    ids = [51, 52]
+    p = I.Params(ants=80, iterations=3, seed=23, stall_mod=1, cost_mode=0)
     s = _sched()
     s.load(regs, ids).run(p, no_prune=True, dump=True)
     dump_parity(s, regs, ids, p)
