@@ -375,6 +375,35 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
     for (uint32_t j = 0; j < n; ++j)
       for (uint32_t q = sp[j]; q < sp[j + 1]; ++q) pred[fill[outs[q]]++] = j | (lats[q] << 16);
   }
+  // predecessor groups: per instruction, {bitset word, mask of its
+  // predecessors in that word} (readiness test of pass 1 / compact pass 2)
+  std::vector<uint32_t> pgp(n + 1, 0), pgv;
+  for (uint32_t v = 0; v < n; ++v) {
+    std::vector<std::pair<uint32_t, uint32_t>> gr;
+    for (uint32_t q = pp[v]; q < pp[v + 1]; ++q) {
+      const uint32_t p = pred[q] & 0xFFFFu;
+      bool found = false;
+      for (auto &g : gr)
+        if (g.first == p >> 5) {
+          g.second |= 1u << (p & 31);
+          found = true;
+        }
+      if (!found) gr.push_back({p >> 5, 1u << (p & 31)});
+    }
+    std::sort(gr.begin(), gr.end());
+    for (auto &g : gr) {
+      pgv.push_back(g.first);
+      pgv.push_back(g.second);
+    }
+    pgp[v + 1] = (uint32_t)(pgv.size() / 2);
+  }
+  // the per-predecessor list is needed only by the u16/u32-cycle pass-2
+  // layouts (ready time = max over predecessors at readiness)
+  const bool compact = mach.issue_width <= 1 && n_classes <= 2 && max_lat <= 511u && mc_max <= 7u;
+  if (compact) {
+    pred.clear();
+    pp.assign(n + 1, 0);
+  }
   // initial per-ant state
   const uint32_t nwr = (n + 31) / 32;
   std::vector<uint32_t> rb0(nwr, 0), rem0((nctr + 1) / 2, 0);
@@ -399,6 +428,8 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   R.img.pred = img_put(img, pred);
   R.img.rb0 = img_put(img, rb0);
   R.img.rem0 = img_put(img, rem0);
+  R.img.pg_ptr = img_put(img, pgp);
+  R.img.pg = img_put(img, pgv);
   img.resize(align16(img.size()) + 16, 0);
   R.img.bytes = (uint32_t)img.size();
   R.n = n;
@@ -425,6 +456,7 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   R.max_cycle_bound = (uint32_t)std::min<uint64_t>(0xFFFFFFFFull, (uint64_t)n * (max_lat + 1ull) + 1);
   R.max_lat = max_lat;
   R.mc_max = mc_max;
+  R.compact = compact ? 1u : 0u;
   for (uint32_t c = 0; c < 4; ++c) {
     R.livein[c] = livein[c];
     R.lbvec[c] = lbvec[c];

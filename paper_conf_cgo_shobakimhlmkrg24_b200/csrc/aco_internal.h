@@ -48,11 +48,12 @@ struct ImageLayout {
   uint32_t succ_ptr;  // u32 [n+1]
   uint32_t succ;      // u32 [E]
   uint32_t pred_ptr;  // u32 [n+1]
-  uint32_t pred;      // u32 [E]: p | latency << 16
+  uint32_t pred;      // u32 [E]: p | latency << 16 (only for the u16/u32-cycle pass-2 layouts)
   uint32_t rb0;       // u32 [nwr]: roots bitset
   uint32_t rem0;      // u32 [nremw]: u16 use counts of >= 3-use registers
   uint32_t bytes;     // total, multiple of 16
-  uint32_t pad[2];
+  uint32_t pg_ptr;    // u32 [n+1]: predecessor groups of each instruction
+  uint32_t pg;        // uint2 [..]: {bitset word, mask of the predecessors in that word}
 };
 
 // Per-region statics (arena header array).
@@ -69,6 +70,8 @@ struct RegionDev {
   uint32_t lbvec[4]; // per-class PRP lower bound vector (R30)
   uint32_t max_lat;  // largest edge latency
   uint32_t mc_max;   // max over instructions and classes of multi-use registers read
+  uint32_t compact;  // pass 2 uses the compact layout (the image has no per-predecessor list)
+  uint32_t pad1;
   uint64_t o_image;  // byte offset of the block image in the arena
   ImageLayout img;
 };

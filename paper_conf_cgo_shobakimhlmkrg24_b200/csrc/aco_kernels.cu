@@ -121,7 +121,8 @@ __device__ void target_of(uint32_t mode, const uint32_t best[4], uint32_t tgt[4]
 struct SV {
   const uint4 *info;
   const uint4 *ds;
-  const uint32_t *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0;
+  const uint32_t *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0, *pg_ptr;
+  const uint2 *pg;
   const uint16_t *eta1, *eta2;
   uint32_t n, nwr, nremw, region_id, L1;
   uint32_t livein01, livein23;  // u16 x 2
@@ -140,6 +141,8 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   V.succ = (const uint32_t *)(img + rd->img.succ);
   V.pred_ptr = (const uint32_t *)(img + rd->img.pred_ptr);
   V.pred = (const uint32_t *)(img + rd->img.pred);
+  V.pg_ptr = (const uint32_t *)(img + rd->img.pg_ptr);
+  V.pg = (const uint2 *)(img + rd->img.pg);
   V.rb0 = (const uint32_t *)(img + rd->img.rb0);
   V.rem0 = (const uint32_t *)(img + rd->img.rem0);
   V.n = rd->n;
@@ -483,7 +486,17 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
     bool ready = true;
     uint32_t rdy = t + (e >> 16);
     if (CT) x_push_rt(A, v, rdy - B);  // ready time = max over placed predecessors
-    if (!(e & kSuccSingle)) {
+    if (!(e & kSuccSingle) && (PASS == 1 || CT)) {
+      // v is ready iff all its predecessors are placed: one scheduled-set
+      // word per group of predecessors sharing a bitset word
+      for (uint32_t k = V.pg_ptr[v]; k < V.pg_ptr[v + 1]; ++k) {
+        const uint2 g = V.pg[k];
+        if ((A.SCH[g.x * A.S] & g.y) != g.y) {
+          ready = false;
+          break;
+        }
+      }
+    } else if (!(e & kSuccSingle)) {
       const uint32_t p0 = V.pred_ptr[v], p1 = V.pred_ptr[v + 1];
       if (PASS == 2 && !CT) rdy = 0;
       for (uint32_t k = p0; k < p1; ++k) {
@@ -1322,10 +1335,16 @@ __global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   if (!A.state[blockIdx.x].active) return;
   extern __shared__ uint4 smem4[];
   __shared__ uint32_t s_prp[3], s_flag;
-  if (A.rws[blockIdx.x].gs)
-    select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
-  else
-    select_body<PASS, MASK, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+  // a batch with some u32-cycle regions launches the T32 variant; its compact
+  // regions replay with the compact layout (their image has no predecessor list)
+  const bool ct = PASS == 2 && T32 && !NC4 && A.regions[blockIdx.x].compact;
+  if (A.rws[blockIdx.x].gs) {
+    if (ct) select_body<PASS, false, false, false, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    else select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+  } else {
+    if (ct) select_body<PASS, MASK, false, false, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    else select_body<PASS, MASK, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+  }
 }
 
 // Shared colony: per-region local argmin over this context's ants, written as
