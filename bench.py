@@ -5,8 +5,17 @@ One STEP = one full two-pass ACO run (aco_schedule_batch: every pass and
 iteration of every region: construction, argmin + winner replay, pheromone
 update, epilogue) over one batch of synthetic regions.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c3|c2|c1]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c3|c2|c1|c4|c5]
+                  [--machine gfx906|dual] [--passes 3|4 --ws-weight W] [--policy off|paper]
+                  [--heur-mix 0|1] [--stall-num k]
   python bench.py --impl reference ...     # the CPU oracle on a bounded sample
+
+Workloads (BASELINE.json configs): c1 FIX10-A; c2 one n = 100 region; c3
+(default, the metric's config) 5,000 rocPRIM-shaped regions per GPU (weak
+scaling); c4 one n = 2,000 region with 8,192 ants per iteration as ONE shared
+colony across the N ranks (strong scaling: 8,192 / N ants per rank, one int64
+MIN allreduce per iteration over NCCL); c5 the full-suite sweep, 1,000
+regions per GPU up to 4,000 instructions (weak scaling).
 
 Multi-GPU: launched by torchrun, one process per GPU.  Regions shard with no
 data-path collective (each rank schedules its own batch with globally unique
@@ -15,6 +24,7 @@ region ids); NCCL is used only for the barrier and the max-over-ranks time.
 from __future__ import annotations
 
 import argparse
+import dataclasses
 import json
 import os
 import subprocess
@@ -39,7 +49,13 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="c3", choices=["c3", "c2", "c1"])
+    ap.add_argument("--workload", default="c3", choices=["c3", "c2", "c1", "c4", "c5"])
+    ap.add_argument("--machine", default="gfx906", choices=["gfx906", "dual"])
+    ap.add_argument("--passes", type=int, default=3, choices=[1, 2, 3, 4])
+    ap.add_argument("--ws-weight", type=int, default=4)
+    ap.add_argument("--policy", default="off", choices=["off", "paper"])
+    ap.add_argument("--heur-mix", type=int, default=0)
+    ap.add_argument("--stall-num", type=int, default=1)
     ap.add_argument("--regions", type=int, default=C3_REGIONS, help="regions per rank (c3)")
     ap.add_argument("--ants", type=int, default=None)
     ap.add_argument("--iterations", type=int, default=None)
@@ -64,14 +80,47 @@ def workload(args, rank: int):
         ids = [rank]
         p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 100, seed=2)
         cfg = {"workload": "c2-single-region-n100", "regions_per_gpu": 1, "latency": "mixed"}
+    elif args.workload == "c4":
+        regs = [I.gen_region(2000, I.region_seed(4, 0))]
+        ids = [0]  # ONE region shared by all ranks (shared colony)
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        total = args.ants or 8192
+        p = I.Params(ants=total // world, iterations=args.iterations or 10, seed=4)
+        cfg = {"workload": "c4-shared-colony-n2000", "regions": 1, "ants_total": total,
+               "ants_per_gpu": total // world, "latency": "mixed"}
+    elif args.workload == "c5":
+        n = args.regions if args.regions != C3_REGIONS else 1000
+        first = rank * n
+        sizes = I.c5_sizes(first + n, base_seed=5)[first:]
+        regs = I.gen_batch(n, base_seed=5, first_id=first, sizes=sizes)
+        ids = list(range(first, first + n))
+        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 5, seed=5)
+        cfg = {"workload": "c5-suite-sweep", "regions_per_gpu": n, "sizes": "20-4000 (c3 mix + 15% tail 500-4000)",
+               "max_n": int(max(r.n_insts for r in regs)), "latency": "mixed"}
     else:
         regs = [I.fix10a()]
         ids = [rank]
         p = I.Params(ants=args.ants or 64, iterations=args.iterations or 20, seed=0, cost_mode=0)
         cfg = {"workload": "c1-fix10a", "regions_per_gpu": 1}
-    cfg.update({"ants": p.ants, "iterations_per_pass": p.iterations, "passes": "RP+ILP",
-                "cost": ["PRP_SUM", "APRP_SUM", "OCC", "PERP"][p.cost_mode], "stop_rules": "off (fixed work)"})
+    p = dataclasses.replace(p, passes=args.passes, ws_weight=args.ws_weight if args.passes == 4 else 0,
+                            heur_mix=args.heur_mix, stall_num=args.stall_num)
+    if args.policy == "paper":
+        p = I.paper_policy(p)
+    passes = {1: "RP", 2: "ILP", 3: "RP+ILP", 4: f"weighted single pass (W={p.ws_weight})"}[p.passes]
+    cfg.update({"ants": p.ants, "iterations_per_pass": p.iterations, "passes": passes,
+                "cost": ["PRP_SUM", "APRP_SUM", "OCC", "PERP"][p.cost_mode],
+                "stop_rules": "paper policy (LB, size classes, gap 21, revert 3/63)" if args.policy == "paper"
+                else "off (fixed work)",
+                "machine": "gfx906 single issue" if args.machine == "gfx906" else "dual issue (VALU/SALU/MEM)"})
+    if args.heur_mix:
+        cfg["heur_mix"] = 1
+    if args.stall_num != 1:
+        cfg["stall_groups"] = f"{args.stall_num}/{p.stall_mod}"
     return regs, ids, p, cfg
+
+
+def machine_of(args):
+    return I.DUAL_ISSUE if args.machine == "dual" else I.GFX906
 
 
 class ClockSampler:
@@ -138,7 +187,18 @@ def bytes_per_ant_step(stats: np.ndarray) -> float:
     return float(b / max(pl, 1.0))
 
 
-def cpu_baseline(regs, ids, p, sample: int):
+def cpu_sample_params(args, p):
+    """Bounded oracle sample: fewer ants / iterations where the full workload
+    would take minutes on the host (c4: one n = 2,000 region; c5: regions up
+    to 4,000 instructions); the per-ant-schedule cost is what is measured."""
+    if args.workload == "c4":
+        return dataclasses.replace(p, ants=64, iterations=2), "64 ants x 2 iterations per pass of the n = 2,000 region"
+    if args.workload == "c5":
+        return dataclasses.replace(p, ants=32, iterations=2), "32 ants x 2 iterations per pass"
+    return p, "full A x I x passes"
+
+
+def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes"):
     """The oracle as it stands on a bounded, stratified sample of the same workload."""
     from oracle import pyoracle as O
     k = min(sample, len(regs))
@@ -148,11 +208,11 @@ def cpu_baseline(regs, ids, p, sample: int):
     sid = [ids[i] for i in pick]
     threads = os.cpu_count() or 1
     t0 = time.perf_counter()
-    _, _, stats, _ = O.schedule_many(sub, sid, I.GFX906, p, n_threads=threads)
+    _, _, stats, _ = O.schedule_many(sub, sid, machine, p, n_threads=threads)
     dt = time.perf_counter() - t0
     scheds = float(stats[:, O.ORS["ant_scheds"]].sum())
-    return {"value": scheds / dt, "unit": METRIC, "cores": threads, "kind": "oracle",
-            "sample": f"{len(sub)} of {len(regs)} regions (stratified by size), full A x I x 2 passes, "
+    return {"value": scheds / dt, "unit": METRIC, "cores": min(threads, len(sub)), "kind": "oracle",
+            "sample": f"{len(sub)} of {len(regs)} regions (stratified by size), {note}, "
                       f"{scheds:.0f} ant-schedules in {dt:.1f} s"}, stats
 
 
@@ -173,8 +233,10 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     regs, ids, p, cfg = workload(args, rank)
+    machine = machine_of(args)
+    colony = args.workload == "c4" and world > 1  # one region, ants split across ranks
     batch = HostBatch(regs, ids)
-    sched = Scheduler(I.GFX906, device=local)
+    sched = Scheduler(machine, device=local)
     stream = torch.cuda.current_stream()
     sched.load(regs, ids, batch=batch)
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{local}")
@@ -183,8 +245,14 @@ def main():
         if world > 1:
             dist.barrier()
 
+    def run(timing=False):
+        if colony:
+            sched.run_colony(p, rank, world, timing=timing)
+        else:
+            sched.run(p, timing=timing)
+
     for _ in range(max(3, args.warmup)):
-        sched.run(p)
+        run()
     torch.cuda.synchronize()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)]
@@ -198,7 +266,7 @@ def main():
     for k in range(args.steps):
         flush.zero_()  # L2 flush between timed steps (outside the events)
         ev[k][0].record(stream)
-        sched.run(p, timing=True)
+        run(timing=True)
         ev[k][1].record(stream)
         ms, ln = sched.timing()  # syncs; events inside the library, same stream
         phase_ms += ms
@@ -231,7 +299,7 @@ def main():
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         sched.load(regs, ids, batch=batch)
-        sched.run(p)
+        run()
         sched.results_raw(0, len(regs), orders, cycles)
         e2e_ms.append((time.perf_counter() - t0) * 1000.0)
     h2d = int(sched.arena.numel()) if sched.arena is not None else 0
@@ -247,7 +315,9 @@ def main():
         cpu = None
         bpas = None
         if world == 1 and not args.no_cpu_baseline:
-            cpu, stats = cpu_baseline(regs, ids, p, args.cpu_sample)
+            ps, note = cpu_sample_params(args, p)
+            cpu, stats = cpu_baseline(regs, ids, ps, args.cpu_sample if args.workload != "c5" else 24,
+                                      machine, note)
             bpas = bytes_per_ant_step(stats)
         # roofline of the dominant kernel (ant construction):
         # algorithmic shared-memory bytes (SURVEY 8(d) per ant-step figure from
@@ -272,9 +342,12 @@ def main():
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup),
-            "ms_per_step": round(max_ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": round(max_ms / args.steps, 3), "higher_is_better": True,
+            "scaling": "strong" if args.workload == "c4" else "weak",
             "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)", "data": "synthetic",
-            "config": dict(cfg, l2="flushed between timed steps (256 MB write)", parallelism=f"regions x{world}"),
+            "config": dict(cfg, l2="flushed between timed steps (256 MB write)",
+                           parallelism=f"shared colony x{world} (NCCL int64 MIN allreduce per iteration)"
+                           if args.workload == "c4" else f"regions x{world}"),
             "aco_ms_per_batch": round(max_ms / args.steps, 3),
             "phase_ms_per_step": {"construct": round(phase_ms[0] / args.steps, 3),
                                   "finalize": round(phase_ms[1] / args.steps, 3),
@@ -299,10 +372,11 @@ def reference_arm(args, world, rank):
     regs, ids, p, cfg = workload(args, 0)
     cpu_times = []
     scheds = 0.0
+    ps, note = cpu_sample_params(args, p)
     for _ in range(args.warmup):
         pass  # the oracle has no warm-up state
     for _ in range(args.steps):
-        cpu, stats = cpu_baseline(regs, ids, p, max(4, args.cpu_sample // max(1, args.steps)))
+        cpu, stats = cpu_baseline(regs, ids, ps, max(4, args.cpu_sample // max(1, args.steps)), machine_of(args), note)
         from oracle.pyoracle import ORS
         s = float(stats[:, ORS["ant_scheds"]].sum())
         scheds += s
@@ -311,7 +385,7 @@ def reference_arm(args, world, rank):
     value = scheds / tot_s
     out = {"metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(1000 * tot_s / args.steps, 3), "higher_is_better": True,
-           "scaling": "weak", "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
+           "scaling": "strong" if args.workload == "c4" else "weak", "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
            "data": "synthetic", "config": cfg, "impl": "reference",
            "cpu_baseline": {"value": round(value, 1), "unit": METRIC, "cores": os.cpu_count(), "kind": "oracle",
                             "sample": f"per step a stratified sample of {max(4, args.cpu_sample // max(1, args.steps))} "

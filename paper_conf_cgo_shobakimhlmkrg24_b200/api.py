@@ -161,10 +161,11 @@ class Scheduler:
         return self
 
     # ---------------------------------------------------------------- shared colony
-    def colony_begin(self, p: Params, ant_base: int, stream: Optional[torch.cuda.Stream] = None):
+    def colony_begin(self, p: Params, ant_base: int, stream: Optional[torch.cuda.Stream] = None,
+                     timing: bool = False):
         """Plan a shared-colony run: this context builds ants [ant_base, ant_base + p.ants)."""
         need = C.c_size_t(0)
-        ps = params_struct(p, 0)
+        ps = params_struct(p, _lib.ACO_FLAG_TIMING if timing else 0)
         _lib.check(self.lib.aco_colony_begin(self.ctx, C.byref(ps), ant_base, None, 0, C.byref(need), None),
                    "aco_colony_begin(size)")
         if self.ws is None or self.ws.numel() < need.value:
@@ -187,11 +188,11 @@ class Scheduler:
     def colony_end(self, stream: Optional[torch.cuda.Stream] = None):
         _lib.check(self.lib.aco_colony_end(self.ctx, _stream_handle(stream)), "aco_colony_end")
 
-    def run_colony(self, p: Params, rank: int, world: int, group=None):
+    def run_colony(self, p: Params, rank: int, world: int, group=None, timing: bool = False):
         """Shared colony over torch.distributed (NCCL): p.ants per rank, global
         ants = p.ants * world; one int64 MIN allreduce per region per iteration."""
         import torch.distributed as dist
-        keys = self.colony_begin(p, rank * p.ants)
+        keys = self.colony_begin(p, rank * p.ants, timing=timing)
         pmask = 2 if p.passes == 4 else p.passes  # pass 4 runs on the pass-2 machinery (R41)
         for pass_ in (1, 2):
             if not (pmask & pass_):

@@ -299,6 +299,18 @@ def c3_sizes(count: int, base_seed: int = 3) -> np.ndarray:
     return np.where(bucket == 0, small, np.where(bucket == 1, mid, big)).astype(np.int64)
 
 
+def c5_sizes(count: int, base_seed: int = 5) -> np.ndarray:
+    """Region sizes for the full-suite sweep (config 5): the config-3 mix
+    (85 %) plus a heavy tail log-uniform in [500, 4000] (15 %) -- Table 1
+    reports regions up to 1,176 / 2,223 instructions (L240-L241); the sweep
+    extends to ~4,000 (BASELINE.json)."""
+    rng = np.random.default_rng(np.uint64(base_seed) + np.uint64(17))
+    base = c3_sizes(count, base_seed)
+    tail = np.floor(np.exp(rng.uniform(np.log(500), np.log(4001), size=count))).astype(np.int64)
+    pick = rng.random(count) < 0.15
+    return np.where(pick, np.clip(tail, 500, 4000), base).astype(np.int64)
+
+
 def gen_batch(count: int, base_seed: int = 3, profile: str = "mixed", first_id: int = 0,
               sizes: Optional[np.ndarray] = None) -> List[Region]:
     """Regions first_id .. first_id+count-1 of the config-3 batch."""

@@ -1,0 +1,18 @@
+# Bench lines for every config and SURVEY 8(f) mode (run under gpurun, 1 GPU).
+# Each JSON line goes to gpurun_out/bench_<name>.json.
+python paper_conf_cgo_shobakimhlmkrg24_b200/build.py
+run() {  # name, args...
+  name=$1; shift
+  timeout 900 python bench.py --steps 3 --warmup 3 "$@" 2>gpurun_out/bench_$name.err | tail -1 > gpurun_out/bench_$name.json
+  echo "== $name: $(cut -c1-160 gpurun_out/bench_$name.json)"
+}
+for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix}; do
+  case $w in
+    c1|c2|c3|c4|c5) run $w --workload $w ;;
+    dual) run c3_dual --machine dual ;;
+    weighted) run c3_weighted --passes 4 --ws-weight 4 ;;
+    policy) run c3_paper_policy --policy paper ;;
+    mix) run c3_heur_mix --heur-mix 1 ;;
+    stall50) run c3_stall50 --stall-num 2 ;;
+  esac
+done
