@@ -14,6 +14,7 @@ if os.environ.get("ACO_LIB_VARIANT"):  # A/B builds of the same sources (tools/,
     LIB_PATH = os.path.join(HERE, f"libaco_b200_{os.environ['ACO_LIB_VARIANT']}.so")
 
 ACO_OK = 0
+ACO_E_WORKSPACE = -6
 ACO_FLAG_NO_PRUNE = 1
 ACO_FLAG_DUMP = 2
 ACO_FLAG_TIMING = 4

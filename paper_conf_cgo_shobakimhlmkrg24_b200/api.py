@@ -105,12 +105,18 @@ class Scheduler:
         b = batch if batch is not None else HostBatch(regions, region_ids)
         need = C.c_size_t(0)
         sh = _stream_handle(stream)
-        _lib.check(self.lib.aco_load_regions(self.ctx, b.descs, len(regions), None, 0, C.byref(need), sh),
-                   "aco_load_regions(size)")
-        if self.arena is None or self.arena.numel() < need.value:
+        st = _lib.ACO_E_WORKSPACE
+        if self.arena is not None:  # one preprocessing pass when the arena is already large enough
+            st = self.lib.aco_load_regions(self.ctx, b.descs, len(regions), C.c_void_p(self.arena.data_ptr()),
+                                           self.arena.numel(), C.byref(need), sh)
+        if st == _lib.ACO_E_WORKSPACE:
+            if need.value == 0:
+                _lib.check(self.lib.aco_load_regions(self.ctx, b.descs, len(regions), None, 0, C.byref(need), sh),
+                           "aco_load_regions(size)")
             self.arena = torch.empty(max(256, need.value), dtype=torch.uint8, device=f"cuda:{self.device}")
-        _lib.check(self.lib.aco_load_regions(self.ctx, b.descs, len(regions), C.c_void_p(self.arena.data_ptr()),
-                                             self.arena.numel(), C.byref(need), sh), "aco_load_regions")
+            st = self.lib.aco_load_regions(self.ctx, b.descs, len(regions), C.c_void_p(self.arena.data_ptr()),
+                                           self.arena.numel(), C.byref(need), sh)
+        _lib.check(st, "aco_load_regions")
         self.batch = b
         self.count = len(regions)
         return self

@@ -13,7 +13,7 @@ HEADERS = [os.path.join(CSRC, "aco_internal.h"),
            os.path.join(os.path.dirname(HERE), "include", "aco.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
-         "-Xcompiler", "-fPIC", "-shared"]
+         "-Xcompiler", "-fPIC", "-Xcompiler", "-pthread", "-shared"]
 
 
 def stale() -> bool:

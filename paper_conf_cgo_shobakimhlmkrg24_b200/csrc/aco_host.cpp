@@ -6,11 +6,13 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <map>
 #include <new>
+#include <thread>
 #include <tuple>
 #include <vector>
 
@@ -526,11 +528,27 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
     for (uint32_t i = 1; i < count; ++i)
       if (ids[i] == ids[i - 1]) return ACO_E_ARG;
   }
+  // host preprocessing of the regions in parallel (independent per region)
   std::vector<Prepped> P(count);
-  for (uint32_t i = 0; i < count; ++i) {
-    aco_status st = prep_region(regions[i], ctx->mach, P[i]);
-    if (st != ACO_OK) return st;
+  std::vector<aco_status> stv(count, ACO_OK);
+  {
+    const uint32_t hw = std::max(1u, std::thread::hardware_concurrency());
+    const uint32_t nt = std::min<uint32_t>(hw, std::max<uint32_t>(1, count / 16));
+    std::atomic<uint32_t> next(0);
+    auto work = [&]() {
+      for (;;) {
+        const uint32_t i = next.fetch_add(1);
+        if (i >= count) break;
+        stv[i] = prep_region(regions[i], ctx->mach, P[i]);
+      }
+    };
+    std::vector<std::thread> th;
+    for (uint32_t t = 1; t < nt; ++t) th.emplace_back(work);
+    work();
+    for (auto &t : th) t.join();
   }
+  for (uint32_t i = 0; i < count; ++i)
+    if (stv[i] != ACO_OK) return stv[i];
   std::vector<unsigned char> blob(align16(sizeof(RegionDev) * (size_t)count + 16), 0);
   for (uint32_t i = 0; i < count; ++i) {
     RegionDev &R = P[i].rd;
@@ -745,7 +763,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       if (fs > kSmemPerSM - 2048) gs[r] = 1;  // replay scratch in the workspace too
       scratch_words[r] = std::max(scratch_words[r], need_words);
       if (!gs[r]) {
-        P.fin_smem[pass] = std::max(P.fin_smem[pass], fs);
+        P.fin_smem[pass] = std::max(P.fin_smem[pass], 4 * need_words + 64);  // replay state only (k_select)
         if (pass == 1) P.init_smem = std::max(P.init_smem, fs);
       }
     }
