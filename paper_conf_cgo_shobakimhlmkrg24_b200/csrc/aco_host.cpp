@@ -606,6 +606,7 @@ namespace {
 struct Shape {
   uint32_t apb, lanes, smem;
   bool ts;
+  uint32_t resident = 0;  // resident threads per SM of this shape
 };
 
 // Shared memory per SM and per-block reservation (sm_100: 228 KB per SM,
@@ -650,7 +651,7 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
                                (ants << 12) | (uint64_t)(4095 - k);
         if (score > best_score) {
           best_score = score;
-          best = Shape{apb, L, smem_for_k(k), ts != 0};
+          best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads};
         }
       }
     }
@@ -699,6 +700,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
   uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
+  uint32_t gs_min_threads[2] = {128, 64};  // measured: tools/probe_sizes.sh
+  if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
   // registers of the construct kernels bound the resident threads per SM
   static uint32_t s_mt[16][2][2];
@@ -735,6 +738,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
                             p->group_size, coin_words(pass, R.n));
       bool g = false;
+      // Huge regions whose image + state leave fewer than gs_min_threads
+      // resident per SM are latency-starved in shared memory: the
+      // global-state kernels (all ants resident, state through L1/L2) win
+      // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
+      if (sh.apb != 0 && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
       if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
         sh = Shape{64, 4, 0, false};
         g = true;
