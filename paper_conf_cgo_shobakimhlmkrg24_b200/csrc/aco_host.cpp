@@ -701,6 +701,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
   uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
   uint32_t gs_min_threads[2] = {128, 64};  // measured: tools/probe_sizes.sh
+  uint32_t gs_lanes[2] = {16, 16};
+  if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
   // registers of the construct kernels bound the resident threads per SM
@@ -744,7 +746,16 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
       if (sh.apb != 0 && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
       if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
-        sh = Shape{64, 4, 0, false};
+        // all ants are resident (state in the workspace); 16 lanes per ant
+        // and 512-thread blocks measured best (tools/probe_gs_lanes.sh:
+        // n = 2000, 8192 ants: 4 lanes x 64 ants 206 + 53 ms -> 45 + 34 ms
+        // per 2 iterations), fewer ants per block when A is small
+        uint32_t gl = gs_lanes[pass - 1];
+        if (pass == 2 && (t32 || P.nc4)) gl = 4;  // the u16/u32-cycle GS variants have 4 lanes
+        uint32_t gapb = std::min(kMaxBlockThreads / gl, std::max(8u, (A / 148) & ~7u));
+        if (const char *e = getenv("ACO_GS_APB")) gapb = (uint32_t)atoi(e);
+        while (gapb * gl > kMaxBlockThreads) gapb /= 2;
+        sh = Shape{gapb, gl, 0, false};
         g = true;
         gs[r] = 1;
         gs_words[r] = std::max(gs_words[r], W);

@@ -1405,6 +1405,7 @@ using ConstructFn = void (*)(KArgs, const BlockItem *, uint32_t);
 __host__ __device__ constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4,
                                                      bool gs, bool wd) {
   return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
+         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) |
          ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((uint32_t)gs << 1) | (uint32_t)wd;
 }
 
@@ -1447,12 +1448,16 @@ static void for_each_construct(F &&f) {
   // huge regions: per-ant state in the workspace, 4 lanes per ant
   reg1<1, 4, false, false, false, false, true, false>(f);
   reg1<2, 4, false, false, false, false, true, false>(f);
+  reg1<1, 8, false, false, false, false, true, false>(f);
+  reg1<2, 8, false, false, false, false, true, false>(f);
+  reg1<1, 16, false, false, false, false, true, false>(f);
+  reg1<2, 16, false, false, false, false, true, false>(f);
   reg1<2, 4, false, false, true, false, true, false>(f);
   reg1<2, 4, false, false, false, true, true, false>(f);
   reg1<2, 4, false, false, true, true, true, false>(f);
 }
 
-static ConstructFn g_construct[512];
+static ConstructFn g_construct[2048];
 static bool g_table_ready = false;
 static void build_table() {
   if (g_table_ready) return;
@@ -1478,7 +1483,7 @@ int construct_max_threads(int device, uint32_t out[2][2]) {
       ok = false;
       return;
     }
-    const uint32_t p = code >> 8, w = code & 1u;
+    const uint32_t p = (code >> 8) & 1u, w = code & 1u;
     regs[p][w] = std::max(regs[p][w], (uint32_t)fa.numRegs);
   });
   if (!ok) {
@@ -1549,7 +1554,7 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
   build_table();
   const bool mask = c.max_n <= 1024 && !c.gs;
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
-  const uint32_t lg = c.gs ? 4u : c.lanes;
+  const uint32_t lg = c.lanes;
   const uint32_t code = variant_code(pass, lg, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32,
                                      pass == 2 && c.nc4, c.gs, c.wide && mask);
   const ConstructFn f = g_construct[code];
