@@ -26,7 +26,7 @@ struct Plan {
   uint32_t fin_smem[3] = {0, 0, 0};
   uint32_t init_smem = 0, p2_smem = 0, max_n = 0, n_upd = 0;
   uint32_t pass_mask = 0, iterations = 0;
-  bool any_t32 = false, nc4 = false, timing = false, p2_done = false;
+  bool any_t32 = false, nc4 = false, timing = false, p2_done = false, stage_img = false;
   uint64_t o_state = 0, o_rws = 0, o_upd = 0, o_gb2 = 0, o_gb2c = 0, o_keys = 0;
   LaunchCtx L{};
 };
@@ -773,18 +773,32 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     }
     P.p2_smem = std::max(P.p2_smem, 4 * R.n + 16);  // also k_post
   }
+  // Replay (k_select) and greedy (k_init): one warp per region.  With many
+  // regions the image is read through L1 and only the replay state is in
+  // shared memory (many replays resident per SM); with few regions (a huge
+  // region, config 4) the image is staged too (latency-bound serial replay).
+  // Regions whose image + replay state exceed shared memory use the workspace.
+  P.stage_img = count <= 2 * 148;
+  std::vector<uint8_t> sgs(count, 0);
   for (uint32_t r = 0; r < count; ++r) {
     const RegionDev &R = ctx->regions[r];
     for (uint32_t pass = 1; pass <= 2; ++pass) {
       const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && P.any_t32, P.nc4);
       const uint32_t need_words = W + R.n + (R.n + 1) / 2 + 4;  // state + cycles + order
       const uint32_t fs = R.img.bytes + 4 * need_words + 64;
-      if (fs > kSmemPerSM - 2048) gs[r] = 1;  // replay scratch in the workspace too
+      if (fs > kSmemPerSM - 2048) sgs[r] = 1;  // replay scratch in the workspace too
       scratch_words[r] = std::max(scratch_words[r], need_words);
-      if (!gs[r]) {
-        P.fin_smem[pass] = std::max(P.fin_smem[pass], 4 * need_words + 64);  // replay state only (k_select)
-        if (pass == 1) P.init_smem = std::max(P.init_smem, fs);
-      }
+    }
+  }
+  for (uint32_t r = 0; r < count; ++r) {
+    const RegionDev &R = ctx->regions[r];
+    if (sgs[r]) continue;
+    for (uint32_t pass = 1; pass <= 2; ++pass) {
+      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && P.any_t32, P.nc4);
+      const uint32_t need_words = W + R.n + (R.n + 1) / 2 + 4;
+      const uint32_t fs = R.img.bytes + 4 * need_words + 64;
+      P.fin_smem[pass] = std::max(P.fin_smem[pass], P.stage_img ? fs : 4 * need_words + 64);
+      if (pass == 1) P.init_smem = std::max(P.init_smem, fs);
     }
   }
   // ---- workspace layout
@@ -838,11 +852,13 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     w.o_dump = (uint64_t)A * ctx->inst_off[r];
     w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
     w.o_heur = o_heur + 2 * ctx->inst_off[r];
-    w.gs = gs[r];
-    if (gs[r]) {
+    w.gs = sgs[r];  // k_init / k_select: image and replay state in the workspace
+    if (gs[r]) {  // global-state construct kernels
       off = align256(off);
       w.o_gstate = off;
       off += 4ull * A * gs_words[r];
+    }
+    if (sgs[r]) {
       off = align256(off);
       w.o_scratch = off;
       off = align256(off + 4ull * scratch_words[r]);
@@ -966,6 +982,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.revert_len = p->revert_len;
   cfg.heur_mix = p->heur_mix;
   cfg.stall_num = p->stall_num;
+  cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;
   cfg.keys = nullptr;
   L.stream = cuda_stream;

@@ -133,6 +133,8 @@ struct RunCfg {
   uint32_t ws_weight;
   uint32_t pass2_gap, revert_occ, revert_len;  // compile policy (R39, R40)
   uint32_t heur_mix, stall_num;                // R43, R44
+  uint32_t stage_img;   // k_select stages the region image in shared memory (few regions)
+  uint32_t pad_cfg;
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
   int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };

@@ -1247,10 +1247,18 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
   const unsigned char *img = A.arena + rd->o_image;
   uint32_t *stw = (uint32_t *)(A.ws + W.o_scratch);
   if (!GS) {
-    // the replay is one warp per region: the image is read through L1 (no
-    // per-block staging), only the replay state lives in shared memory, so
-    // many regions' replays are resident per SM
-    stw = (uint32_t *)smem;
+    // the replay is one warp per region: with many regions the image is read
+    // through L1 (no per-block staging) and only the replay state lives in
+    // shared memory, so many replays are resident per SM; with few regions
+    // the image is staged as well (latency-bound serial replay)
+    if (A.cfg.stage_img) {
+      stage((uint4 *)smem, (const uint4 *)img, rd->img.bytes);
+      img = smem;
+      stw = (uint32_t *)(smem + rd->img.bytes);
+      __syncwarp();
+    } else {
+      stw = (uint32_t *)smem;
+    }
   }
   unsigned long long best = ~0ull;
   if (A.cfg.keys) {
