@@ -752,7 +752,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         // per 2 iterations), fewer ants per block when A is small
         uint32_t gl = gs_lanes[pass - 1];
         if (pass == 2 && (t32 || P.nc4)) gl = 4;  // the u16/u32-cycle GS variants have 4 lanes
-        uint32_t gapb = std::min(kMaxBlockThreads / gl, std::max(8u, (A / 148) & ~7u));
+        uint32_t gapb = std::min<uint64_t>(kMaxBlockThreads / gl, std::max<uint64_t>(8u, ((uint64_t)A * count / 148) & ~7ull));
         if (const char *e = getenv("ACO_GS_APB")) gapb = (uint32_t)atoi(e);
         while (gapb * gl > kMaxBlockThreads) gapb /= 2;
         sh = Shape{gapb, gl, 0, false};

@@ -1124,7 +1124,9 @@ template <bool MASK>
 __global__ void __launch_bounds__(128) k_init(KArgs A) {
   extern __shared__ uint4 smem4[];
   if (A.rws[blockIdx.x].gs) init_body<false, true>(A, (unsigned char *)smem4);
-  else init_body<MASK, false>(A, (unsigned char *)smem4);
+  else if (A.regions[blockIdx.x].n <= 1024) init_body<true, false>(A, (unsigned char *)smem4);
+  else init_body<false, false>(A, (unsigned char *)smem4);
+  (void)MASK;
 }
 
 // ASAP timing of an order (R29) on the general machine model (R42): in-order
@@ -1350,10 +1352,14 @@ __global__ void __launch_bounds__(32) k_select(KArgs A, uint32_t iter) {
   if (A.rws[blockIdx.x].gs) {
     if (ct) select_body<PASS, false, false, false, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
     else select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+  } else if (A.regions[blockIdx.x].n <= 1024) {  // word-mask scan per region (MASK: n <= 1024)
+    if (ct) select_body<PASS, true, false, false, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    else select_body<PASS, true, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
   } else {
-    if (ct) select_body<PASS, MASK, false, false, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
-    else select_body<PASS, MASK, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    if (ct) select_body<PASS, false, false, false, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    else select_body<PASS, false, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
   }
+  (void)MASK;
 }
 
 // Shared colony: per-region local argmin over this context's ants, written as
