@@ -607,6 +607,7 @@ struct Shape {
   uint32_t apb, lanes, smem;
   bool ts;
   uint32_t resident = 0;  // resident threads per SM of this shape
+  bool ig = false;        // image read through L1 instead of staged in shared memory
 };
 
 // Shared memory per SM and per-block reservation (sm_100: 228 KB per SM,
@@ -625,19 +626,25 @@ uint32_t smem_for_k(uint32_t k) { return std::min(kSmemPerSM, (kSmemSM / k - kBl
 // fewer lanes per ant (less reduction overhead), then tau in shared memory,
 // then more resident USEFUL ants (A ants of a region fill ceil(A/apb) blocks),
 // then fewer blocks (one image copy per block).
+// allow_ig: the image may instead be read through L1 (large regions; wide
+// variants), which frees its shared memory for more resident ants; ranked
+// after everything else, so it is taken only when it adds resident threads.
 Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
-                 uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w) {
-  Shape best{0, 1, 0, false};
+                 uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w,
+                 bool allow_ig = false) {
+  Shape bests[2] = {Shape{0, 1, 0, false}, Shape{0, 1, 0, false}};
+  for (int ig = 0; ig <= (allow_ig ? 1 : 0); ++ig) {
+  Shape &best = bests[ig];
   uint64_t best_score = 0;
   for (int ts = 1; ts >= 0; --ts) {
-    if (ts && !allow_ts) continue;
+    if (ts && (!allow_ts || ig)) continue;  // the image-through-L1 variants keep tau in global memory
     for (uint32_t L : {1u, 2u, 4u, 8u}) {
       if (lanes14 && L != 1 && L != 4) continue;
       if (L > max_lanes) continue;
       for (uint32_t threads : {32u, 64u, 96u, 128u, 192u, 256u, 384u, 512u}) {
         if (threads > kMaxBlockThreads) break;
         const uint32_t apb = threads / L;
-        const uint64_t bytes = (uint64_t)img + (ts ? tb : 0u) + (uint64_t)ant_stride(apb, L) * W * 4 +
+        const uint64_t bytes = (uint64_t)(ig ? 0u : img) + (ts ? tb : 0u) + (uint64_t)ant_stride(apb, L) * W * 4 +
                                (uint64_t)coin_groups(apb, gsz) * coin_w * 4;
         if (bytes > kSmemPerSM) break;
         uint32_t k = kSmemSM / ((uint32_t)bytes + kBlockReserve);
@@ -649,14 +656,18 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
         const uint64_t ants = std::min<uint64_t>((uint64_t)k * std::max(1u, A) / ((std::max(1u, A) + apb - 1) / apb), 4095);
         const uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) |
                                (ants << 12) | (uint64_t)(4095 - k);
-        if (score > best_score) {
+        if (score > best_score) {  // strict: the staged image wins ties
           best_score = score;
-          best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads};
+          best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads, ig != 0};
         }
       }
     }
   }
-  return best;
+  }
+  // Reading the image through L1 costs ~15 % per ant-step (measured, n = 300
+  // and 450 pass 2); it pays only with >= 20 % more resident ants.
+  if (bests[1].apb && (!bests[0].apb || 5ull * bests[1].resident >= 6ull * bests[0].resident)) return bests[1];
+  return bests[0];
 }
 
 }  // namespace
@@ -692,7 +703,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     uint32_t smem;
     std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t, bool>;
+  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t, bool, bool>;
   std::map<Key, Cls> classes;
   P.nc4 = ctx->mach.n_classes > 2;
   // launch-shape policy (tuning knobs; defaults measured on B200)
@@ -702,6 +713,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
   uint32_t gs_min_threads[2] = {128, 64};  // measured: tools/probe_sizes.sh
   uint32_t gs_lanes[2] = {16, 16};
+  uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
+  if (const char *e = getenv("ACO_IMG_L1")) sscanf(e, "%u,%u", &img_l1[0], &img_l1[1]);
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
@@ -738,7 +751,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       const bool wide = R.n >= kWideN && R.n <= 1024;
       Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
-                            p->group_size, coin_words(pass, R.n));
+                            p->group_size, coin_words(pass, R.n), wide && !rare && img_l1[pass - 1]);
       bool g = false;
       // Huge regions whose image + state leave fewer than gs_min_threads
       // resident per SM are latency-starved in shared memory: the
@@ -761,7 +774,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         gs_words[r] = std::max(gs_words[r], W);
       }
       const bool mask = R.n <= 1024 && !g;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask);
+      if (g) sh.ig = false;
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask, sh.ig);
       Cls &c = classes[key];
       c.wide = wide && mask;
       c.sh = sh;
@@ -917,6 +931,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       cl.nc4 = P.nc4;
       cl.gs = c.gs;
       cl.wide = c.wide;
+      cl.img_l1 = c.sh.ig;
       P.launches[std::get<0>(kv.first)].push_back(cl);
       class_work[std::get<0>(kv.first)].push_back(0);
       for (auto &pr : c.regs) class_work[std::get<0>(kv.first)].back() += ~pr.first;
@@ -933,9 +948,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       for (size_t i = 0; i < idx.size(); ++i)
         fprintf(stderr,
                 "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d gs %d "
-                "wide %d work %.3g\n",
+                "wide %d img_l1 %d work %.3g\n",
                 pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes,
                 (int)sorted[i].tau_smem, (int)sorted[i].t32, (int)sorted[i].gs, (int)sorted[i].wide,
+                (int)sorted[i].img_l1,
                 (double)class_work[pass][idx[i]]);
   }
   if (plan_only) {

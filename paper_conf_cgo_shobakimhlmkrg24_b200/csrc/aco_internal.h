@@ -229,6 +229,7 @@ struct ClassLaunch {
   bool nc4;                // 3-4 register classes (u16 last-use counts)
   bool gs;                 // per-ant state in global memory (huge regions)
   bool wide;               // 4-wide candidate scan (n >= kWideN, word-mask variant)
+  bool img_l1 = false;     // the block image is read through L1 (not staged): more ants per SM
 };
 
 int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success

@@ -924,7 +924,11 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
 // Launch bounds: the 1-wide variants keep <= 64 registers (2 x 512 threads per
 // SM); the 4-wide ones (large regions, few ants per SM by shared memory) may
 // use up to 128.
-template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, bool GS, bool WIDE>
+// GS: 0 = image and per-ant state in shared memory; 1 = huge region, both
+// through L1/L2 (state in the workspace); 2 = image read through L1 (it is
+// small next to the state of large regions), per-ant state (and tau when
+// staged) in shared memory: more ants resident per SM.
+template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS, bool WIDE>
 __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
@@ -943,13 +947,13 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
   uint32_t stride;
   const uint32_t *coins = nullptr;
   uint32_t coin_t = 0;
-  if (GS) {  // huge region: statics through L1/L2, per-ant state in the workspace
+  if (GS == 1) {  // huge region: statics through L1/L2, per-ant state in the workspace
     if (ai >= A.cfg.ants) return;
     stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
     stride = A.cfg.ants;
   } else {
-    const uint32_t img_bytes = rd->img.bytes;
-    stage(smem4, (const uint4 *)img, img_bytes);
+    const uint32_t img_bytes = GS == 0 ? rd->img.bytes : 0u;
+    if (GS == 0) stage(smem4, (const uint4 *)img, img_bytes);
     uint32_t state_off = img_bytes;
     if (TAU_SMEM) {
       const uint32_t tb = tau_smem_bytes(rd->n);
@@ -978,7 +982,7 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
     }
     __syncthreads();
     if (ai >= A.cfg.ants) return;  // whole lane group
-    img = smem;
+    if (GS == 0) img = smem;
     stbase = (uint32_t *)(smem + state_off) + local;
   }
   const Grp<LG> G(threadIdx.x);
@@ -1417,13 +1421,13 @@ int last_cuda_error() { return check(); }
 using ConstructFn = void (*)(KArgs, const BlockItem *, uint32_t);
 
 __host__ __device__ constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4,
-                                                     bool gs, bool wd) {
+                                                     int gs, bool wd) {
   return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
-         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) |
-         ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((uint32_t)gs << 1) | (uint32_t)wd;
+         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) | ((gs == 2 ? 1u : 0u) << 11) |
+         ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((gs == 1 ? 1u : 0u) << 1) | (uint32_t)wd;
 }
 
-template <int P, int LG, bool M, bool TS, bool T3, bool N4, bool GS, bool WD, typename F>
+template <int P, int LG, bool M, bool TS, bool T3, bool N4, int GS, bool WD, typename F>
 static void reg1(F &f) {
   f(&k_construct<P, LG, M, TS, T3, N4, GS, WD>, variant_code(P, LG, M, TS, T3, N4, GS, WD));
 }
@@ -1434,6 +1438,8 @@ static void reg_w(F &f) {  // the 4-wide scan exists only with the word mask (n 
 }
 template <int LG, typename F>
 static void reg_lg(F &f) {
+  reg1<1, LG, true, false, false, false, 2, true>(f);  // large regions, image through L1
+  reg1<2, LG, true, false, false, false, 2, true>(f);
   reg_w<1, LG, true, true, false, false>(f);
   reg_w<1, LG, true, false, false, false>(f);
   reg_w<1, LG, false, true, false, false>(f);
@@ -1460,18 +1466,18 @@ static void for_each_construct(F &&f) {
   reg_rare<4, true>(f);
   reg_rare<4, false>(f);
   // huge regions: per-ant state in the workspace, 4 lanes per ant
-  reg1<1, 4, false, false, false, false, true, false>(f);
-  reg1<2, 4, false, false, false, false, true, false>(f);
-  reg1<1, 8, false, false, false, false, true, false>(f);
-  reg1<2, 8, false, false, false, false, true, false>(f);
-  reg1<1, 16, false, false, false, false, true, false>(f);
-  reg1<2, 16, false, false, false, false, true, false>(f);
-  reg1<2, 4, false, false, true, false, true, false>(f);
-  reg1<2, 4, false, false, false, true, true, false>(f);
-  reg1<2, 4, false, false, true, true, true, false>(f);
+  reg1<1, 4, false, false, false, false, 1, false>(f);
+  reg1<2, 4, false, false, false, false, 1, false>(f);
+  reg1<1, 8, false, false, false, false, 1, false>(f);
+  reg1<2, 8, false, false, false, false, 1, false>(f);
+  reg1<1, 16, false, false, false, false, 1, false>(f);
+  reg1<2, 16, false, false, false, false, 1, false>(f);
+  reg1<2, 4, false, false, true, false, 1, false>(f);
+  reg1<2, 4, false, false, false, true, 1, false>(f);
+  reg1<2, 4, false, false, true, true, 1, false>(f);
 }
 
-static ConstructFn g_construct[2048];
+static ConstructFn g_construct[4096];
 static bool g_table_ready = false;
 static void build_table() {
   if (g_table_ready) return;
@@ -1570,7 +1576,7 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   const uint32_t lg = c.lanes;
   const uint32_t code = variant_code(pass, lg, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32,
-                                     pass == 2 && c.nc4, c.gs, c.wide && mask);
+                                     pass == 2 && c.nc4, c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask);
   const ConstructFn f = g_construct[code];
   if (!f) return (int)cudaErrorInvalidDeviceFunction;
   f<<<c.n_blocks, c.ants_pb * lg, c.smem_bytes, (cudaStream_t)L.stream>>>(kargs(L), c.items, iter);
