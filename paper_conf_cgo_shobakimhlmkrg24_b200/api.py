@@ -197,7 +197,7 @@ class Scheduler:
     def run_colony(self, p: Params, rank: int, world: int, group=None, timing: bool = False):
         """Shared colony over torch.distributed (NCCL): p.ants per rank, global
         ants = p.ants * world; one int64 MIN allreduce per region per iteration."""
-        import torch.distributed as dist
+        from .sharding import colony_allreduce
         keys = self.colony_begin(p, rank * p.ants, timing=timing)
         pmask = 2 if p.passes == 4 else p.passes  # pass 4 runs on the pass-2 machinery (R41)
         for pass_ in (1, 2):
@@ -206,7 +206,7 @@ class Scheduler:
             for it in range(p.iterations):
                 self.colony_construct(pass_, it)
                 if world > 1:
-                    dist.all_reduce(keys, op=dist.ReduceOp.MIN, group=group)
+                    colony_allreduce(keys, group)
                 self.colony_finalize(pass_, it)
         self.colony_end()
         return self

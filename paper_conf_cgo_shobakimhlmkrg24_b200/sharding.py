@@ -53,3 +53,42 @@ def gather_results(local: Dict[int, dict], world: int, rank: int, group=None) ->
             assert k not in out, f"region {k} scheduled twice"
             out[k] = v
     return out
+
+
+# ---------------------------------------------------------------- shared colony (config 4)
+# The only data-path exchange of the shared colony: per
+# region and iteration every rank contributes ONE int64, its local best ant's
+# key, and a MIN all-reduce picks the global iteration winner.  The key is
+# (cost << 32 | global ant) XOR 2^63 (csrc/aco_internal.h kKeyBias), so a
+# signed int64 MIN orders keys like the unsigned (cost, ant) pair: lowest
+# cost, ties to the lowest ant id (R10); an invalid ant has cost 0xFFFFFFFF
+# (R35).  The kernels build these keys on the device (k_local_keys); the
+# helpers below are the host-side statement of the encoding.
+KEY_BIAS = 1 << 63
+INVALID_COST = 0xFFFFFFFF
+
+
+def colony_key(cost: int, ant: int) -> int:
+    """Biased winner key as a signed int64 value."""
+    u = ((int(cost) << 32) | int(ant)) ^ KEY_BIAS
+    return u - (1 << 64) if u >= (1 << 63) else u
+
+
+def colony_decode(key: int):
+    """(cost, global ant) of a biased key."""
+    u = (int(key) + (1 << 64)) % (1 << 64) ^ KEY_BIAS
+    return u >> 32, u & 0xFFFFFFFF
+
+
+def local_best_key(costs: Sequence[int], ant_base: int) -> int:
+    """The key of this rank's best ant: lexicographic (cost, ant) minimum."""
+    best = min(range(len(costs)), key=lambda a: (int(costs[a]), a))
+    return colony_key(int(costs[best]), ant_base + best)
+
+
+def colony_allreduce(keys, group=None):
+    """MIN all-reduce of a per-region int64 key tensor, in place (the shared
+    colony's exchange; NCCL on the GPU path, any backend here)."""
+    import torch.distributed as dist
+    dist.all_reduce(keys, op=dist.ReduceOp.MIN, group=group)
+    return keys
