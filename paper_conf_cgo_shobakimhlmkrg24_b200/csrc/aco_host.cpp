@@ -353,7 +353,12 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
     ds[4 * j + 1] = info[(size_t)j * 4 + 1];
   }
   for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j];
-  for (uint32_t j = 0; j < n; ++j) ds[4 * j + 3] = d.inst_type ? d.inst_type[j] : 0u;  // issue type (R42)
+  // ds.w = issue type (R42, bits 0-3) | multi-use register count << 4 |
+  // their start in the multi-use list << 8 (the lean pass-2 layout derives
+  // the dynamic kills from them)
+  for (uint32_t j = 0; j < n; ++j)
+    ds[4 * j + 3] = (d.inst_type ? d.inst_type[j] : 0u) | ((info[(size_t)j * 4 + 3] & 0xFFu) << 4) |
+                    (info[(size_t)j * 4 + 3] & ~0xFFu);
   // users of each counter register (to find the last remaining user)
   std::vector<uint32_t> cu_ptr(nctr + 1, 0), cu;
   for (uint32_t g = 0; g < G; ++g)
@@ -699,11 +704,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // ---- per-pass construct classes
   struct Cls {
     Shape sh;
-    bool mask, t32, gs, wide = false;
+    bool mask, t32, gs, wide = false, lean = false;
     uint32_t smem;
     std::vector<std::pair<uint64_t, uint32_t>> regs;  // (~work, region)
   };
-  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t, bool, bool>;
+  using Key = std::tuple<uint32_t, uint32_t, uint32_t, bool, bool, bool, bool, uint32_t, bool, bool, bool>;
   std::map<Key, Cls> classes;
   P.nc4 = ctx->mach.n_classes > 2;
   // launch-shape policy (tuning knobs; defaults measured on B200)
@@ -715,13 +720,17 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t gs_lanes[2] = {16, 16};
   uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
   if (const char *e = getenv("ACO_IMG_L1")) sscanf(e, "%u,%u", &img_l1[0], &img_l1[1]);
+  bool lean_on = true;  // pass-2 lean layout for large regions
+  if (const char *e = getenv("ACO_LEAN")) lean_on = atoi(e) != 0;
+  uint32_t lean_gain = 0;  // % more resident ants the lean layout must reach (C3: 0 measured best)
+  if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
   // registers of the construct kernels bound the resident threads per SM
-  static uint32_t s_mt[16][2][2];
+  static uint32_t s_mt[16][2][3];
   static bool s_mt_ok[16];
-  uint32_t mt[2][2];
+  uint32_t mt[2][3];
   {
     const int dv = ctx->device >= 0 && ctx->device < 16 ? ctx->device : 0;
     if (!s_mt_ok[dv]) s_mt_ok[dv] = construct_max_threads(ctx->device, s_mt[dv]) == 0;
@@ -742,16 +751,34 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                      (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
     P.any_t32 |= t32;
     for (uint32_t pass = 1; pass <= 2; ++pass) {
-      const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
+      const bool wide = R.n >= kWideN && R.n <= 1024;
+      // lean pass-2 layout (u8 ready times, kills derived at evaluation):
+      // large regions, single issue, 2 classes, latencies < 128
+      bool lean = pass == 2 && lean_on && wide && !t32 && !P.nc4 && ctx->mach.issue_width <= 1 && R.max_lat < 128u;
+      uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);  // lean: decided below
       if (!(pmask & pass)) continue;
       if (getenv("ACO_DEBUG_REGIONS"))
         fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
                 R.nremw, R.L);
       const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
-      const bool wide = R.n >= kWideN && R.n <= 1024;
       Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
                             p->group_size, coin_words(pass, R.n), wide && !rare && img_l1[pass - 1]);
+      if (lean) {
+        // the lean layout costs per ant-step (kills derived at every
+        // evaluation) and gains resident ants; on the mixed C3 batch it wins
+        // whenever it fits at least as many ants (B200: 684 -> 645 ms/batch;
+        // ACO_LEAN_GAIN = 20 / 50 %: 654 ms)
+        const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true);
+        const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[1][2], false, false,
+                                     tgt_threads[1], 1, A, p->group_size, coin_words(pass, R.n), img_l1[1] != 0);
+        if (shl.apb && 100ull * shl.resident >= (100ull + lean_gain) * sh.resident) {
+          sh = shl;
+          W = Wl;
+        } else {
+          lean = false;
+        }
+      }
       bool g = false;
       // Huge regions whose image + state leave fewer than gs_min_threads
       // resident per SM are latency-starved in shared memory: the
@@ -771,17 +798,20 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         sh = Shape{gapb, gl, 0, false};
         g = true;
         gs[r] = 1;
+        lean = false;
+        W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
         gs_words[r] = std::max(gs_words[r], W);
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask, sh.ig);
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask, sh.ig, lean);
       Cls &c = classes[key];
       c.wide = wide && mask;
       c.sh = sh;
       c.mask = mask;
       c.t32 = pass == 2 && t32;
       c.gs = g;
+      c.lean = lean;
       c.smem = std::max(c.smem, sh.smem);
       c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
     }
@@ -932,6 +962,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       cl.gs = c.gs;
       cl.wide = c.wide;
       cl.img_l1 = c.sh.ig;
+      cl.lean = c.lean;
       P.launches[std::get<0>(kv.first)].push_back(cl);
       class_work[std::get<0>(kv.first)].push_back(0);
       for (auto &pr : c.regs) class_work[std::get<0>(kv.first)].back() += ~pr.first;
@@ -948,10 +979,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       for (size_t i = 0; i < idx.size(); ++i)
         fprintf(stderr,
                 "[aco plan] pass %d class %zu: blocks %u ants/blk %u lanes %u smem %u tau_smem %d t32 %d gs %d "
-                "wide %d img_l1 %d work %.3g\n",
+                "wide %d img_l1 %d lean %d work %.3g\n",
                 pass, i, sorted[i].n_blocks, sorted[i].ants_pb, sorted[i].lanes, sorted[i].smem_bytes,
                 (int)sorted[i].tau_smem, (int)sorted[i].t32, (int)sorted[i].gs, (int)sorted[i].wide,
-                (int)sorted[i].img_l1,
+                (int)sorted[i].img_l1, (int)sorted[i].lean,
                 (double)class_work[pass][idx[i]]);
   }
   if (plan_only) {

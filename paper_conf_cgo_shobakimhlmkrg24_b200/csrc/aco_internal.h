@@ -166,15 +166,19 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 //           per class and instruction):
 //           X  [ceil(n/2)] u16: windowed ready time (10 bits) | last-use
 //                           counts (2 classes x 3 bits) << 10
+//   pass 2, lean (large regions, latencies < 128):
+//           X8 [ceil(n/4)] u8 windowed ready time; last-use counts derived
+//                           from REM / SCH at evaluation (dyn_kills)
 //   pass 2, otherwise:
 //           T  [ceil(n/2)] u16 (or [n] u32 if t32): issue cycle (placed) or
 //                           ready time (ready instruction)
 //           DK [ceil(n/4)] u8 = 2 classes x 4 bits (or [ceil(n/2)] u16 = 4
 //                           classes x 4 bits if nc4): per-class last-use counts
 ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32_t nremw, bool t32,
-                                 bool nc4) {
+                                 bool nc4, bool lean = false) {
   const uint32_t w = 2 * nwr + nremw;
   if (pass == 1) return w + (n + 7) / 8;
+  if (lean) return w + (n + 3) / 4;  // lean: u8 windowed ready time (kills derived, not stored)
   if (!t32 && !nc4) return w + (n + 1) / 2;  // compact: u16 (windowed ready time | last uses)
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }
@@ -230,12 +234,13 @@ struct ClassLaunch {
   bool gs;                 // per-ant state in global memory (huge regions)
   bool wide;               // 4-wide candidate scan (n >= kWideN, word-mask variant)
   bool img_l1 = false;     // the block image is read through L1 (not staged): more ants per SM
+  bool lean = false;       // pass 2: lean per-ant layout (u8 ready times, dynamic kills)
 };
 
 int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success
 // Resident threads per SM that the construct kernels' registers allow, per
 // [pass-1][wide]; returns nonzero (and conservative defaults) without a device.
-int construct_max_threads(int device, uint32_t out[2][2]);
+int construct_max_threads(int device, uint32_t out[2][3]);  // [pass-1][plain, wide, lean]
 int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);

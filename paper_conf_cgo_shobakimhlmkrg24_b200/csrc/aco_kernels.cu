@@ -36,6 +36,9 @@
 #ifndef ACO_PREFETCH
 #define ACO_PREFETCH 0
 #endif
+#ifndef ACO_LEAN_LB  // launch bound of the lean pass-2 variants (caps registers: 65536 / bound per thread)
+#define ACO_LEAN_LB 512
+#endif
 #ifndef ACO_BRANCHLESS1  // pass-1 4-wide evaluation without branches (measured faster)
 #define ACO_BRANCHLESS1 1
 #endif
@@ -164,7 +167,7 @@ struct St {
   uint32_t S;
 };
 
-template <int PASS, bool T32, bool NC4>
+template <int PASS, bool T32, bool NC4, bool LEAN = false>
 __device__ __forceinline__ St make_st(uint32_t *st, uint32_t S, const SV &V) {
   St A;
   A.S = S;
@@ -255,6 +258,70 @@ __device__ __forceinline__ void x_push_rt(const St &A, uint32_t v, uint32_t rt) 
 // rt >= 512 -> rt & 0x1FF, else 0 (rt < 1024).
 __device__ __forceinline__ uint32_t x_slide2(uint32_t w) {
   return (w & 0xFC00FC00u) | (w & (((w >> 9) & 0x00010001u) * 0x1FFu));
+}
+
+// ---- pass-2 LEAN layout (large regions: more ants per SM): one u8 per
+// instruction = ready time relative to the window base B (window kWin8 = 128,
+// latencies < 128, so a stored value is <= 254), and NO stored last-use
+// counts: the dynamic kills of a candidate are derived from its multi-use
+// registers' remaining-use counters / partners' scheduled bits (dyn_kills).
+constexpr uint32_t kWin8 = 128;
+__device__ __forceinline__ uint32_t r8_get(const St &A, uint32_t j) {
+  return (A.T[(j >> 2) * A.S] >> ((j & 3u) * 8)) & 0xFFu;
+}
+__device__ __forceinline__ void r8_push(const St &A, uint32_t v, uint32_t rt) {
+  uint32_t *p = A.T + (v >> 2) * A.S;
+  *p = __vmaxu4(*p, rt << ((v & 3u) * 8));  // byte-wise max (push-style ready time)
+}
+// kills_c(j) - static kills_c(j) as packed u8 x 4: registers read by j with >= 2
+// users whose last unscheduled user j is (R14): a counter register with one
+// remaining use, or a 2-user register whose partner is scheduled.
+// dsw = ds.w of j (multi-use count << 4 | start << 8).
+__device__ __forceinline__ uint32_t dyn_kills(const SV &V, const St &A, uint32_t dsw) {
+  uint32_t K = 0;
+  const uint32_t mc = (dsw >> 4) & 0xFu, m0 = dsw >> 8;
+  for (uint32_t q = 0; q < mc; ++q) {
+    const uint32_t e = V.muse[m0 + q];
+    uint32_t last;
+    if (e & kMuseCounter) {
+      const uint32_t m = e & 0xFFFFu;
+      last = ((A.REM[(m >> 1) * A.S] >> ((m & 1u) * 16)) & 0xFFFFu) == 1u;
+    } else {
+      last = sch_bit(A, e & 0x1FFFu);
+    }
+    K += last << (8 * ((e >> 16) & 3u));
+  }
+  return K;
+}
+// dyn_kills of four candidates at once: level q of every candidate's
+// multi-use list is fetched together (two dependent shared/L1 loads per
+// level for all four, instead of four serial chains).
+__device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4 (&ds)[4], uint32_t (&dk)[4]) {
+  uint32_t mc[4], m0[4], mx = 0;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    mc[u] = (ds[u].w >> 4) & 0xFu;
+    m0[u] = ds[u].w >> 8;
+    dk[u] = 0;
+    mx = ::max(mx, mc[u]);
+  }
+  for (uint32_t q = 0; q < mx; ++q) {
+    uint32_t e[4], w[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) e[u] = q < mc[u] ? V.muse[m0[u] + q] : 0u;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {  // counter word (>= 3 users) or the partner's scheduled-set word
+      const uint32_t m = e[u] & 0xFFFFu, pa = e[u] & 0x1FFFu;
+      w[u] = (e[u] & kMuseCounter) ? A.REM[(m >> 1) * A.S] : A.SCH[(pa >> 5) * A.S];
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t m = e[u] & 0xFFFFu, pa = e[u] & 0x1FFFu;
+      const uint32_t last = (e[u] & kMuseCounter) ? (((w[u] >> ((m & 1u) * 16)) & 0xFFFFu) == 1u)
+                                                  : ((w[u] >> (pa & 31u)) & 1u);
+      dk[u] += (q < mc[u] ? last : 0u) << (8 * ((e[u] >> 16) & 3u));
+    }
+  }
 }
 
 // ---- lane groups: LG consecutive lanes of a warp build one ant together.
@@ -427,11 +494,11 @@ __device__ __forceinline__ uint32_t cost_of(uint32_t mode, uint32_t prp01, uint3
 // Commit of instruction j at cycle t (both passes): scheduled / ready sets,
 // the RP update (R14, R15), last-use bookkeeping of the registers j reads,
 // and the successors that become ready (pass 2: with their ready times).
-template <int PASS, bool MASK, bool T32, bool NC4>
+template <int PASS, bool MASK, bool T32, bool NC4, bool LEAN = false>
 __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uint32_t t, uint32_t &wmask,
                                        uint32_t &live01, uint32_t &live23, uint32_t &prp01,
                                        uint32_t &prp23, uint32_t B = 0) {
-  constexpr bool CT = PASS == 2 && !T32 && !NC4;
+  constexpr bool CT = PASS == 2 && !T32 && !NC4;  // push-style ready times (compact or lean)
   {
     const uint32_t wi = j >> 5, bit = 1u << (j & 31u);
     const uint32_t nw = A.RB[wi * A.S] & ~bit;
@@ -455,7 +522,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
         const uint32_t left = (w >> sh) & 0xFFFFu;  // users left including j
         if (left == 1u) {
           K += 1u << (8 * c);  // j is the last user: the register dies here
-        } else if (left == 2u) {  // one user remains: it becomes the last user
+        } else if (!LEAN && left == 2u) {  // one user remains: it becomes the last user
           for (uint32_t k = V.cu_ptr[m]; k < V.cu_ptr[m + 1]; ++k) {
             const uint32_t u = V.cu[k];
             if (!sch_bit(A, u)) {
@@ -467,7 +534,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
       } else {  // 2 users: the partner
         const uint32_t p = e & 0x1FFFu;
         if (sch_bit(A, p)) K += 1u << (8 * c);
-        else dk_add<PASS, T32, NC4>(A, p, c);
+        else if (!LEAN) dk_add<PASS, T32, NC4>(A, p, c);
       }
     }
   }
@@ -485,7 +552,10 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
     const uint32_t v = e & 0x1FFFu;
     bool ready = true;
     uint32_t rdy = t + (e >> 16);
-    if (CT) x_push_rt(A, v, rdy - B);  // ready time = max over placed predecessors
+    if (CT) {  // ready time = max over placed predecessors
+      if (LEAN) r8_push(A, v, rdy - B);
+      else x_push_rt(A, v, rdy - B);
+    }
     if (!(e & kSuccSingle) && (PASS == 1 || CT)) {
       // v is ready iff all its predecessors are placed: one scheduled-set
       // word per group of predecessors sharing a bitset word
@@ -517,7 +587,7 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
   }
 }
 
-template <int PASS, bool MASK, bool T32, bool NC4>
+template <int PASS, bool MASK, bool T32, bool NC4, bool LEAN = false>
 __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
   uint32_t wmask = 0;
   for (uint32_t w = 0; w < V.nwr; ++w) {
@@ -529,7 +599,7 @@ __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
   for (uint32_t w = 0; w < V.nremw; ++w) A.REM[w * A.S] = V.rem0[w];
   const uint32_t n = V.n;
   const bool ct = PASS == 2 && !T32 && !NC4;
-  const uint32_t tw = PASS == 1 ? 0 : (T32 ? n : (n + 1) / 2);
+  const uint32_t tw = PASS == 1 ? 0 : (LEAN ? (n + 3) / 4 : (T32 ? n : (n + 1) / 2));
   const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
   for (uint32_t w = 0; w < tw + dw; ++w) A.T[w * A.S] = 0;  // T and DK are contiguous
   return wmask;
@@ -684,7 +754,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
 // instruction whose slot (width / type) is full counts as semi-ready with
 // ready time t + 1; the Philox step is t * issue_width + used.
 // Weighted single pass (pass 4, R41): no target, cost = length + W * cost_rp.
-template <int LG, bool MASK, bool T32, bool NC4, bool WIDE = false>
+template <int LG, bool MASK, bool T32, bool NC4, bool WIDE = false, bool LEAN = false>
 __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
@@ -692,7 +762,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
                                             const uint32_t *coins = nullptr, uint32_t coin_t = 0) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   uint32_t wmask = 0;
-  if (G.leader()) wmask = init_state<2, MASK, T32, NC4>(V, A);
+  if (G.leader()) wmask = init_state<2, MASK, T32, NC4, LEAN>(V, A);
   wmask = G.bcast(wmask);
   G.sync();
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
@@ -709,9 +779,13 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   const uint32_t slots = c_mach.type_slots;  // u8 x 4
   uint32_t used = 0, used_t = 0;              // placed in cycle t: total, per type (u8 x 4)
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0, B = 0;
-  // ready time and per-class last-use counts of instruction j
+  // ready time and per-class last-use counts of instruction j (LEAN: the
+  // counts come from dyn_kills once ds is loaded)
   auto rd_dk = [&](uint32_t j, uint32_t &rd, uint32_t &dk) {
-    if constexpr (CT) {
+    if constexpr (LEAN) {
+      rd = B + r8_get(A, j);
+      dk = 0;
+    } else if constexpr (CT) {
       const uint32_t x = x_get(A, j);
       rd = B + (x & 0x3FFu);
       dk = x_dk(x);
@@ -728,7 +802,11 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   o.prp01 = o.prp23 = 0;
   o.len = kInvalid;
   while (placed < n) {
-    if (CT && t - B >= kWin) {  // slide the ready-time window (t - B <= 2 kWin - 2 here)
+    if (LEAN && t - B >= kWin8) {  // slide the u8 window: saturating byte subtract
+      for (uint32_t q = G.lane; q < (n + 3) / 4; q += LG) A.T[q * A.S] = __vsubus4(A.T[q * A.S], 0x80808080u);
+      B += kWin8;
+      G.sync();
+    } else if (!LEAN && CT && t - B >= kWin) {  // slide the ready-time window (t - B <= 2 kWin - 2 here)
       for (uint32_t q = G.lane; q < (n + 1) / 2; q += LG) A.T[q * A.S] = x_slide2(A.T[q * A.S]);
       B += kWin;
       G.sync();
@@ -763,7 +841,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     auto eval = [&](uint32_t j, uint32_t rdy, const uint4 &ds, uint32_t dk, uint32_t tv) {
       const uint32_t K = ds.y + dk;                   // kills per class (R14)
       const bool lat_ok = rdy <= t;
-      if (lat_ok && (!mi || ((avail >> (8 * ds.w)) & 1u))) {
+      if (lat_ok && (!mi || ((avail >> (8 * (ds.w & 0xFu))) & 1u))) {
         counts += 1u;
         if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
           const uint32_t s = tv * eta_of(j, ds.z, dk);
@@ -791,6 +869,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
           ds[u] = V.ds[j[u]];                         // defs, static kills, eta2, type
           tv[u] = trow[j[u]];
         }
+        if (LEAN) dyn_kills4(V, A, ds, dk);
 #pragma unroll
         for (int u = 0; u < 4; ++u)
           if (v[u]) eval(j[u], rd[u], ds[u], dk[u], tv[u]);
@@ -799,7 +878,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
         uint32_t rd, dk;
         rd_dk(j, rd, dk);
-        eval(j, rd, V.ds[j], dk, trow[j]);
+        const uint4 ds = V.ds[j];
+        if (LEAN) dk = dyn_kills(V, A, ds.w);
+        eval(j, rd, ds, dk, trow[j]);
         return false;
       });
     }
@@ -857,7 +938,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
           rd_dk(j, rd, dk);
           if (rd > t) return false;
           const uint4 ds = V.ds[j];
-          if (mi && !((avail >> (8 * ds.w)) & 1u)) return false;
+          if (LEAN) dk = dyn_kills(V, A, ds.w);
+          if (mi && !((avail >> (8 * (ds.w & 0xFu))) & 1u)) return false;
           if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u) return false;
           pre += (uint32_t)trow[j] * eta_of(j, ds.z, dk);
           if (pre > r) {
@@ -870,7 +952,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       jstar = G.bcast(jstar);
     }
     if (G.leader()) {
-      commit<2, MASK, T32, NC4>(V, A, jstar, t, wmask, live01, live23, prp01, prp23, B);
+      commit<2, MASK, T32, NC4, LEAN>(V, A, jstar, t, wmask, live01, live23, prp01, prp23, B);
       if (rec_o) {
         rec_o[placed] = (uint16_t)jstar;
         rec_c[placed] = t;
@@ -884,7 +966,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     prev = jstar;
     if (mi) {  // R42: the cycle is complete after issue_width placements
       ++used;
-      used_t += 1u << (8 * V.ds[jstar].w);
+      used_t += 1u << (8 * (V.ds[jstar].w & 0xFu));
       if (used == w) {
         ++t;
         used = used_t = 0;
@@ -928,8 +1010,9 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
 // through L1/L2 (state in the workspace); 2 = image read through L1 (it is
 // small next to the state of large regions), per-ant state (and tau when
 // staged) in shared memory: more ants resident per SM.
-template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS, bool WIDE>
-__global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
+// LEAN: pass-2 lean per-ant layout (u8 ready times, dynamic kills).
+template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS, bool WIDE, bool LEAN = false>
+__global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 1 : 2)
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
@@ -969,7 +1052,7 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
       const uint32_t gsz = A.cfg.group_size, abase = A.cfg.ant_base + bi.ant0, g0 = abase / gsz;
       const uint32_t ng = (abase + apb - 1) / gsz - g0 + 1, cw = coin_words(PASS, rd->n);
       uint32_t *cz = (uint32_t *)(smem + state_off) +
-                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4);
+                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4, LEAN);
       const uint32_t lane = threadIdx.x & 31u, c2 = PASS == 1 ? iter : (0x80000000u | iter);
       for (uint32_t task = threadIdx.x >> 5; task < ng * cw; task += blockDim.x >> 5) {
         const uint32_t gi = task / cw, k = (task - gi * cw) * 32 + lane;
@@ -987,7 +1070,7 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
   }
   const Grp<LG> G(threadIdx.x);
   const SV V = make_sv(img, rd);
-  const St S = make_st<PASS, T32, NC4>(stbase, stride, V);
+  const St S = make_st<PASS, T32, NC4, LEAN>(stbase, stride, V);
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
   if (PASS == 1) {
@@ -1008,7 +1091,7 @@ __global__ void __launch_bounds__(kMaxBlockThreads, WIDE ? 1 : 2)
       rec_o = A.dump_order + base;
       rec_c = A.dump_cycle + base;
     }
-    o = ant_pass2<LG, MASK, T32, NC4, WIDE>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
+    o = ant_pass2<LG, MASK, T32, NC4, WIDE, LEAN>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
                                       rec_c, coins, coin_t);
   }
   if (G.leader()) {
@@ -1142,7 +1225,7 @@ __device__ uint32_t asap_order(const SV &V, const uint16_t *order, uint16_t *out
   const uint32_t n = V.n, w = c_mach.issue_width;
   uint32_t t = 0, used = 0, used_t = 0;
   for (uint32_t k = 0; k < n; ++k) {
-    const uint32_t j = order[k], y = V.ds[j].w;
+    const uint32_t j = order[k], y = V.ds[j].w & 0xFu;
     uint32_t c = k == 0 ? rdyv[j] : max(t, rdyv[j]);
     if (k > 0 && c == t && (used >= w || ((used_t >> (8 * y)) & 0xFFu) >= ((c_mach.type_slots >> (8 * y)) & 0xFFu)))
       c = t + 1;
@@ -1421,15 +1504,15 @@ int last_cuda_error() { return check(); }
 using ConstructFn = void (*)(KArgs, const BlockItem *, uint32_t);
 
 __host__ __device__ constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4,
-                                                     int gs, bool wd) {
+                                                     int gs, bool wd, bool lean = false) {
   return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
-         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) | ((gs == 2 ? 1u : 0u) << 11) |
+         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) | ((gs == 2 ? 1u : 0u) << 11) | ((uint32_t)lean << 12) |
          ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((gs == 1 ? 1u : 0u) << 1) | (uint32_t)wd;
 }
 
-template <int P, int LG, bool M, bool TS, bool T3, bool N4, int GS, bool WD, typename F>
+template <int P, int LG, bool M, bool TS, bool T3, bool N4, int GS, bool WD, typename F, bool LN = false>
 static void reg1(F &f) {
-  f(&k_construct<P, LG, M, TS, T3, N4, GS, WD>, variant_code(P, LG, M, TS, T3, N4, GS, WD));
+  f(&k_construct<P, LG, M, TS, T3, N4, GS, WD, LN>, variant_code(P, LG, M, TS, T3, N4, GS, WD, LN));
 }
 template <int P, int LG, bool M, bool TS, bool T3, bool N4, typename F>
 static void reg_w(F &f) {  // the 4-wide scan exists only with the word mask (n <= 1024)
@@ -1440,6 +1523,10 @@ template <int LG, typename F>
 static void reg_lg(F &f) {
   reg1<1, LG, true, false, false, false, 2, true>(f);  // large regions, image through L1
   reg1<2, LG, true, false, false, false, 2, true>(f);
+  if constexpr (LG == 1) {  // pass-2 lean layout (large regions), image staged or through L1
+    reg1<2, 1, true, false, false, false, 0, true, F, true>(f);
+    reg1<2, 1, true, false, false, false, 2, true, F, true>(f);
+  }
   reg_w<1, LG, true, true, false, false>(f);
   reg_w<1, LG, true, false, false, false>(f);
   reg_w<1, LG, false, true, false, false>(f);
@@ -1477,7 +1564,7 @@ static void for_each_construct(F &&f) {
   reg1<2, 4, false, false, true, true, 1, false>(f);
 }
 
-static ConstructFn g_construct[4096];
+static ConstructFn g_construct[8192];
 static bool g_table_ready = false;
 static void build_table() {
   if (g_table_ready) return;
@@ -1486,16 +1573,17 @@ static void build_table() {
 }
 
 // Resident threads per SM the registers of the construct kernels allow, per
-// (pass, wide); conservative defaults when no device is visible.
-int construct_max_threads(int device, uint32_t out[2][2]) {
+// (pass, plain | wide | lean); conservative defaults when no device is visible.
+int construct_max_threads(int device, uint32_t out[2][3]) {
   out[0][0] = out[1][0] = 1024;
   out[0][1] = out[1][1] = 512;
+  out[0][2] = out[1][2] = 512;
   int cur = -1;
   if (cudaGetDevice(&cur) != cudaSuccess || (device >= 0 && cur != device && cudaSetDevice(device) != cudaSuccess)) {
     cudaGetLastError();
     return 1;
   }
-  uint32_t regs[2][2] = {{0, 0}, {0, 0}};
+  uint32_t regs[2][3] = {{0, 0, 0}, {0, 0, 0}};
   bool ok = true;
   for_each_construct([&](ConstructFn f, uint32_t code) {
     cudaFuncAttributes fa;
@@ -1503,7 +1591,7 @@ int construct_max_threads(int device, uint32_t out[2][2]) {
       ok = false;
       return;
     }
-    const uint32_t p = (code >> 8) & 1u, w = code & 1u;
+    const uint32_t p = (code >> 8) & 1u, w = ((code >> 12) & 1u) ? 2u : (code & 1u);
     regs[p][w] = std::max(regs[p][w], (uint32_t)fa.numRegs);
   });
   if (!ok) {
@@ -1511,7 +1599,7 @@ int construct_max_threads(int device, uint32_t out[2][2]) {
     return 1;
   }
   for (int p = 0; p < 2; ++p)
-    for (int w = 0; w < 2; ++w) {
+    for (int w = 0; w < 3; ++w) {
       const uint32_t r8 = std::max(8u, (regs[p][w] + 7u) & ~7u);  // allocation unit: 8 registers per thread
       const uint32_t warps = std::min(64u, 65536u / (32u * r8));
       out[p][w] = warps * 32u;
@@ -1576,7 +1664,8 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   const uint32_t lg = c.lanes;
   const uint32_t code = variant_code(pass, lg, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32,
-                                     pass == 2 && c.nc4, c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask);
+                                     pass == 2 && c.nc4, c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask,
+                                     pass == 2 && c.lean);
   const ConstructFn f = g_construct[code];
   if (!f) return (int)cudaErrorInvalidDeviceFunction;
   f<<<c.n_blocks, c.ants_pb * lg, c.smem_bytes, (cudaStream_t)L.stream>>>(kargs(L), c.items, iter);

@@ -344,3 +344,37 @@ def test_many_multiuse_registers_every_ant(torch_cuda):
     s = _sched()
     s.load(regs, ids).run(p, no_prune=True, dump=True)
     dump_parity(s, regs, ids, p)
+
+
+@pytest.mark.parametrize("mode,mix", [(0, 0), (1, 0), (1, 1)])
+def test_lean_layout_every_ant(torch_cuda, mode, mix):
+    """Large regions (n >= 160) run pass 2 in the lean layout (u8 ready times
+    relative to a 128-cycle window, kills derived from the remaining-use
+    counters at evaluation): every ant bit-exact, including latencies of
+    exactly 127 (the lean window's bound) and per-group mixed heuristics."""
+    regs = [I.gen_region(160, 1601), _relat(I.gen_region(211, 1602), lambda x: 127 if x >= 20 else x, "-l127"),
+            I.gen_region(333, 1603, "unit"), I.gen_region(420, 1604)]
+    ids = [61, 62, 63, 64]
+    p = I.Params(ants=96, iterations=2, seed=24 + mode, cost_mode=mode, stall_mod=2, heur_mix=mix)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_lean_equals_compact_layout(torch_cuda, monkeypatch):
+    """Production mode (pruning on, no dump): the lean and the 10-bit compact
+    pass-2 layouts give the same results (the layout is an implementation
+    choice, not semantics)."""
+    regs = [I.gen_region(n, 1700 + n) for n in (170, 260, 480)]
+    ids = [71, 72, 73]
+    p = I.Params(ants=256, iterations=4, seed=31)
+    out = []
+    for lean in ("0", "1"):
+        monkeypatch.setenv("ACO_LEAN", lean)
+        s = _sched()
+        s.load(regs, ids).run(p)
+        out.append(s.results())
+    for k in range(len(regs)):
+        ora = O.schedule(regs[k], ids[k], I.GFX906, p)
+        for g in out:
+            compare_results(g[k], ora, f"region {k}")
