@@ -658,57 +658,137 @@ typedef struct {
 } ant_out;
 
 /* Pass-1 ant (L108, L116-L118, L145; R19): latencies ignored, one
- * instruction per step, candidates = all ready instructions. */
-static void ant_pass1(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *tau, int greedy,
-                      uint32_t *order, ant_out *out) {
+ * instruction per step, candidates = all ready instructions.  Written as
+ * steps (begin / ready list / choose-and-commit) so that the ants of one
+ * wavefront can also run in lockstep for the ready-list size limit (R45). */
+static void p1_begin(ant_ctx *a) {
   const model *m = a->m;
-  uint32_t n = m->n;
-  for (uint32_t j = 0; j < n; ++j) { a->pred_left[j] = m->indeg[j]; a->scheduled[j] = 0; }
+  for (uint32_t j = 0; j < m->n; ++j) { a->pred_left[j] = m->indeg[j]; a->scheduled[j] = 0; }
   rp_init(m, &a->rp);
-  uint32_t prev = ROOT_ROW(n);
-  for (uint32_t k = 0; k < n; ++k) {
-    uint32_t cnt = 0;
-    for (uint32_t j = 0; j < n; ++j) /* ascending index order (R25) */
-      if (!a->scheduled[j] && a->pred_left[j] == 0) {
-        a->cand[cnt] = j;
-        /* R43: with heur_mix, odd ant groups are guided by the ILP heuristic
-         * (CP, eta2) instead of LUC-then-CP; the greedy schedule never is */
-        uint32_t e = (!greedy && a->p->heur_mix && ((ant / a->p->group_size) & 1u)) ? eta2(m, j)
-                                                                                    : eta1(m, &a->rp, j);
-        a->score[cnt] = (uint32_t)tau[(size_t)prev * n + j] * e;
-        cnt++;
-      }
-    int exploit;
-    uint64_t r64 = 0;
-    if (greedy) {
-      exploit = 1;
-    } else {
-      uint32_t coin = draw_group_coin(a->p->seed, a->region_id, 1, iter, ant / a->p->group_size, k);
-      exploit = (uint64_t)coin < a->p->q0_t; /* R1-R3 */
-      if (!exploit) {
-        uint32_t x[4];
-        draw_ant(a->p->seed, a->region_id, 1, iter, ant, k, x);
-        r64 = ((uint64_t)x[1] << 32) | x[0];
-      }
+}
+
+/* The ready list in ascending index order (R25) with its scores
+ * tau[prev][j] * eta(j) (R1, R4); returns its size. */
+static uint32_t p1_ready(ant_ctx *a, uint32_t ant, uint32_t prev, const uint16_t *tau, int greedy) {
+  const model *m = a->m;
+  uint32_t n = m->n, cnt = 0;
+  for (uint32_t j = 0; j < n; ++j)
+    if (!a->scheduled[j] && a->pred_left[j] == 0) {
+      a->cand[cnt] = j;
+      /* R43: with heur_mix, odd ant groups are guided by the ILP heuristic
+       * (CP, eta2) instead of LUC-then-CP; the greedy schedule never is */
+      uint32_t e = (!greedy && a->p->heur_mix && ((ant / a->p->group_size) & 1u)) ? eta2(m, j)
+                                                                                  : eta1(m, &a->rp, j);
+      a->score[cnt] = (uint32_t)tau[(size_t)prev * n + j] * e;
+      cnt++;
     }
-    uint32_t j = a->cand[orc_select(a->score, cnt, exploit, r64)];
-    if (a->stats && !greedy) {
-      a->stats[ORS_SUM_R] += cnt;
-      a->stats[ORS_SUM_F] += cnt;
-      a->stats[ORS_SUM_DEG] += m->succ_ptr[j + 1] - m->succ_ptr[j];
-      a->stats[ORS_SUM_USE] += m->src->use_ptr[j + 1] - m->src->use_ptr[j];
-      a->stats[ORS_SUM_DEF] += m->src->def_ptr[j + 1] - m->src->def_ptr[j];
-      a->stats[ORS_PLACEMENTS]++;
+  return cnt;
+}
+
+/* Step k: select among the first `lim` ready instructions (all of them
+ * unless the ready-list limit R45 is on) and commit; returns the choice. */
+static uint32_t p1_commit(ant_ctx *a, uint32_t iter, uint32_t ant, uint32_t k, uint32_t cnt, uint32_t lim,
+                          int greedy) {
+  const model *m = a->m;
+  int exploit;
+  uint64_t r64 = 0;
+  if (greedy) {
+    exploit = 1;
+  } else {
+    uint32_t coin = draw_group_coin(a->p->seed, a->region_id, 1, iter, ant / a->p->group_size, k);
+    exploit = (uint64_t)coin < a->p->q0_t; /* R1-R3 */
+    if (!exploit) {
+      uint32_t x[4];
+      draw_ant(a->p->seed, a->region_id, 1, iter, ant, k, x);
+      r64 = ((uint64_t)x[1] << 32) | x[0];
     }
-    rp_issue(m, &a->rp, j);
-    order[k] = j;
-    a->scheduled[j] = 1;
-    for (uint32_t q = m->succ_ptr[j]; q < m->succ_ptr[j + 1]; ++q) a->pred_left[m->succ[q]]--;
-    prev = j;
   }
+  uint32_t j = a->cand[orc_select(a->score, lim, exploit, r64)];
+  if (a->stats && !greedy) {
+    a->stats[ORS_SUM_R] += cnt;
+    a->stats[ORS_SUM_F] += lim;
+    a->stats[ORS_SUM_DEG] += m->succ_ptr[j + 1] - m->succ_ptr[j];
+    a->stats[ORS_SUM_USE] += m->src->use_ptr[j + 1] - m->src->use_ptr[j];
+    a->stats[ORS_SUM_DEF] += m->src->def_ptr[j + 1] - m->src->def_ptr[j];
+    a->stats[ORS_PLACEMENTS]++;
+  }
+  rp_issue(m, &a->rp, j);
+  a->scheduled[j] = 1;
+  for (uint32_t q = m->succ_ptr[j]; q < m->succ_ptr[j + 1]; ++q) a->pred_left[m->succ[q]]--;
+  return j;
+}
+
+static void p1_end(ant_ctx *a, ant_out *out) {
   for (uint32_t c = 0; c < 4; ++c) out->prp[c] = a->rp.prp[c];
   out->cost = orc_cost_rp(a->mach, a->p->cost_mode, a->rp.prp);
   out->length = 0;
+}
+
+static void ant_pass1(ant_ctx *a, uint32_t iter, uint32_t ant, const uint16_t *tau, int greedy,
+                      uint32_t *order, ant_out *out) {
+  uint32_t n = a->m->n, prev = ROOT_ROW(n);
+  p1_begin(a);
+  for (uint32_t k = 0; k < n; ++k) {
+    uint32_t cnt = p1_ready(a, ant, prev, tau, greedy);
+    prev = order[k] = p1_commit(a, iter, ant, k, cnt, cnt, greedy);
+  }
+  p1_end(a, out);
+}
+
+/* Scratch of one ant context (the per-ant arrays of ant_ctx). */
+static int ant_scratch_alloc(ant_ctx *a, const model *m) {
+  uint32_t n = m->n;
+  a->pred_left = malloc(sizeof(uint32_t) * (n + 1));
+  a->rdy = malloc(sizeof(uint32_t) * (n + 1));
+  a->cand = malloc(sizeof(uint32_t) * (n + 1));
+  a->score = malloc(sizeof(uint32_t) * (n + 1));
+  a->flist = malloc(sizeof(uint32_t) * (n + 1));
+  a->scheduled = malloc(n + 1);
+  a->rp.rem = calloc(m->n_regs + 1, sizeof(uint32_t));
+  return a->pred_left && a->rdy && a->cand && a->score && a->flist && a->scheduled && a->rp.rem;
+}
+static void ant_scratch_free(ant_ctx *a) {
+  free(a->pred_left); free(a->rdy); free(a->cand); free(a->score); free(a->flist); free(a->scheduled);
+  free(a->rp.rem);
+}
+
+/* Ready-list size limit (L214; R45): the ants of one wavefront -- the group
+ * of G = group_size consecutive ant ids (R3) -- build their pass-1 schedules
+ * in lockstep; at step k every ant of the group considers only the first K
+ * instructions of its ready list (ascending index, R25), with K = the
+ * smallest ready-list size in the group at step k (rl_limit = 1) or the
+ * midpoint floor((min + max) / 2) of the smallest and largest (rl_limit = 2).
+ * Ants [a0, a0 + cnt) of the group; orders[i * n ..] and outs[i] receive
+ * ant a0 + i's schedule and result. */
+static int pass1_group_lockstep(const ant_ctx *proto, uint32_t iter, uint32_t a0, uint32_t cnt,
+                                const uint16_t *tau, uint32_t *orders, ant_out *outs) {
+  const model *m = proto->m;
+  uint32_t n = m->n;
+  ant_ctx *g = calloc(cnt, sizeof(ant_ctx));
+  uint32_t *prev = malloc(sizeof(uint32_t) * cnt), *size = malloc(sizeof(uint32_t) * cnt);
+  int ok = g && prev && size;
+  for (uint32_t i = 0; ok && i < cnt; ++i) {
+    g[i] = *proto;
+    ok = ant_scratch_alloc(&g[i], m);
+    if (ok) p1_begin(&g[i]);
+    prev[i] = ROOT_ROW(n);
+  }
+  for (uint32_t k = 0; ok && k < n; ++k) {
+    uint32_t lo = UINT32_MAX, hi = 0;
+    for (uint32_t i = 0; i < cnt; ++i) {
+      size[i] = p1_ready(&g[i], a0 + i, prev[i], tau, 0);
+      if (size[i] < lo) lo = size[i];
+      if (size[i] > hi) hi = size[i];
+    }
+    uint32_t lim = proto->p->rl_limit == 1 ? lo : (lo + hi) / 2;
+    for (uint32_t i = 0; i < cnt; ++i) /* (a midpoint above an ant's own size does not bind) */
+      prev[i] = orders[(size_t)i * n + k] = p1_commit(&g[i], iter, a0 + i, k, size[i], lim < size[i] ? lim : size[i], 0);
+  }
+  for (uint32_t i = 0; ok && i < cnt; ++i) p1_end(&g[i], &outs[i]);
+  if (g)
+    for (uint32_t i = 0; i < cnt; ++i) ant_scratch_free(&g[i]);
+  free(g); free(prev); free(size);
+  return ok ? ORC_OK : ORC_E_ARG;
 }
 
 /* Is ant group g allowed optional stalls?  (L202-L204; R23, R44) */
@@ -960,7 +1040,7 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
                  uint32_t *dump_cycle, uint16_t *tau_out) {
   if (p->pass < 1 || p->pass > 4 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
       p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->ws_weight > 1024u ||
-      p->heur_mix > 1u)
+      p->heur_mix > 1u || p->rl_limit > 2u)
     return ORC_E_ARG;
   int st = machine_check(r, mach);
   if (st != ORC_OK) return st;
@@ -990,6 +1070,9 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
   uint32_t *best_cycle_of = malloc(sizeof(uint32_t) * (n + 1));
   uint32_t *win_cycle_of = malloc(sizeof(uint32_t) * (n + 1));
   uint32_t *tmp_cycle = malloc(sizeof(uint32_t) * (n + 1));
+  /* R45: one wavefront's lockstep pass-1 schedules */
+  uint32_t *grp_order = p->rl_limit ? malloc(sizeof(uint32_t) * ((size_t)p->group_size * n + 1)) : NULL;
+  ant_out *grp_out = p->rl_limit ? malloc(sizeof(ant_out) * p->group_size) : NULL;
 
   uint32_t lb_cost, lb_len, ub, final_len = 0;
   orc_lower_bounds(r, mach, p->cost_mode, &lb_cost, &lb_len, &ub);
@@ -1027,7 +1110,18 @@ int orc_schedule(const orc_region *r, uint32_t region_id, const orc_machine *mac
       memset(&wout, 0, sizeof(wout));
       for (uint32_t ant = 0; ant < p->ants; ++ant) {
         ant_out o;
-        ant_pass1(&a, it, ant, tau, 0, ant_order, &o);
+        if (p->rl_limit) { /* R45: the ant's wavefront was built in lockstep */
+          uint32_t gs = p->group_size, a0 = ant - ant % gs;
+          uint32_t gc = (a0 + gs <= p->ants ? gs : p->ants - a0);
+          if (ant == a0 && pass1_group_lockstep(&a, it, a0, gc, tau, grp_order, grp_out) != ORC_OK) {
+            st = ORC_E_ARG;
+            goto report;
+          }
+          memcpy(ant_order, grp_order + (size_t)(ant - a0) * n, sizeof(uint32_t) * n);
+          o = grp_out[ant - a0];
+        } else {
+          ant_pass1(&a, it, ant, tau, 0, ant_order, &o);
+        }
         stats[ORS_ANT_SCHEDS]++;
         if (dump_cost) dump_cost[((size_t)0 * p->iterations + it) * p->ants + ant] = o.cost;
         if (dump_order)
@@ -1147,7 +1241,7 @@ report:
 
   free(a.pred_left); free(a.rdy); free(a.cand); free(a.score); free(a.flist); free(a.scheduled); free(a.rp.rem);
   free(tau); free(ant_order); free(ant_cycle_of); free(best_order); free(win_order);
-  free(best_cycle_of); free(win_cycle_of); free(tmp_cycle); free(heur_order);
+  free(best_cycle_of); free(win_cycle_of); free(tmp_cycle); free(heur_order); free(grp_order); free(grp_out);
   model_free(&m);
   return st;
 }

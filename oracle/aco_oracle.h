@@ -71,6 +71,7 @@ typedef struct {
   uint32_t ws_weight;              /* pass 4: cost = length + ws_weight * cost_rp (R41) */
   uint32_t heur_mix;               /* 1: odd ant groups use the other pass's heuristic (L216-L218; R43) */
   uint32_t stall_num;              /* group g may stall iff (g - stall_rem) mod stall_mod < stall_num (R44) */
+  uint32_t rl_limit;               /* pass-1 ready-list size limit per wavefront (L214; R45): 0 off, 1 min, 2 mid */
 } orc_params;
 
 /* Indices into the u64 result vector filled by orc_schedule. */

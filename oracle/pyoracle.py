@@ -69,6 +69,7 @@ class _Params(C.Structure):
         ("stop_no_improve", C.c_uint32), ("stop_at_lb", C.c_uint32),
         ("pass2_gap", C.c_uint32), ("revert_occ", C.c_uint32), ("revert_len", C.c_uint32),
         ("ws_weight", C.c_uint32), ("heur_mix", C.c_uint32), ("stall_num", C.c_uint32),
+        ("rl_limit", C.c_uint32),
     ]
 
 
@@ -156,7 +157,7 @@ def params_struct(p) -> _Params:
     return _Params(p.ants, p.iterations, p.seed, p.passes, p.cost_mode, p.q0_t, p.group_size,
                    p.stall_mod, p.stall_rem, p.tau0, p.rho_q16, p.delta, p.tau_min, p.tau_max,
                    p.stop_no_improve, p.stop_at_lb, p.pass2_gap, p.revert_occ, p.revert_len,
-                   p.ws_weight, p.heur_mix, p.stall_num)
+                   p.ws_weight, p.heur_mix, p.stall_num, p.rl_limit)
 
 
 def philox(ctr: Sequence[int], key: Sequence[int]):

@@ -150,6 +150,7 @@ class Params:
     ws_weight: int = 0  # passes == 4: cost = length + ws_weight * cost_rp (L74; R41)
     heur_mix: int = 0  # 1: odd ant groups use the other pass's heuristic (L216-L218; R43)
     stall_num: int = 1  # group g may stall iff (g - stall_rem) % stall_mod < stall_num (R44)
+    rl_limit: int = 0  # pass-1 ready-list size limit per ant group (L214; R45): 0 off, 1 min, 2 mid
 
 
 def paper_policy(p: "Params") -> "Params":

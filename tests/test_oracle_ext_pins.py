@@ -354,3 +354,75 @@ def test_weighted_pass_fix10a():
                                                    ws_weight=W))
         assert brute.optimum_machine(x, I.GFX906, 0, weight=W)[1] == opt == r["ws_cost"]
     assert brute.optimum_machine(x, I.GFX906, 0, weight=10)[1] == 63
+
+
+# ---------------------------------------------------------------- R45: ready-list size limit (L214)
+def _ready_lists(region, order):
+    """Ready list (ascending) before every step of a pass-1 order, recomputed
+    from the edges alone (latencies ignored, R19)."""
+    n = region.n_insts
+    preds = brute.preds_of(region)
+    done, out = set(), []
+    for j in order:
+        out.append([v for v in range(n) if v not in done and all(p in done for p, _ in preds.get(v, []))])
+        done.add(j)
+    return out
+
+
+def _pass1_dump(region, p):
+    o = O.schedule(region, 3, I.GFX906, p, dump=True, dump_orders=True)
+    return o, o["dump_order"][0], o["dump_cost"][0]
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+def test_rl_limit_group_of_one_is_unlimited(mode):
+    """A wavefront of one ant: min = max = its own ready-list size, so the
+    limit never binds and every ant equals the unlimited one."""
+    r = I.gen_region(50, 4501)
+    base = dict(ants=24, iterations=3, seed=5, cost_mode=0, group_size=1)
+    a = O.schedule(r, 3, I.GFX906, I.Params(**base), dump=True, dump_orders=True)
+    b = O.schedule(r, 3, I.GFX906, I.Params(**base, rl_limit=mode), dump=True, dump_orders=True)
+    assert np.array_equal(a["dump_order"], b["dump_order"]) and a["trace_hash"] == b["trace_hash"]
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+def test_rl_limit_antichain_is_unlimited(mode):
+    """No edges: every ant's ready list at step k has n - k entries, the
+    group's min = max, so the limit never binds."""
+    n = 12
+    r = I.Region.from_lists(n, [], [0] * n, [2] * n, [[g] for g in range(n)], [[] for _ in range(n)], name="anti")
+    base = dict(ants=40, iterations=2, seed=8, cost_mode=0, group_size=16)
+    a = O.schedule(r, 3, I.GFX906, I.Params(**base), dump=True, dump_orders=True)
+    b = O.schedule(r, 3, I.GFX906, I.Params(**base, rl_limit=mode), dump=True, dump_orders=True)
+    assert np.array_equal(a["dump_order"], b["dump_order"])
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+def test_rl_limit_choices_respect_group_limit(mode):
+    """Every pass-1 choice of every ant lies within the first K entries of its
+    ready list, K = the minimum (mode 1) or the min/max midpoint (mode 2) of
+    the ready-list sizes of its group (G consecutive ants, partial last group)
+    at that step -- all recomputed here from the dumped orders and the edges.
+    The limit must bind somewhere (non-vacuous) and change some schedule."""
+    G = 8
+    binds = changed = 0
+    for seed, n in ((1, 30), (2, 45)):
+        r = I.gen_region(n, 4600 + seed)
+        p = I.Params(ants=20, iterations=2, seed=seed, cost_mode=0, group_size=G, rl_limit=mode)
+        o, orders, costs = _pass1_dump(r, p)
+        free = O.schedule(r, 3, I.GFX906, dataclasses.replace(p, rl_limit=0), dump=True, dump_orders=True)
+        changed += int(not np.array_equal(free["dump_order"][0], orders))
+        for it in range(o["iters1"]):
+            rl = [_ready_lists(r, list(orders[it, a])) for a in range(p.ants)]
+            for g0 in range(0, p.ants, G):
+                grp = range(g0, min(g0 + G, p.ants))
+                for k in range(n):
+                    sizes = [len(rl[a][k]) for a in grp]
+                    K = min(sizes) if mode == 1 else (min(sizes) + max(sizes)) // 2
+                    for a in grp:
+                        ready = rl[a][k]
+                        assert int(orders[it, a, k]) in ready[:K], (seed, it, a, k, K)
+                        binds += K < len(ready)
+            for a in range(p.ants):  # the cost is the order's PRP cost (independent recompute)
+                assert costs[it, a] == brute.cost(I.GFX906, 0, checker.prp(r, list(orders[it, a])))
+    assert binds > 0 and changed > 0
