@@ -7,7 +7,7 @@ update, epilogue) over one batch of synthetic regions.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c3|c2|c1|c4|c5]
                   [--machine gfx906|dual] [--passes 3|4 --ws-weight W] [--policy off|paper]
-                  [--heur-mix 0|1] [--stall-num k]
+                  [--heur-mix 0|1] [--stall-num k] [--rl-limit 0|1|2]
   python bench.py --impl reference ...     # the CPU oracle on a bounded sample
 
 Workloads (BASELINE.json configs): c1 FIX10-A; c2 one n = 100 region; c3
@@ -56,6 +56,7 @@ def parse():
     ap.add_argument("--policy", default="off", choices=["off", "paper"])
     ap.add_argument("--heur-mix", type=int, default=0)
     ap.add_argument("--stall-num", type=int, default=1)
+    ap.add_argument("--rl-limit", type=int, default=0, help="pass-1 ready-list size limit (R45): 1 min, 2 mid")
     ap.add_argument("--regions", type=int, default=C3_REGIONS, help="regions per rank (c3)")
     ap.add_argument("--ants", type=int, default=None)
     ap.add_argument("--iterations", type=int, default=None)
@@ -103,7 +104,8 @@ def workload(args, rank: int):
         p = I.Params(ants=args.ants or 64, iterations=args.iterations or 20, seed=0, cost_mode=0)
         cfg = {"workload": "c1-fix10a", "regions_per_gpu": 1}
     p = dataclasses.replace(p, passes=args.passes, ws_weight=args.ws_weight if args.passes == 4 else 0,
-                            heur_mix=args.heur_mix, stall_num=args.stall_num)
+                            heur_mix=args.heur_mix, stall_num=args.stall_num,
+                            rl_limit=args.rl_limit)
     if args.policy == "paper":
         p = I.paper_policy(p)
     passes = {1: "RP", 2: "ILP", 3: "RP+ILP", 4: f"weighted single pass (W={p.ws_weight})"}[p.passes]
@@ -116,6 +118,8 @@ def workload(args, rank: int):
         cfg["heur_mix"] = 1
     if args.stall_num != 1:
         cfg["stall_groups"] = f"{args.stall_num}/{p.stall_mod}"
+    if args.rl_limit:
+        cfg["ready_list_limit"] = {1: "group min", 2: "group min/max midpoint"}[args.rl_limit]
     return regs, ids, p, cfg
 
 

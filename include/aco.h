@@ -117,6 +117,10 @@ typedef struct {
   uint32_t ws_weight;       /* pass 4: cost = length + ws_weight * cost_rp (<= 1024; R41) */
   uint32_t heur_mix;        /* 1: odd ant groups use the other pass's heuristic (L216-L218; R43) */
   uint32_t stall_num;       /* group g may stall iff (g - stall_rem) % stall_mod < stall_num (R44; paper 1) */
+  uint32_t rl_limit;        /* pass-1 ready-list size limit per ant group (L214; R45): 0 off (default),
+                               1 = the group's minimum ready-list size, 2 = midpoint of its min and max.
+                               Not with the shared colony, nor for regions that need the
+                               global-state kernels (ACO_E_ARG) */
 } aco_params;
 
 /* Per-region result (sizes fixed; the schedule itself is returned through

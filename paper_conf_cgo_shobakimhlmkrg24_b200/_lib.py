@@ -57,6 +57,7 @@ class Params(C.Structure):
         ("stop_no_improve", C.c_uint32), ("stop_at_lb", C.c_uint32), ("flags", C.c_uint32),
         ("pass2_gap", C.c_uint32), ("revert_occ", C.c_uint32), ("revert_len", C.c_uint32),
         ("ws_weight", C.c_uint32), ("heur_mix", C.c_uint32), ("stall_num", C.c_uint32),
+        ("rl_limit", C.c_uint32),
     ]
 
 

@@ -44,7 +44,7 @@ def params_struct(p: Params, flags: int = 0) -> _lib.Params:
     return _lib.Params(p.ants, p.iterations, p.seed, p.passes, p.cost_mode, p.q0_t, p.group_size,
                        p.stall_mod, p.stall_rem, p.tau0, p.rho_q16, p.delta, p.tau_min, p.tau_max,
                        p.stop_no_improve, p.stop_at_lb, flags, p.pass2_gap, p.revert_occ, p.revert_len,
-                       p.ws_weight, p.heur_mix, p.stall_num)
+                       p.ws_weight, p.heur_mix, p.stall_num, p.rl_limit)
 
 
 class HostBatch:

@@ -636,7 +636,7 @@ uint32_t smem_for_k(uint32_t k) { return std::min(kSmemPerSM, (kSmemSM / k - kBl
 // after everything else, so it is taken only when it adds resident threads.
 Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
                  uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w,
-                 bool allow_ig = false) {
+                 bool allow_ig = false, uint32_t apb_mult = 1) {
   Shape bests[2] = {Shape{0, 1, 0, false}, Shape{0, 1, 0, false}};
   for (int ig = 0; ig <= (allow_ig ? 1 : 0); ++ig) {
   Shape &best = bests[ig];
@@ -649,6 +649,7 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
       for (uint32_t threads : {32u, 64u, 96u, 128u, 192u, 256u, 384u, 512u}) {
         if (threads > kMaxBlockThreads) break;
         const uint32_t apb = threads / L;
+        if (apb % apb_mult) continue;  // R45: whole ant groups per block
         const uint64_t bytes = (uint64_t)(ig ? 0u : img) + (ts ? tb : 0u) + (uint64_t)ant_stride(apb, L) * W * 4 +
                                (uint64_t)coin_groups(apb, gsz) * coin_w * 4;
         if (bytes > kSmemPerSM) break;
@@ -681,7 +682,7 @@ namespace {
 
 aco_status check_params(const aco_params *p) {
   if (p->pass < 1 || p->pass > 4 || p->cost_mode > 3 || p->group_size == 0 || p->stall_mod == 0 ||
-      p->ws_weight > 1024u || p->heur_mix > 1u ||
+      p->ws_weight > 1024u || p->heur_mix > 1u || p->rl_limit > 2u ||
       p->ants == 0 || p->tau_min > p->tau_max || p->tau_max > 65535u || p->tau0 > 65535u ||
       p->tau0 < p->tau_min || p->tau0 > p->tau_max || p->q0_t > (1ull << 32) || p->rho_q16 > 65536u ||
       p->iterations > 0x7FFFFFFFu)
@@ -698,6 +699,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // passes that run construct/finalize launches: pass 4 (weighted, R41) uses the pass-2 machinery
   const uint32_t pmask = p->pass == 4 ? 2u : p->pass;
   const uint32_t count = ctx->count, A = p->ants;
+  // R45 (pass-1 ready-list limit): ant groups in lockstep inside one block;
+  // not with the shared colony (a group would span ranks)
+  const bool rl1 = p->rl_limit != 0 && (pmask & 1u);
+  if (p->rl_limit && colony) return ACO_E_ARG;
   Plan saved = ctx->plan;  // a sizing call must not disturb a planned run
   Plan &P = ctx->plan;
   P = Plan();
@@ -763,7 +768,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
       Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
-                            p->group_size, coin_words(pass, R.n), wide && !rare && img_l1[pass - 1]);
+                            p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
+                            wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u);
       if (lean) {
         // the lean layout costs per ant-step (kills derived at every
         // evaluation) and gains resident ants; on the mixed C3 batch it wins
@@ -785,6 +791,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // global-state kernels (all ants resident, state through L1/L2) win
       // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
       if (sh.apb != 0 && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
+      if (sh.apb == 0 && rl1 && pass == 1) {  // R45 needs a block-wide lockstep: shared-memory kernels only
+        ctx->plan = saved;
+        return ACO_E_ARG;
+      }
       if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
         // all ants are resident (state in the workspace); 16 lanes per ant
         // and 512-thread blocks measured best (tools/probe_gs_lanes.sh:
@@ -879,6 +889,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   off = align256(off + 2 * (sum_n + count) + 16);
   const uint64_t o_cost = off;
   off = align256(off + 4ull * A * count);
+  const uint64_t n_grp = rl1 ? ((uint64_t)A + p->group_size - 1) / p->group_size : 0;
+  const uint64_t o_rlk = off;  // R45: K per (ant group, step)
+  off = align256(off + 2 * n_grp * sum_n + 16);
   P.o_keys = off;
   off = align256(off + 8ull * count);
   std::vector<RegionWs> rws(count);
@@ -896,6 +909,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     w.o_dump = (uint64_t)A * ctx->inst_off[r];
     w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
     w.o_heur = o_heur + 2 * ctx->inst_off[r];
+    w.o_rlk = o_rlk + 2 * n_grp * ctx->inst_off[r];
     w.gs = sgs[r];  // k_init / k_select: image and replay state in the workspace
     if (gs[r]) {  // global-state construct kernels
       off = align256(off);
@@ -1029,6 +1043,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.revert_len = p->revert_len;
   cfg.heur_mix = p->heur_mix;
   cfg.stall_num = p->stall_num;
+  cfg.rl_limit = p->rl_limit;
   cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;
   cfg.keys = nullptr;

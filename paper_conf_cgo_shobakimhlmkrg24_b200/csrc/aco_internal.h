@@ -108,6 +108,7 @@ struct RegionWs {
   uint64_t o_gstate; // global-state regions: per-ant state [word][ant] (ants x words u32)
   uint64_t o_scratch;// global-state regions: replay scratch (words + cycles + order)
   uint64_t o_heur;   // u16 [n]  the heuristic (greedy pass-1) order, R40
+  uint64_t o_rlk;    // u16 [ceil(ants/G)][n]: ready-list limit K per (ant group, step), R45 (rl_limit only)
   uint32_t tau_len;  // (n+1)*n rounded up to a multiple of 8
   uint32_t gs;       // 1: the region's state does not fit shared memory (global-state kernels)
 };
@@ -133,6 +134,8 @@ struct RunCfg {
   uint32_t ws_weight;
   uint32_t pass2_gap, revert_occ, revert_len;  // compile policy (R39, R40)
   uint32_t heur_mix, stall_num;                // R43, R44
+  uint32_t rl_limit;                           // R45: 0 off, 1 min, 2 mid
+  uint32_t pad_rl;
   uint32_t stage_img;   // k_select stages the region image in shared memory (few regions)
   uint32_t pad_cfg;
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n

@@ -611,6 +611,42 @@ __device__ __forceinline__ unsigned long long akey(uint32_t s, uint32_t j) {
 }
 
 // ------------------------------------------------------------ pass-1 ant
+// Ready-list size limit (L214; R45): the ants of one group of G consecutive
+// ids (the paper's wavefront) run pass 1 in lockstep inside one block; at
+// step k each ant considers only its first K ready instructions (ascending),
+// K = the group's smallest ready-list size (mode 1) or the midpoint of the
+// smallest and largest (mode 2).  buf: per-block shared counters, triple
+// buffered by step (one barrier per step); out: K per step of the group
+// (written by its first ant, read by the winner replay through `in`).
+struct RL {
+  uint32_t *buf;       // [3][ng][2] {min, max}; nullptr: no limit
+  uint32_t gi, ng, mode;
+  uint16_t *out;       // K per step of this ant's group, or nullptr
+  const uint16_t *in;  // replay: the recorded K per step (no barriers)
+};
+
+// Block barrier for the lockstep steps: NOT the .aligned form of
+// __syncthreads, because a warp may hold both live ants (in ant_pass1) and
+// ghost lanes past the ant count (in k_construct's matching loop), which
+// reach it from different code.
+__device__ __forceinline__ void rl_barrier() { asm volatile("barrier.sync 0;" ::: "memory"); }
+
+// Index of the K-th (1-based) set bit of the ready bitset in ascending order
+// (the last candidate an ant may consider); n if there are fewer.
+__device__ __forceinline__ uint32_t kth_ready(const St &A, uint32_t nwr, uint32_t K, uint32_t n) {
+  for (uint32_t w = 0; w < nwr; ++w) {
+    const uint32_t x = A.RB[w * A.S], c = __popc(x);
+    if (K <= c) return w * 32u + __fns(x, 0, K);
+    K -= c;
+  }
+  return n;
+}
+__device__ __forceinline__ uint32_t ready_count(const St &A, uint32_t nwr) {
+  uint32_t c = 0;
+  for (uint32_t w = 0; w < nwr; ++w) c += __popc(A.RB[w * A.S]);
+  return c;
+}
+
 // RP pass (L108, L145; R19): latencies ignored, candidates = ready list,
 // score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
 // Philox step (R26).  rec (leader, may be NULL) receives the order.  The
@@ -619,8 +655,9 @@ template <int LG, bool MASK, bool WIDE = false>
 __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const bool greedy, uint16_t *rec,
-                                            const uint32_t *coins = nullptr) {
+                                            const uint32_t *coins = nullptr, const RL rl = RL{nullptr, 0, 0, 0, nullptr, nullptr}) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
+  const bool limit = rl.buf != nullptr || rl.in != nullptr;  // R45
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<1, MASK, false, false>(V, A);
   wmask = G.bcast(wmask);
@@ -643,6 +680,34 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       }
     }
     const uint16_t *trow = tau + prev * n;
+    // R45: the last candidate index this ant may consider at step k
+    uint32_t jmax = n;
+    if (limit) {
+      uint32_t K;
+      if (rl.in) {
+        K = rl.in[k];
+      } else {
+        uint32_t *slot = rl.buf + ((k % 3u) * rl.ng + rl.gi) * 2u;
+        if (G.leader()) {
+          const uint32_t c = ready_count(A, nwr);
+          atomicMin(slot, c);
+          atomicMax(slot + 1, c);
+        }
+        if (threadIdx.x == 0) {  // reset the buffer of step k + 1 (last read at step k - 2)
+          uint32_t *nb = rl.buf + ((k + 1u) % 3u) * rl.ng * 2u;
+          for (uint32_t g = 0; g < rl.ng; ++g) {
+            nb[2 * g] = 0xFFFFFFFFu;
+            nb[2 * g + 1] = 0u;
+          }
+        }
+        rl_barrier();
+        const uint32_t lo = slot[0], hi = slot[1];
+        K = rl.mode == 1 ? lo : (lo + hi) / 2u;
+        if (rl.out && G.leader()) rl.out[k] = (uint16_t)K;
+      }
+      if (G.leader()) jmax = kth_ready(A, nwr, K, n);
+      jmax = G.bcast(jmax);
+    }
     // score(j) = tau[prev][j] * eta1(j, sk(j) + d(j)) (R1, R4)
     auto score = [&](uint32_t j) -> uint32_t {
       return (uint32_t)trow[j] * (mix ? V.ds[j].z : (uint32_t)V.eta1[j * L1 + dk1_get(A, j)]);
@@ -653,10 +718,12 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     uint32_t bs1 = 0, bj = 0;
     unsigned long long sum = 0;
     if constexpr (wide) {
-      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v)[4]) {
+      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v0)[4]) {
         uint32_t tv[4], dk[4];
+        bool v[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
+          v[u] = v0[u] && j[u] <= jmax;  // R45 (jmax = n: no limit)
           tv[u] = trow[j[u]];
           dk[u] = A.DK[(j[u] >> 3) * A.S];
         }
@@ -696,6 +763,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
+        if (j > jmax) return true;  // R45: ascending, nothing further is allowed
         const uint32_t sc = score(j);
         if (sc + 1u > bs1) {
           bs1 = sc + 1u;
@@ -719,7 +787,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
         const uint64_t r = __umul64hi(((uint64_t)x.y << 32) | x.x, sum);
         uint64_t pre = 0;
         scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
-          pre += score(j);
+          pre += score(j);  // (j <= jmax: the prefix exceeds r within the allowed candidates)
           if (pre > r) {
             jstar = j;
             return true;
@@ -1030,6 +1098,7 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
   uint32_t stride;
   const uint32_t *coins = nullptr;
   uint32_t coin_t = 0;
+  RL rl{nullptr, 0, 0, A.cfg.rl_limit, nullptr, nullptr};
   if (GS == 1) {  // huge region: statics through L1/L2, per-ant state in the workspace
     if (ai >= A.cfg.ants) return;
     stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
@@ -1062,9 +1131,23 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
       }
       coins = cz + (ant / gsz - g0) * cw;
       coin_t = PASS == 1 ? 0xFFFFFFFFu : cw * 32;
+      if (PASS == 1 && A.cfg.rl_limit) {  // R45: group min/max counters after the coin table
+        rl.buf = cz + ng * cw;
+        rl.gi = ant / gsz - g0;
+        rl.ng = ng;
+        for (uint32_t i = threadIdx.x; i < 3 * ng; i += blockDim.x) {
+          rl.buf[2 * i] = 0xFFFFFFFFu;
+          rl.buf[2 * i + 1] = 0u;
+        }
+        if (ai < A.cfg.ants && ai % gsz == 0) rl.out = (uint16_t *)(A.ws + W.o_rlk) + (size_t)(ai / gsz) * rd->n;
+      }
     }
     __syncthreads();
-    if (ai >= A.cfg.ants) return;  // whole lane group
+    if (ai >= A.cfg.ants) {  // whole lane group
+      if (PASS == 1 && rl.buf)  // the block's lockstep steps need every thread at the barrier (R45)
+        for (uint32_t k = 0; k < rd->n; ++k) rl_barrier();
+      return;
+    }
     if (GS == 0) img = smem;
     stbase = (uint32_t *)(smem + state_off) + local;
   }
@@ -1077,7 +1160,7 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
     uint16_t *rec = nullptr;
     if (dump && A.dump_order)
       rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
-    o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins);
+    o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -1370,7 +1453,10 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
     const Grp<32> G32(threadIdx.x);
     AntOut o;
     if (PASS == 1) {
-      o = ant_pass1<32, MASK>(V, tau, S, G32, want, iter, A.cfg, false, ord);
+      RL rl{nullptr, 0, 0, A.cfg.rl_limit, nullptr, nullptr};
+      if (A.cfg.rl_limit)  // R45: the winner's group limits as recorded by the construct kernel
+        rl.in = (const uint16_t *)(A.ws + W.o_rlk) + (size_t)((want - A.cfg.ant_base) / A.cfg.group_size) * n;
+      o = ant_pass1<32, MASK>(V, tau, S, G32, want, iter, A.cfg, false, ord, nullptr, rl);
     } else {
       uint32_t tgt[4];
       for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];

@@ -378,3 +378,31 @@ def test_lean_equals_compact_layout(torch_cuda, monkeypatch):
         ora = O.schedule(regs[k], ids[k], I.GFX906, p)
         for g in out:
             compare_results(g[k], ora, f"region {k}")
+
+
+@pytest.mark.parametrize("mode", [1, 2])
+def test_ready_list_limit_every_ant(torch_cuda, mode):
+    """Pass-1 ready-list size limit (L214; R45): the ants of each group of 64
+    run in lockstep and consider only the first K ready instructions, K = the
+    group's minimum (mode 1) or min/max midpoint (mode 2) ready-list size;
+    100 ants = a full and a partial group; regions from a single bitset word
+    to the 4-wide large-region kernels."""
+    regs = [I.fix10a(), I.gen_region(45, 1801), I.gen_region(130, 1802, "unit"), I.gen_region(230, 1803)]
+    ids = [81, 82, 83, 84]
+    p = I.Params(ants=100, iterations=3, seed=40 + mode, cost_mode=0, rl_limit=mode)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    dump_parity(s, regs, ids, p)
+
+
+def test_ready_list_limit_production(torch_cuda):
+    """R45 in production mode (pruning on, winner replay with the recorded
+    per-group limits) at 1024 ants: results equal the oracle's."""
+    regs = [I.gen_region(n, 1900 + n) for n in (60, 180, 400)]
+    ids = [91, 92, 93]
+    p = I.Params(ants=1024, iterations=3, seed=47, rl_limit=1)
+    s = _sched()
+    s.load(regs, ids).run(p)
+    got = s.results()
+    for k in range(len(regs)):
+        compare_results(got[k], O.schedule(regs[k], ids[k], I.GFX906, p), f"region {k}")

@@ -6,13 +6,15 @@ run() {  # name, args...
   timeout 900 python bench.py --steps 3 --warmup 3 "$@" 2>gpurun_out/bench_$name.err | tail -1 > gpurun_out/bench_$name.json
   echo "== $name: $(cut -c1-160 gpurun_out/bench_$name.json)"
 }
-for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix}; do
+for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix rlmin}; do
   case $w in
     c1|c2|c3|c4|c5) run $w --workload $w ;;
     dual) run c3_dual --machine dual ;;
     weighted) run c3_weighted --passes 4 --ws-weight 4 ;;
     policy) run c3_paper_policy --policy paper ;;
     mix) run c3_heur_mix --heur-mix 1 ;;
+    rlmin) run c3_rl_min --rl-limit 1 ;;
+    rlmid) run c3_rl_mid --rl-limit 2 ;;
     stall50) run c3_stall50 --stall-num 2 ;;
   esac
 done
