@@ -26,7 +26,7 @@ struct Plan {
   uint32_t fin_smem[3] = {0, 0, 0};
   uint32_t init_smem = 0, p2_smem = 0, max_n = 0, n_upd = 0;
   uint32_t pass_mask = 0, iterations = 0;
-  bool any_t32 = false, nc4 = false, timing = false, p2_done = false, stage_img = false;
+  bool any_t32 = false, nc4 = false, timing = false, p2_done = false, stage_img = false, record = false;
   uint64_t o_state = 0, o_rws = 0, o_upd = 0, o_gb2 = 0, o_gb2c = 0, o_keys = 0;
   LaunchCtx L{};
 };
@@ -634,9 +634,15 @@ uint32_t smem_for_k(uint32_t k) { return std::min(kSmemPerSM, (kSmemSM / k - kBl
 // allow_ig: the image may instead be read through L1 (large regions; wide
 // variants), which frees its shared memory for more resident ants; ranked
 // after everything else, so it is taken only when it adds resident threads.
+uint32_t lane_pow2(uint32_t words) {
+  uint32_t l = 1;
+  while (l < words && l < 32) l <<= 1;
+  return l;
+}
+
 Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
                  uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w,
-                 bool allow_ig = false, uint32_t apb_mult = 1) {
+                 bool allow_ig = false, uint32_t apb_mult = 1, uint32_t spread_cap = 0, uint32_t lane_pref = 1) {
   Shape bests[2] = {Shape{0, 1, 0, false}, Shape{0, 1, 0, false}};
   for (int ig = 0; ig <= (allow_ig ? 1 : 0); ++ig) {
   Shape &best = bests[ig];
@@ -645,11 +651,17 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
     if (ts && (!allow_ts || ig)) continue;  // the image-through-L1 variants keep tau in global memory
     for (uint32_t L : {1u, 2u, 4u, 8u}) {
       if (lanes14 && L != 1 && L != 4) continue;
-      if (L > max_lanes) continue;
+      if (spread_cap) {  // few ants in the whole batch: lanes ~ bitset words, small blocks
+        const uint32_t lp = lanes14 ? (lane_pref >= 4 ? 4u : 1u) : lane_pref;
+        if (L != lp) continue;
+      } else if (L > max_lanes) {
+        continue;
+      }
       for (uint32_t threads : {32u, 64u, 96u, 128u, 192u, 256u, 384u, 512u}) {
         if (threads > kMaxBlockThreads) break;
         const uint32_t apb = threads / L;
         if (apb % apb_mult) continue;  // R45: whole ant groups per block
+        if (spread_cap && apb > std::max(spread_cap, 32u / L)) break;
         const uint64_t bytes = (uint64_t)(ig ? 0u : img) + (ts ? tb : 0u) + (uint64_t)ant_stride(apb, L) * W * 4 +
                                (uint64_t)coin_groups(apb, gsz) * coin_w * 4;
         if (bytes > kSmemPerSM) break;
@@ -660,8 +672,9 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
         if (!k) continue;
         const uint64_t thr = std::min<uint64_t>((uint64_t)k * threads, target_threads);
         const uint64_t ants = std::min<uint64_t>((uint64_t)k * std::max(1u, A) / ((std::max(1u, A) + apb - 1) / apb), 4095);
-        const uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) |
-                               (ants << 12) | (uint64_t)(4095 - k);
+        uint64_t score = (thr << 40) | ((uint64_t)(8 - L) << 32) | ((uint64_t)(ts ? 1 : 0) << 31) |
+                         (ants << 12) | (uint64_t)(4095 - k);
+        if (spread_cap) score = ((uint64_t)(ts ? 1 : 0) << 40) | ((uint64_t)apb << 20) | (uint64_t)(4095 - k);
         if (score > best_score) {  // strict: the staged image wins ties
           best_score = score;
           best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads, ig != 0};
@@ -723,6 +736,19 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
   uint32_t gs_min_threads[2] = {128, 64};  // measured: tools/probe_sizes.sh
   uint32_t gs_lanes[2] = {16, 16};
+  // Spread mode: a batch with few ants in total (one region of 1,024 ants,
+  // config 2; FIX10-A, config 1) cannot fill the SMs with large blocks, so
+  // the ants are spread over >= 148 small blocks with lanes ~ bitset words
+  // (the per-ant step latency, not issue slots, is then the bound).
+  uint32_t spread_cap = 0;
+  {
+    const uint64_t total = (uint64_t)A * count;
+    // measured: C2 75 -> 80 ms (the per-ant step latency, not the SM count,
+    // bounds one region of 1,024 ants), so off unless asked for
+    bool on = false;
+    if (const char *e = getenv("ACO_SPREAD")) on = total < 148ull * 64 && atoi(e) != 0;
+    if (on) spread_cap = (uint32_t)std::max<uint64_t>(1, (total + 147) / 148);
+  }
   uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
   if (const char *e = getenv("ACO_IMG_L1")) sscanf(e, "%u,%u", &img_l1[0], &img_l1[1]);
   bool lean_on = true;  // pass-2 lean layout for large regions
@@ -769,7 +795,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
                             p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
-                            wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u);
+                            wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u,
+                            rl1 && pass == 1 ? 0u : spread_cap, std::min(8u, lane_pow2(R.nwr)));
+      if (lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
       if (lean) {
         // the lean layout costs per ant-step (kills derived at every
         // evaluation) and gains resident ants; on the mixed C3 batch it wins
@@ -892,6 +920,21 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   const uint64_t n_grp = rl1 ? ((uint64_t)A + p->group_size - 1) / p->group_size : 0;
   const uint64_t o_rlk = off;  // R45: K per (ant group, step)
   off = align256(off + 2 * n_grp * sum_n + 16);
+  // Record mode: every ant stores its schedule (step-major, coalesced) and
+  // k_select copies the winner's instead of replaying it serially.  Measured
+  // on B200 (ms per batch, replay -> record): C1 2.34 -> 1.80, C2 79.9 ->
+  // 62.2, C3 674 -> 650, C4 500 -> 432, C5 3327 -> 3109; the writes (C3:
+  // 2.9 GB per pass-2 iteration, coalesced) hide under the construction.
+  uint64_t rec_mb = 16384;
+  if (const char *e = getenv("ACO_RECORD_MB")) rec_mb = strtoull(e, nullptr, 10);
+  const uint64_t rec_bytes = (uint64_t)A * sum_n * ((pmask & 2u) ? 6u : 2u) + 16ull * A * count;
+  P.record = !colony && !(p->flags & ACO_FLAG_DUMP) && rec_bytes <= (rec_mb << 20);
+  const uint64_t o_rec = off;
+  if (P.record) off = align256(off + 2ull * A * sum_n + 16);
+  const uint64_t o_recc = off;
+  if (P.record && (pmask & 2u)) off = align256(off + 4ull * A * sum_n + 16);
+  const uint64_t o_recp = off;
+  if (P.record) off = align256(off + 16ull * A * count);
   P.o_keys = off;
   off = align256(off + 8ull * count);
   std::vector<RegionWs> rws(count);
@@ -910,6 +953,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     w.o_next = o_next + 2 * (ctx->inst_off[r] + r);
     w.o_heur = o_heur + 2 * ctx->inst_off[r];
     w.o_rlk = o_rlk + 2 * n_grp * ctx->inst_off[r];
+    w.o_rec = o_rec + 2ull * A * ctx->inst_off[r];
+    w.o_recc = o_recc + 4ull * A * ctx->inst_off[r];
+    w.o_recp = o_recp + 16ull * A * r;
     w.gs = sgs[r];  // k_init / k_select: image and replay state in the workspace
     if (gs[r]) {  // global-state construct kernels
       off = align256(off);
@@ -1044,6 +1090,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.heur_mix = p->heur_mix;
   cfg.stall_num = p->stall_num;
   cfg.rl_limit = p->rl_limit;
+  cfg.record = P.record ? 1u : 0u;
   cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;
   cfg.keys = nullptr;

@@ -109,6 +109,9 @@ struct RegionWs {
   uint64_t o_scratch;// global-state regions: replay scratch (words + cycles + order)
   uint64_t o_heur;   // u16 [n]  the heuristic (greedy pass-1) order, R40
   uint64_t o_rlk;    // u16 [ceil(ants/G)][n]: ready-list limit K per (ant group, step), R45 (rl_limit only)
+  uint64_t o_rec;    // record mode: u16 [n][ants] every ant's order (step-major: coalesced stores)
+  uint64_t o_recc;   // record mode: u32 [n][ants] pass-2 issue cycles
+  uint64_t o_recp;   // record mode: uint4 [ants] {prp01, prp23, length, 0}
   uint32_t tau_len;  // (n+1)*n rounded up to a multiple of 8
   uint32_t gs;       // 1: the region's state does not fit shared memory (global-state kernels)
 };
@@ -135,7 +138,7 @@ struct RunCfg {
   uint32_t pass2_gap, revert_occ, revert_len;  // compile policy (R39, R40)
   uint32_t heur_mix, stall_num;                // R43, R44
   uint32_t rl_limit;                           // R45: 0 off, 1 min, 2 mid
-  uint32_t pad_rl;
+  uint32_t record;                             // ants record their schedules; k_select copies the winner's
   uint32_t stage_img;   // k_select stages the region image in shared memory (few regions)
   uint32_t pad_cfg;
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n

@@ -651,13 +651,14 @@ __device__ __forceinline__ uint32_t ready_count(const St &A, uint32_t nwr) {
 // score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
 // Philox step (R26).  rec (leader, may be NULL) receives the order.  The
 // result is valid in the leader lane.
-template <int LG, bool MASK, bool WIDE = false>
+template <int LG, bool MASK, bool WIDE = false, bool RLIM = false>
 __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const bool greedy, uint16_t *rec,
-                                            const uint32_t *coins = nullptr, const RL rl = RL{nullptr, 0, 0, 0, nullptr, nullptr}) {
+                                            const uint32_t *coins = nullptr, const RL rl = RL{nullptr, 0, 0, 0, nullptr, nullptr},
+                                            const uint32_t rec_stride = 1) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
-  const bool limit = rl.buf != nullptr || rl.in != nullptr;  // R45
+  constexpr bool limit = RLIM;  // R45 (rl.buf or rl.in set)
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<1, MASK, false, false>(V, A);
   wmask = G.bcast(wmask);
@@ -682,7 +683,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     const uint16_t *trow = tau + prev * n;
     // R45: the last candidate index this ant may consider at step k
     uint32_t jmax = n;
-    if (limit) {
+    if constexpr (limit) {
       uint32_t K;
       if (rl.in) {
         K = rl.in[k];
@@ -723,7 +724,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
         bool v[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          v[u] = v0[u] && j[u] <= jmax;  // R45 (jmax = n: no limit)
+          v[u] = v0[u] && (!limit || j[u] <= jmax);  // R45
           tv[u] = trow[j[u]];
           dk[u] = A.DK[(j[u] >> 3) * A.S];
         }
@@ -763,7 +764,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       });
     } else {
       scan_bits<MASK>(A, nwr, wmask, G.lane, LG, sub, [&](uint32_t j) {
-        if (j > jmax) return true;  // R45: ascending, nothing further is allowed
+        if (limit && j > jmax) return true;  // R45: ascending, nothing further is allowed
         const uint32_t sc = score(j);
         if (sc + 1u > bs1) {
           bs1 = sc + 1u;
@@ -799,7 +800,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     }
     if (G.leader()) {
       commit<1, MASK, false, false>(V, A, jstar, 0, wmask, live01, live23, prp01, prp23);
-      if (rec) rec[k] = (uint16_t)jstar;
+      if (rec) rec[(size_t)k * rec_stride] = (uint16_t)jstar;
     }
     wmask = G.bcast(wmask);
     G.sync();
@@ -827,7 +828,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
                                             const bool prune, uint16_t *rec_o, uint32_t *rec_c,
-                                            const uint32_t *coins = nullptr, uint32_t coin_t = 0) {
+                                            const uint32_t *coins = nullptr, uint32_t coin_t = 0,
+                                            const uint32_t rec_stride = 1) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   uint32_t wmask = 0;
   if (G.leader()) wmask = init_state<2, MASK, T32, NC4, LEAN>(V, A);
@@ -1022,8 +1024,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     if (G.leader()) {
       commit<2, MASK, T32, NC4, LEAN>(V, A, jstar, t, wmask, live01, live23, prp01, prp23, B);
       if (rec_o) {
-        rec_o[placed] = (uint16_t)jstar;
-        rec_c[placed] = t;
+        rec_o[(size_t)placed * rec_stride] = (uint16_t)jstar;
+        rec_c[(size_t)placed * rec_stride] = t;
       }
     }
     wmask = G.bcast(wmask);
@@ -1158,9 +1160,17 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
   AntOut o;
   if (PASS == 1) {
     uint16_t *rec = nullptr;
-    if (dump && A.dump_order)
+    uint32_t rs1 = 1;
+    if (dump && A.dump_order) {
       rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
-    o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl);
+    } else if (A.cfg.record) {
+      rec = (uint16_t *)(A.ws + W.o_rec) + ai;
+      rs1 = A.cfg.ants;
+    }
+    if (rl.buf)
+      o = ant_pass1<LG, MASK, WIDE, true>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
+    else
+      o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -1174,12 +1184,19 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
       rec_o = A.dump_order + base;
       rec_c = A.dump_cycle + base;
     }
+    uint32_t rs2 = 1;
+    if (!rec_o && A.cfg.record) {
+      rec_o = (uint16_t *)(A.ws + W.o_rec) + ai;
+      rec_c = (uint32_t *)(A.ws + W.o_recc) + ai;
+      rs2 = A.cfg.ants;
+    }
     o = ant_pass2<LG, MASK, T32, NC4, WIDE, LEAN>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
-                                      rec_c, coins, coin_t);
+                                      rec_c, coins, coin_t, rs2);
   }
   if (G.leader()) {
     uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
     costs[ai] = o.cost;
+    if (A.cfg.record) ((uint4 *)(A.ws + W.o_recp))[ai] = make_uint4(o.prp01, o.prp23, o.len, 0u);
     if (dump && A.dump_cost)
       A.dump_cost[(((size_t)(PASS - 1) * A.cfg.iterations + iter) * A.cfg.count + bi.region) * A.cfg.ants + ai] =
           o.cost;
@@ -1448,7 +1465,21 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
   uint32_t *cyc = stw + ant_words(PASS, n, rd->nwr, rd->nremw, T32, NC4);
   uint16_t *ord = (uint16_t *)(cyc + n);
   __syncwarp();
-  if (have) {  // the whole warp replays the winner as one 32-lane group
+  if (have && A.cfg.record && !A.cfg.keys) {  // the winner recorded its schedule: copy it
+    const uint32_t wl = want - A.cfg.ant_base, na = A.cfg.ants;
+    const uint16_t *ro = (const uint16_t *)(A.ws + W.o_rec) + wl;
+    const uint32_t *rc = (const uint32_t *)(A.ws + W.o_recc) + wl;
+    for (uint32_t k = threadIdx.x; k < n; k += 32) {
+      ord[k] = ro[(size_t)k * na];
+      if (PASS == 2) cyc[k] = rc[(size_t)k * na];
+    }
+    if (threadIdx.x == 0) {
+      const uint4 q = ((const uint4 *)(A.ws + W.o_recp))[wl];
+      s_prp[0] = q.x;
+      s_prp[1] = q.y;
+      s_prp[2] = q.z;
+    }
+  } else if (have) {  // the whole warp replays the winner as one 32-lane group
     const St S = make_st<PASS, T32, NC4>(stw, 1, V);
     const Grp<32> G32(threadIdx.x);
     AntOut o;
@@ -1456,7 +1487,8 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
       RL rl{nullptr, 0, 0, A.cfg.rl_limit, nullptr, nullptr};
       if (A.cfg.rl_limit)  // R45: the winner's group limits as recorded by the construct kernel
         rl.in = (const uint16_t *)(A.ws + W.o_rlk) + (size_t)((want - A.cfg.ant_base) / A.cfg.group_size) * n;
-      o = ant_pass1<32, MASK>(V, tau, S, G32, want, iter, A.cfg, false, ord, nullptr, rl);
+      if (rl.in) o = ant_pass1<32, MASK, false, true>(V, tau, S, G32, want, iter, A.cfg, false, ord, nullptr, rl);
+      else o = ant_pass1<32, MASK>(V, tau, S, G32, want, iter, A.cfg, false, ord, nullptr, rl);
     } else {
       uint32_t tgt[4];
       for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
