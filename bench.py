@@ -336,17 +336,20 @@ def main():
         if bpas is not None and construct_ms > 0:
             n_launch = phase_launches[0] / max(1, args.steps)
             achieved = bpas * ant_steps / (construct_ms / 1000.0) / 1e9
-            traffic, tsrc = None, None
+            traffic, tsrc, issue = None, None, None
             try:  # DRAM bytes per construct launch from the committed ncu --set full capture
                 with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
                     tj = json.load(f)
                 if args.workload == "c3":
                     traffic, tsrc = tj["dram_bytes_per_launch"], tj["source"]
+                    # the bound that actually binds: SM issue slots, from ncu
+                    issue = {"util_pct": tj.get("issue_util_pct"), "warps_active_pct": tj.get("warps_active_pct"),
+                             "source": tj.get("issue_source")}
             except Exception:
                 pass
             roof = {"bound": "smem", "achieved": round(achieved, 1), "peak": round(smem_peak, 1),
                     "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": traffic,
-                    "traffic_source": tsrc,
+                    "traffic_source": tsrc, "issue_slots_ncu": issue,
                     "algorithmic_bytes_per_launch": round(bpas * ant_steps / max(1.0, n_launch)),
                     "kernel": "k_construct (all classes)", "bytes_per_ant_step": round(bpas, 2),
                     "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,
