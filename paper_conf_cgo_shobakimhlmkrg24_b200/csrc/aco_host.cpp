@@ -1164,7 +1164,12 @@ int run_construct(aco_ctx ctx, uint32_t pass, uint32_t it) {
   if (cls.size() <= 1) {
     for (const ClassLaunch &cl : cls) err |= launch_construct(L, pass, it, cl);
   } else {  // fork: classes round-robin over the internal streams, join on the main stream
-    const int k = (int)std::min<size_t>(cls.size(), aco_ctx_s::kStreams);
+    static const int ks = [] {  // fork streams (A/B knob; 4 measured best, 8: C5 3109 -> 3996 ms)
+      const char *e = getenv("ACO_STREAMS");
+      const int v = e ? atoi(e) : aco_ctx_s::kStreams;
+      return std::max(1, std::min(v, aco_ctx_s::kStreams));
+    }();
+    const int k = (int)std::min<size_t>(cls.size(), (size_t)ks);
     err |= cudaEventRecord(ctx->fork_ev, s) != cudaSuccess;
     for (int i = 0; i < k; ++i) err |= cudaStreamWaitEvent(ctx->side[i], ctx->fork_ev, 0) != cudaSuccess;
     for (size_t c = 0; c < cls.size(); ++c) {
