@@ -6,7 +6,7 @@ run() {  # name, args...
   timeout 900 python bench.py --steps 3 --warmup 3 "$@" 2>gpurun_out/bench_$name.err | tail -1 > gpurun_out/bench_$name.json
   echo "== $name: $(cut -c1-160 gpurun_out/bench_$name.json)"
 }
-for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix rlmin}; do
+for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix rlmin rlmid}; do
   case $w in
     c1|c2|c3|c4|c5) run $w --workload $w ;;
     dual) run c3_dual --machine dual ;;
