@@ -748,7 +748,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     bool on = false;
     if (const char *e = getenv("ACO_SPREAD")) on = total < 148ull * 64 && atoi(e) != 0;
     if (on) spread_cap = (uint32_t)std::max<uint64_t>(1, (total + 147) / 148);
+    if (const char *e = getenv("ACO_SPREAD_CAP")) spread_cap = on ? (uint32_t)atoi(e) : 0u;
   }
+  uint32_t spread_lanes = 0;  // 0: lanes ~ bitset words
+  if (const char *e = getenv("ACO_SPREAD_LANES")) spread_lanes = (uint32_t)atoi(e);
   uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
   if (const char *e = getenv("ACO_IMG_L1")) sscanf(e, "%u,%u", &img_l1[0], &img_l1[1]);
   bool lean_on = true;  // pass-2 lean layout for large regions
@@ -796,7 +799,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                             pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
                             p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
                             wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u,
-                            rl1 && pass == 1 ? 0u : spread_cap, std::min(8u, lane_pow2(R.nwr)));
+                            rl1 && pass == 1 ? 0u : spread_cap, spread_lanes ? spread_lanes : std::min(8u, lane_pow2(R.nwr)));
       if (lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
       if (lean) {
         // the lean layout costs per ant-step (kills derived at every
