@@ -93,3 +93,50 @@ def test_too_large_region(lib):
     big = I.Region.from_lists(n, [], [], [], [[] for _ in range(n)], [[] for _ in range(n)])
     st, _ = _size_status(lib, [big])
     assert st == -5
+
+
+def _plan_status(lib, regions, p, colony=False):
+    """Sizing calls only (NULL arena / workspace): no CUDA call is made
+    (ACO_DEBUG_PLAN keeps the host metadata of a sizing-only load and prints
+    the launch plan to stderr)."""
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch, params_struct
+    os.environ["ACO_DEBUG_PLAN"] = "1"
+    ctx, m = _ctx(lib)
+    b = HostBatch(regions, list(range(len(regions))))
+    need = C.c_size_t(0)
+    assert lib.aco_load_regions(ctx, b.descs, len(regions), None, 0, C.byref(need), None) == 0
+    ps = params_struct(p)
+    ws = C.c_size_t(0)
+    if colony:
+        st = lib.aco_colony_begin(ctx, C.byref(ps), 0, None, 0, C.byref(ws), None)
+    else:
+        st = lib.aco_schedule_batch(ctx, C.byref(ps), None, 0, C.byref(ws), None)
+    lib.aco_destroy(ctx)
+    del os.environ["ACO_DEBUG_PLAN"]
+    return st, ws.value
+
+
+def test_ready_list_limit_params(lib):
+    """R45: modes 0-2 plan; 3 is rejected; the shared colony rejects any
+    limit (a wavefront would span ranks)."""
+    regs = I.gen_batch(6, base_seed=5)
+    for mode in (0, 1, 2):
+        assert _plan_status(lib, regs, I.Params(ants=128, iterations=2, rl_limit=mode))[0] == 0
+    assert _plan_status(lib, regs, I.Params(ants=128, iterations=2, rl_limit=3))[0] == -1
+    assert _plan_status(lib, regs, I.Params(ants=128, iterations=2, rl_limit=1), colony=True)[0] == -1
+    assert _plan_status(lib, regs, I.Params(ants=128, iterations=2), colony=True)[0] == 0
+
+
+def test_record_mode_workspace(lib, monkeypatch):
+    """Record mode (winner copied, not replayed) adds exactly the recorded
+    schedules to the workspace: A x sum(n) x (2 + 4) bytes (order u16, pass-2
+    cycles u32) plus A x 16 bytes per region, up to 256-byte alignment."""
+    regs = I.gen_batch(12, base_seed=6)
+    p = I.Params(ants=256, iterations=2)
+    monkeypatch.setenv("ACO_RECORD_MB", "0")
+    st0, ws0 = _plan_status(lib, regs, p)
+    monkeypatch.setenv("ACO_RECORD_MB", "16384")
+    st1, ws1 = _plan_status(lib, regs, p)
+    assert st0 == st1 == 0
+    want = p.ants * sum(r.n_insts for r in regs) * 6 + 16 * p.ants * len(regs)
+    assert want <= ws1 - ws0 <= want + 3 * 256 + 3 * 16
