@@ -730,7 +730,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   std::map<Key, Cls> classes;
   P.nc4 = ctx->mach.n_classes > 2;
   // launch-shape policy (tuning knobs; defaults measured on B200)
-  uint32_t tgt_threads[2] = {512, 768}, max_lanes[2] = {8, 1};
+  uint32_t tgt_threads[2] = {384, 768}, max_lanes[2] = {8, 1};  // pass 1: 384 (C3 320/384/448/512: 615/615/625/625 ms)
   if (const char *e = getenv("ACO_TARGET_THREADS")) sscanf(e, "%u,%u", &tgt_threads[0], &tgt_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES")) sscanf(e, "%u,%u", &max_lanes[0], &max_lanes[1]);
   uint32_t max_lanes_w[2] = {max_lanes[0], max_lanes[1]};  // wide (large-region) classes
