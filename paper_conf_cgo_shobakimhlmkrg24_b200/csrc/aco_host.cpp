@@ -758,6 +758,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_LEAN")) lean_on = atoi(e) != 0;
   uint32_t lean_gain = 0;  // % more resident ants the lean layout must reach (C3: 0 measured best)
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
+  const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
@@ -770,6 +771,33 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     if (!s_mt_ok[dv]) s_mt_ok[dv] = construct_max_threads(ctx->device, s_mt[dv]) == 0;
     if (s_mt_ok[dv]) std::memcpy(mt, s_mt[dv], sizeof(mt));
     else construct_max_threads(-2, mt);  // conservative defaults (no device: sizing only)
+  }
+  // Lanes per ant of the global-state (huge-region) kernels: enough lanes to
+  // fill the SMs when few ants take that path (config 4: one region, 8,192
+  // ants -> 16 lanes), fewer when many do (config 5: every n >= ~1,500 region
+  // -> 4 lanes): ~148 x 1,024 threads in flight.  Measured (ms): C4 16/8/4
+  // lanes 423/583/827, C5 2,961/2,529/2,328.
+  if (!gs_lanes_env) {
+    uint64_t gs_ants[2] = {0, 0};
+    for (uint32_t r = 0; r < count; ++r) {
+      const RegionDev &R = ctx->regions[r];
+      if (R.n <= 600) continue;  // (host time: smaller regions always fit shared memory)
+      const bool t32 = ctx->mach.issue_width > 1 ||
+                       (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
+      for (uint32_t pass = 1; pass <= 2; ++pass) {
+        if (!(pmask & pass)) continue;
+        const bool wide = R.n >= kWideN && R.n <= 1024, rare = pass == 2 && (t32 || P.nc4);
+        const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
+        const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
+                                    pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1],
+                                    A, p->group_size, coin_words(pass, R.n));
+        if (sh.apb == 0 || sh.resident < gs_min_threads[pass - 1]) gs_ants[pass - 1] += A;
+      }
+    }
+    for (int q = 0; q < 2; ++q) {
+      const uint64_t per = gs_ants[q] ? (148ull * 1024) / gs_ants[q] : 16;
+      gs_lanes[q] = per >= 16 ? 16u : (per >= 8 ? 8u : 4u);
+    }
   }
   std::vector<uint8_t> gs(count, 0);
   std::vector<uint32_t> gs_words(count, 0), scratch_words(count, 0);
