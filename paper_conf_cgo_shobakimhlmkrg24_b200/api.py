@@ -9,6 +9,7 @@ hot path runs in the CUDA library).  PyTorch provides device memory and streams.
 from __future__ import annotations
 
 import ctypes as C
+import dataclasses
 from typing import List, Optional, Sequence
 
 import numpy as np
@@ -86,6 +87,7 @@ class Scheduler:
         self.ws: Optional[torch.Tensor] = None
         self.batch: Optional[HostBatch] = None
         self.count = 0
+        self._need = {}  # workspace bytes per (params, flags) for the loaded regions
         self.params: Optional[Params] = None
         self.dump = None
 
@@ -118,6 +120,7 @@ class Scheduler:
                                            self.arena.numel(), C.byref(need), sh)
         _lib.check(st, "aco_load_regions")
         self.batch = b
+        self._need = {}
         self.count = len(regions)
         return self
 
@@ -155,7 +158,11 @@ class Scheduler:
                      (self.params.ants, self.params.iterations) != (p.ants, p.iterations) or
                      self.dump[0].shape[2] != self.count):
             self.set_dump(p)
-        need = self.workspace_bytes(p, flags)
+        key = (dataclasses.astuple(p), flags)
+        need = self._need.get(key)
+        if need is None:  # sizing call (host planning) only for new parameters or regions
+            need = self.workspace_bytes(p, flags)
+            self._need[key] = need
         if self.ws is None or self.ws.numel() < need:
             self.ws = torch.empty(max(256, need), dtype=torch.uint8, device=f"cuda:{self.device}")
         ps = params_struct(p, flags)

@@ -35,6 +35,16 @@ struct aco_ctx_s {
   int device = 0;
   Plan plan;
   bool planned = false;
+  // plan cache: a run with the same parameters, workspace and loaded regions
+  // as the previous one reuses its plan (launch classes, workspace layout and
+  // the plan blob already in the workspace) -- ~11 ms of host time on C3
+  bool cache_ok = false;
+  aco_params cache_params{};
+  void *cache_ws = nullptr;
+  size_t cache_ws_bytes = 0, cache_need = 0;
+  uint32_t cache_ant_base = 0;
+  bool cache_colony = false;
+  const void *cache_dump[3] = {nullptr, nullptr, nullptr};
   MachineDev mach{};
   bool machine_uploaded = false;
   // loaded batch
@@ -526,6 +536,7 @@ void aco_destroy(aco_ctx ctx) { delete ctx; }
 aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_t count, void *d_arena,
                             size_t arena_bytes, size_t *arena_needed, void *cuda_stream) {
   if (!ctx || (count && !regions)) return ACO_E_ARG;
+  ctx->cache_ok = false;
   {  // unique region ids
     std::vector<uint32_t> ids(count);
     for (uint32_t i = 0; i < count; ++i) ids[i] = regions[i].region_id;
@@ -708,6 +719,25 @@ aco_status check_params(const aco_params *p) {
 aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *d_workspace, size_t ws_bytes,
                      size_t *ws_needed, void *cuda_stream, bool colony) {
   if (aco_status st = check_params(p)) return st;
+  if (d_workspace && ctx->cache_ok && std::memcmp(p, &ctx->cache_params, sizeof(aco_params)) == 0 &&
+      d_workspace == ctx->cache_ws && ws_bytes == ctx->cache_ws_bytes && ant_base == ctx->cache_ant_base &&
+      colony == ctx->cache_colony && ctx->cache_dump[0] == ctx->dump_cost &&
+      ctx->cache_dump[1] == ctx->dump_order && ctx->cache_dump[2] == ctx->dump_cycle) {
+    Plan &P = ctx->plan;  // same run again: the plan and its blob in the workspace are current
+    if (ws_needed) *ws_needed = ctx->cache_need;
+    P.L.stream = cuda_stream;
+    P.L.launches = 0;
+    ctx->ev_used = 0;
+    for (int ph = 0; ph < 3; ++ph) {
+      ctx->ev_pairs[ph].clear();
+      ctx->phase_launches[ph] = 0;
+    }
+    ctx->stream = cuda_stream;
+    ctx->have_run = true;
+    ctx->planned = true;
+    return ACO_OK;
+  }
+  if (d_workspace) ctx->cache_ok = false;  // (a sizing call leaves the cached plan intact)
   if ((p->flags & ACO_FLAG_DUMP) && (!ctx->dump_cost || colony)) return ACO_E_ARG;
   // passes that run construct/finalize launches: pass 4 (weighted, R41) uses the pass-2 machinery
   const uint32_t pmask = p->pass == 4 ? 2u : p->pass;
@@ -1145,6 +1175,16 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   ctx->o_gb2c = P.o_gb2c;
   ctx->have_run = true;
   ctx->planned = true;
+  ctx->cache_ok = !getenv("ACO_NO_PLAN_CACHE");
+  ctx->cache_params = *p;
+  ctx->cache_ws = d_workspace;
+  ctx->cache_ws_bytes = ws_bytes;
+  ctx->cache_need = need;
+  ctx->cache_ant_base = ant_base;
+  ctx->cache_colony = colony;
+  ctx->cache_dump[0] = ctx->dump_cost;
+  ctx->cache_dump[1] = ctx->dump_order;
+  ctx->cache_dump[2] = ctx->dump_cycle;
   return ACO_OK;
 }
 

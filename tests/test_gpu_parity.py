@@ -406,3 +406,20 @@ def test_ready_list_limit_production(torch_cuda):
     got = s.results()
     for k in range(len(regs)):
         compare_results(got[k], O.schedule(regs[k], ids[k], I.GFX906, p), f"region {k}")
+
+
+def test_plan_cache_reruns(torch_cuda):
+    """Re-running a context with the same parameters reuses its plan (host
+    planning skipped); changing a parameter re-plans.  Every run equals the
+    oracle for its parameters."""
+    regs = [I.gen_region(n, 2000 + n) for n in (35, 120, 260)]
+    ids = [101, 102, 103]
+    pa = I.Params(ants=128, iterations=3, seed=51)
+    pb = I.Params(ants=128, iterations=3, seed=52, cost_mode=0)
+    s = _sched()
+    s.load(regs, ids)
+    for p in (pa, pa, pb, pa, pb):
+        s.run(p)
+        got = s.results()
+        for k in range(len(regs)):
+            compare_results(got[k], O.schedule(regs[k], ids[k], I.GFX906, p), f"region {k} seed {p.seed}")
