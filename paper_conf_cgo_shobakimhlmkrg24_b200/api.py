@@ -160,13 +160,25 @@ class Scheduler:
             self.set_dump(p)
         key = (dataclasses.astuple(p), flags)
         need = self._need.get(key)
-        if need is None:  # sizing call (host planning) only for new parameters or regions
-            need = self.workspace_bytes(p, flags)
-            self._need[key] = need
-        if self.ws is None or self.ws.numel() < need:
-            self.ws = torch.empty(max(256, need), dtype=torch.uint8, device=f"cuda:{self.device}")
         ps = params_struct(p, flags)
         n = C.c_size_t(0)
+        if need is None and self.ws is not None:
+            # new parameters or regions: try the workspace we have -- the library
+            # plans once and reports the size it needs if it is too small
+            st = self.lib.aco_schedule_batch(self.ctx, C.byref(ps), C.c_void_p(self.ws.data_ptr()),
+                                             self.ws.numel(), C.byref(n), _stream_handle(stream))
+            if st == 0:
+                self._need[key] = int(n.value)
+                self.params = p
+                return self
+            if st != _lib.ACO_E_WORKSPACE:
+                _lib.check(st, "aco_schedule_batch")
+            need = int(n.value)
+        if need is None:  # sizing call (host planning)
+            need = self.workspace_bytes(p, flags)
+        self._need[key] = need
+        if self.ws is None or self.ws.numel() < need:
+            self.ws = torch.empty(max(256, need), dtype=torch.uint8, device=f"cuda:{self.device}")
         _lib.check(self.lib.aco_schedule_batch(self.ctx, C.byref(ps), C.c_void_p(self.ws.data_ptr()),
                                                self.ws.numel(), C.byref(n), _stream_handle(stream)),
                    "aco_schedule_batch")
