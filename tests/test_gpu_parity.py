@@ -416,9 +416,10 @@ def test_plan_cache_reruns(torch_cuda):
     ids = [101, 102, 103]
     pa = I.Params(ants=128, iterations=3, seed=51)
     pb = I.Params(ants=128, iterations=3, seed=52, cost_mode=0)
+    pc = I.Params(ants=320, iterations=2, seed=53)  # a larger workspace: the binding re-sizes it
     s = _sched()
     s.load(regs, ids)
-    for p in (pa, pa, pb, pa, pb):
+    for p in (pa, pa, pb, pa, pc, pb, pc):
         s.run(p)
         got = s.results()
         for k in range(len(regs)):
