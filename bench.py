@@ -202,12 +202,21 @@ def cpu_sample_params(args, p):
     return p, "full A x I x passes"
 
 
-def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes"):
-    """The oracle as it stands on a bounded, stratified sample of the same workload."""
-    from oracle import pyoracle as O
+def stratified_pick(regs, sample: int):
+    """Indices of a size-stratified sample, largest region first (the oracle's
+    thread pool takes regions in the order given: largest first keeps one big
+    region from running alone at the end; per-region results do not depend on it)."""
     k = min(sample, len(regs))
     order = np.argsort([r.n_insts for r in regs], kind="stable")
-    pick = sorted(set(int(order[int(i)]) for i in np.linspace(0, len(regs) - 1, k)))
+    pick = set(int(order[int(i)]) for i in np.linspace(0, len(regs) - 1, k))
+    return sorted(pick, key=lambda i: (-regs[i].n_insts, i))
+
+
+def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes", pick=None):
+    """The oracle as it stands on a bounded, stratified sample of the same workload."""
+    from oracle import pyoracle as O
+    if pick is None:
+        pick = stratified_pick(regs, sample)
     sub = [regs[i] for i in pick]
     sid = [ids[i] for i in pick]
     threads = os.cpu_count() or 1
@@ -392,8 +401,12 @@ def reference_arm(args, world, rank):
     ps, note = cpu_sample_params(args, p)
     for _ in range(args.warmup):
         pass  # the oracle has no warm-up state
-    for _ in range(args.steps):
-        cpu, stats = cpu_baseline(regs, ids, ps, max(4, args.cpu_sample // max(1, args.steps)), machine_of(args), note)
+    # the --cpu-sample stratified sample, dealt round-robin over the steps
+    # (each step a smaller stratified sample, largest region first)
+    full = stratified_pick(regs, max(args.cpu_sample, 4 * args.steps))
+    per_step = [full[s::args.steps] or full for s in range(args.steps)]
+    for s in range(args.steps):
+        cpu, stats = cpu_baseline(regs, ids, ps, 0, machine_of(args), note, pick=per_step[s])
         from oracle.pyoracle import ORS
         s = float(stats[:, ORS["ant_scheds"]].sum())
         scheds += s
@@ -405,8 +418,8 @@ def reference_arm(args, world, rank):
            "scaling": "strong" if args.workload == "c4" else "weak", "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
            "data": "synthetic", "config": cfg, "impl": "reference",
            "cpu_baseline": {"value": round(value, 1), "unit": METRIC, "cores": os.cpu_count(), "kind": "oracle",
-                            "sample": f"per step a stratified sample of {max(4, args.cpu_sample // max(1, args.steps))} "
-                                      f"regions of the {cfg['workload']} workload"},
+                            "sample": f"per step about {max(1, len(full) // args.steps)} regions (a stratified sample of "
+                                      f"{len(full)} dealt over the steps, largest first) of the {cfg['workload']} workload, {note}"},
            "e2e": {"value": round(value, 1), "unit": METRIC, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
     return out
