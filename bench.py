@@ -212,6 +212,12 @@ def stratified_pick(regs, sample: int):
     return sorted(pick, key=lambda i: (-regs[i].n_insts, i))
 
 
+def deal_over_steps(full, steps: int):
+    """Round-robin the sample over the steps (a sample smaller than the step
+    count is reused whole by the steps it does not reach)."""
+    return [full[s::steps] or full for s in range(steps)]
+
+
 def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes", pick=None):
     """The oracle as it stands on a bounded, stratified sample of the same workload."""
     from oracle import pyoracle as O
@@ -404,7 +410,7 @@ def reference_arm(args, world, rank):
     # the --cpu-sample stratified sample, dealt round-robin over the steps
     # (each step a smaller stratified sample, largest region first)
     full = stratified_pick(regs, max(args.cpu_sample, 4 * args.steps))
-    per_step = [full[s::args.steps] or full for s in range(args.steps)]
+    per_step = deal_over_steps(full, args.steps)
     for s in range(args.steps):
         cpu, stats = cpu_baseline(regs, ids, ps, 0, machine_of(args), note, pick=per_step[s])
         from oracle.pyoracle import ORS
