@@ -169,12 +169,16 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
 aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_result *out,
                            uint32_t *orders, uint32_t *cycles);
 
-/* Dump buffers for ACO_FLAG_DUMP (device pointers, caller-owned):
+/* Dump buffers for ACO_FLAG_DUMP (device pointers, caller-owned), with their
+ * sizes in ELEMENTS:
  *   costs : u32 [2][iterations][count][ants]            (INVALID = 0xFFFFFFFF)
  *   orders: u16 [2][iterations][sum over regions of ants * n]   (may be NULL)
  *   cycles: u32 same shape as orders, pass-2 issue cycles       (may be NULL)
- * Region r's block in a (pass, iteration) slice starts at ants * sum_{q<r} n_q. */
-aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint32_t *d_cycles);
+ * Region r's block in a (pass, iteration) slice starts at ants * sum_{q<r} n_q.
+ * aco_schedule_batch with ACO_FLAG_DUMP returns ACO_E_WORKSPACE when a given
+ * buffer is smaller than the loaded batch and parameters need. */
+aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint64_t costs_len, uint16_t *d_orders,
+                        uint64_t orders_len, uint32_t *d_cycles, uint64_t cycles_len);
 
 /* ---- Shared colony (config 4): the ants of the loaded regions are split
  * across ranks (one context per GPU).  Ant ids are global: this context runs

@@ -11,7 +11,7 @@
  * instruction scheduling of one basic-block DDG, in the two-pass form of
  * Shobaki et al., "Instruction Scheduling for the GPU on the GPU", CGO 2024
  * (PAPER.md L106-L164, L198-L206, L226), with every point the paper leaves
- * open fixed by the readings R1..R40 listed in DESIGN.md section 3.
+ * open fixed by the readings R1..R45 listed in DESIGN.md section 3.
  */
 #ifndef ACO_ORACLE_H
 #define ACO_ORACLE_H

@@ -15,6 +15,7 @@ if os.environ.get("ACO_LIB_VARIANT"):  # A/B builds of the same sources (tools/,
 
 ACO_OK = 0
 ACO_E_WORKSPACE = -6
+ACO_E_STATE = -8
 ACO_FLAG_NO_PRUNE = 1
 ACO_FLAG_DUMP = 2
 ACO_FLAG_TIMING = 4
@@ -84,12 +85,12 @@ def load(path: str = LIB_PATH):
             f"{path} is missing: build it with `python -m paper_conf_cgo_shobakimhlmkrg24_b200.build` "
             "(there is no CPU fallback)")
     L = C.CDLL(path)
-    vp, u32, sz = C.c_void_p, C.c_uint32, C.c_size_t
+    vp, u32, u64, sz = C.c_void_p, C.c_uint32, C.c_uint64, C.c_size_t
     L.aco_create.argtypes = [C.c_int, vp, C.POINTER(vp)]
     L.aco_load_regions.argtypes = [vp, vp, u32, vp, sz, C.POINTER(sz), vp]
     L.aco_schedule_batch.argtypes = [vp, vp, vp, sz, C.POINTER(sz), vp]
     L.aco_get_results.argtypes = [vp, u32, u32, vp, vp, vp]
-    L.aco_set_dump.argtypes = [vp, vp, vp, vp]
+    L.aco_set_dump.argtypes = [vp, vp, u64, vp, u64, vp, u64]
     L.aco_last_launch_count.argtypes = [vp, C.POINTER(C.c_uint64)]
     L.aco_get_timing.argtypes = [vp, vp, vp]
     L.aco_colony_begin.argtypes = [vp, vp, u32, vp, sz, C.POINTER(sz), vp]

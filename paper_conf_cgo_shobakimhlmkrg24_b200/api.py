@@ -90,6 +90,7 @@ class Scheduler:
         self._need = {}  # workspace bytes per (params, flags) for the loaded regions
         self.params: Optional[Params] = None
         self.dump = None
+        self.dump_key = None
 
     def __del__(self):
         try:
@@ -122,6 +123,7 @@ class Scheduler:
         self.batch = b
         self._need = {}
         self.count = len(regions)
+        self.dump = None  # dump buffers are sized for the loaded batch (sum of n)
         return self
 
     # ---------------------------------------------------------------- run
@@ -145,18 +147,19 @@ class Scheduler:
             od = torch.zeros(size, dtype=torch.int16, device=dev)
             cy = torch.zeros(size, dtype=torch.int32, device=dev)
         self.dump = (costs, od, cy)
-        _lib.check(self.lib.aco_set_dump(self.ctx, C.c_void_p(costs.data_ptr()),
+        self.dump_key = (p.ants, p.iterations)
+        _lib.check(self.lib.aco_set_dump(self.ctx, C.c_void_p(costs.data_ptr()), costs.numel(),
                                          C.c_void_p(od.data_ptr()) if od is not None else None,
-                                         C.c_void_p(cy.data_ptr()) if cy is not None else None),
+                                         od.numel() if od is not None else 0,
+                                         C.c_void_p(cy.data_ptr()) if cy is not None else None,
+                                         cy.numel() if cy is not None else 0),
                    "aco_set_dump")
 
     def run(self, p: Params, stream: Optional[torch.cuda.Stream] = None, no_prune: bool = False,
             dump: bool = False, timing: bool = False):
         flags = ((_lib.ACO_FLAG_NO_PRUNE if no_prune else 0) | (_lib.ACO_FLAG_DUMP if dump else 0)
                  | (_lib.ACO_FLAG_TIMING if timing else 0))
-        if dump and (self.dump is None or self.params is None or
-                     (self.params.ants, self.params.iterations) != (p.ants, p.iterations) or
-                     self.dump[0].shape[2] != self.count):
+        if dump and (self.dump is None or self.dump_key != (p.ants, p.iterations)):
             self.set_dump(p)
         key = (dataclasses.astuple(p), flags)
         need = self._need.get(key)

@@ -11,6 +11,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <mutex>
 #include <new>
 #include <thread>
 #include <tuple>
@@ -19,6 +20,57 @@
 #include "aco_internal.h"
 
 using namespace aco;
+
+// Machine slots per device (c_mach[kMachSlots] in aco_kernels.cu): contexts
+// with the same machine share a slot; a slot is rewritten only when no live
+// context holds it (after a device synchronisation), so contexts with
+// different machines can run on one device in any order.
+namespace {
+constexpr int kMaxDevices = 64;
+struct MachineSlots {
+  std::mutex mu;
+  MachineDev m[kMaxDevices][kMachSlots]{};
+  uint32_t refs[kMaxDevices][kMachSlots]{};
+  bool written[kMaxDevices][kMachSlots]{};
+  bool attrs[kMaxDevices]{};
+};
+MachineSlots &machine_slots() {
+  static MachineSlots s;
+  return s;
+}
+// Bind a machine to a slot of `device` (the current device); -1 on failure.
+int acquire_machine_slot(int device, const MachineDev &m) {
+  if (device < 0 || device >= kMaxDevices) return -1;
+  MachineSlots &S = machine_slots();
+  std::lock_guard<std::mutex> lk(S.mu);
+  if (!S.attrs[device]) {
+    if (init_kernel_attrs() != 0) return -1;
+    S.attrs[device] = true;
+  }
+  for (uint32_t k = 0; k < kMachSlots; ++k)
+    if (S.written[device][k] && std::memcmp(&S.m[device][k], &m, sizeof(m)) == 0) {
+      S.refs[device][k]++;
+      return (int)k;
+    }
+  for (uint32_t k = 0; k < kMachSlots; ++k)
+    if (S.refs[device][k] == 0) {
+      // kernels of a destroyed context may still read this slot
+      if (S.written[device][k] && cudaDeviceSynchronize() != cudaSuccess) return -1;
+      if (set_machine(k, m) != 0) return -1;
+      S.m[device][k] = m;
+      S.written[device][k] = true;
+      S.refs[device][k] = 1;
+      return (int)k;
+    }
+  return -1;  // more than kMachSlots distinct machines live on this device
+}
+void release_machine_slot(int device, int slot) {
+  if (device < 0 || device >= kMaxDevices || slot < 0) return;
+  MachineSlots &S = machine_slots();
+  std::lock_guard<std::mutex> lk(S.mu);
+  if (S.refs[device][slot]) S.refs[device][slot]--;
+}
+}  // namespace
 
 // A planned run: launch classes, workspace offsets and the launch context.
 struct Plan {
@@ -46,7 +98,7 @@ struct aco_ctx_s {
   bool cache_colony = false;
   const void *cache_dump[3] = {nullptr, nullptr, nullptr};
   MachineDev mach{};
-  bool machine_uploaded = false;
+  int mslot = -1;  // machine slot on `device` (acquire_machine_slot)
   // loaded batch
   uint32_t count = 0;
   std::vector<RegionDev> regions;  // host copy (offsets valid in the arena)
@@ -62,6 +114,7 @@ struct aco_ctx_s {
   bool have_run = false;
   uint64_t launches = 0;
   uint32_t *dump_cost = nullptr;
+  uint64_t dump_len[3] = {0, 0, 0};  // elements of the dump buffers (costs, orders, cycles)
   uint16_t *dump_order = nullptr;
   uint32_t *dump_cycle = nullptr;
   std::vector<unsigned char> plan_blob;  // host staging of RegionWs + BlockItems
@@ -91,6 +144,7 @@ struct aco_ctx_s {
     return true;
   }
   ~aco_ctx_s() {
+    release_machine_slot(device, mslot);
     for (int i = 0; i < kStreams; ++i) {
       if (side[i]) cudaStreamDestroy(side[i]);
       if (join_ev[i]) cudaEventDestroy(join_ev[i]);
@@ -600,11 +654,16 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   ctx->arena = (unsigned char *)d_arena;
   ctx->arena_bytes = arena_bytes;
   ctx->have_run = false;
+  ctx->planned = false;  // colony calls need a new aco_colony_begin
   return ACO_OK;
 }
 
-aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint16_t *d_orders, uint32_t *d_cycles) {
+aco_status aco_set_dump(aco_ctx ctx, uint32_t *d_costs, uint64_t costs_len, uint16_t *d_orders,
+                        uint64_t orders_len, uint32_t *d_cycles, uint64_t cycles_len) {
   if (!ctx) return ACO_E_ARG;
+  ctx->dump_len[0] = d_costs ? costs_len : 0;
+  ctx->dump_len[1] = d_orders ? orders_len : 0;
+  ctx->dump_len[2] = d_cycles ? cycles_len : 0;
   ctx->dump_cost = d_costs;
   ctx->dump_order = d_orders;
   ctx->dump_cycle = d_cycles;
@@ -727,6 +786,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     if (ws_needed) *ws_needed = ctx->cache_need;
     P.L.stream = cuda_stream;
     P.L.launches = 0;
+    P.p2_done = false;  // per-run flags of the plan
+    P.L.cfg.keys = nullptr;
     ctx->ev_used = 0;
     for (int ph = 0; ph < 3; ++ph) {
       ctx->ev_pairs[ph].clear();
@@ -739,6 +800,13 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   }
   if (d_workspace) ctx->cache_ok = false;  // (a sizing call leaves the cached plan intact)
   if ((p->flags & ACO_FLAG_DUMP) && (!ctx->dump_cost || colony)) return ACO_E_ARG;
+  if (p->flags & ACO_FLAG_DUMP) {  // the dump buffers must hold every (pass, iteration) slice
+    const uint64_t sn = ctx->inst_off.empty() ? 0 : ctx->inst_off[ctx->count];
+    const uint64_t slices = 2ull * p->iterations;
+    if (ctx->dump_len[0] < slices * ctx->count * p->ants) return ACO_E_WORKSPACE;
+    if (ctx->dump_order && ctx->dump_len[1] < slices * p->ants * sn) return ACO_E_WORKSPACE;
+    if (ctx->dump_cycle && ctx->dump_len[2] < slices * p->ants * sn) return ACO_E_WORKSPACE;
+  }
   // passes that run construct/finalize launches: pass 4 (weighted, R41) uses the pass-2 machinery
   const uint32_t pmask = p->pass == 4 ? 2u : p->pass;
   const uint32_t count = ctx->count, A = p->ants;
@@ -1047,10 +1115,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       return ACO_E_WORKSPACE;
     }
     if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
-    if (!ctx->machine_uploaded) {
-      if (set_machine(ctx->mach) != 0) return ACO_E_CUDA;
-      ctx->machine_uploaded = true;
-    }
+    if (ctx->mslot < 0 && (ctx->mslot = acquire_machine_slot(ctx->device, ctx->mach)) < 0) return ACO_E_CUDA;
     if (!ctx->make_side()) return ACO_E_CUDA;
   }
   unsigned char *ws = (unsigned char *)d_workspace;
@@ -1151,6 +1216,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.heur_mix = p->heur_mix;
   cfg.stall_num = p->stall_num;
   cfg.rl_limit = p->rl_limit;
+  cfg.mslot = (uint32_t)ctx->mslot;
   cfg.record = P.record ? 1u : 0u;
   cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;

@@ -140,7 +140,7 @@ struct RunCfg {
   uint32_t rl_limit;                           // R45: 0 off, 1 min, 2 mid
   uint32_t record;                             // ants record their schedules; k_select copies the winner's
   uint32_t stage_img;   // k_select stages the region image in shared memory (few regions)
-  uint32_t pad_cfg;
+  uint32_t mslot;       // machine slot (c_mach[mslot]) of this context
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
   int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };
@@ -243,7 +243,9 @@ struct ClassLaunch {
   bool lean = false;       // pass 2: lean per-ant layout (u8 ready times, dynamic kills)
 };
 
-int set_machine(const MachineDev &m);  // cudaMemcpyToSymbol; 0 on success
+constexpr uint32_t kMachSlots = 8;  // distinct machine models resident per device
+int set_machine(uint32_t slot, const MachineDev &m);  // cudaMemcpyToSymbol into slot; 0 on success
+int init_kernel_attrs();                              // shared-memory opt-in of every kernel (once per device)
 // Resident threads per SM that the construct kernels' registers allow, per
 // [pass-1][wide]; returns nonzero (and conservative defaults) without a device.
 int construct_max_threads(int device, uint32_t out[2][3]);  // [pass-1][plain, wide, lean]

@@ -45,7 +45,10 @@
 
 namespace aco {
 
-__constant__ MachineDev c_mach;
+// Machine models (occupancy tables, issue width), one per slot: every context
+// is bound to the slot holding its machine (aco_host.cpp: MachineSlots), so
+// contexts with different machines can share a device (cfg.mslot).
+__constant__ MachineDev c_mach[kMachSlots];
 
 // ---------------------------------------------------------------- Philox
 // Philox4x32-10 (Salmon et al., SC'11) -- R26.
@@ -70,27 +73,29 @@ __device__ __forceinline__ uint4 philox(uint32_t c0, uint32_t c1, uint32_t c2, u
 }
 
 // ---------------------------------------------------------------- costs (R16-R18)
-__device__ __forceinline__ uint32_t occ_of(uint32_t c, uint32_t x) {
-  for (uint32_t i = 0; i < c_mach.step_count[c]; ++i)
-    if (x <= c_mach.step_max[c][i]) return c_mach.occ_max - i;
+__device__ __forceinline__ uint32_t occ_of(const MachineDev &M, uint32_t c, uint32_t x) {
+  for (uint32_t i = 0; i < M.step_count[c]; ++i)
+    if (x <= M.step_max[c][i]) return M.occ_max - i;
   return 0;
 }
-__device__ __forceinline__ uint32_t aprp_of(uint32_t c, uint32_t x) {
-  for (uint32_t i = 0; i < c_mach.step_count[c]; ++i)
-    if (x <= c_mach.step_max[c][i]) return c_mach.step_max[c][i];
+__device__ __forceinline__ uint32_t aprp_of(const MachineDev &M, uint32_t c, uint32_t x) {
+  for (uint32_t i = 0; i < M.step_count[c]; ++i)
+    if (x <= M.step_max[c][i]) return M.step_max[c][i];
   return x;
 }
-__device__ __noinline__ uint32_t cost_rp(uint32_t mode, uint32_t p0, uint32_t p1, uint32_t p2, uint32_t p3) {
+__device__ __noinline__ uint32_t cost_rp(uint32_t ms, uint32_t mode, uint32_t p0, uint32_t p1, uint32_t p2,
+                                         uint32_t p3) {
+  const MachineDev &c_mach = aco::c_mach[ms];
   const uint32_t prp[4] = {p0, p1, p2, p3};
   const uint32_t nc = c_mach.n_classes;
   uint32_t cost = 0;
   if (mode == ACO_COST_PRP_SUM) {
     for (uint32_t c = 0; c < nc; ++c) cost += prp[c];
   } else if (mode == ACO_COST_APRP_SUM) {
-    for (uint32_t c = 0; c < nc; ++c) cost += aprp_of(c, prp[c]);
+    for (uint32_t c = 0; c < nc; ++c) cost += aprp_of(c_mach, c, prp[c]);
   } else if (mode == ACO_COST_OCC) {
     uint32_t occ = c_mach.occ_max;
-    for (uint32_t c = 0; c < nc; ++c) occ = min(occ, occ_of(c, prp[c]));
+    for (uint32_t c = 0; c < nc; ++c) occ = min(occ, occ_of(c_mach, c, prp[c]));
     cost = c_mach.occ_max - occ;
   } else {
     for (uint32_t c = 0; c < nc; ++c)
@@ -98,16 +103,17 @@ __device__ __noinline__ uint32_t cost_rp(uint32_t mode, uint32_t p0, uint32_t p1
   }
   return cost;
 }
-__device__ void target_of(uint32_t mode, const uint32_t best[4], uint32_t tgt[4]) {
+__device__ void target_of(uint32_t ms, uint32_t mode, const uint32_t best[4], uint32_t tgt[4]) {
+  const MachineDev &c_mach = aco::c_mach[ms];
   const uint32_t nc = c_mach.n_classes;
   for (uint32_t c = 0; c < 4; ++c) tgt[c] = kInvalid;
   if (mode == ACO_COST_PRP_SUM) {
     for (uint32_t c = 0; c < nc; ++c) tgt[c] = best[c];
   } else if (mode == ACO_COST_APRP_SUM) {
-    for (uint32_t c = 0; c < nc; ++c) tgt[c] = aprp_of(c, best[c]);
+    for (uint32_t c = 0; c < nc; ++c) tgt[c] = aprp_of(c_mach, c, best[c]);
   } else if (mode == ACO_COST_OCC) {
     uint32_t occ = c_mach.occ_max;
-    for (uint32_t c = 0; c < nc; ++c) occ = min(occ, occ_of(c, best[c]));
+    for (uint32_t c = 0; c < nc; ++c) occ = min(occ, occ_of(c_mach, c, best[c]));
     if (occ > 0)
       for (uint32_t c = 0; c < nc; ++c) {
         const uint32_t idx = c_mach.occ_max - occ;
@@ -487,8 +493,8 @@ __device__ __forceinline__ bool stall_group(const RunCfg &cfg, uint32_t g) {
 // Sum of the four u8 lanes (per-class last-use counts -> LUC).
 __device__ __forceinline__ uint32_t sum_u8x4(uint32_t x) { return __dp4a(x, 0x01010101u, 0u); }
 
-__device__ __forceinline__ uint32_t cost_of(uint32_t mode, uint32_t prp01, uint32_t prp23) {
-  return cost_rp(mode, prp01 & 0xFFFFu, prp01 >> 16, prp23 & 0xFFFFu, prp23 >> 16);
+__device__ __forceinline__ uint32_t cost_of(uint32_t ms, uint32_t mode, uint32_t prp01, uint32_t prp23) {
+  return cost_rp(ms, mode, prp01 & 0xFFFFu, prp01 >> 16, prp23 & 0xFFFFu, prp23 >> 16);
 }
 
 // Commit of instruction j at cycle t (both passes): scheduled / ready sets,
@@ -810,7 +816,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
   o.prp01 = prp01;
   o.prp23 = prp23;
   o.len = 0;
-  o.cost = G.leader() ? cost_of(cfg.cost_mode, prp01, prp23) : 0u;
+  o.cost = G.leader() ? cost_of(cfg.mslot, cfg.cost_mode, prp01, prp23) : 0u;
   return o;
 }
 
@@ -844,9 +850,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   constexpr bool wide = MASK && WIDE;
   constexpr bool CT = !T32 && !NC4;  // compact layout (x_get)
   // general machine model (R42): runtime, only in the u32-cycle variants
-  const uint32_t w = T32 ? c_mach.issue_width : 1u;
+  const uint32_t w = T32 ? c_mach[cfg.mslot].issue_width : 1u;
   const bool mi = T32 && w > 1u;
-  const uint32_t slots = c_mach.type_slots;  // u8 x 4
+  const uint32_t slots = c_mach[cfg.mslot].type_slots;  // u8 x 4
   uint32_t used = 0, used_t = 0;              // placed in cycle t: total, per type (u8 x 4)
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0, B = 0;
   // ready time and per-class last-use counts of instruction j (LEAN: the
@@ -1051,7 +1057,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   o.prp23 = prp23;
   o.len = len;
   o.cost = len;
-  if (cfg.weighted && G.leader()) o.cost = len + cfg.ws_weight * cost_of(cfg.cost_mode, prp01, prp23);  // R41
+  if (cfg.weighted && G.leader()) o.cost = len + cfg.ws_weight * cost_of(cfg.mslot, cfg.cost_mode, prp01, prp23);  // R41
   return o;
 }
 
@@ -1293,7 +1299,7 @@ __device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
     uint16_t *heur = (uint16_t *)(A.ws + W.o_heur);  // the heuristic order, kept for R40
     for (uint32_t k = threadIdx.x; k < rd->n; k += 32) heur[k] = gb1[k];
     if (threadIdx.x != 0) return;
-    rs.lb_cost = cost_rp(A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
+    rs.lb_cost = cost_rp(A.cfg.mslot, A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
     rs.init[0] = rs.best[0] = o.cost;
     const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
     for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = rs.heur_prp[c] = prp[c];
@@ -1320,14 +1326,14 @@ __global__ void __launch_bounds__(128) k_init(KArgs A) {
 // issue, c_k = max(c_{k-1}, ready time), moved to c_{k-1} + 1 when cycle
 // c_{k-1} has no free slot (width or the instruction's type).  One thread;
 // rdyv[n] is zeroed scratch.  Returns the length.
-__device__ uint32_t asap_order(const SV &V, const uint16_t *order, uint16_t *out_o, uint32_t *out_c,
-                               uint32_t *rdyv) {
-  const uint32_t n = V.n, w = c_mach.issue_width;
+__device__ uint32_t asap_order(const MachineDev &M, const SV &V, const uint16_t *order, uint16_t *out_o,
+                               uint32_t *out_c, uint32_t *rdyv) {
+  const uint32_t n = V.n, w = M.issue_width;
   uint32_t t = 0, used = 0, used_t = 0;
   for (uint32_t k = 0; k < n; ++k) {
     const uint32_t j = order[k], y = V.ds[j].w & 0xFu;
     uint32_t c = k == 0 ? rdyv[j] : max(t, rdyv[j]);
-    if (k > 0 && c == t && (used >= w || ((used_t >> (8 * y)) & 0xFFu) >= ((c_mach.type_slots >> (8 * y)) & 0xFFu)))
+    if (k > 0 && c == t && (used >= w || ((used_t >> (8 * y)) & 0xFFu) >= ((M.type_slots >> (8 * y)) & 0xFFu)))
       c = t + 1;
     if (k == 0 || c != t) used = used_t = 0;
     t = c;
@@ -1363,17 +1369,17 @@ __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
     const uint16_t *gb1 = (const uint16_t *)(A.ws + W.o_gb1);
     uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
     uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
-    const uint32_t len = asap_order(V, gb1, gb2, gb2c, rdyv);
+    const uint32_t len = asap_order(c_mach[A.cfg.mslot], V, gb1, gb2, gb2c, rdyv);
     for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.prp1[c];
     rs.len2 = len;
     uint32_t tgt[4];
     uint32_t best = len, lb = rd->lb_len;
     if (A.cfg.weighted) {  // R41: cost = length + W * cost_rp, no RP target
       for (int c = 0; c < 4; ++c) tgt[c] = kInvalid;
-      best = len + A.cfg.ws_weight * cost_rp(A.cfg.cost_mode, rs.prp1[0], rs.prp1[1], rs.prp1[2], rs.prp1[3]);
+      best = len + A.cfg.ws_weight * cost_rp(A.cfg.mslot, A.cfg.cost_mode, rs.prp1[0], rs.prp1[1], rs.prp1[2], rs.prp1[3]);
       lb = rd->lb_len + A.cfg.ws_weight * rs.lb_cost;
     } else {
-      target_of(A.cfg.cost_mode, rs.prp1, tgt);
+      target_of(A.cfg.mslot, A.cfg.cost_mode, rs.prp1, tgt);
     }
     rs.init[1] = rs.best[1] = best;
     for (int c = 0; c < 4; ++c) rs.target[c] = tgt[c];
@@ -1402,17 +1408,18 @@ __global__ void __launch_bounds__(32) k_post(KArgs A) {
   if (threadIdx.x != 0) return;
   const SV V = make_sv(A.arena + rd->o_image, rd);
   const uint16_t *heur = (const uint16_t *)(A.ws + W.o_heur);
-  const uint32_t hlen = asap_order(V, heur, nullptr, nullptr, rdyv);
+  const MachineDev &M = c_mach[A.cfg.mslot];
+  const uint32_t hlen = asap_order(M, V, heur, nullptr, nullptr, rdyv);
   rs.heur_len = hlen;
   if (A.cfg.revert_occ == 0) return;
-  uint32_t of = c_mach.occ_max, oh = c_mach.occ_max;
-  for (uint32_t c = 0; c < c_mach.n_classes; ++c) {
-    of = min(of, occ_of(c, rs.prp2[c]));
-    oh = min(oh, occ_of(c, rs.heur_prp[c]));
+  uint32_t of = M.occ_max, oh = M.occ_max;
+  for (uint32_t c = 0; c < M.n_classes; ++c) {
+    of = min(of, occ_of(M, c, rs.prp2[c]));
+    oh = min(oh, occ_of(M, c, rs.heur_prp[c]));
   }
   if (of >= oh + A.cfg.revert_occ && (uint64_t)rs.len2 > (uint64_t)hlen + A.cfg.revert_len) {
     for (uint32_t i = 0; i < n; ++i) rdyv[i] = 0;
-    asap_order(V, heur, (uint16_t *)(A.ws + W.o_gb2), (uint32_t *)(A.ws + W.o_gb2c), rdyv);
+    asap_order(M, V, heur, (uint16_t *)(A.ws + W.o_gb2), (uint32_t *)(A.ws + W.o_gb2c), rdyv);
     for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.heur_prp[c];
     rs.len2 = hlen;
     rs.policy |= 2u;
@@ -1740,8 +1747,13 @@ static void big_smem(K kernel) {
     g_attr_err = 1;
 }
 
-int set_machine(const MachineDev &m) {
-  if (cudaMemcpyToSymbol(c_mach, &m, sizeof(m)) != cudaSuccess) return 1;
+int set_machine(uint32_t slot, const MachineDev &m) {
+  if (slot >= kMachSlots) return 1;
+  if (cudaMemcpyToSymbol(c_mach, &m, sizeof(m), sizeof(m) * slot) != cudaSuccess) return 1;
+  return check();
+}
+
+int init_kernel_attrs() {
   g_attr_err = 0;
   big_smem(k_init<true>);
   big_smem(k_init<false>);
