@@ -139,7 +139,7 @@ typedef struct {
   uint32_t policy;       /* bit0: pass 2 filtered by the cycle gap (R39); bit1: reverted (R40) */
   uint32_t heur_len;     /* length of the heuristic schedule (greedy order timed ASAP, R40) */
   uint32_t ws_cost;      /* pass 4: final weighted cost (R41), else 0 */
-  uint32_t pad;
+  uint32_t ants_pruned;  /* pass-2 ants cut short by the winner-invariant prune (R24), all iterations */
 } aco_result;
 
 /* Create a context on CUDA device `device` for machine model *m (copied). */
@@ -210,6 +210,19 @@ aco_status aco_get_timing(aco_ctx ctx, double ms[3], uint64_t launches[3]);
 
 /* Number of kernel launches enqueued by the last aco_schedule_batch. */
 aco_status aco_last_launch_count(aco_ctx ctx, uint64_t *launches);
+
+/* Construct-kernel variants (the instantiation of the ant-construction
+ * kernel each launch class uses) planned by the last aco_schedule_batch or
+ * aco_colony_begin on this context, sizing calls included (the plan is made
+ * without running).  codes: caller buffer of cap entries (may be NULL when
+ * cap == 0); *count = number of distinct codes (ascending).  Code bits:
+ * 0 4-wide candidate scan, 1 per-ant state in global memory, 2 3-4 register
+ * classes, 3 u32 pass-2 cycles, 4 pheromone staged in shared memory, 5
+ * word-mask bitset scan (n <= 1024), 6-7 lanes per ant (0:1 1:2 2:4 3:>=8),
+ * 8 pass 2, 9 lanes >= 16, 10 lanes 32, 11 block image read through L1,
+ * 12 lean pass-2 layout.  Used by the tests to prove that every variant a
+ * benchmark launches is covered by an every-ant parity test. */
+aco_status aco_last_variants(aco_ctx ctx, uint32_t *codes, uint32_t cap, uint32_t *count);
 
 /* Human-readable name of a status code (static storage). */
 const char *aco_status_string(aco_status st);

@@ -23,7 +23,7 @@ INVALID = 0xFFFFFFFF
 
 EXPORTS = [
     "aco_create", "aco_load_regions", "aco_schedule_batch", "aco_get_results", "aco_set_dump",
-    "aco_last_launch_count", "aco_get_timing", "aco_status_string", "aco_destroy",
+    "aco_last_launch_count", "aco_last_variants", "aco_get_timing", "aco_status_string", "aco_destroy",
     "aco_colony_begin", "aco_colony_construct", "aco_colony_finalize", "aco_colony_end",
 ]
 
@@ -68,7 +68,7 @@ class Result(C.Structure):
         ("prp", C.c_uint32 * 4), ("iters_run", C.c_uint32 * 2), ("best_cost", C.c_uint32 * 2),
         ("init_cost", C.c_uint32 * 2), ("lb_cost", C.c_uint32), ("lb_len", C.c_uint32),
         ("target", C.c_uint32 * 4), ("trace_hash", C.c_uint64),
-        ("policy", C.c_uint32), ("heur_len", C.c_uint32), ("ws_cost", C.c_uint32), ("pad", C.c_uint32),
+        ("policy", C.c_uint32), ("heur_len", C.c_uint32), ("ws_cost", C.c_uint32), ("ants_pruned", C.c_uint32),
     ]
 
 
@@ -92,6 +92,7 @@ def load(path: str = LIB_PATH):
     L.aco_get_results.argtypes = [vp, u32, u32, vp, vp, vp]
     L.aco_set_dump.argtypes = [vp, vp, u64, vp, u64, vp, u64]
     L.aco_last_launch_count.argtypes = [vp, C.POINTER(C.c_uint64)]
+    L.aco_last_variants.argtypes = [vp, vp, u32, C.POINTER(u32)]
     L.aco_get_timing.argtypes = [vp, vp, vp]
     L.aco_colony_begin.argtypes = [vp, vp, u32, vp, sz, C.POINTER(sz), vp]
     L.aco_colony_construct.argtypes = [vp, u32, u32, vp, vp]
@@ -102,7 +103,7 @@ def load(path: str = LIB_PATH):
     L.aco_destroy.argtypes = [vp]
     L.aco_destroy.restype = None
     for f in ("aco_create", "aco_load_regions", "aco_schedule_batch", "aco_get_results",
-              "aco_set_dump", "aco_last_launch_count", "aco_get_timing", "aco_colony_begin",
+              "aco_set_dump", "aco_last_launch_count", "aco_last_variants", "aco_get_timing", "aco_colony_begin",
               "aco_colony_construct", "aco_colony_finalize", "aco_colony_end"):
         getattr(L, f).restype = C.c_int32
     _lib = L

@@ -245,6 +245,19 @@ class Scheduler:
         _lib.check(self.lib.aco_last_launch_count(self.ctx, C.byref(v)), "aco_last_launch_count")
         return int(v.value)
 
+    def variants(self) -> List[int]:
+        """Construct-kernel variant codes of the last plan (aco_last_variants)."""
+        cnt = C.c_uint32(0)
+        _lib.check(self.lib.aco_last_variants(self.ctx, None, 0, C.byref(cnt)), "aco_last_variants")
+        buf = (C.c_uint32 * max(1, cnt.value))()
+        _lib.check(self.lib.aco_last_variants(self.ctx, buf, cnt.value, C.byref(cnt)), "aco_last_variants")
+        return [int(buf[i]) for i in range(cnt.value)]
+
+    def plan_variants(self, p: Params, flags: int = 0) -> List[int]:
+        """Variants a run with these parameters would launch (a sizing call: plans, runs nothing)."""
+        self.workspace_bytes(p, flags)
+        return self.variants()
+
     # ---------------------------------------------------------------- results
     def results_raw(self, first: int = 0, count: Optional[int] = None, orders=None, cycles=None):
         """Fill caller-provided host arrays (for the e2e path); returns the Result array."""
@@ -274,7 +287,7 @@ class Scheduler:
                 iters1=r.iters_run[0], iters2=r.iters_run[1], best1=r.best_cost[0], best2=r.best_cost[1],
                 init1=r.init_cost[0], init2=r.init_cost[1], lb1=r.lb_cost, lblen=r.lb_len,
                 target=list(r.target), trace_hash=int(r.trace_hash),
-                policy=r.policy, heur_len=r.heur_len, ws_cost=r.ws_cost,
+                policy=r.policy, heur_len=r.heur_len, ws_cost=r.ws_cost, ants_pruned=r.ants_pruned,
                 order=orders[a:b].copy(), cycle=cycles[a:b].copy()))
         return res
 

@@ -118,6 +118,7 @@ struct aco_ctx_s {
   uint16_t *dump_order = nullptr;
   uint32_t *dump_cycle = nullptr;
   std::vector<unsigned char> plan_blob;  // host staging of RegionWs + BlockItems
+  std::vector<uint32_t> variants;        // construct variants of the last plan
   // ACO_FLAG_TIMING: event pairs per phase
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
@@ -1171,6 +1172,14 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                 (int)sorted[i].img_l1, (int)sorted[i].lean,
                 (double)class_work[pass][idx[i]]);
   }
+  ctx->variants.clear();  // construct-kernel variants of this plan (aco_last_variants)
+  for (int pass = 1; pass <= 2; ++pass)
+    for (const ClassLaunch &cl : P.launches[pass]) {
+      const uint32_t code = class_variant((uint32_t)pass, cl);
+      if (std::find(ctx->variants.begin(), ctx->variants.end(), code) == ctx->variants.end())
+        ctx->variants.push_back(code);
+    }
+  std::sort(ctx->variants.begin(), ctx->variants.end());
   if (plan_only) {
     ctx->plan = saved;
     return ACO_OK;
@@ -1420,6 +1429,13 @@ aco_status aco_get_timing(aco_ctx ctx, double ms[3], uint64_t launches[3]) {
   return ACO_OK;
 }
 
+aco_status aco_last_variants(aco_ctx ctx, uint32_t *codes, uint32_t cap, uint32_t *count) {
+  if (!ctx || !count || (cap && !codes)) return ACO_E_ARG;
+  *count = (uint32_t)ctx->variants.size();
+  for (uint32_t i = 0; i < cap && i < ctx->variants.size(); ++i) codes[i] = ctx->variants[i];
+  return ACO_OK;
+}
+
 aco_status aco_last_launch_count(aco_ctx ctx, uint64_t *launches) {
   if (!ctx || !launches) return ACO_E_ARG;
   *launches = ctx->launches;
@@ -1496,6 +1512,7 @@ aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_resu
     o.policy = S.policy;
     o.heur_len = S.heur_len;
     o.ws_cost = ctx->cfg.weighted ? S.best[1] : 0u;
+    o.ants_pruned = S.pruned;
   }
   for (uint64_t q = 0; q < i1 - i0; ++q) {
     if (orders) orders[q] = o16[q];

@@ -87,12 +87,12 @@ struct RegionState {
   uint32_t prp2[4];      // PRP of the pass-2 global best (final)
   uint32_t target[4];    // pass-2 target (R18)
   uint32_t prune_len;    // best completed length of the running iteration (R24)
+  uint32_t pruned;       // pass-2 ants pruned (R24), summed over iterations; must follow prune_len
   uint32_t lb_cost;
   uint32_t len2;         // length of the pass-2 global best (pass 4: best[1] is the weighted cost)
   uint32_t policy;       // bit0 gap-filtered (R39), bit1 reverted (R40)
   uint32_t heur_len;     // the heuristic schedule's length (R40)
   uint32_t heur_prp[4];  // the heuristic schedule's PRP
-  uint32_t pad;
   uint64_t hash;         // FNV-1a trace
 };
 
@@ -244,6 +244,24 @@ struct ClassLaunch {
 };
 
 constexpr uint32_t kMachSlots = 8;  // distinct machine models resident per device
+// Construct-kernel variant code (the template arguments of k_construct, see
+// include/aco.h aco_last_variants): bit 0 4-wide scan, 1 global state, 2 3-4
+// classes, 3 u32 cycles, 4 tau in smem, 5 word mask, 6-7 lanes (1,2,4,8),
+// 8 pass-1, 9 lanes >= 16, 10 lanes 32, 11 image through L1, 12 lean.
+ACO_HD constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4, int gs, bool wd,
+                                       bool lean = false) {
+  return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
+         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) | ((gs == 2 ? 1u : 0u) << 11) |
+         ((uint32_t)lean << 12) | ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) |
+         ((gs == 1 ? 1u : 0u) << 1) | (uint32_t)wd;
+}
+inline uint32_t class_variant(uint32_t pass, const ClassLaunch &c) {
+  const bool mask = c.max_n <= 1024 && !c.gs;
+  const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
+  return variant_code(pass, c.lanes, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32, pass == 2 && c.nc4,
+                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask, pass == 2 && c.lean);
+}
+
 int set_machine(uint32_t slot, const MachineDev &m);  // cudaMemcpyToSymbol into slot; 0 on success
 int init_kernel_attrs();                              // shared-memory opt-in of every kernel (once per device)
 // Resident threads per SM that the construct kernels' registers allow, per

@@ -16,13 +16,18 @@
 // shared-memory loads overlap (ILP).
 //
 // Per pass and iteration (L135-L139):
-//   k_construct : every ant builds a schedule and writes its cost (K1a)
-//   k_finalize  : per region: argmin over (cost, ant) (K1b), replay of the
-//                 winner to recover its order (no per-ant order is stored),
-//                 pheromone evaporate + deposit (K1c), global-best epilogue and
-//                 termination (K1d).
-// Plus k_init (tau0, greedy heuristic schedule) and k_pass2_init (target, ASAP
-// of the pass-1 best, tau reset).
+//   k_construct : every ant builds a schedule and writes its cost (K1a); in
+//                 record mode (the default) it also stores its order (and
+//                 pass-2 cycles) step-major, coalesced across the ants
+//   k_select    : per region: argmin over (cost, ant) (K1b); copy of the
+//                 winner's recorded schedule -- or, in the shared colony and
+//                 dump mode, a whole-warp replay of the winner from the same
+//                 pheromone table and Philox counters; winner successor table;
+//                 global-best epilogue (K1d)
+//   k_update    : pheromone evaporate + deposit (K1c) over all tables
+//   k_stop      : termination (K1d)
+// Plus k_init (tau0, greedy heuristic schedule), k_pass2_init (target, ASAP
+// of the pass-1 best, tau reset) and k_post (heuristic length, R40).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -893,6 +898,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       bl = G.bcast(bl);
       const uint32_t lbf = mi ? t + (n - placed + used + w - 1) / w : t + (n - placed);
       if (lbf > bl) {
+        if (G.leader()) atomicAdd(prune_len + 1, 1u);  // RegionState::pruned follows prune_len
         o.cost = kInvalid;
         return o;
       }
@@ -1308,6 +1314,7 @@ __device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
     rs.iters[0] = rs.iters[1] = 0;
     rs.no_imp = 0;
     rs.prune_len = kInvalid;
+    rs.pruned = 0;
     rs.hash = 0xcbf29ce484222325ull;
     rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
   }
@@ -1628,13 +1635,6 @@ int last_cuda_error() { return check(); }
 // launch dispatch (a class launch looks its kernel up by variant code).
 using ConstructFn = void (*)(KArgs, const BlockItem *, uint32_t);
 
-__host__ __device__ constexpr uint32_t variant_code(uint32_t pass, uint32_t lg, bool m, bool ts, bool t3, bool n4,
-                                                     int gs, bool wd, bool lean = false) {
-  return ((pass - 1) << 8) | ((lg == 1 ? 0u : lg == 2 ? 1u : lg == 4 ? 2u : 3u) << 6) | ((uint32_t)m << 5) |
-         ((lg >= 16 ? 1u : 0u) << 9) | ((lg == 32 ? 1u : 0u) << 10) | ((gs == 2 ? 1u : 0u) << 11) | ((uint32_t)lean << 12) |
-         ((uint32_t)ts << 4) | ((uint32_t)t3 << 3) | ((uint32_t)n4 << 2) | ((gs == 1 ? 1u : 0u) << 1) | (uint32_t)wd;
-}
-
 template <int P, int LG, bool M, bool TS, bool T3, bool N4, int GS, bool WD, typename F, bool LN = false>
 static void reg1(F &f) {
   f(&k_construct<P, LG, M, TS, T3, N4, GS, WD, LN>, variant_code(P, LG, M, TS, T3, N4, GS, WD, LN));
@@ -1790,12 +1790,8 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c) {
   if (!c.n_blocks) return 0;
   build_table();
-  const bool mask = c.max_n <= 1024 && !c.gs;
-  const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   const uint32_t lg = c.lanes;
-  const uint32_t code = variant_code(pass, lg, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32,
-                                     pass == 2 && c.nc4, c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask,
-                                     pass == 2 && c.lean);
+  const uint32_t code = class_variant(pass, c);
   const ConstructFn f = g_construct[code];
   if (!f) return (int)cudaErrorInvalidDeviceFunction;
   f<<<c.n_blocks, c.ants_pb * lg, c.smem_bytes, (cudaStream_t)L.stream>>>(kargs(L), c.items, iter);

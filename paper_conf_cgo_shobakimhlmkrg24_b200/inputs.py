@@ -10,9 +10,13 @@ Workload recipe:
   * instruction mix shaped like a GPU basic block: VALU 55 %, SALU 15 %,
     VMEM load 12 %, SMEM load 8 %, LDS load 5 %, store 5 %;
   * operands pick recent values of the needed class with geometric recency
-    (p = 0.3) or, for SGPR operands, a long-lived live-in base (20 %);
+    (p = 0.15) or, for SGPR operands, a long-lived live-in base (20 %);
   * memory ordering: every load and store depends on the last store (lat 1);
-  * 4 SGPR + 2 VGPR live-in registers; unused defs are live-out with p = 0.7;
+  * 4 SGPR + 8 VGPR live-in registers; unused defs are live-out with p = 0.7;
+  * calibration: with recency 0.15 and 8 VGPR live-ins, 56 % of
+    the n >= 50 regions of the config-3 batch have a greedy-heuristic VGPR PRP
+    above 24 (round 1's 0.3 / 2 gave 35 %), so under APRP_SUM the RP pass has
+    occupancy bands to search (tools/calibrate_generator.py);
   * latency profiles "mixed" (VMEM 20-80, SMEM 8-20, LDS 4-8, transcendental
     VALU 4, else 1) and "unit" (all 1);
   * region sizes for the rocPRIM-shaped batch follow Table 3.a's bucket counts
@@ -168,7 +172,8 @@ _KINDS = ("valu", "salu", "vmem", "smem", "lds", "store")
 _MIX = np.array([0.55, 0.15, 0.12, 0.08, 0.05, 0.05])
 
 
-def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "") -> Region:
+def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "", recency: float = 0.15,
+               v_livein: int = 8) -> Region:
     """A synthetic GPU-basic-block-like region of n instructions (2 classes)."""
     rng = np.random.default_rng(np.uint64(seed))
     reg_class: List[int] = []
@@ -182,7 +187,7 @@ def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "") -> Reg
 
     for _ in range(4):
         pools[SGPR].append(new_reg(SGPR, LIVE_IN))
-    for _ in range(2):
+    for _ in range(v_livein):
         pools[VGPR].append(new_reg(VGPR, LIVE_IN))
     base = pools[SGPR][0]
 
@@ -190,7 +195,7 @@ def gen_region(n: int, seed: int, profile: str = "mixed", name: str = "") -> Reg
         if c == SGPR and rng.random() < 0.2:
             return base
         pool = pools[c]
-        back = int(rng.geometric(0.3)) - 1
+        back = int(rng.geometric(recency)) - 1
         return pool[max(0, len(pool) - 1 - back)]
 
     def lat_of(kind):
