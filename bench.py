@@ -2,24 +2,27 @@
 """Benchmark: region-batch ACO throughput (ant-schedules/s) on 1..N B200s.
 
 One STEP = one full two-pass ACO run (aco_schedule_batch: every pass and
-iteration of every region: construction, argmin + winner replay, pheromone
+iteration of every region: construction, argmin + winner copy, pheromone
 update, epilogue) over one batch of synthetic regions.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c3|c2|c1|c4|c5]
+                  [--scaling strong|weak] [--parity sample|all|off]
                   [--machine gfx906|dual] [--passes 3|4 --ws-weight W] [--policy off|paper]
                   [--heur-mix 0|1] [--stall-num k] [--rl-limit 0|1|2]
   python bench.py --impl reference ...     # the CPU oracle on a bounded sample
 
 Workloads (BASELINE.json configs): c1 FIX10-A; c2 one n = 100 region; c3
-(default, the metric's config) 5,000 rocPRIM-shaped regions per GPU (weak
-scaling); c4 one n = 2,000 region with 8,192 ants per iteration as ONE shared
-colony across the N ranks (strong scaling: 8,192 / N ants per rank, one int64
-MIN allreduce per iteration over NCCL); c5 the full-suite sweep, 1,000
-regions per GPU up to 4,000 instructions (weak scaling).
+(default, the metric's config) the 5,000 rocPRIM-shaped regions, LPT-
+partitioned across the N ranks (strong scaling; --scaling weak gives every
+rank its own 5,000); c4 one n = 2,000 region with 8,192 ants x 20 iterations
+per pass, ONE shared colony across the N ranks (one int64 MIN allreduce per
+iteration over NCCL); c5 the SURVEY 8(d) sweep n in {10..4000} x {unit,
+mixed} x 3 seeds (I = 10, 5 for n >= 2,000), LPT-partitioned.
 
 Multi-GPU: launched by torchrun, one process per GPU.  Regions shard with no
-data-path collective (each rank schedules its own batch with globally unique
-region ids); NCCL is used only for the barrier and the max-over-ranks time.
+data-path collective (global region ids key the Philox streams, so a region's
+result does not depend on the rank running it); NCCL carries only the
+barrier, the max-over-ranks time and the result gather for the parity check.
 """
 from __future__ import annotations
 
@@ -38,18 +41,24 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 from paper_conf_cgo_shobakimhlmkrg24_b200 import inputs as I  # noqa: E402
+from paper_conf_cgo_shobakimhlmkrg24_b200 import sharding  # noqa: E402
 
 METRIC = "ant-schedules/s"
 C3_REGIONS = 5000
+# result fields compared bit for bit by the parity check (oracle vs GPU)
+PARITY_FIELDS = ("order", "cycle", "prp", "length", "cost_rp", "iters1", "iters2", "best1", "best2",
+                 "init1", "init2", "lb1", "lblen", "trace_hash")
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="c3", choices=["c3", "c2", "c1", "c4", "c5"])
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="c3/c5 at N > 1: partition the same batch (strong) or one batch per rank (weak)")
     ap.add_argument("--machine", default="gfx906", choices=["gfx906", "dual"])
     ap.add_argument("--passes", type=int, default=3, choices=[1, 2, 3, 4])
     ap.add_argument("--ws-weight", type=int, default=4)
@@ -57,59 +66,96 @@ def parse():
     ap.add_argument("--heur-mix", type=int, default=0)
     ap.add_argument("--stall-num", type=int, default=1)
     ap.add_argument("--rl-limit", type=int, default=0, help="pass-1 ready-list size limit (R45): 1 min, 2 mid")
-    ap.add_argument("--regions", type=int, default=C3_REGIONS, help="regions per rank (c3)")
+    ap.add_argument("--regions", type=int, default=C3_REGIONS, help="regions of the c3 batch")
     ap.add_argument("--ants", type=int, default=None)
     ap.add_argument("--iterations", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=160, help="regions in the oracle sample")
-    return ap.parse_args()
+    ap.add_argument("--parity", default="sample", choices=["sample", "all", "off"],
+                    help="compare GPU results with the oracle on the cpu_baseline sample, on every region, or not")
+    ap.add_argument("--parity-log", default=None, help="write the per-region parity log here (--parity all)")
+    return ap.parse_args(argv)
 
 
-def workload(args, rank: int):
-    """(regions, region_ids, params, config dict) for this rank."""
-    if args.workload == "c3":
-        n = args.regions
-        first = rank * n
-        regs = I.gen_batch(n, base_seed=3, first_id=first)
-        ids = list(range(first, first + n))
-        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 10, seed=3)
-        cfg = {"workload": "c3-rocprim-shaped-batch", "regions_per_gpu": n,
-               "sizes": "20-500 (Table 3.a buckets)", "latency": "mixed"}
-    elif args.workload == "c2":
-        regs = [I.gen_region(100, I.region_seed(2, rank))]
-        ids = [rank]
-        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 100, seed=2)
-        cfg = {"workload": "c2-single-region-n100", "regions_per_gpu": 1, "latency": "mixed"}
-    elif args.workload == "c4":
-        regs = [I.gen_region(2000, I.region_seed(4, 0))]
-        ids = [0]  # ONE region shared by all ranks (shared colony)
-        world = int(os.environ.get("WORLD_SIZE", "1"))
-        total = args.ants or 8192
-        p = I.Params(ants=total // world, iterations=args.iterations or 10, seed=4)
-        cfg = {"workload": "c4-shared-colony-n2000", "regions": 1, "ants_total": total,
-               "ants_per_gpu": total // world, "latency": "mixed"}
-    elif args.workload == "c5":
-        n = args.regions if args.regions != C3_REGIONS else 1000
-        first = rank * n
-        sizes = I.c5_sizes(first + n, base_seed=5)[first:]
-        regs = I.gen_batch(n, base_seed=5, first_id=first, sizes=sizes)
-        ids = list(range(first, first + n))
-        p = I.Params(ants=args.ants or 1024, iterations=args.iterations or 5, seed=5)
-        cfg = {"workload": "c5-suite-sweep", "regions_per_gpu": n, "sizes": "20-4000 (c3 mix + 15% tail 500-4000)",
-               "max_n": int(max(r.n_insts for r in regs)), "latency": "mixed"}
-    else:
-        regs = [I.fix10a()]
-        ids = [rank]
-        p = I.Params(ants=args.ants or 64, iterations=args.iterations or 20, seed=0, cost_mode=0)
-        cfg = {"workload": "c1-fix10a", "regions_per_gpu": 1}
+# ---------------------------------------------------------------- workloads
+@dataclasses.dataclass
+class Batch:
+    regs: list
+    ids: list
+    p: I.Params
+
+
+def base_params(args, p):
     p = dataclasses.replace(p, passes=args.passes, ws_weight=args.ws_weight if args.passes == 4 else 0,
-                            heur_mix=args.heur_mix, stall_num=args.stall_num,
-                            rl_limit=args.rl_limit)
+                            heur_mix=args.heur_mix, stall_num=args.stall_num, rl_limit=args.rl_limit)
     if args.policy == "paper":
         p = I.paper_policy(p)
+    return p
+
+
+def workload(args, rank: int, world: int, gen: bool = True):
+    """(batches for this rank, config dict, scaling) -- every batch is one
+    aco_schedule_batch call per step (c5: one per iteration count).
+    gen=False: parameters only (no regions generated)."""
+    strong = args.scaling == "strong"
+    if args.workload == "c3":
+        R = args.regions
+        p = base_params(args, I.Params(ants=args.ants or 1024, iterations=args.iterations or 10, seed=3))
+        if strong or world == 1:
+            sizes = I.c3_sizes(R, 3)
+            ids = sharding.lpt_partition(sizes, world, p.ants, p.iterations)[rank]
+            regs = I.gen_regions(ids, sizes, 3) if gen else []
+            cfg = {"workload": "c3-rocprim-shaped-batch", "regions": R, "regions_this_rank_0": None}
+        else:
+            regs = I.gen_batch(R, base_seed=3, first_id=rank * R) if gen else []
+            ids = list(range(rank * R, (rank + 1) * R))
+            cfg = {"workload": "c3-rocprim-shaped-batch", "regions_per_gpu": R}
+        cfg.update({"sizes": "20-500 (Table 3.a buckets)", "latency": "mixed"})
+        batches = [Batch(regs, list(ids), p)]
+        scaling = "strong" if strong else "weak"
+    elif args.workload == "c5":
+        grid = I.c5_grid()
+        p10 = base_params(args, I.Params(ants=args.ants or 1024, iterations=args.iterations or 10, seed=5))
+        p5 = dataclasses.replace(p10, iterations=args.iterations or 5)
+        batches = []
+        for big, p in ((False, p10), (True, p5)):
+            sel = [g for g in grid if (g[1] >= 2000) == big]
+            sizes = {g[0]: g[1] for g in sel}
+            gids = [g[0] for g in sel]
+            if world > 1:
+                part = sharding.lpt_partition([sizes[i] for i in gids], world, p.ants, p.iterations)[rank]
+                gids = [gids[k] for k in part]
+            regs = [I.c5_region(g[0], g[1], g[2]) for g in sel if g[0] in set(gids)] if gen else []
+            batches.append(Batch(regs, [g[0] for g in sel if g[0] in set(gids)], p))
+        cfg = {"workload": "c5-suite-sweep", "regions": len(grid), "sizes": list(I.C5_SIZES),
+               "latency": list(I.C5_PROFILES), "seeds": len(I.C5_SEEDS),
+               "iterations_per_pass": "10 (n < 2000), 5 (n >= 2000)"}
+        scaling = "strong"
+    elif args.workload == "c4":
+        total = args.ants or 8192
+        p = base_params(args, I.Params(ants=total // world, iterations=args.iterations or 20, seed=4))
+        batches = [Batch([I.gen_region(2000, I.region_seed(4, 0))], [0], p)]
+        cfg = {"workload": "c4-shared-colony-n2000", "regions": 1, "ants_total": total,
+               "ants_per_gpu": total // world, "latency": "mixed"}
+        scaling = "strong"
+    elif args.workload == "c2":
+        p = base_params(args, I.Params(ants=args.ants or 1024, iterations=args.iterations or 100, seed=2))
+        batches = [Batch([I.gen_region(100, I.region_seed(2, 0))], [rank], p)]
+        cfg = {"workload": "c2-single-region-n100", "regions_per_gpu": 1, "latency": "mixed",
+               "multi_gpu": "replicas only (one region does not shard)"}
+        scaling = "weak"
+    else:
+        p = base_params(args, I.Params(ants=args.ants or 64, iterations=args.iterations or 20, seed=0, cost_mode=0))
+        batches = [Batch([I.fix10a()], [rank], p)]
+        cfg = {"workload": "c1-fix10a", "regions_per_gpu": 1,
+               "multi_gpu": "replicas only (one region does not shard)"}
+        scaling = "weak"
+    p = batches[0].p
     passes = {1: "RP", 2: "ILP", 3: "RP+ILP", 4: f"weighted single pass (W={p.ws_weight})"}[p.passes]
-    cfg.update({"ants": p.ants, "iterations_per_pass": p.iterations, "passes": passes,
+    cfg.pop("regions_this_rank_0", None)
+    cfg.update({"ants": p.ants if args.workload != "c4" else cfg["ants_total"],
+                "iterations_per_pass": cfg.get("iterations_per_pass", p.iterations), "passes": passes,
                 "cost": ["PRP_SUM", "APRP_SUM", "OCC", "PERP"][p.cost_mode],
                 "stop_rules": "paper policy (LB, size classes, gap 21, revert 3/63)" if args.policy == "paper"
                 else "off (fixed work)",
@@ -120,13 +166,14 @@ def workload(args, rank: int):
         cfg["stall_groups"] = f"{args.stall_num}/{p.stall_mod}"
     if args.rl_limit:
         cfg["ready_list_limit"] = {1: "group min", 2: "group min/max midpoint"}[args.rl_limit]
-    return regs, ids, p, cfg
+    return batches, cfg, scaling
 
 
 def machine_of(args):
     return I.DUAL_ISSUE if args.machine == "dual" else I.GFX906
 
 
+# ---------------------------------------------------------------- helpers
 class ClockSampler:
     """nvidia-smi clocks + throttle reasons during the timed region."""
 
@@ -180,6 +227,19 @@ def measured_peaks():
         return {}
 
 
+def host_cpu():
+    """CPU model and thread count of the host (lscpu)."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.lower().startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return {"model": model, "threads": os.cpu_count()}
+
+
 def bytes_per_ant_step(stats: np.ndarray) -> float:
     """SURVEY 8(d) algorithmic bytes per ant-step from oracle instrumentation:
     8.5|F| + 2|R| + 12 deg + 6 |Use| + 2 |Def| + 16 per placed instruction."""
@@ -213,30 +273,64 @@ def stratified_pick(regs, sample: int):
 
 
 def deal_over_steps(full, steps: int):
-    """Round-robin the sample over the steps (a sample smaller than the step
+    """Round-robin a sample over the steps (a sample smaller than the step
     count is reused whole by the steps it does not reach)."""
     return [full[s::steps] or full for s in range(steps)]
 
 
-def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes", pick=None):
-    """The oracle as it stands on a bounded, stratified sample of the same workload."""
+def run_oracle(regs, ids, p, machine, threads=None):
+    """The oracle as it stands over regions on the host's threads: (per-region
+    result dicts, stats, seconds, ant-schedules)."""
     from oracle import pyoracle as O
+    threads = threads or os.cpu_count() or 1
+    t0 = time.perf_counter()
+    order, cyc, stats, off = O.schedule_many(regs, ids, machine, p, n_threads=threads)
+    dt = time.perf_counter() - t0
+    res = []
+    for k in range(len(regs)):
+        d = {n: int(stats[k, i]) for n, i in O.ORS.items()}
+        d["prp"] = [d["prp0"], d["prp1"], d["prp2"], d["prp3"]]
+        a, b = int(off[k]), int(off[k + 1])
+        d["order"] = [int(x) for x in order[a:b]]
+        d["cycle"] = [int(x) for x in cyc[a:b]]
+        res.append(d)
+    return res, stats, dt, float(stats[:, O.ORS["ant_scheds"]].sum())
+
+
+def cpu_baseline(regs, ids, p, sample: int, machine=I.GFX906, note="full A x I x passes", pick=None):
+    """The oracle as it stands on a bounded, stratified sample of the same
+    workload: (baseline dict, stats, picked indices, oracle results, seconds,
+    ant-schedules)."""
     if pick is None:
         pick = stratified_pick(regs, sample)
     sub = [regs[i] for i in pick]
     sid = [ids[i] for i in pick]
     threads = os.cpu_count() or 1
-    t0 = time.perf_counter()
-    _, _, stats, _ = O.schedule_many(sub, sid, machine, p, n_threads=threads)
-    dt = time.perf_counter() - t0
-    scheds = float(stats[:, O.ORS["ant_scheds"]].sum())
-    return {"value": scheds / dt, "unit": METRIC, "cores": min(threads, len(sub)), "kind": "oracle",
-            "sample": f"{len(sub)} of {len(regs)} regions (stratified by size), {note}, "
-                      f"{scheds:.0f} ant-schedules in {dt:.1f} s"}, stats
+    res, stats, dt, scheds = run_oracle(sub, sid, p, machine, threads)
+    base = {"value": scheds / dt, "unit": METRIC, "cores": min(threads, len(sub)), "kind": "oracle",
+            "host": host_cpu(),
+            "sample": f"{len(sub)} of {len(regs)} regions (stratified by size, largest first), {note}, "
+                      f"{scheds:.0f} ant-schedules in {dt:.1f} s on {min(threads, len(sub))} host threads"}
+    return base, stats, pick, res, dt, scheds
 
 
-def main():
-    args = parse()
+def gpu_digest(r: dict) -> dict:
+    """The fields of a GPU result compared with the oracle (plain Python types)."""
+    return {"order": [int(x) for x in r["order"]], "cycle": [int(x) for x in r["cycle"]],
+            "prp": [int(x) for x in r["prp"]], "length": r["length"], "cost_rp": r["cost_rp"],
+            "iters1": r["iters1"], "iters2": r["iters2"], "best1": r["best1"], "best2": r["best2"],
+            "init1": r["init1"], "init2": r["init2"], "lb1": r["lb1"], "lblen": r["lblen"],
+            "trace_hash": r["trace_hash"]}
+
+
+def parity_compare(gpu: dict, ora: dict):
+    """Names of the fields where the GPU result differs from the oracle's."""
+    return [f for f in PARITY_FIELDS if gpu[f] != ora[f]]
+
+
+# ---------------------------------------------------------------- main arm
+def main(argv=None):
+    args = parse(argv)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -251,13 +345,14 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    regs, ids, p, cfg = workload(args, rank)
+    batches, cfg, scaling = workload(args, rank, world)
     machine = machine_of(args)
     colony = args.workload == "c4" and world > 1  # one region, ants split across ranks
-    batch = HostBatch(regs, ids)
-    sched = Scheduler(machine, device=local)
+    hosts = [HostBatch(b.regs, b.ids) for b in batches]
+    scheds = [Scheduler(machine, device=local) for _ in batches]
     stream = torch.cuda.current_stream()
-    sched.load(regs, ids, batch=batch)
+    for s, b, h in zip(scheds, batches, hosts):
+        s.load(b.regs, b.ids, batch=h)
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{local}")
 
     def barrier():
@@ -265,18 +360,21 @@ def main():
             dist.barrier()
 
     def run(timing=False):
-        if colony:
-            sched.run_colony(p, rank, world, timing=timing)
-        else:
-            sched.run(p, timing=timing)
+        for s, b in zip(scheds, batches):
+            if not b.regs and not colony:
+                continue
+            if colony:
+                s.run_colony(b.p, rank, world, timing=timing)
+            else:
+                s.run(b.p, timing=timing)
 
     for _ in range(max(3, args.warmup)):
         run()
     torch.cuda.synchronize()
+
+    # ---- timed region: K steps, no per-phase events inside (ACO_FLAG_TIMING off)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)]
-    phase_ms = np.zeros(3)
-    phase_launches = np.zeros(3)
     launches = 0
     clk = ClockSampler(local)
     clk.start()
@@ -285,12 +383,9 @@ def main():
     for k in range(args.steps):
         flush.zero_()  # L2 flush between timed steps (outside the events)
         ev[k][0].record(stream)
-        run(timing=True)
+        run()
         ev[k][1].record(stream)
-        ms, ln = sched.timing()  # syncs; events inside the library, same stream
-        phase_ms += ms
-        phase_launches += ln
-        launches += sched.launch_count()
+        launches += sum(s.launch_count() for s, b in zip(scheds, batches) if b.regs or colony)
     torch.cuda.synchronize()
     barrier()
     clocks = clk.stop()
@@ -299,95 +394,187 @@ def main():
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     max_ms = float(t.item())
-    res = sched.results()
-    iters = sum(r["iters1"] + r["iters2"] for r in res)
-    scheds_rank = p.ants * iters * args.steps
-    tot = torch.tensor([float(scheds_rank)], dtype=torch.float64, device=f"cuda:{local}")
+    res = {}  # global id -> GPU result (this rank)
+    for s, b in zip(scheds, batches):
+        if b.regs:
+            for rid, r in zip(b.ids, s.results()):
+                res[rid] = r
+    scheds_rank = sum(b.p.ants * (r["iters1"] + r["iters2"]) for s, b in zip(scheds, batches)
+                      for r in (res[i] for i in b.ids)) * args.steps
+    if colony:  # every rank holds the same region: count its own ants once
+        scheds_rank = batches[0].p.ants * sum(res[i]["iters1"] + res[i]["iters2"] for i in batches[0].ids) * args.steps
+    pruned = sum(r["ants_pruned"] for r in res.values())
+    p2_ants = sum(b.p.ants * res[i]["iters2"] for b in batches for i in b.ids)
+    tot = torch.tensor([float(scheds_rank), float(pruned), float(p2_ants)], dtype=torch.float64,
+                       device=f"cuda:{local}")
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.SUM)
-    value = float(tot.item()) / (max_ms / 1000.0)
+    total_scheds = float(tot[0].item())
+    value = total_scheds / (max_ms / 1000.0)
+    prune_frac = float(tot[1].item()) / max(1.0, float(tot[2].item()))
+
+    # ---- phase split and construct time (roofline): the same K steps again
+    # with per-phase CUDA events on the launching streams (ACO_FLAG_TIMING)
+    phase_ms = np.zeros(3)
+    phase_launches = np.zeros(3)
+    for k in range(args.steps):
+        flush.zero_()
+        run(timing=True)
+        for s, b in zip(scheds, batches):
+            if b.regs or colony:
+                ms, ln = s.timing()
+                phase_ms += ms
+                phase_launches += ln
+    torch.cuda.synchronize()
 
     # ---- end to end through the public API: host inputs -> H2D -> run -> D2H results
     e2e_ms = []
-    h2d = d2h = 0
-    sum_n = int(batch.offsets[-1])
-    orders = np.zeros(max(1, sum_n), np.uint32)
-    cycles = np.zeros(max(1, sum_n), np.uint32)
+    sum_n = sum(int(h.offsets[-1]) for h in hosts)
+    outs = [(np.zeros(max(1, int(h.offsets[-1])), np.uint32), np.zeros(max(1, int(h.offsets[-1])), np.uint32))
+            for h in hosts]
     for _ in range(max(1, args.e2e_steps)):
         barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        sched.load(regs, ids, batch=batch)
+        for s, b, h in zip(scheds, batches, hosts):
+            s.load(b.regs, b.ids, batch=h)
         run()
-        sched.results_raw(0, len(regs), orders, cycles)
+        for s, b, (o, c) in zip(scheds, batches, outs):
+            if b.regs:
+                s.results_raw(0, len(b.regs), o, c)
         e2e_ms.append((time.perf_counter() - t0) * 1000.0)
-    h2d = int(sched.arena.numel()) if sched.arena is not None else 0
-    d2h = int(len(regs) * 64 + 4 * 2 * sum_n)
+    h2d = sum(int(s.arena.numel()) for s in scheds if s.arena is not None)
+    n_regs = sum(len(b.regs) for b in batches)
+    d2h = int(n_regs * 72 + 4 * 2 * sum_n)  # aco_result + orders + cycles
     e = torch.tensor([float(np.median(e2e_ms))], dtype=torch.float64, device=f"cuda:{local}")
     if world > 1:
         dist.all_reduce(e, op=dist.ReduceOp.MAX)
-    e2e_value = float(tot.item()) / args.steps / (float(e.item()) / 1000.0)
+    e2e_value = total_scheds / args.steps / (float(e.item()) / 1000.0)
+
+    # ---- gather every rank's results (global id -> digest) to rank 0 for the parity check
+    local_digest = {rid: gpu_digest(r) for rid, r in res.items()}
+    if world > 1 and not colony:
+        all_digest = sharding.gather_results(local_digest, world, rank)
+    else:
+        all_digest = local_digest
 
     out = None
     if rank == 0:
         peaks = measured_peaks()
-        cpu = None
-        bpas = None
+        cpu, bpas, parity = None, None, None
+        n_cmp, n_ok, bad, log = 0, 0, [], []
+
+        def check(rid, n, gdig, ora):
+            nonlocal n_cmp, n_ok
+            diff = parity_compare(gdig, ora)
+            n_cmp += 1
+            n_ok += not diff
+            if diff:
+                bad.append({"region": rid, "fields": diff})
+            log.append(f"{rid} n={n} {'ok' if not diff else 'MISMATCH ' + ','.join(diff)} "
+                       f"len={ora['length']} cost={ora['cost_rp']} hash={ora['trace_hash']:016x}")
+
+        parity_note = None
         if world == 1 and not args.no_cpu_baseline:
-            ps, note = cpu_sample_params(args, p)
-            cpu, stats = cpu_baseline(regs, ids, ps, args.cpu_sample if args.workload != "c5" else 24,
-                                      machine, note)
-            bpas = bytes_per_ant_step(stats)
+            # the oracle on a stratified sample (per batch; c5 has two), on all host threads
+            share = max(4, args.cpu_sample if args.workload != "c5" else 24)
+            parts, stats_all, secs, scheds_cpu = [], [], 0.0, 0.0
+            for s, b in zip(scheds, batches):
+                ps, note = cpu_sample_params(args, b.p)
+                k = share if len(batches) == 1 else max(2, share // len(batches))
+                base, stats, pick, ores, dt, sc = cpu_baseline(b.regs, b.ids, ps, k, machine, note)
+                parts.append(base)
+                stats_all.append(stats)
+                secs += dt
+                scheds_cpu += sc
+                if args.parity == "off":
+                    continue
+                if ps == b.p:  # the timed run's own results
+                    gd = {b.ids[i]: all_digest[b.ids[i]] for i in pick}
+                else:  # reduced sample parameters: one more GPU run with them, same regions
+                    s.run(ps)
+                    rr = s.results()
+                    gd = {b.ids[i]: gpu_digest(rr[i]) for i in pick}
+                    parity_note = f"GPU re-run with the cpu_baseline sample parameters ({note})"
+                for q, i in enumerate(pick):
+                    check(b.ids[i], b.regs[i].n_insts, gd[b.ids[i]], ores[q])
+            cpu = dict(parts[0])
+            cpu["value"] = round(scheds_cpu / max(secs, 1e-9), 1)
+            if len(parts) > 1:
+                cpu["sample"] = " + ".join(x["sample"] for x in parts)
+            bpas = bytes_per_ant_step(np.concatenate(stats_all))
+        if args.parity != "off" and (n_cmp == 0 or args.parity == "all") and args.workload not in ("c4", "c5"):
+            # the oracle with the run's own parameters on a small stratified
+            # sample (N > 1: every rank's results gathered to rank 0), or on
+            # every region of the batch (--parity all)
+            all_regs = [(r, i, b.p) for b in batches for r, i in zip(b.regs, b.ids)]
+            if world > 1 and args.workload == "c3":  # rank 0 holds its share: regenerate the batch
+                all_regs = [(r, i, b.p) for b in workload(args, 0, 1)[0] for r, i in zip(b.regs, b.ids)
+                            if i in all_digest]
+            regs_ = [x[0] for x in all_regs]
+            pick = list(range(len(regs_))) if args.parity == "all" else stratified_pick(regs_, 24)
+            if args.parity == "all":
+                n_cmp, n_ok, bad, log = 0, 0, [], []
+            t0 = time.perf_counter()
+            pp = all_regs[0][2]
+            ores, _, _, _ = run_oracle([all_regs[i][0] for i in pick], [all_regs[i][1] for i in pick], pp, machine)
+            for q, i in enumerate(pick):
+                check(all_regs[i][1], all_regs[i][0].n_insts, all_digest[all_regs[i][1]], ores[q])
+            parity_note = (f"every region ({time.perf_counter() - t0:.0f} s of oracle)" if args.parity == "all"
+                           else f"{len(pick)} regions stratified by size, all ranks' results gathered to rank 0")
+        elif args.parity != "off" and n_cmp == 0:
+            parity_note = "not in this run (c4/c5 at N > 1: every-ant parity of these variants is in tests/)"
+        if n_cmp or parity_note:
+            parity = {"regions": n_cmp, "bit_exact": n_ok, "mismatches": bad[:8], "fields": list(PARITY_FIELDS),
+                      "sample": parity_note or "the cpu_baseline sample (stratified by size)"}
+        if args.parity_log and log:
+            with open(args.parity_log, "w") as f:
+                f.write(f"# parity {args.workload} N={world}: {n_ok}/{n_cmp} regions bit-exact vs the oracle "
+                        f"({', '.join(PARITY_FIELDS)})\n")
+                f.write("\n".join(log) + "\n")
         # roofline of the dominant kernel (ant construction):
         # algorithmic shared-memory bytes (SURVEY 8(d) per ant-step figure from
         # the oracle's instrumentation of the sample) x ant-steps per launch,
         # over the construct launches' CUDA-event time; peak = the SM shared
         # memory crossbar, 148 SMs x 128 B/clk x the SM clock seen under load.
         construct_ms = phase_ms[0] / max(1, args.steps)
-        ant_steps = p.ants * sum(r["n"] * (r["iters1"] + r["iters2"]) for r in res)
+        ant_steps = sum(b.p.ants * sum(r.n_insts * (res[i]["iters1"] + res[i]["iters2"])
+                                       for r, i in zip(b.regs, b.ids)) for b in batches)
         sm_mhz = clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
         smem_peak = 148 * 128 * sm_mhz * 1e6 / 1e9  # GB/s
         roof = None
         if bpas is not None and construct_ms > 0:
             n_launch = phase_launches[0] / max(1, args.steps)
             achieved = bpas * ant_steps / (construct_ms / 1000.0) / 1e9
-            traffic, tsrc, issue = None, None, None
-            try:  # DRAM bytes per construct launch from the committed ncu --set full capture
-                with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
-                    tj = json.load(f)
-                if args.workload == "c3":
-                    traffic, tsrc = tj["dram_bytes_per_launch"], tj["source"]
-                    # the bound that actually binds: SM issue slots, from ncu
-                    issue = {"util_pct": tj.get("issue_util_pct"), "warps_active_pct": tj.get("warps_active_pct"),
-                             "source": tj.get("issue_source")}
-            except Exception:
-                pass
             roof = {"bound": "smem", "achieved": round(achieved, 1), "peak": round(smem_peak, 1),
-                    "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": traffic,
-                    "traffic_source": tsrc, "issue_slots_ncu": issue,
+                    "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": None,
+                    "traffic_note": "ncu --set full DRAM bytes per construct launch: profiles/r02_*_ncu_summary.md",
                     "algorithmic_bytes_per_launch": round(bpas * ant_steps / max(1.0, n_launch)),
                     "kernel": "k_construct (all classes)", "bytes_per_ant_step": round(bpas, 2),
                     "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,
                     "construct_ms_per_step": round(construct_ms, 3),
                     "ant_steps_per_s": round(ant_steps / (construct_ms / 1000.0), 1),
                     "peak_source": f"guide: 148 SM x 128 B/clk x {sm_mhz:.0f} MHz (smem crossbar, no measured peak)"}
+        par = (f"shared colony x{world} (NCCL int64 MIN allreduce per iteration)" if args.workload == "c4"
+               else (f"regions LPT-partitioned x{world}" if scaling == "strong" else f"regions x{world}")
+               if args.workload in ("c3", "c5") else f"replicas x{world}")
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup),
             "ms_per_step": round(max_ms / args.steps, 3), "higher_is_better": True,
-            "scaling": "strong" if args.workload == "c4" else "weak",
-            "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)", "data": "synthetic",
-            "config": dict(cfg, l2="flushed between timed steps (256 MB write)",
-                           parallelism=f"shared colony x{world} (NCCL int64 MIN allreduce per iteration)"
-                           if args.workload == "c4" else f"regions x{world}"),
+            "scaling": scaling, "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
+            "data": "synthetic",
+            "config": dict(cfg, l2="flushed between timed steps (256 MB write)", parallelism=par),
             "aco_ms_per_batch": round(max_ms / args.steps, 3),
             "phase_ms_per_step": {"construct": round(phase_ms[0] / args.steps, 3),
                                   "finalize": round(phase_ms[1] / args.steps, 3),
-                                  "init": round(phase_ms[2] / args.steps, 3)},
+                                  "init": round(phase_ms[2] / args.steps, 3),
+                                  "note": "from K further steps with per-phase events (value is timed without them)"},
+            "pruned_pass2_ant_frac": round(prune_frac, 4),
             "gpu_launches": int(launches),
             "e2e": {"value": round(e2e_value, 1), "unit": METRIC, "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "ms_per_step": round(float(e.item()), 3)},
-            "clocks": clocks, "roofline": roof, "cpu_baseline": cpu,
+            "clocks": clocks, "roofline": roof, "cpu_baseline": cpu, "parity": parity,
         }
         print(json.dumps(out), flush=True)
     if world > 1:
@@ -396,36 +583,44 @@ def main():
     return out
 
 
+# ---------------------------------------------------------------- reference arm
 def reference_arm(args, world, rank):
-    """--impl reference: the oracle (as it stands) on the host cores, on a
-    bounded sample of this arm's workload per step."""
+    """--impl reference: the oracle (as it stands) on the host cores.  Every
+    step runs the SAME stratified sample of this arm's workload (the value
+    does not depend on --steps); the sample is shrunk only when K steps of it
+    would exceed the time budget, never below 4 regions per host thread."""
     if rank != 0:
         return None
-    regs, ids, p, cfg = workload(args, 0)
-    cpu_times = []
-    scheds = 0.0
-    ps, note = cpu_sample_params(args, p)
-    for _ in range(args.warmup):
-        pass  # the oracle has no warm-up state
-    # the --cpu-sample stratified sample, dealt round-robin over the steps
-    # (each step a smaller stratified sample, largest region first)
-    full = stratified_pick(regs, max(args.cpu_sample, 4 * args.steps))
-    per_step = deal_over_steps(full, args.steps)
-    for s in range(args.steps):
-        cpu, stats = cpu_baseline(regs, ids, ps, 0, machine_of(args), note, pick=per_step[s])
-        from oracle.pyoracle import ORS
-        s = float(stats[:, ORS["ant_scheds"]].sum())
+    batches, cfg, scaling = workload(args, 0, 1)
+    threads = os.cpu_count() or 1
+    budget_s = float(os.environ.get("ACO_REF_BUDGET_S", "240"))
+    b = max(batches, key=lambda x: sum(r.n_insts for r in x.regs))
+    ps, note = cpu_sample_params(args, b.p)
+    full = stratified_pick(b.regs, args.cpu_sample)
+    # size the per-step sample: time one step of the full sample, shrink if K of them would not fit
+    times, scheds = [], 0.0
+    res0, _, dt0, s0 = run_oracle([b.regs[i] for i in full], [b.ids[i] for i in full], ps, machine_of(args), threads)
+    pick = full
+    if dt0 * args.steps > budget_s:
+        keep = max(4 * threads, int(len(full) * budget_s / (dt0 * args.steps)))
+        pick = stratified_pick([b.regs[i] for i in full], min(len(full), keep))
+        pick = [full[i] for i in pick]
+    for _ in range(args.steps):
+        _, _, dt, s = run_oracle([b.regs[i] for i in pick], [b.ids[i] for i in pick], ps, machine_of(args), threads)
+        times.append(dt)
         scheds += s
-        cpu_times.append(s / cpu["value"])
-    tot_s = sum(cpu_times)
+    tot_s = sum(times)
     value = scheds / tot_s
     out = {"metric": METRIC, "value": round(value, 1), "unit": METRIC, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(1000 * tot_s / args.steps, 3), "higher_is_better": True,
-           "scaling": "strong" if args.workload == "c4" else "weak", "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
+           "scaling": scaling, "vs_baseline": None, "dtype": "u32/u16 fixed-point (integer only)",
            "data": "synthetic", "config": cfg, "impl": "reference",
-           "cpu_baseline": {"value": round(value, 1), "unit": METRIC, "cores": os.cpu_count(), "kind": "oracle",
-                            "sample": f"per step about {max(1, len(full) // args.steps)} regions (a stratified sample of "
-                                      f"{len(full)} dealt over the steps, largest first) of the {cfg['workload']} workload, {note}"},
+           "cpu_baseline": {"value": round(value, 1), "unit": METRIC, "cores": min(threads, len(pick)),
+                            "kind": "oracle", "host": host_cpu(),
+                            "regions_per_step": len(pick), "threads": threads,
+                            "sample": f"every step: the same {len(pick)} regions (stratified by size, largest first) "
+                                      f"of the {cfg['workload']} workload, {note}; {scheds / args.steps:.0f} "
+                                      f"ant-schedules per step on {threads} host threads"},
            "e2e": {"value": round(value, 1), "unit": METRIC, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
     return out

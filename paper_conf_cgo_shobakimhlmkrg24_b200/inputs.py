@@ -326,6 +326,33 @@ def gen_batch(count: int, base_seed: int = 3, profile: str = "mixed", first_id: 
                        name=f"c3-{first_id + i}") for i in range(count)]
 
 
+def gen_regions(ids: Sequence[int], sizes: Sequence[int], base_seed: int = 3, profile: str = "mixed",
+                tag: str = "c3") -> List[Region]:
+    """Regions with the given global ids of a batch whose region i has size
+    sizes[i] (strong scaling: any subset of the same batch, same regions)."""
+    return [gen_region(int(sizes[i]), region_seed(base_seed, int(i)), profile, name=f"{tag}-{int(i)}") for i in ids]
+
+
+# Config 5 (SURVEY 8(d)): n x latency profile x seed grid.
+C5_SIZES = (10, 20, 50, 100, 200, 500, 1000, 2000, 4000)
+C5_PROFILES = ("unit", "mixed")
+C5_SEEDS = (0, 1, 2)
+
+
+def c5_grid():
+    """[(global id, n, profile, seed index)] of the config-5 sweep."""
+    out = []
+    for n in C5_SIZES:
+        for prof in C5_PROFILES:
+            for s in C5_SEEDS:
+                out.append((len(out), n, prof, s))
+    return out
+
+
+def c5_region(gid: int, n: int, profile: str) -> Region:
+    return gen_region(n, region_seed(5, gid), profile, name=f"c5-n{n}-{profile}-{gid}")
+
+
 # --------------------------------------------------------------------------
 # Hand-built fixtures (data only).  FIG1-R reconstructs PAPER.md Fig. 1 from
 # its text (L143-L155, L184, L200); FIX10-A is config 1 (SURVEY.md 8(c)).

@@ -38,3 +38,23 @@ def test_reference_steps_partition_the_sample():
 def test_deal_over_steps_reuses_a_small_sample():
     assert bench.deal_over_steps([7], 3) == [[7], [7], [7]]
     assert bench.deal_over_steps([1, 2, 3, 4, 5], 2) == [[1, 3, 5], [2, 4]]
+
+
+def test_strong_partition_covers_the_batch_once():
+    """bench.py c3 at N ranks: the LPT shares of the same batch are disjoint,
+    cover every region, and regenerate the world-1 regions exactly."""
+    a = bench.parse(["--workload", "c3", "--regions", "60"])
+    one = bench.workload(a, 0, 1)[0][0]
+    shares = [bench.workload(a, r, 3)[0][0] for r in range(3)]
+    ids = sorted(i for b in shares for i in b.ids)
+    assert ids == list(range(60))
+    by_id = {i: r for b in shares for i, r in zip(b.ids, b.regs)}
+    for i, r in zip(one.ids, one.regs):
+        assert by_id[i].n_insts == r.n_insts and (by_id[i].edge_src == r.edge_src).all()
+
+
+def test_c5_grid_batches():
+    a = bench.parse(["--workload", "c5"])
+    b = bench.workload(a, 0, 1, gen=False)[0]
+    assert [x.p.iterations for x in b] == [10, 5]
+    assert len(bench.I.c5_grid()) == 9 * 2 * 3

@@ -43,7 +43,14 @@ def compare_results(gpu, ora, ctx=""):
     assert gpu["ws_cost"] == ora["ws_cost"], ctx
 
 
+# construct-kernel variants exercised by every-ant (dump) parity in this
+# session; tests/test_zz_variant_coverage.py checks the benchmarks' variants
+# against it
+DUMP_VARIANTS = set()
+
+
 def dump_parity(s, regions, ids, p, machine=I.GFX906):
+    DUMP_VARIANTS.update(s.variants())
     c, o, y = s.dump_arrays()
     A, n_it = p.ants, p.iterations
     for k, (reg, rid) in enumerate(zip(regions, ids)):
@@ -188,12 +195,15 @@ def test_config3_sampled(torch_cuda):
     g = s.results()
     sizes = np.array([r.n_insts for r in regs])
     sample = sorted(set([int(np.argmax(sizes)), int(np.argmin(sizes))] + list(range(0, 5000, 499))))
-    _, _, stats, off = O.schedule_many([regs[k] for k in sample], [ids[k] for k in sample], I.GFX906, p)
+    order, cyc, stats, off = O.schedule_many([regs[k] for k in sample], [ids[k] for k in sample], I.GFX906, p)
     for q, k in enumerate(sample):
         ora = {n: int(stats[q, i]) for n, i in O.ORS.items()}
         assert g[k]["trace_hash"] == ora["trace_hash"], k
         assert g[k]["length"] == ora["length"] and g[k]["cost_rp"] == ora["cost_rp"], k
         assert g[k]["prp"] == [ora["prp0"], ora["prp1"], ora["prp2"], ora["prp3"]], k
+        a, b = int(off[q]), int(off[q + 1])  # the final schedule itself: order and issue cycles
+        assert list(g[k]["order"]) == [int(x) for x in order[a:b]], k
+        assert list(g[k]["cycle"]) == [int(x) for x in cyc[a:b]], k
     # every region's final schedule is valid (independent checker)
     for k in range(0, 5000, 97):
         checker.check_schedule(regs[k], g[k]["order"], g[k]["cycle"], g[k]["length"])
