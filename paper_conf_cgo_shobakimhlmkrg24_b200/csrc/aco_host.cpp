@@ -968,7 +968,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         gs[r] = 1;
         lean = false;
         W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
-        gs_words[r] = std::max(gs_words[r], W);
+        gs_words[r] = std::max(gs_words[r], (W + 3u) & ~3u);  // (ant-major rows padded to 16 B)
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;
@@ -1226,6 +1226,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   cfg.stall_num = p->stall_num;
   cfg.rl_limit = p->rl_limit;
   cfg.mslot = (uint32_t)ctx->mslot;
+  cfg.gs_ant_major = 1;  // measured: DESIGN.md 5 (ACO_GS_LAYOUT=0: [word][ant])
+  if (const char *e = getenv("ACO_GS_LAYOUT")) cfg.gs_ant_major = atoi(e) != 0;
   cfg.record = P.record ? 1u : 0u;
   cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;

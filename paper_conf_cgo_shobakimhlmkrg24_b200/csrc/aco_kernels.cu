@@ -598,21 +598,29 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
   }
 }
 
-template <int PASS, bool MASK, bool T32, bool NC4, bool LEAN = false>
-__device__ __forceinline__ uint32_t init_state(const SV &V, const St &A) {
+// Initial per-ant state, written by the LG lanes of the ant's group (lane l
+// takes words l, l + LG, ...); returns the non-empty-word mask (MASK) in
+// every lane.
+template <int PASS, bool MASK, bool T32, bool NC4, bool LEAN = false, int LG = 1>
+__device__ __forceinline__ uint32_t init_state(const SV &V, const St &A, const Grp<LG> &G) {
   uint32_t wmask = 0;
-  for (uint32_t w = 0; w < V.nwr; ++w) {
+  for (uint32_t w = G.lane; w < V.nwr; w += LG) {
     const uint32_t x = V.rb0[w];
     A.RB[w * A.S] = x;
     A.SCH[w * A.S] = 0;
     if (MASK && x) wmask |= 1u << w;
   }
-  for (uint32_t w = 0; w < V.nremw; ++w) A.REM[w * A.S] = V.rem0[w];
+  for (uint32_t w = G.lane; w < V.nremw; w += LG) A.REM[w * A.S] = V.rem0[w];
   const uint32_t n = V.n;
   const bool ct = PASS == 2 && !T32 && !NC4;
   const uint32_t tw = PASS == 1 ? 0 : (LEAN ? (n + 3) / 4 : (T32 ? n : (n + 1) / 2));
   const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
-  for (uint32_t w = 0; w < tw + dw; ++w) A.T[w * A.S] = 0;  // T and DK are contiguous
+  for (uint32_t w = G.lane; w < tw + dw; w += LG) A.T[w * A.S] = 0;  // T and DK are contiguous
+  if (MASK && LG > 1) {
+#pragma unroll
+    for (int o = LG / 2; o > 0; o >>= 1) wmask |= __shfl_xor_sync(G.mask, wmask, o, LG);
+  }
+  G.sync();
   return wmask;
 }
 
@@ -670,10 +678,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
                                             const uint32_t rec_stride = 1) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   constexpr bool limit = RLIM;  // R45 (rl.buf or rl.in set)
-  uint32_t wmask = 0;
-  if (G.leader()) wmask = init_state<1, MASK, false, false>(V, A);
-  wmask = G.bcast(wmask);
-  G.sync();
+  uint32_t wmask = init_state<1, MASK, false, false, false, LG>(V, A, G);
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const uint32_t sub = lane_words<LG>(G.lane);
@@ -842,10 +847,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
                                             const uint32_t *coins = nullptr, uint32_t coin_t = 0,
                                             const uint32_t rec_stride = 1) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
-  uint32_t wmask = 0;
-  if (G.leader()) wmask = init_state<2, MASK, T32, NC4, LEAN>(V, A);
-  wmask = G.bcast(wmask);
-  G.sync();
+  uint32_t wmask = init_state<2, MASK, T32, NC4, LEAN, LG>(V, A, G);
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const bool stall_en = stall_group(cfg, group);      // R23, R44
@@ -1115,8 +1117,14 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 
   RL rl{nullptr, 0, 0, A.cfg.rl_limit, nullptr, nullptr};
   if (GS == 1) {  // huge region: statics through L1/L2, per-ant state in the workspace
     if (ai >= A.cfg.ants) return;
-    stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
-    stride = A.cfg.ants;
+    if (A.cfg.gs_ant_major) {  // ant-major: the lanes of one ant read consecutive words (coalesced scan)
+      const uint32_t wpa = (ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4) + 3u) & ~3u;
+      stbase = (uint32_t *)(A.ws + W.o_gstate) + (size_t)ai * wpa;
+      stride = 1;
+    } else {  // word-major [word][ant]
+      stbase = (uint32_t *)(A.ws + W.o_gstate) + ai;
+      stride = A.cfg.ants;
+    }
   } else {
     const uint32_t img_bytes = GS == 0 ? rd->img.bytes : 0u;
     if (GS == 0) stage(smem4, (const uint4 *)img, img_bytes);

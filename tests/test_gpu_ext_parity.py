@@ -102,7 +102,7 @@ def test_compile_policy_filters(torch_cuda):
     regs = [I.gen_region((60, 100, 150, 200, 250, 300)[i % 6], 1300 + i) for i in range(12, 18)]
     ids = list(range(12, 18))
     base = I.Params(ants=64, iterations=4, cost_mode=1)
-    for q in (dataclasses.replace(base, pass2_gap=21), dataclasses.replace(base, pass2_gap=400),
+    for q in (dataclasses.replace(base, pass2_gap=21), dataclasses.replace(base, pass2_gap=100000),
               dataclasses.replace(base, revert_occ=1, revert_len=0), I.paper_policy(base)):
         s = _sched()
         s.load(regs, ids).run(q)
@@ -112,7 +112,7 @@ def test_compile_policy_filters(torch_cuda):
             ora = O.schedule(regs[k], ids[k], I.GFX906, q)
             compare_results(g, ora, f"{q} region {k}")
             pol |= g["policy"]
-        if q.pass2_gap == 400:
+        if q.pass2_gap == 100000:
             assert all(g["policy"] & 1 and g["iters2"] == 0 for g in got)
         if q.revert_occ == 1:
             assert pol & 2  # region 14 reverts (see test_oracle_ext_pins)
