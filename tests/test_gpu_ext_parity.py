@@ -99,7 +99,10 @@ def test_stall_fraction_every_ant(torch_cuda, num, rem):
 def test_compile_policy_filters(torch_cuda):
     """Cycle-gap filter and revert filter (production mode) on a batch whose
     regions straddle the thresholds; policy bits and heuristic lengths."""
-    regs = [I.gen_region((60, 100, 150, 200, 250, 300)[i % 6], 1300 + i) for i in range(12, 18)]
+    # regions of the round-1 generator calibration (recency 0.3, 2 VGPR
+    # live-ins), where region 14 reverts under (revert_occ 1, revert_len 0)
+    regs = [I.gen_region((60, 100, 150, 200, 250, 300)[i % 6], 1300 + i, recency=0.3, v_livein=2)
+            for i in range(12, 18)]
     ids = list(range(12, 18))
     base = I.Params(ants=64, iterations=4, cost_mode=1)
     for q in (dataclasses.replace(base, pass2_gap=21), dataclasses.replace(base, pass2_gap=100000),
