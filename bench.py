@@ -323,6 +323,34 @@ def gpu_digest(r: dict) -> dict:
             "trace_hash": r["trace_hash"]}
 
 
+# APRP bands of the gfx906 VGPR table (R17): upper bound of each band
+VGPR_BANDS = (24, 28, 32, 36, 40, 48, 64, 84, 128, 256)
+
+
+def schedule_quality(res: dict) -> dict:
+    """Histogram of the heuristic (greedy, R28) and final ACO VGPR PRP over the
+    regions' occupancy bands, plus how many regions the RP pass improved
+    (final cost below the heuristic cost) and the mean / max pass-2 length
+    gain over its input schedule -- the RP pass visibly doing work."""
+    def band(x):
+        for i, b in enumerate(VGPR_BANDS):
+            if x <= b:
+                return i
+        return len(VGPR_BANDS)
+    h = [0] * (len(VGPR_BANDS) + 1)
+    a = [0] * (len(VGPR_BANDS) + 1)
+    for r in res.values():
+        h[band(r["heur_prp"][0])] += 1
+        a[band(r["prp"][0])] += 1
+    imp = sum(1 for r in res.values() if r["best1"] < r["init1"])
+    gains = [(r["init2"] - r["length"]) / r["init2"] for r in res.values() if r["init2"]]
+    return {"vgpr_band_upper": list(VGPR_BANDS) + ["more"], "regions_by_heuristic_vgpr_band": h,
+            "regions_by_aco_vgpr_band": a, "regions": len(res), "rp_pass_improved_cost": imp,
+            "heuristic_vgpr_prp_above_24": sum(h[1:]), "aco_vgpr_prp_above_24": sum(a[1:]),
+            "pass2_len_gain_mean_pct": round(100 * float(np.mean(gains)), 2) if gains else None,
+            "pass2_len_gain_max_pct": round(100 * float(np.max(gains)), 2) if gains else None}
+
+
 def parity_compare(gpu: dict, ora: dict):
     """Names of the fields where the GPU result differs from the oracle's."""
     return [f for f in PARITY_FIELDS if gpu[f] != ora[f]]
@@ -575,6 +603,7 @@ def main(argv=None):
             "e2e": {"value": round(e2e_value, 1), "unit": METRIC, "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "ms_per_step": round(float(e.item()), 3)},
             "clocks": clocks, "roofline": roof, "cpu_baseline": cpu, "parity": parity,
+            "schedule_quality": schedule_quality(res) if args.workload != "c4" or not colony else None,
         }
         print(json.dumps(out), flush=True)
     if world > 1:

@@ -140,6 +140,7 @@ typedef struct {
   uint32_t heur_len;     /* length of the heuristic schedule (greedy order timed ASAP, R40) */
   uint32_t ws_cost;      /* pass 4: final weighted cost (R41), else 0 */
   uint32_t ants_pruned;  /* pass-2 ants cut short by the winner-invariant prune (R24), all iterations */
+  uint32_t heur_prp[4];  /* PRP per class of the greedy heuristic schedule (R28), the RP pass's start */
 } aco_result;
 
 /* Create a context on CUDA device `device` for machine model *m (copied). */

@@ -69,6 +69,7 @@ class Result(C.Structure):
         ("init_cost", C.c_uint32 * 2), ("lb_cost", C.c_uint32), ("lb_len", C.c_uint32),
         ("target", C.c_uint32 * 4), ("trace_hash", C.c_uint64),
         ("policy", C.c_uint32), ("heur_len", C.c_uint32), ("ws_cost", C.c_uint32), ("ants_pruned", C.c_uint32),
+        ("heur_prp", C.c_uint32 * 4),
     ]
 
 

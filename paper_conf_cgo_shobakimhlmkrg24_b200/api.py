@@ -287,7 +287,7 @@ class Scheduler:
                 iters1=r.iters_run[0], iters2=r.iters_run[1], best1=r.best_cost[0], best2=r.best_cost[1],
                 init1=r.init_cost[0], init2=r.init_cost[1], lb1=r.lb_cost, lblen=r.lb_len,
                 target=list(r.target), trace_hash=int(r.trace_hash),
-                policy=r.policy, heur_len=r.heur_len, ws_cost=r.ws_cost, ants_pruned=r.ants_pruned,
+                policy=r.policy, heur_len=r.heur_len, ws_cost=r.ws_cost, ants_pruned=r.ants_pruned, heur_prp=list(r.heur_prp),
                 order=orders[a:b].copy(), cycle=cycles[a:b].copy()))
         return res
 

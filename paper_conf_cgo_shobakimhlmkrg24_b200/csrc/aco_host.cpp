@@ -91,6 +91,18 @@ struct aco_ctx_s {
   // as the previous one reuses its plan (launch classes, workspace layout and
   // the plan blob already in the workspace) -- ~11 ms of host time on C3
   bool cache_ok = false;
+  bool cache_hit = false;  // the last make_plan reused the cached plan
+  // CUDA graph of a whole aco_schedule_batch (every launch of both passes),
+  // captured on the second run of a cached plan and replayed while the plan
+  // stays cached (the launch-free iteration loop)
+  cudaGraphExec_t gexec = nullptr;
+  bool gexec_ok = false;
+  uint64_t gexec_launches = 0;
+  void drop_graph() {
+    if (gexec) cudaGraphExecDestroy(gexec);
+    gexec = nullptr;
+    gexec_ok = false;
+  }
   aco_params cache_params{};
   void *cache_ws = nullptr;
   size_t cache_ws_bytes = 0, cache_need = 0;
@@ -133,9 +145,17 @@ struct aco_ctx_s {
   static constexpr int kStreams = 4;
   cudaStream_t side[kStreams] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t fork_ev = nullptr, join_ev[kStreams] = {nullptr, nullptr, nullptr, nullptr};
+  // graph stream: the captured run is launched here, ordered after / before
+  // the caller's stream by two events (the caller's stream may be the legacy
+  // default stream, which cannot be captured)
+  cudaStream_t gstream = nullptr;
+  cudaEvent_t g_in = nullptr, g_out = nullptr;
   bool side_ok = false;
   bool make_side() {
     if (side_ok) return true;
+    if (cudaStreamCreateWithFlags(&gstream, cudaStreamNonBlocking) != cudaSuccess) return false;
+    if (cudaEventCreateWithFlags(&g_in, cudaEventDisableTiming) != cudaSuccess) return false;
+    if (cudaEventCreateWithFlags(&g_out, cudaEventDisableTiming) != cudaSuccess) return false;
     for (int i = 0; i < kStreams; ++i) {
       if (cudaStreamCreateWithFlags(&side[i], cudaStreamNonBlocking) != cudaSuccess) return false;
       if (cudaEventCreateWithFlags(&join_ev[i], cudaEventDisableTiming) != cudaSuccess) return false;
@@ -145,12 +165,16 @@ struct aco_ctx_s {
     return true;
   }
   ~aco_ctx_s() {
+    drop_graph();
     release_machine_slot(device, mslot);
     for (int i = 0; i < kStreams; ++i) {
       if (side[i]) cudaStreamDestroy(side[i]);
       if (join_ev[i]) cudaEventDestroy(join_ev[i]);
     }
     if (fork_ev) cudaEventDestroy(fork_ev);
+    if (gstream) cudaStreamDestroy(gstream);
+    if (g_in) cudaEventDestroy(g_in);
+    if (g_out) cudaEventDestroy(g_out);
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
     for (int i = 0; i < 2; ++i) {
       if (pin_ev[i]) cudaEventDestroy(pin_ev[i]);
@@ -490,6 +514,24 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   R.img.info = img_put(img, info);
   R.img.ds = img_put(img, ds);
   R.img.muse = img_put(img, muse);
+  {  // kill tests of the multi-use entries on the per-ant state (lean pass 2):
+     // a counter register (RB, SCH, then REM: word 2 nwr + m / 2, half m % 2)
+     // is last-used at 1 remaining use; a 2-user register when its partner's
+     // scheduled bit (SCH word nwr + p / 32) is set; word < 2 * 256 + 32768 fits 16 bits
+    const uint32_t nwr0 = (n + 31) / 32;
+    std::vector<uint32_t> mk(muse.size());
+    for (size_t q = 0; q < muse.size(); ++q) {
+      const uint32_t e = muse[q], c = (e >> 16) & 3u;
+      if (e & kMuseCounter) {
+        const uint32_t m = e & 0xFFFFu;
+        mk[q] = (2 * nwr0 + (m >> 1)) | (((m & 1u) * 16) << 16) | kMkCounter | (c << 22);
+      } else {
+        const uint32_t pa = e & 0x1FFFu;
+        mk[q] = (nwr0 + (pa >> 5)) | ((pa & 31u) << 16) | (c << 22);
+      }
+    }
+    R.img.mk = img_put(img, mk);
+  }
   R.img.cu_ptr = img_put(img, cu_ptr);
   R.img.cu = img_put(img, cu);
   R.img.eta1 = img_put(img, eta1);
@@ -592,6 +634,7 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
                             size_t arena_bytes, size_t *arena_needed, void *cuda_stream) {
   if (!ctx || (count && !regions)) return ACO_E_ARG;
   ctx->cache_ok = false;
+  ctx->drop_graph();
   {  // unique region ids
     std::vector<uint32_t> ids(count);
     for (uint32_t i = 0; i < count; ++i) ids[i] = regions[i].region_id;
@@ -797,9 +840,14 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     ctx->stream = cuda_stream;
     ctx->have_run = true;
     ctx->planned = true;
+    ctx->cache_hit = true;
     return ACO_OK;
   }
-  if (d_workspace) ctx->cache_ok = false;  // (a sizing call leaves the cached plan intact)
+  if (d_workspace) {  // (a sizing call leaves the cached plan intact)
+    ctx->cache_ok = false;
+    ctx->cache_hit = false;
+    ctx->drop_graph();
+  }
   if ((p->flags & ACO_FLAG_DUMP) && (!ctx->dump_cost || colony)) return ACO_E_ARG;
   if (p->flags & ACO_FLAG_DUMP) {  // the dump buffers must hold every (pass, iteration) slice
     const uint64_t sn = ctx->inst_off.empty() ? 0 : ctx->inst_off[ctx->count];
@@ -858,6 +906,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t lean_gain = 0;  // % more resident ants the lean layout must reach (C3: 0 measured best)
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
+  bool gs_wide = true;  // 4-wide scan in the global-state kernels
+  if (const char *e = getenv("ACO_GS_WIDE")) gs_wide = atoi(e) != 0;
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
@@ -972,9 +1022,13 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wide && mask, sh.ig, lean);
+      // global-state kernels: 4-wide candidate scan over strided words (not in
+      // the u32-cycle / 3-4 class instantiations)
+      const bool gwide = g && gs_wide && !(pass == 2 && (t32 || P.nc4));
+      const bool wk = (wide && mask) || gwide;
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];
-      c.wide = wide && mask;
+      c.wide = wk;
       c.sh = sh;
       c.mask = mask;
       c.t32 = pass == 2 && t32;
@@ -1352,18 +1406,58 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   if (!ctx || !p) return ACO_E_ARG;
   aco_status st = make_plan(ctx, p, 0, d_workspace, ws_bytes, ws_needed, cuda_stream, false);
   if (st != ACO_OK || !d_workspace) return st;
-  int err = run_init(ctx);
-  for (uint32_t pass = 1; pass <= 2 && !err; ++pass) {
-    if (pass == 2) err |= run_pass2_init(ctx);
-    if (!(ctx->plan.pass_mask & pass)) continue;
-    for (uint32_t it = 0; it < p->iterations && !err; ++it) {
-      err |= run_construct(ctx, pass, it);
-      err |= run_finalize(ctx, pass, it, nullptr);
-    }
+  cudaStream_t s = (cudaStream_t)cuda_stream;
+  // Replay of the captured graph: the plan is cached (same parameters,
+  // workspace, regions and dump buffers), so every launch and its arguments
+  // are identical to the captured run's; the kernels take every data-dependent
+  // decision (stop rules, active regions) on the device.
+  static const bool graphs = [] {
+    const char *e = getenv("ACO_GRAPH");
+    return e ? atoi(e) != 0 : true;
+  }();
+  const bool use_graph = graphs && ctx->cache_hit && !ctx->plan.timing;
+  // graph launch on the graph stream, ordered after and before the caller's stream
+  auto launch_graph = [&]() {
+    return cudaEventRecord(ctx->g_in, s) != cudaSuccess || cudaStreamWaitEvent(ctx->gstream, ctx->g_in, 0) != cudaSuccess ||
+           cudaGraphLaunch(ctx->gexec, ctx->gstream) != cudaSuccess ||
+           cudaEventRecord(ctx->g_out, ctx->gstream) != cudaSuccess || cudaStreamWaitEvent(s, ctx->g_out, 0) != cudaSuccess;
+  };
+  if (use_graph && ctx->gexec_ok) {
+    ctx->launches = ctx->gexec_launches;
+    return launch_graph() ? ACO_E_CUDA : ACO_OK;
   }
-  if (!err) err |= run_post(ctx);
-  ctx->launches = ctx->plan.L.launches;
-  return err ? ACO_E_CUDA : ACO_OK;
+  auto issue = [&]() {  // the launch sequence of L135-L139
+    int e = run_init(ctx);
+    for (uint32_t pass = 1; pass <= 2 && !e; ++pass) {
+      if (pass == 2) e |= run_pass2_init(ctx);
+      if (!(ctx->plan.pass_mask & pass)) continue;
+      for (uint32_t it = 0; it < p->iterations && !e; ++it) {
+        e |= run_construct(ctx, pass, it);
+        e |= run_finalize(ctx, pass, it, nullptr);
+      }
+    }
+    if (!e) e |= run_post(ctx);
+    ctx->launches = ctx->plan.L.launches;
+    return e;
+  };
+  if (use_graph && cudaStreamBeginCapture(ctx->gstream, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
+    ctx->plan.L.stream = ctx->gstream;  // the launch sequence is recorded on the graph stream
+    const int ce = issue();
+    ctx->plan.L.stream = cuda_stream;
+    cudaGraph_t g = nullptr;
+    const bool ended = cudaStreamEndCapture(ctx->gstream, &g) == cudaSuccess && g;
+    if (!ce && ended && cudaGraphInstantiate(&ctx->gexec, g, 0) == cudaSuccess) {
+      ctx->gexec_ok = true;
+      ctx->gexec_launches = ctx->launches;
+    } else {
+      ctx->drop_graph();
+    }
+    if (g) cudaGraphDestroy(g);
+    cudaGetLastError();
+    if (ctx->gexec_ok) return launch_graph() ? ACO_E_CUDA : ACO_OK;
+    ctx->plan.L.launches = 0;  // capture failed: nothing ran, launch directly
+  }
+  return issue() ? ACO_E_CUDA : ACO_OK;
 }
 
 aco_status aco_colony_begin(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *d_workspace, size_t ws_bytes,
@@ -1517,6 +1611,7 @@ aco_status aco_get_results(aco_ctx ctx, uint32_t first, uint32_t count, aco_resu
     o.heur_len = S.heur_len;
     o.ws_cost = ctx->cfg.weighted ? S.best[1] : 0u;
     o.ants_pruned = S.pruned;
+    for (int c = 0; c < 4; ++c) o.heur_prp[c] = S.heur_prp[c];
   }
   for (uint64_t q = 0; q < i1 - i0; ++q) {
     if (orders) orders[q] = o16[q];

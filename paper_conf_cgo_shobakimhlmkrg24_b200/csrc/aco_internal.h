@@ -54,7 +54,12 @@ struct ImageLayout {
   uint32_t bytes;     // total, multiple of 16
   uint32_t pg_ptr;    // u32 [n+1]: predecessor groups of each instruction
   uint32_t pg;        // uint2 [..]: {bitset word, mask of the predecessors in that word}
+  uint32_t mk;        // u32 [nm]: muse entry as a kill test on the per-ant state (lean layout):
+                      //   word (bits 0-15, relative to the state base) | shift << 16 |
+                      //   counter << 21 | class << 22; last use iff ((w >> shift) & (counter ? 0xFFFF : 1)) == 1
+  uint32_t pad_img;
 };
+constexpr uint32_t kMkCounter = 1u << 21;
 
 // Per-region statics (arena header array).
 struct RegionDev {
@@ -240,7 +245,7 @@ struct ClassLaunch {
   bool t32;                // u32 pass-2 cycle array
   bool nc4;                // 3-4 register classes (u16 last-use counts)
   bool gs;                 // per-ant state in global memory (huge regions)
-  bool wide;               // 4-wide candidate scan (n >= kWideN, word-mask variant)
+  bool wide;               // 4-wide candidate scan (n >= kWideN: word-mask variant; global state: strided words)
   bool img_l1 = false;     // the block image is read through L1 (not staged): more ants per SM
   bool lean = false;       // pass 2: lean per-ant layout (u8 ready times, dynamic kills)
 };
@@ -261,7 +266,7 @@ inline uint32_t class_variant(uint32_t pass, const ClassLaunch &c) {
   const bool mask = c.max_n <= 1024 && !c.gs;
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   return variant_code(pass, c.lanes, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32, pass == 2 && c.nc4,
-                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && mask, pass == 2 && c.lean);
+                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && (mask || c.gs), pass == 2 && c.lean);
 }
 
 int set_machine(uint32_t slot, const MachineDev &m);  // cudaMemcpyToSymbol into slot; 0 on success

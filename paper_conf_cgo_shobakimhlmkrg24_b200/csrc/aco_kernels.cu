@@ -135,7 +135,7 @@ __device__ void target_of(uint32_t ms, uint32_t mode, const uint32_t best[4], ui
 struct SV {
   const uint4 *info;
   const uint4 *ds;
-  const uint32_t *muse, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0, *pg_ptr;
+  const uint32_t *muse, *mk, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0, *pg_ptr;
   const uint2 *pg;
   const uint16_t *eta1, *eta2;
   uint32_t n, nwr, nremw, region_id, L1;
@@ -147,6 +147,7 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   V.info = (const uint4 *)(img + rd->img.info);
   V.ds = (const uint4 *)(img + rd->img.ds);
   V.muse = (const uint32_t *)(img + rd->img.muse);
+  V.mk = (const uint32_t *)(img + rd->img.mk);
   V.cu_ptr = (const uint32_t *)(img + rd->img.cu_ptr);
   V.cu = (const uint32_t *)(img + rd->img.cu);
   V.eta1 = (const uint16_t *)(img + rd->img.eta1);
@@ -288,25 +289,23 @@ __device__ __forceinline__ void r8_push(const St &A, uint32_t v, uint32_t rt) {
 // users whose last unscheduled user j is (R14): a counter register with one
 // remaining use, or a 2-user register whose partner is scheduled.
 // dsw = ds.w of j (multi-use count << 4 | start << 8).
+__device__ __forceinline__ uint32_t mk_last(const St &A, uint32_t e) {  // e: an mk entry (ImageLayout::mk)
+  const uint32_t w = A.RB[(e & 0xFFFFu) * A.S];  // RB is the state base
+  return ((w >> ((e >> 16) & 31u)) & ((e & kMkCounter) ? 0xFFFFu : 1u)) == 1u;
+}
 __device__ __forceinline__ uint32_t dyn_kills(const SV &V, const St &A, uint32_t dsw) {
   uint32_t K = 0;
   const uint32_t mc = (dsw >> 4) & 0xFu, m0 = dsw >> 8;
   for (uint32_t q = 0; q < mc; ++q) {
-    const uint32_t e = V.muse[m0 + q];
-    uint32_t last;
-    if (e & kMuseCounter) {
-      const uint32_t m = e & 0xFFFFu;
-      last = ((A.REM[(m >> 1) * A.S] >> ((m & 1u) * 16)) & 0xFFFFu) == 1u;
-    } else {
-      last = sch_bit(A, e & 0x1FFFu);
-    }
-    K += last << (8 * ((e >> 16) & 3u));
+    const uint32_t e = V.mk[m0 + q];
+    K += mk_last(A, e) << (8 * ((e >> 22) & 3u));
   }
   return K;
 }
 // dyn_kills of four candidates at once: level q of every candidate's
 // multi-use list is fetched together (two dependent shared/L1 loads per
-// level for all four, instead of four serial chains).
+// level for all four, instead of four serial chains).  An exhausted list
+// reads state word 0 (in bounds) and is masked out.
 __device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4 (&ds)[4], uint32_t (&dk)[4]) {
   uint32_t mc[4], m0[4], mx = 0;
 #pragma unroll
@@ -319,18 +318,13 @@ __device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4
   for (uint32_t q = 0; q < mx; ++q) {
     uint32_t e[4], w[4];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) e[u] = q < mc[u] ? V.muse[m0[u] + q] : 0u;
+    for (int u = 0; u < 4; ++u) e[u] = q < mc[u] ? V.mk[m0[u] + q] : 0u;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {  // counter word (>= 3 users) or the partner's scheduled-set word
-      const uint32_t m = e[u] & 0xFFFFu, pa = e[u] & 0x1FFFu;
-      w[u] = (e[u] & kMuseCounter) ? A.REM[(m >> 1) * A.S] : A.SCH[(pa >> 5) * A.S];
-    }
+    for (int u = 0; u < 4; ++u) w[u] = A.RB[(e[u] & 0xFFFFu) * A.S];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      const uint32_t m = e[u] & 0xFFFFu, pa = e[u] & 0x1FFFu;
-      const uint32_t last = (e[u] & kMuseCounter) ? (((w[u] >> ((m & 1u) * 16)) & 0xFFFFu) == 1u)
-                                                  : ((w[u] >> (pa & 31u)) & 1u);
-      dk[u] += (q < mc[u] ? last : 0u) << (8 * ((e[u] >> 16) & 3u));
+      const uint32_t last = ((w[u] >> ((e[u] >> 16) & 31u)) & ((e[u] & kMkCounter) ? 0xFFFFu : 1u)) == 1u;
+      dk[u] += (q < mc[u] && last ? 1u : 0u) << (8 * ((e[u] >> 22) & 3u));
     }
   }
 }
@@ -482,6 +476,38 @@ __device__ __forceinline__ void scan4(const St &A, uint32_t m, F &&visit) {
     if (!v[3] || (!bits && !m)) return;
   }
 #endif
+}
+
+// Batched scan without a word mask (huge regions, global-state kernels):
+// this lane's words first, first + stride, ... < nwr, four set bits at a time
+// in ascending order (same contract as scan4).
+template <typename F>
+__device__ __forceinline__ void scan4s(const St &A, uint32_t first, uint32_t stride, uint32_t nwr, F &&visit) {
+  uint32_t w = 0, bits = 0, nw = first;
+  while (true) {
+    uint32_t j[4];
+    bool v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      while (!bits && nw < nwr) {
+        w = nw;
+        bits = A.RB[w * A.S];
+        nw += stride;
+      }
+      v[u] = bits != 0u;
+      j[u] = v[u] ? w * 32u + (__ffs(bits) - 1) : j[0];
+      bits &= bits - 1;
+    }
+    if (!v[0]) return;
+    visit(j, v);
+    if (!v[3] || (!bits && nw >= nwr)) return;
+  }
+}
+template <bool MASK, typename F>
+__device__ __forceinline__ void scan4_any(const St &A, uint32_t m, uint32_t first, uint32_t stride, uint32_t nwr,
+                                          F &&visit) {
+  if constexpr (MASK) scan4(A, m, visit);
+  else scan4s(A, first, stride, nwr, visit);
 }
 
 struct AntOut {
@@ -682,7 +708,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const uint32_t sub = lane_words<LG>(G.lane);
-  constexpr bool wide = MASK && WIDE;
+  constexpr bool wide = WIDE;  // 4-wide scan (word mask or strided words)
   // R43: odd groups are guided by the ILP heuristic (CP, eta2) instead
   const bool mix = !greedy && cfg.heur_mix && (group & 1u);
   uint32_t prev = n;
@@ -735,7 +761,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     uint32_t bs1 = 0, bj = 0;
     unsigned long long sum = 0;
     if constexpr (wide) {
-      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v0)[4]) {
+      scan4_any<MASK>(A, wmask & sub, G.lane, LG, nwr, [&](const uint32_t(&j)[4], const bool(&v0)[4]) {
         uint32_t tv[4], dk[4];
         bool v[4];
 #pragma unroll
@@ -854,7 +880,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   const bool mix = cfg.heur_mix && (group & 1u);      // R43: odd groups use eta1 (LUC, CP)
   const uint32_t c2 = 0x80000000u | iter;
   const uint32_t sub = lane_words<LG>(G.lane);
-  constexpr bool wide = MASK && WIDE;
+  constexpr bool wide = WIDE;  // 4-wide scan (word mask or strided words)
   constexpr bool CT = !T32 && !NC4;  // compact layout (x_get)
   // general machine model (R42): runtime, only in the u32-cycle variants
   const uint32_t w = T32 ? c_mach[cfg.mslot].issue_width : 1u;
@@ -944,7 +970,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       }
     };
     if constexpr (wide) {
-      scan4(A, wmask & sub, [&](const uint32_t(&j)[4], const bool(&v)[4]) {
+      scan4_any<MASK>(A, wmask & sub, G.lane, LG, nwr, [&](const uint32_t(&j)[4], const bool(&v)[4]) {
         uint32_t rd[4], dk[4], tv[4];
         uint4 ds[4];
 #pragma unroll
@@ -1096,7 +1122,7 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
 // staged) in shared memory: more ants resident per SM.
 // LEAN: pass-2 lean per-ant layout (u8 ready times, dynamic kills).
 template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS, bool WIDE, bool LEAN = false>
-__global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, WIDE ? 1 : 2)
+__global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE && GS != 1) ? 1 : 2)
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
@@ -1685,13 +1711,20 @@ static void for_each_construct(F &&f) {
   reg_rare<1, false>(f);
   reg_rare<4, true>(f);
   reg_rare<4, false>(f);
-  // huge regions: per-ant state in the workspace, 4 lanes per ant
+  // huge regions: per-ant state in the workspace, 4 / 8 / 16 lanes per ant,
+  // 1-wide or 4-wide candidate scan (strided words, scan4s)
   reg1<1, 4, false, false, false, false, 1, false>(f);
   reg1<2, 4, false, false, false, false, 1, false>(f);
   reg1<1, 8, false, false, false, false, 1, false>(f);
   reg1<2, 8, false, false, false, false, 1, false>(f);
   reg1<1, 16, false, false, false, false, 1, false>(f);
   reg1<2, 16, false, false, false, false, 1, false>(f);
+  reg1<1, 4, false, false, false, false, 1, true>(f);
+  reg1<2, 4, false, false, false, false, 1, true>(f);
+  reg1<1, 8, false, false, false, false, 1, true>(f);
+  reg1<2, 8, false, false, false, false, 1, true>(f);
+  reg1<1, 16, false, false, false, false, 1, true>(f);
+  reg1<2, 16, false, false, false, false, 1, true>(f);
   reg1<2, 4, false, false, true, false, 1, false>(f);
   reg1<2, 4, false, false, false, true, 1, false>(f);
   reg1<2, 4, false, false, true, true, 1, false>(f);

@@ -131,3 +131,28 @@ def test_plan_cache_colony_then_batch(torch_cuda):
         got = s.results()
         for k in range(len(regs)):
             compare_results(got[k], ora[k], f"{mode} region {k}")
+
+
+def test_graph_replay_equals_oracle(torch_cuda, monkeypatch):
+    """Identical runs: the 1st launches directly, the 2nd captures the whole
+    run as a CUDA graph, the 3rd+ replay it (also on another stream); every
+    run equals the oracle, and the graph run reports the same launch count."""
+    regs = [I.gen_region(n, 3800 + n) for n in (12, 40, 130, 300, 1200)]
+    ids = [20, 21, 22, 23, 24]
+    p = I.Params(ants=96, iterations=3, seed=66)
+    ora = [O.schedule(r, i, I.GFX906, p) for r, i in zip(regs, ids)]
+    s = _sched()
+    s.load(regs, ids)
+    counts = []
+    side = torch_cuda.cuda.Stream()
+    for k in range(5):
+        if k == 3:
+            with torch_cuda.cuda.stream(side):
+                s.run(p, stream=side)
+        else:
+            s.run(p)
+        got = s.results()
+        counts.append(s.launch_count())
+        for q in range(len(regs)):
+            compare_results(got[q], ora[q], f"run {k} region {q}")
+    assert len(set(counts)) == 1, counts
