@@ -1022,9 +1022,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;
-      // global-state kernels: 4-wide candidate scan over strided words (not in
-      // the u32-cycle / 3-4 class instantiations)
-      const bool gwide = g && gs_wide && !(pass == 2 && (t32 || P.nc4));
+      // global-state kernels: 4-wide candidate scan over strided words with
+      // <= 8 lanes per ant (not in the u32-cycle / 3-4 class instantiations).
+      // Measured (r02d, ms per step): C5 (4 lanes) 1963 -> 1808; C4 (16 lanes,
+      // few candidates per lane) 855 -> 872, so 16-lane classes stay 1-wide
+      const bool gwide = g && gs_wide && sh.lanes <= 8 && !(pass == 2 && (t32 || P.nc4));
       const bool wk = (wide && mask) || gwide;
       const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];
