@@ -79,6 +79,8 @@ struct Plan {
   uint32_t init_smem = 0, p2_smem = 0, max_n = 0, n_upd = 0;
   uint32_t pass_mask = 0, iterations = 0;
   bool any_t32 = false, nc4 = false, timing = false, p2_done = false, stage_img = false, record = false;
+  bool fused = false;  // the whole run in one k_fused launch (one block per region)
+  uint32_t fused_threads = 0, fused_smem = 0;
   uint64_t o_state = 0, o_rws = 0, o_upd = 0, o_gb2 = 0, o_gb2c = 0, o_keys = 0;
   LaunchCtx L{};
 };
@@ -1228,8 +1230,31 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                 (int)sorted[i].img_l1, (int)sorted[i].lean,
                 (double)class_work[pass][idx[i]]);
   }
+  // Fused single-block run (k_fused): every region's ants fit one block and
+  // its image, pheromone table, ant states and recorded schedules fit shared
+  // memory; a batch with few ants in total (config 1), where the per-launch
+  // latency of the multi-launch path dominates.  Word-mask scan, compact
+  // pass-2 layout; not the shared colony nor the ready-list limit.
+  {
+    uint32_t fused_ants = 512;
+    if (const char *e = getenv("ACO_FUSED_ANTS")) fused_ants = (uint32_t)atoi(e);
+    bool ok = !colony && p->rl_limit == 0 && count > 0 && A <= 512 && (uint64_t)count * A <= fused_ants &&
+              ctx->mach.issue_width <= 1 && !P.nc4;
+    uint32_t smem = 0;
+    for (uint32_t r = 0; r < count && ok; ++r) {
+      const RegionDev &R = ctx->regions[r];
+      ok = R.n <= 1024 && R.max_lat <= 511u && R.mc_max <= 7u;
+      if (ok) smem = std::max(smem, fused_layout(R.n, R.nwr, R.nremw, R.img.bytes, A).bytes);
+    }
+    if (ok && smem <= kSmemPerSM) {
+      P.fused = true;
+      P.fused_threads = std::max(32u, (A + 31u) & ~31u);
+      P.fused_smem = smem;
+    }
+  }
   ctx->variants.clear();  // construct-kernel variants of this plan (aco_last_variants)
-  for (int pass = 1; pass <= 2; ++pass)
+  if (P.fused) ctx->variants.push_back(kFusedVariant);
+  for (int pass = 1; pass <= 2 && !P.fused; ++pass)
     for (const ClassLaunch &cl : P.launches[pass]) {
       const uint32_t code = class_variant((uint32_t)pass, cl);
       if (std::find(ctx->variants.begin(), ctx->variants.end(), code) == ctx->variants.end())
@@ -1427,6 +1452,12 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   if (use_graph && ctx->gexec_ok) {
     ctx->launches = ctx->gexec_launches;
     return launch_graph() ? ACO_E_CUDA : ACO_OK;
+  }
+  if (ctx->plan.fused) {  // the whole run in one launch (no graph needed)
+    Bracket b(ctx, 0);
+    const int e = launch_fused(ctx->plan.L, ctx->plan.fused_threads, ctx->plan.fused_smem);
+    ctx->launches = ctx->plan.L.launches;
+    return e ? ACO_E_CUDA : ACO_OK;
   }
   auto issue = [&]() {  // the launch sequence of L135-L139
     int e = run_init(ctx);

@@ -219,6 +219,32 @@ ACO_HD inline uint32_t coin_words(uint32_t pass, uint32_t n) {
 // Bytes of the pheromone table as staged in shared memory.
 ACO_HD inline uint32_t tau_smem_bytes(uint32_t n) { return (((n + 1) * n * 2) + 15) & ~15u; }
 
+// Shared-memory layout of the fused single-block run (k_fused: all ants of a
+// region in one block, every pass and iteration in one launch), offsets in
+// bytes from the block's dynamic shared memory.
+struct FusedLayout {
+  uint32_t o_tau, o_state, o_reco, o_recc, o_costs, o_recp, o_ord, o_cyc, o_next, bytes, words;
+};
+ACO_HD inline uint32_t round16(uint32_t x) { return (x + 15u) & ~15u; }
+ACO_HD inline FusedLayout fused_layout(uint32_t n, uint32_t nwr, uint32_t nremw, uint32_t img_bytes, uint32_t ants) {
+  FusedLayout L;
+  const uint32_t w1 = ant_words(1, n, nwr, nremw, false, false), w2 = ant_words(2, n, nwr, nremw, false, false);
+  L.words = w1 > w2 ? w1 : w2;                         // per-ant state words (stride = ants)
+  uint32_t off = round16(img_bytes);                   // the region's block image
+  L.o_tau = off;   off += tau_smem_bytes(n);           // pheromone (n+1) x n u16
+  L.o_state = off; off += round16(4u * L.words * ants);
+  L.o_reco = off;  off += round16(2u * n * ants);      // every ant's order, [step][ant]
+  L.o_recc = off;  off += round16(4u * (n * ants > n ? n * ants : n));  // pass-2 cycles (also ASAP scratch)
+  L.o_costs = off; off += round16(4u * ants);
+  L.o_recp = off;  off += 16u * ants;                  // {prp01, prp23, length, 0}
+  L.o_ord = off;   off += round16(2u * n);             // the iteration winner's order / cycles
+  L.o_cyc = off;   off += round16(4u * n);
+  L.o_next = off;  off += round16(2u * (n + 1));       // its successor table (deposit links)
+  L.bytes = off;
+  return L;
+}
+constexpr uint32_t kFusedVariant = 1u << 13;  // variant code of k_fused (aco_last_variants)
+
 // ---- launch interface implemented in aco_kernels.cu ----
 struct LaunchCtx {
   const unsigned char *arena;
@@ -280,7 +306,8 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
 int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
                     bool nc4, const UpdItem *upd, uint32_t n_upd);
 int launch_local_keys(LaunchCtx &L, int64_t *keys);
-int launch_post(LaunchCtx &L, uint32_t smem);  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys
+int launch_post(LaunchCtx &L, uint32_t smem);
+int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem);  // the whole run, one block per region  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys
 
 // Biased winner key: (cost << 32 | global ant) XOR 2^63, so that a signed
 // int64 MIN (NCCL / torch) orders keys like the unsigned (cost, ant) pair.

@@ -1313,6 +1313,38 @@ __global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restri
 
 // Per-region initialisation: tau0, the greedy pass-1 heuristic schedule
 // (R28: the q0 = 1 ant on a uniform tau), LB check (L251).
+// The greedy heuristic schedule (warp 0 as one 32-lane group, scratch state
+// stw) and the region state at the start of a run.  tau is uniform (tau0).
+template <bool MASK>
+__device__ __forceinline__ void init_greedy(const KArgs &A, const RegionDev *rd, const RegionWs &W, RegionState &rs,
+                                            const unsigned char *img, const uint16_t *tau, uint32_t *stw) {
+  if (threadIdx.x >= 32) return;
+  const SV V = make_sv(img, rd);
+  const St S = make_st<1, false, false>(stw, 1, V);
+  uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
+  const Grp<32> G32(threadIdx.x);
+  AntOut o = ant_pass1<32, MASK>(V, tau, S, G32, 0, 0, A.cfg, true, gb1);
+  __syncwarp();
+  uint16_t *heur = (uint16_t *)(A.ws + W.o_heur);  // the heuristic order, kept for R40
+  for (uint32_t k = threadIdx.x; k < rd->n; k += 32) heur[k] = gb1[k];
+  if (threadIdx.x == 0) {
+    rs.lb_cost = cost_rp(A.cfg.mslot, A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
+    rs.init[0] = rs.best[0] = o.cost;
+    const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
+    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = rs.heur_prp[c] = prp[c];
+    rs.policy = 0;
+    rs.heur_len = 0;
+    rs.iters[0] = rs.iters[1] = 0;
+    rs.no_imp = 0;
+    rs.prune_len = kInvalid;
+    rs.pruned = 0;
+    rs.hash = 0xcbf29ce484222325ull;
+    rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
+  }
+}
+
+// Per-region initialisation: tau0, the greedy pass-1 heuristic schedule
+// (R28: the q0 = 1 ant on a uniform tau), LB check (L251).
 template <bool MASK, bool GS>
 __device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
   const uint32_t r = blockIdx.x;
@@ -1329,29 +1361,7 @@ __device__ __forceinline__ void init_body(const KArgs &A, unsigned char *smem) {
   }
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   __syncthreads();
-  if (threadIdx.x < 32) {  // warp 0 builds the greedy schedule as one 32-lane group
-    const SV V = make_sv(img, rd);
-    const St S = make_st<1, false, false>(stw, 1, V);
-    uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
-    const Grp<32> G32(threadIdx.x);
-    AntOut o = ant_pass1<32, MASK>(V, tau, S, G32, 0, 0, A.cfg, true, gb1);
-    __syncwarp();
-    uint16_t *heur = (uint16_t *)(A.ws + W.o_heur);  // the heuristic order, kept for R40
-    for (uint32_t k = threadIdx.x; k < rd->n; k += 32) heur[k] = gb1[k];
-    if (threadIdx.x != 0) return;
-    rs.lb_cost = cost_rp(A.cfg.mslot, A.cfg.cost_mode, rd->lbvec[0], rd->lbvec[1], rd->lbvec[2], rd->lbvec[3]);
-    rs.init[0] = rs.best[0] = o.cost;
-    const uint32_t prp[4] = {o.prp01 & 0xFFFFu, o.prp01 >> 16, o.prp23 & 0xFFFFu, o.prp23 >> 16};
-    for (int c = 0; c < 4; ++c) rs.prp1[c] = rs.prp2[c] = rs.heur_prp[c] = prp[c];
-    rs.policy = 0;
-    rs.heur_len = 0;
-    rs.iters[0] = rs.iters[1] = 0;
-    rs.no_imp = 0;
-    rs.prune_len = kInvalid;
-    rs.pruned = 0;
-    rs.hash = 0xcbf29ce484222325ull;
-    rs.active = (A.cfg.pass_mask & 1u) && A.cfg.iterations > 0 && !(A.cfg.stop_at_lb && o.cost == rs.lb_cost);
-  }
+  init_greedy<MASK>(A, rd, W, rs, img, tau, stw);
 }
 
 template <bool MASK>
@@ -1394,19 +1404,15 @@ __device__ uint32_t asap_order(const MachineDev &M, const SV &V, const uint16_t 
 // Pass transition (L147; R13, R18, R29): target from the pass-1 best, the
 // initial pass-2 schedule = ASAP(pass-1 best order), tau reset, the cycle-gap
 // filter (R39).  Weighted pass (R41): no target, weighted initial cost.
-__global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
-  const uint32_t r = blockIdx.x;
-  const RegionDev *rd = A.regions + r;
-  const RegionWs &W = A.rws[r];
-  RegionState &rs = A.state[r];
-  uint16_t *tau = (uint16_t *)(A.ws + W.o_tau);
-  extern __shared__ uint32_t rdyv[];  // rdy[n]
+// (block-wide: every thread of the block calls it)
+__device__ __forceinline__ void pass2_init_body(const KArgs &A, const RegionDev *rd, const RegionWs &W, RegionState &rs,
+                                                const unsigned char *img, uint16_t *tau, uint32_t *rdyv) {
   const uint32_t n = rd->n;
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) rdyv[i] = 0;
   __syncthreads();
   if (threadIdx.x == 0) {
-    const SV V = make_sv(A.arena + rd->o_image, rd);
+    const SV V = make_sv(img, rd);
     const uint16_t *gb1 = (const uint16_t *)(A.ws + W.o_gb1);
     uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
     uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
@@ -1434,20 +1440,22 @@ __global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
   }
 }
 
-// After the last pass (L366; R40): the heuristic schedule's length, and the
-// revert filter -- report the heuristic schedule when the result gained at
-// least revert_occ occupancy but is more than revert_len cycles longer.
-__global__ void __launch_bounds__(32) k_post(KArgs A) {
+__global__ void __launch_bounds__(128) k_pass2_init(KArgs A) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
-  RegionState &rs = A.state[r];
   extern __shared__ uint32_t rdyv[];  // rdy[n]
+  pass2_init_body(A, rd, W, A.state[r], A.arena + rd->o_image, (uint16_t *)(A.ws + W.o_tau), rdyv);
+}
+
+// After the last pass (L366; R40): the heuristic schedule's length, and the
+// revert filter -- report the heuristic schedule when the result gained at
+// least revert_occ occupancy but is more than revert_len cycles longer.
+// (thread 0 works; rdyv must be zeroed by the caller)
+__device__ __forceinline__ void post_body(const KArgs &A, const RegionDev *rd, const RegionWs &W, RegionState &rs,
+                                          const unsigned char *img, uint32_t *rdyv) {
   const uint32_t n = rd->n;
-  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) rdyv[i] = 0;
-  __syncwarp();
-  if (threadIdx.x != 0) return;
-  const SV V = make_sv(A.arena + rd->o_image, rd);
+  const SV V = make_sv(img, rd);
   const uint16_t *heur = (const uint16_t *)(A.ws + W.o_heur);
   const MachineDev &M = c_mach[A.cfg.mslot];
   const uint32_t hlen = asap_order(M, V, heur, nullptr, nullptr, rdyv);
@@ -1464,6 +1472,66 @@ __global__ void __launch_bounds__(32) k_post(KArgs A) {
     for (int c = 0; c < 4; ++c) rs.prp2[c] = rs.heur_prp[c];
     rs.len2 = hlen;
     rs.policy |= 2u;
+  }
+}
+
+__global__ void __launch_bounds__(32) k_post(KArgs A) {
+  const uint32_t r = blockIdx.x;
+  const RegionDev *rd = A.regions + r;
+  extern __shared__ uint32_t rdyv[];  // rdy[n]
+  for (uint32_t i = threadIdx.x; i < rd->n; i += blockDim.x) rdyv[i] = 0;
+  __syncwarp();
+  if (threadIdx.x == 0) post_body(A, rd, A.rws[r], A.state[r], A.arena + rd->o_image, rdyv);
+}
+
+// The iteration winner's successor table (pheromone deposit links, R8-R9)
+// and the global-best epilogue (L139; R11): one warp.
+template <int PASS>
+__device__ __forceinline__ void epilogue_body(const KArgs &A, uint32_t iter, RegionState &rs, const RegionWs &W,
+                                              uint32_t n, bool have, uint32_t wcost, uint32_t want, const uint16_t *ord,
+                                              const uint32_t *cyc, uint16_t *next, const uint32_t *s_prp,
+                                              uint32_t &s_flag) {
+  for (uint32_t i = threadIdx.x; i <= n; i += 32) next[i] = 0xFFFFu;
+  __syncwarp();
+  if (have) {
+    for (uint32_t k = threadIdx.x; k + 1 < n; k += 32) next[ord[k]] = ord[k + 1];
+    if (threadIdx.x == 0 && n) next[n] = ord[0];
+  }
+  // ---- epilogue (first thread, L139)
+  if (threadIdx.x == 0) {
+    rs.hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(rs.hash, PASS == 2 && A.cfg.weighted ? 4u : PASS), iter),
+                              have ? wcost : kInvalid),
+                      have ? want : kInvalid);
+    const bool improved = have && wcost < rs.best[PASS - 1];  // strict (R11)
+    s_flag = improved;
+    if (improved) {
+      rs.best[PASS - 1] = wcost;
+      rs.no_imp = 0;
+      uint32_t *prp = PASS == 1 ? rs.prp1 : rs.prp2;
+      prp[0] = s_prp[0] & 0xFFFFu;
+      prp[1] = s_prp[0] >> 16;
+      prp[2] = s_prp[1] & 0xFFFFu;
+      prp[3] = s_prp[1] >> 16;
+      if (PASS == 2) rs.len2 = s_prp[2];
+    } else {
+      rs.no_imp++;
+    }
+    rs.iters[PASS - 1] = iter + 1;
+    rs.prune_len = kInvalid;
+  }
+  __syncwarp();
+  if (s_flag) {
+    if (PASS == 1) {
+      uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
+      for (uint32_t k = threadIdx.x; k < n; k += 32) gb1[k] = ord[k];
+    } else {
+      uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
+      uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
+      for (uint32_t k = threadIdx.x; k < n; k += 32) {
+        gb2[k] = ord[k];
+        gb2c[k] = cyc[k];
+      }
+    }
   }
 }
 
@@ -1549,49 +1617,7 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
     }
   }
   __syncwarp();
-  uint16_t *next = (uint16_t *)(A.ws + W.o_next);
-  for (uint32_t i = threadIdx.x; i <= n; i += 32) next[i] = 0xFFFFu;
-  __syncwarp();
-  if (have) {
-    for (uint32_t k = threadIdx.x; k + 1 < n; k += 32) next[ord[k]] = ord[k + 1];
-    if (threadIdx.x == 0 && n) next[n] = ord[0];
-  }
-  // ---- epilogue (first thread, L139)
-  if (threadIdx.x == 0) {
-    rs.hash = fnv_u32(fnv_u32(fnv_u32(fnv_u32(rs.hash, PASS == 2 && A.cfg.weighted ? 4u : PASS), iter),
-                              have ? wcost : kInvalid),
-                      have ? want : kInvalid);
-    const bool improved = have && wcost < rs.best[PASS - 1];  // strict (R11)
-    s_flag = improved;
-    if (improved) {
-      rs.best[PASS - 1] = wcost;
-      rs.no_imp = 0;
-      uint32_t *prp = PASS == 1 ? rs.prp1 : rs.prp2;
-      prp[0] = s_prp[0] & 0xFFFFu;
-      prp[1] = s_prp[0] >> 16;
-      prp[2] = s_prp[1] & 0xFFFFu;
-      prp[3] = s_prp[1] >> 16;
-      if (PASS == 2) rs.len2 = s_prp[2];
-    } else {
-      rs.no_imp++;
-    }
-    rs.iters[PASS - 1] = iter + 1;
-    rs.prune_len = kInvalid;
-  }
-  __syncwarp();
-  if (s_flag) {
-    if (PASS == 1) {
-      uint16_t *gb1 = (uint16_t *)(A.ws + W.o_gb1);
-      for (uint32_t k = threadIdx.x; k < n; k += 32) gb1[k] = ord[k];
-    } else {
-      uint16_t *gb2 = (uint16_t *)(A.ws + W.o_gb2);
-      uint32_t *gb2c = (uint32_t *)(A.ws + W.o_gb2c);
-      for (uint32_t k = threadIdx.x; k < n; k += 32) {
-        gb2[k] = ord[k];
-        gb2c[k] = cyc[k];
-      }
-    }
-  }
+  epilogue_body<PASS>(A, iter, rs, W, n, have, wcost, want, ord, cyc, (uint16_t *)(A.ws + W.o_next), s_prp, s_flag);
 }
 
 template <int PASS, bool MASK, bool T32, bool NC4>
@@ -1640,6 +1666,132 @@ __global__ void k_stop(KArgs A, uint32_t pass) {
   if ((A.cfg.stop_at_lb && rs.best[pass - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
       rs.iters[pass - 1] >= A.cfg.iterations)
     rs.active = 0;
+}
+
+// ------------------------------------------------------------ fused run
+// The whole two-pass ACO of one region in ONE block (the
+// paper's cooperative kernel runs construct -> reduce -> update -> epilogue
+// in one launch).  Used for batches whose ants all fit one block per region
+// (config 1): image, pheromone table, every ant's state and its recorded
+// schedule stay in shared memory across the iterations; block barriers
+// replace the kernel boundaries of the multi-launch path, so the sequence of
+// states -- and every result -- is that of the launches it replaces (the
+// same device functions run in the same order).  One ant per thread
+// (word-mask scan, compact pass-2 layout, group coins drawn inline).
+__global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
+  const uint32_t r = blockIdx.x;
+  const RegionDev *rd = A.regions + r;
+  const RegionWs &W = A.rws[r];
+  RegionState &rs = A.state[r];
+  extern __shared__ uint4 smem4[];
+  unsigned char *smem = (unsigned char *)smem4;
+  __shared__ uint32_t s_prp[3], s_flag, s_active;
+  const uint32_t n = rd->n, na = A.cfg.ants, tid = threadIdx.x;
+  const FusedLayout F = fused_layout(n, rd->nwr, rd->nremw, rd->img.bytes, na);
+  stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
+  const unsigned char *img = smem;
+  uint16_t *tau = (uint16_t *)(smem + F.o_tau);
+  uint32_t *st = (uint32_t *)(smem + F.o_state);
+  uint16_t *rec_o = (uint16_t *)(smem + F.o_reco);
+  uint32_t *rec_c = (uint32_t *)(smem + F.o_recc);
+  uint32_t *costs = (uint32_t *)(smem + F.o_costs);
+  uint4 *recp = (uint4 *)(smem + F.o_recp);
+  uint16_t *ord = (uint16_t *)(smem + F.o_ord);
+  uint32_t *cyc = (uint32_t *)(smem + F.o_cyc);
+  uint16_t *next = (uint16_t *)(smem + F.o_next);
+  tau_fill(tau, W.tau_len, A.cfg.tau0);
+  __syncthreads();
+  init_greedy<true>(A, rd, W, rs, img, tau, st);  // (k_init)
+  __syncthreads();
+  const SV V = make_sv(img, rd);
+  const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
+  for (uint32_t pass = 1; pass <= 2; ++pass) {
+    if (pass == 2) {  // (k_pass2_init)
+      pass2_init_body(A, rd, W, rs, img, tau, rec_c);
+      __syncthreads();
+    }
+    if (!(A.cfg.pass_mask & pass)) continue;
+    for (uint32_t it = 0; it < A.cfg.iterations; ++it) {
+      if (tid == 0) s_active = rs.active;
+      __syncthreads();
+      if (!s_active) break;  // block-uniform
+      if (tid < na) {  // (k_construct) ant tid
+        const Grp<1> G(tid);
+        const uint32_t ant = A.cfg.ant_base + tid;
+        AntOut o;
+        if (pass == 1) {
+          const St S = make_st<1, false, false>(st + tid, na, V);
+          o = ant_pass1<1, true>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, nullptr,
+                                 RL{nullptr, 0, 0, 0, nullptr, nullptr}, na);
+        } else {
+          const St S = make_st<2, false, false>(st + tid, na, V);
+          uint32_t tgt[4];
+#pragma unroll
+          for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
+          const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
+          o = ant_pass2<1, true, false, false>(V, tau, S, G, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + tid,
+                                               rec_c + tid, nullptr, 0, na);
+        }
+        costs[tid] = o.cost;
+        recp[tid] = make_uint4(o.prp01, o.prp23, o.len, 0u);
+        if (dump && A.dump_cost) {
+          A.dump_cost[(((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.count + r) * na + tid] = o.cost;
+          const size_t base = ((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.dump_slice + W.o_dump + (size_t)tid * n;
+          if (A.dump_order && o.cost != kInvalid)
+            for (uint32_t k = 0; k < n; ++k) A.dump_order[base + k] = rec_o[k * na + tid];
+          if (A.dump_cycle && pass == 2 && o.cost != kInvalid)
+            for (uint32_t k = 0; k < n; ++k) A.dump_cycle[base + k] = rec_c[k * na + tid];
+        }
+      }
+      __syncthreads();
+      if (tid < 32) {  // (k_select) argmin over (cost, ant), copy of the winner's schedule, epilogue
+        unsigned long long best = ~0ull;
+        for (uint32_t a = tid; a < na; a += 32)
+          best = min(best, ((unsigned long long)costs[a] << 32) | (A.cfg.ant_base + a));
+#pragma unroll
+        for (int off = 16; off; off >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, off));
+        const uint32_t wcost = (uint32_t)(best >> 32), want = (uint32_t)best;
+        const bool have = wcost != kInvalid;
+        if (have) {
+          const uint32_t wl = want - A.cfg.ant_base;
+          for (uint32_t k = tid; k < n; k += 32) {
+            ord[k] = rec_o[k * na + wl];
+            if (pass == 2) cyc[k] = rec_c[k * na + wl];
+          }
+          if (tid == 0) {
+            const uint4 q = recp[wl];
+            s_prp[0] = q.x;
+            s_prp[1] = q.y;
+            s_prp[2] = q.z;
+          }
+        }
+        __syncwarp();
+        if (pass == 1) epilogue_body<1>(A, it, rs, W, n, have, wcost, want, ord, cyc, next, s_prp, s_flag);
+        else epilogue_body<2>(A, it, rs, W, n, have, wcost, want, ord, cyc, next, s_prp, s_flag);
+      }
+      __syncthreads();
+      {  // (k_update) evaporate + deposit + clamp, R6-R9
+        const uint32_t rho = A.cfg.rho_q16, dl = A.cfg.delta, lo = A.cfg.tau_min, hi = A.cfg.tau_max;
+        for (uint32_t e = tid; e < (n + 1) * n; e += blockDim.x) {
+          const uint32_t i = e / n, j = e - i * n;
+          uint32_t x = ((uint32_t)tau[e] * rho) >> 16;
+          if (next[i] == j) x += dl;
+          tau[e] = (uint16_t)min(max(x, lo), hi);
+        }
+      }
+      if (tid == 0) {  // (k_stop) termination, R12
+        const uint32_t lim = no_improve_limit(A.cfg, n);
+        const uint32_t lb = pass == 1 ? rs.lb_cost : rd->lb_len + (A.cfg.weighted ? A.cfg.ws_weight * rs.lb_cost : 0u);
+        if ((A.cfg.stop_at_lb && rs.best[pass - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
+            rs.iters[pass - 1] >= A.cfg.iterations)
+          rs.active = 0;
+      }
+      __syncthreads();
+    }
+  }
+  for (uint32_t i = tid; i < n; i += blockDim.x) rec_c[i] = 0;  // (k_post)
+  __syncthreads();
+  if (tid == 0) post_body(A, rd, W, rs, img, rec_c);
 }
 
 // ------------------------------------------------------------ launchers
@@ -1800,6 +1952,7 @@ int init_kernel_attrs() {
   big_smem(k_init<false>);
   big_smem(k_pass2_init);
   big_smem(k_post);
+  big_smem(k_fused);
 #define ACO_SEL(M) big_smem(k_select<1, M, false, false>); big_smem(k_select<2, M, false, false>); \
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
@@ -1866,6 +2019,13 @@ int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, u
 int launch_post(LaunchCtx &L, uint32_t smem) {
   if (!L.cfg.count) return 0;
   k_post<<<L.cfg.count, 32, smem, (cudaStream_t)L.stream>>>(kargs(L));
+  L.launches++;
+  return check();
+}
+
+int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
+  if (!L.cfg.count) return 0;
+  k_fused<<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
   L.launches++;
   return check();
 }

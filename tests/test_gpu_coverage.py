@@ -88,3 +88,29 @@ def test_size_class_termination_gpu(torch_cuda):
     s.load(regs, ids).run(p)
     for n, g in zip(sizes, s.results()):
         assert g["iters1"] == g["iters2"] == paper_class_limit(n), (n, g["iters1"], g["iters2"])
+
+
+@pytest.mark.parametrize("kind", ["both", "paper", "weighted", "pass1", "pass2", "mix"])
+def test_fused_run_equals_oracle_and_multilaunch(torch_cuda, monkeypatch, kind):
+    """The fused single-block run (k_fused: every pass and iteration of a
+    region in one block) is taken for batches with few
+    ants in total; it equals the oracle and the multi-launch path bit for bit
+    (final schedule, trace, iterations), for every pass mode and policy."""
+    regs = [I.fix10a(), I.gen_region(60, 9700), I.gen_region(130, 9701, "unit")]
+    ids = [50, 51, 52]
+    base = I.Params(ants=128, iterations=6, seed=5)
+    p = {"both": base, "paper": I.paper_policy(base), "weighted": dataclasses.replace(base, passes=4, ws_weight=2),
+         "pass1": dataclasses.replace(base, passes=1), "pass2": dataclasses.replace(base, passes=2),
+         "mix": dataclasses.replace(base, heur_mix=1, stall_num=2, cost_mode=I.COST_OCC)}[kind]
+    s = _sched()
+    s.load(regs, ids).run(p)
+    assert s.variants() == [1 << 13], s.variants()  # k_fused
+    fused = s.results()
+    for k in range(len(regs)):
+        compare_results(fused[k], O.schedule(regs[k], ids[k], I.GFX906, p), f"{kind} region {k}")
+    monkeypatch.setenv("ACO_FUSED_ANTS", "0")
+    m = _sched()
+    m.load(regs, ids).run(p)
+    assert (1 << 13) not in m.variants()
+    for k, g in enumerate(m.results()):
+        compare_results(g, O.schedule(regs[k], ids[k], I.GFX906, p), f"{kind} multi-launch region {k}")

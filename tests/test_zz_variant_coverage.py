@@ -27,6 +27,8 @@ BENCH_LINES = [
 
 
 def decode(code):
+    if code & (1 << 13):
+        return "fused"
     lanes = [1, 2, 4, 8][(code >> 6) & 3]
     if code & (1 << 9):
         lanes = 32 if code & (1 << 10) else 16
