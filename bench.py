@@ -240,6 +240,33 @@ def host_cpu():
     return {"model": model, "threads": os.cpu_count()}
 
 
+def lib_sha256():
+    """sha256 of the loaded CUDA library (matches a profile to its build)."""
+    import hashlib
+    from paper_conf_cgo_shobakimhlmkrg24_b200 import _lib
+    with open(_lib.LIB_PATH, "rb") as f:
+        return hashlib.sha256(f.read()).hexdigest()
+
+
+def ncu_evidence(workload: str):
+    """DRAM traffic and issue-slot figures of the construct launches from the
+    committed ncu --set full capture (profiles/r02_traffic.json) -- used only
+    when that capture profiled this very build (same libaco_b200.so sha256)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
+            tj = json.load(f)
+    except Exception:
+        return None, None, "no committed capture"
+    if workload != "c3":
+        return None, None, "capture is of the c3 batch"
+    sha = lib_sha256()
+    if tj.get("so_sha256") != sha:
+        return None, None, f"committed capture is of another build ({str(tj.get('so_sha256'))[:12]} vs {sha[:12]})"
+    issue = {"util_pct": tj.get("issue_util_pct"), "warps_active_pct": tj.get("warps_active_pct"),
+             "source": tj.get("issue_source")}
+    return tj.get("dram_bytes_per_launch"), issue, tj.get("source")
+
+
 def bytes_per_ant_step(stats: np.ndarray) -> float:
     """SURVEY 8(d) algorithmic bytes per ant-step from oracle instrumentation:
     8.5|F| + 2|R| + 12 deg + 6 |Use| + 2 |Def| + 16 per placed instruction."""
@@ -574,9 +601,10 @@ def main(argv=None):
         if bpas is not None and construct_ms > 0:
             n_launch = phase_launches[0] / max(1, args.steps)
             achieved = bpas * ant_steps / (construct_ms / 1000.0) / 1e9
+            traffic, issue, tsrc = ncu_evidence(args.workload)
             roof = {"bound": "smem", "achieved": round(achieved, 1), "peak": round(smem_peak, 1),
-                    "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": None,
-                    "traffic_note": "ncu --set full DRAM bytes per construct launch: profiles/r02_*_ncu_summary.md",
+                    "unit": "GB/s", "frac": round(achieved / smem_peak, 4), "traffic": traffic,
+                    "traffic_source": tsrc, "issue_slots_ncu": issue,
                     "algorithmic_bytes_per_launch": round(bpas * ant_steps / max(1.0, n_launch)),
                     "kernel": "k_construct (all classes)", "bytes_per_ant_step": round(bpas, 2),
                     "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,

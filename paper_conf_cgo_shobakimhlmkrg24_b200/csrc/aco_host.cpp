@@ -7,6 +7,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -899,6 +900,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     if (on) spread_cap = (uint32_t)std::max<uint64_t>(1, (total + 147) / 148);
     if (const char *e = getenv("ACO_SPREAD_CAP")) spread_cap = on ? (uint32_t)atoi(e) : 0u;
   }
+  bool fill_sms = true;  // spread passes with fewer shared-memory blocks than SMs (below)
+  if (const char *e = getenv("ACO_FILL")) fill_sms = atoi(e) != 0;
   uint32_t spread_lanes = 0;  // 0: lanes ~ bitset words
   if (const char *e = getenv("ACO_SPREAD_LANES")) spread_lanes = (uint32_t)atoi(e);
   uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
@@ -952,9 +955,16 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   }
   std::vector<uint8_t> gs(count, 0);
   std::vector<uint32_t> gs_words(count, 0), scratch_words(count, 0);
-  for (uint32_t r = 0; r < count; ++r) {
+  // Shape of one region in one pass (spread: ants-per-block cap with the
+  // given lanes per ant, 0 = off).
+  struct RegionPlan {
+    Shape sh;
+    bool g = false, lean = false, t32 = false, wide = false, on = false;
+    uint32_t W = 0;
+  };
+  auto plan_region = [&](uint32_t r, uint32_t pass, uint32_t spread, uint32_t lane_pref) {
+    RegionPlan q;
     const RegionDev &R = ctx->regions[r];
-    P.max_n = std::max(P.max_n, R.n);
     // pass-2 state variant: the compact layout (windowed u8 ready times) needs
     // latencies < 512, 2 classes and <= 7 multi-use registers per class and
     // instruction; otherwise u16 cycles (3-4 classes), or u32 when a
@@ -962,65 +972,115 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // the general machine model (R42) runs in the u32-cycle variants
     const bool t32 = ctx->mach.issue_width > 1 ||
                      (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
-    P.any_t32 |= t32;
-    for (uint32_t pass = 1; pass <= 2; ++pass) {
-      const bool wide = R.n >= kWideN && R.n <= 1024;
-      // lean pass-2 layout (u8 ready times, kills derived at evaluation):
-      // large regions, single issue, 2 classes, latencies < 128
-      bool lean = pass == 2 && lean_on && wide && !t32 && !P.nc4 && ctx->mach.issue_width <= 1 && R.max_lat < 128u;
-      uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);  // lean: decided below
-      if (!(pmask & pass)) continue;
-      if (getenv("ACO_DEBUG_REGIONS"))
-        fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
-                R.nremw, R.L);
-      const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
-      Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
-                            pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
-                            p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
-                            wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u,
-                            rl1 && pass == 1 ? 0u : spread_cap, spread_lanes ? spread_lanes : std::min(8u, lane_pow2(R.nwr)));
-      if (lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
-      if (lean) {
-        // the lean layout costs per ant-step (kills derived at every
-        // evaluation) and gains resident ants; on the mixed C3 batch it wins
-        // whenever it fits at least as many ants (B200: 684 -> 645 ms/batch;
-        // ACO_LEAN_GAIN = 20 / 50 %: 654 ms)
-        const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true);
-        const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[1][2], false, false,
-                                     tgt_threads[1], 1, A, p->group_size, coin_words(pass, R.n), img_l1[1] != 0);
-        if (shl.apb && 100ull * shl.resident >= (100ull + lean_gain) * sh.resident) {
-          sh = shl;
-          W = Wl;
-        } else {
-          lean = false;
-        }
+    q.t32 = t32;
+    const bool wide = R.n >= kWideN && R.n <= 1024;
+    q.wide = wide;
+    // lean pass-2 layout (u8 ready times, kills derived at evaluation):
+    // large regions, single issue, 2 classes, latencies < 128
+    bool lean = pass == 2 && lean_on && wide && !t32 && !P.nc4 && ctx->mach.issue_width <= 1 && R.max_lat < 128u;
+    uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);  // lean: decided below
+    if (getenv("ACO_DEBUG_REGIONS"))
+      fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
+              R.nremw, R.L);
+    const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
+    Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
+                          pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
+                          p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
+                          wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u,
+                          rl1 && pass == 1 ? 0u : spread, lane_pref);
+    if (lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
+    if (lean) {
+      // the lean layout costs per ant-step (kills derived at every
+      // evaluation) and gains resident ants; on the mixed C3 batch it wins
+      // whenever it fits at least as many ants (B200: 684 -> 645 ms/batch;
+      // ACO_LEAN_GAIN = 20 / 50 %: 654 ms)
+      const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true);
+      const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[1][2], false, false, tgt_threads[1], 1, A,
+                                   p->group_size, coin_words(pass, R.n), img_l1[1] != 0, 1u, spread, 1u);
+      if (shl.apb && 100ull * shl.resident >= (100ull + lean_gain) * sh.resident) {
+        sh = shl;
+        W = Wl;
+      } else {
+        lean = false;
       }
-      bool g = false;
-      // Huge regions whose image + state leave fewer than gs_min_threads
-      // resident per SM are latency-starved in shared memory: the
-      // global-state kernels (all ants resident, state through L1/L2) win
-      // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
-      if (sh.apb != 0 && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
-      if (sh.apb == 0 && rl1 && pass == 1) {  // R45 needs a block-wide lockstep: shared-memory kernels only
+    }
+    // Huge regions whose image + state leave fewer than gs_min_threads
+    // resident per SM are latency-starved in shared memory: the
+    // global-state kernels (all ants resident, state through L1/L2) win
+    // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
+    // (not for a spread shape: there few resident ants per SM is the point)
+    if (sh.apb != 0 && !spread && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
+    if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
+      // all ants are resident (state in the workspace); 16 lanes per ant
+      // and 512-thread blocks measured best (tools/probe_gs_lanes.sh:
+      // n = 2000, 8192 ants: 4 lanes x 64 ants 206 + 53 ms -> 45 + 34 ms
+      // per 2 iterations), fewer ants per block when A is small
+      uint32_t gl = gs_lanes[pass - 1];
+      if (pass == 2 && (t32 || P.nc4)) gl = 4;  // the u16/u32-cycle GS variants have 4 lanes
+      uint32_t gapb = std::min<uint64_t>(kMaxBlockThreads / gl, std::max<uint64_t>(8u, ((uint64_t)A * count / 148) & ~7ull));
+      if (const char *e = getenv("ACO_GS_APB")) gapb = (uint32_t)atoi(e);
+      while (gapb * gl > kMaxBlockThreads) gapb /= 2;
+      sh = Shape{gapb, gl, 0, false};
+      q.g = true;
+      lean = false;
+      W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
+    }
+    q.sh = sh;
+    q.lean = lean;
+    q.W = W;
+    q.on = true;
+    return q;
+  };
+  std::vector<RegionPlan> rp(2 * (size_t)count);
+  for (uint32_t pass = 1; pass <= 2; ++pass) {
+    if (!(pmask & pass)) continue;
+    uint64_t blocks = 0, ants_smem = 0;
+    for (uint32_t r = 0; r < count; ++r) {
+      RegionPlan &q = rp[2 * r + pass - 1];
+      q = plan_region(r, pass, spread_cap, spread_lanes ? spread_lanes : std::min(8u, lane_pow2(ctx->regions[r].nwr)));
+      if (q.sh.apb == 0 && rl1 && pass == 1) {  // R45 needs a block-wide lockstep: shared-memory kernels only
         ctx->plan = saved;
         return ACO_E_ARG;
       }
-      if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
-        // all ants are resident (state in the workspace); 16 lanes per ant
-        // and 512-thread blocks measured best (tools/probe_gs_lanes.sh:
-        // n = 2000, 8192 ants: 4 lanes x 64 ants 206 + 53 ms -> 45 + 34 ms
-        // per 2 iterations), fewer ants per block when A is small
-        uint32_t gl = gs_lanes[pass - 1];
-        if (pass == 2 && (t32 || P.nc4)) gl = 4;  // the u16/u32-cycle GS variants have 4 lanes
-        uint32_t gapb = std::min<uint64_t>(kMaxBlockThreads / gl, std::max<uint64_t>(8u, ((uint64_t)A * count / 148) & ~7ull));
-        if (const char *e = getenv("ACO_GS_APB")) gapb = (uint32_t)atoi(e);
-        while (gapb * gl > kMaxBlockThreads) gapb /= 2;
-        sh = Shape{gapb, gl, 0, false};
-        g = true;
+      if (!q.g) {
+        blocks += (A + q.sh.apb - 1) / q.sh.apb;
+        ants_smem += A;
+      }
+    }
+    // Fill the SMs in proportion to work: a region holding the share w_r of
+    // the pass's work should spread its ants over >= 148 w_r blocks, else its
+    // few large blocks run alone at the end of the pass while SMs idle (few
+    // large regions: configs 2 and 5).  Such a region keeps its lanes per ant
+    // and caps its ants per block (the ant step is latency-bound at this
+    // scale: more SMs at fewer warps each); many-region batches (config 3)
+    // are unaffected (w_r is tiny).
+    if (fill_sms && !spread_cap && !(rl1 && pass == 1) && ants_smem) {
+      double wtot = 0;
+      for (uint32_t r = 0; r < count; ++r) wtot += (double)ctx->regions[r].n * (ctx->regions[r].n + 16.0);
+      for (uint32_t r = 0; r < count; ++r) {
+        RegionPlan &q = rp[2 * r + pass - 1];
+        if (q.g || wtot <= 0) continue;
+        const double nr = ctx->regions[r].n;
+        const uint32_t need = (uint32_t)std::ceil(148.0 * nr * (nr + 16.0) / wtot);
+        const uint32_t have = (A + q.sh.apb - 1) / q.sh.apb;
+        if (need <= have) continue;
+        const RegionPlan f = plan_region(r, pass, std::max(1u, (A + need - 1) / need), q.sh.lanes);
+        if (!f.g && f.sh.apb && (A + f.sh.apb - 1) / f.sh.apb > have) q = f;
+      }
+    }
+  }
+  for (uint32_t r = 0; r < count; ++r) {
+    const RegionDev &R = ctx->regions[r];
+    P.max_n = std::max(P.max_n, R.n);
+    for (uint32_t pass = 1; pass <= 2; ++pass) {
+      const RegionPlan &q = rp[2 * r + pass - 1];
+      P.any_t32 |= q.t32;
+      if (!q.on) continue;
+      Shape sh = q.sh;
+      const bool g = q.g, t32 = q.t32, wide = q.wide, lean = q.lean;
+      if (g) {
         gs[r] = 1;
-        lean = false;
-        W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
-        gs_words[r] = std::max(gs_words[r], (W + 3u) & ~3u);  // (ant-major rows padded to 16 B)
+        gs_words[r] = std::max(gs_words[r], (q.W + 3u) & ~3u);  // (ant-major rows padded to 16 B)
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;

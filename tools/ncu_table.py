@@ -15,7 +15,7 @@ COLS = [('kernel', 'Kernel Name'), ('grid', 'Grid Size'), ('block', 'Block Size'
 SCALE = {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9, 'nsecond': 1e-6, 'usecond': 1e-3, 'msecond': 1.0}
 
 
-def main(path, traffic_out=None, source=""):
+def main(path, traffic_out=None, source="", so_sha256=None):
     rows = list(csv.reader(open(path)))
     h, u = rows[0], rows[1]
 
@@ -53,9 +53,12 @@ def main(path, traffic_out=None, source=""):
         json.dump({"kernel": "k_construct (all classes)", "dram_bytes_per_launch": int(dram / nc), "launches": nc,
                    "source": source, "issue_util_pct": round(acc / tw, 1), "warps_active_pct": round(accw / tw, 1),
                    "issue_source": "time-weighted sm__inst_issued.avg.pct_of_peak_sustained_active (and "
-                                   "sm__warps_active) over the same construct launches"},
+                                   "sm__warps_active) over the same construct launches",
+                   "so_sha256": so_sha256},
                   open(traffic_out, 'w'), indent=1)
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, sys.argv[3] if len(sys.argv) > 3 else "")
+    # ncu_table.py prof_raw.csv [traffic.json source-text [sha256 of the profiled libaco_b200.so]]
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, sys.argv[3] if len(sys.argv) > 3 else "",
+         sys.argv[4] if len(sys.argv) > 4 else None)
