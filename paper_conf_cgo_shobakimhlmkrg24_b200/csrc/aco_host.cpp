@@ -902,6 +902,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   }
   bool fill_sms = true;  // spread passes with fewer shared-memory blocks than SMs (below)
   if (const char *e = getenv("ACO_FILL")) fill_sms = atoi(e) != 0;
+  uint32_t fill_img_max = 64 * 1024;
+  if (const char *e = getenv("ACO_FILL_IMG")) fill_img_max = (uint32_t)atoi(e);
   uint32_t spread_lanes = 0;  // 0: lanes ~ bitset words
   if (const char *e = getenv("ACO_SPREAD_LANES")) spread_lanes = (uint32_t)atoi(e);
   uint32_t img_l1[2] = {0, 1};  // large regions may read the image through L1 (pass 2; pass 1 measured slower)
@@ -909,6 +911,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   bool lean_on = true;  // pass-2 lean layout for large regions
   if (const char *e = getenv("ACO_LEAN")) lean_on = atoi(e) != 0;
   uint32_t lean_gain = 0;  // % more resident ants the lean layout must reach (C3: 0 measured best)
+  bool lean1_on = true;    // pass-1 lean layout for large regions
+  if (const char *e = getenv("ACO_LEAN1")) lean1_on = atoi(e) != 0;
+  uint32_t lean1_gain = 20;
+  if (const char *e = getenv("ACO_LEAN1_GAIN")) lean1_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
   bool gs_wide = true;  // 4-wide scan in the global-state kernels
@@ -988,8 +994,23 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
                           p->group_size, coin_words(pass, R.n) + (rl1 && pass == 1 ? 6u : 0u),
                           wide && !rare && img_l1[pass - 1], rl1 && pass == 1 ? p->group_size : 1u,
                           rl1 && pass == 1 ? 0u : spread, lane_pref);
-    if (lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
-    if (lean) {
+    if (pass == 1 && lean1_on && wide && !q.t32) {
+      // lean pass-1 layout (no stored last-use counts: derived from the
+      // remaining-use counters and scheduled bits at evaluation, one lane per
+      // ant): taken when it keeps >= lean1_gain % more ants resident
+      const uint32_t Wl = ant_words(1, R.n, R.nwr, R.nremw, false, P.nc4, true);
+      const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[0][2], false, false, tgt_threads[0], 1, A,
+                                   p->group_size, coin_words(1, R.n) + (rl1 ? 6u : 0u), img_l1[0] != 0,
+                                   rl1 ? p->group_size : 1u, rl1 ? 0u : spread, 1u);
+      const uint64_t base_ants = sh.apb ? sh.resident / sh.lanes : 0;
+      if (shl.apb && 100ull * shl.resident >= (100ull + lean1_gain) * base_ants) {
+        sh = shl;
+        W = Wl;
+        lean = true;
+      }
+    }
+    if (pass == 2 && lean && sh.lanes != 1) lean = false;  // (lean variants: one lane per ant)
+    if (pass == 2 && lean) {
       // the lean layout costs per ant-step (kills derived at every
       // evaluation) and gains resident ants; on the mixed C3 batch it wins
       // whenever it fits at least as many ants (B200: 684 -> 645 ms/batch;
@@ -1059,7 +1080,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       for (uint32_t r = 0; r < count; ++r) wtot += (double)ctx->regions[r].n * (ctx->regions[r].n + 16.0);
       for (uint32_t r = 0; r < count; ++r) {
         RegionPlan &q = rp[2 * r + pass - 1];
-        if (q.g || wtot <= 0) continue;
+        // (regions with a large image stay: staging it into more blocks costs
+        // more than the extra SMs give -- C5 n = 1,000: 599 -> 643 ms)
+        if (q.g || wtot <= 0 || ctx->regions[r].img.bytes > fill_img_max) continue;
         const double nr = ctx->regions[r].n;
         const uint32_t need = (uint32_t)std::ceil(148.0 * nr * (nr + 16.0) / wtot);
         const uint32_t have = (A + q.sh.apb - 1) / q.sh.apb;
@@ -1304,7 +1327,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     for (uint32_t r = 0; r < count && ok; ++r) {
       const RegionDev &R = ctx->regions[r];
       ok = R.n <= 1024 && R.max_lat <= 511u && R.mc_max <= 7u;
-      if (ok) smem = std::max(smem, fused_layout(R.n, R.nwr, R.nremw, R.img.bytes, A).bytes);
+      if (ok) smem = std::max(smem, fused_layout(R.n, R.nwr, R.nremw, R.img.bytes, A, p->group_size).bytes);
     }
     if (ok && smem <= kSmemPerSM) {
       P.fused = true;

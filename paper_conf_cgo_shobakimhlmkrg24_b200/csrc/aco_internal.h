@@ -174,7 +174,8 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 // Per-ant state words (u32) of a region for a pass, [word][ant] interleave:
 //   RB [nwr] ready set, SCH [nwr] scheduled set, REM [nremw] u16 counters, then
 //   pass 1: DK [ceil(n/8)]  4-bit count of registers whose last remaining
-//                           user is the instruction (dynamic part of LUC)
+//                           user is the instruction (dynamic part of LUC);
+//                           none in the lean pass-1 layout (derived, dyn_kills)
 //   pass 2, compact (2 classes, latencies < 512, <= 7 multi-use registers
 //           per class and instruction):
 //           X  [ceil(n/2)] u16: windowed ready time (10 bits) | last-use
@@ -190,7 +191,7 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32_t nremw, bool t32,
                                  bool nc4, bool lean = false) {
   const uint32_t w = 2 * nwr + nremw;
-  if (pass == 1) return w + (n + 7) / 8;
+  if (pass == 1) return w + (lean ? 0u : (n + 7) / 8);  // lean pass 1: last-use counts derived, not stored
   if (lean) return w + (n + 3) / 4;  // lean: u8 windowed ready time (kills derived, not stored)
   if (!t32 && !nc4) return w + (n + 1) / 2;  // compact: u16 (windowed ready time | last uses)
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
@@ -223,10 +224,11 @@ ACO_HD inline uint32_t tau_smem_bytes(uint32_t n) { return (((n + 1) * n * 2) + 
 // region in one block, every pass and iteration in one launch), offsets in
 // bytes from the block's dynamic shared memory.
 struct FusedLayout {
-  uint32_t o_tau, o_state, o_reco, o_recc, o_costs, o_recp, o_ord, o_cyc, o_next, bytes, words;
+  uint32_t o_tau, o_state, o_reco, o_recc, o_costs, o_recp, o_ord, o_cyc, o_next, o_coins, bytes, words;
 };
 ACO_HD inline uint32_t round16(uint32_t x) { return (x + 15u) & ~15u; }
-ACO_HD inline FusedLayout fused_layout(uint32_t n, uint32_t nwr, uint32_t nremw, uint32_t img_bytes, uint32_t ants) {
+ACO_HD inline FusedLayout fused_layout(uint32_t n, uint32_t nwr, uint32_t nremw, uint32_t img_bytes, uint32_t ants,
+                                       uint32_t group_size) {
   FusedLayout L;
   const uint32_t w1 = ant_words(1, n, nwr, nremw, false, false), w2 = ant_words(2, n, nwr, nremw, false, false);
   L.words = w1 > w2 ? w1 : w2;                         // per-ant state words (stride = ants)
@@ -240,6 +242,7 @@ ACO_HD inline FusedLayout fused_layout(uint32_t n, uint32_t nwr, uint32_t nremw,
   L.o_ord = off;   off += round16(2u * n);             // the iteration winner's order / cycles
   L.o_cyc = off;   off += round16(4u * n);
   L.o_next = off;  off += round16(2u * (n + 1));       // its successor table (deposit links)
+  L.o_coins = off; off += round16(4u * coin_groups(ants, group_size) * coin_words(2, n));  // group coins (R3)
   L.bytes = off;
   return L;
 }
@@ -273,7 +276,7 @@ struct ClassLaunch {
   bool gs;                 // per-ant state in global memory (huge regions)
   bool wide;               // 4-wide candidate scan (n >= kWideN: word-mask variant; global state: strided words)
   bool img_l1 = false;     // the block image is read through L1 (not staged): more ants per SM
-  bool lean = false;       // pass 2: lean per-ant layout (u8 ready times, dynamic kills)
+  bool lean = false;       // lean per-ant layout: kills derived (pass 1: no last-use counts; pass 2: u8 ready times)
 };
 
 constexpr uint32_t kMachSlots = 8;  // distinct machine models resident per device
@@ -292,7 +295,7 @@ inline uint32_t class_variant(uint32_t pass, const ClassLaunch &c) {
   const bool mask = c.max_n <= 1024 && !c.gs;
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   return variant_code(pass, c.lanes, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32, pass == 2 && c.nc4,
-                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && (mask || c.gs), pass == 2 && c.lean);
+                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && (mask || c.gs), c.lean);
 }
 
 int set_machine(uint32_t slot, const MachineDev &m);  // cudaMemcpyToSymbol into slot; 0 on success

@@ -306,12 +306,12 @@ __device__ __forceinline__ uint32_t dyn_kills(const SV &V, const St &A, uint32_t
 // multi-use list is fetched together (two dependent shared/L1 loads per
 // level for all four, instead of four serial chains).  An exhausted list
 // reads state word 0 (in bounds) and is masked out.
-__device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4 (&ds)[4], uint32_t (&dk)[4]) {
+__device__ __forceinline__ void dyn_kills4w(const SV &V, const St &A, const uint32_t (&dsw)[4], uint32_t (&dk)[4]) {
   uint32_t mc[4], m0[4], mx = 0;
 #pragma unroll
   for (int u = 0; u < 4; ++u) {
-    mc[u] = (ds[u].w >> 4) & 0xFu;
-    m0[u] = ds[u].w >> 8;
+    mc[u] = (dsw[u] >> 4) & 0xFu;
+    m0[u] = dsw[u] >> 8;
     dk[u] = 0;
     mx = ::max(mx, mc[u]);
   }
@@ -327,6 +327,10 @@ __device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4
       dk[u] += (q < mc[u] && last ? 1u : 0u) << (8 * ((e[u] >> 22) & 3u));
     }
   }
+}
+__device__ __forceinline__ void dyn_kills4(const SV &V, const St &A, const uint4 (&ds)[4], uint32_t (&dk)[4]) {
+  const uint32_t dsw[4] = {ds[0].w, ds[1].w, ds[2].w, ds[3].w};
+  dyn_kills4w(V, A, dsw, dk);
 }
 
 // ---- lane groups: LG consecutive lanes of a warp build one ant together.
@@ -640,7 +644,7 @@ __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A, const G
   const uint32_t n = V.n;
   const bool ct = PASS == 2 && !T32 && !NC4;
   const uint32_t tw = PASS == 1 ? 0 : (LEAN ? (n + 3) / 4 : (T32 ? n : (n + 1) / 2));
-  const uint32_t dw = PASS == 1 ? (n + 7) / 8 : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
+  const uint32_t dw = PASS == 1 ? (LEAN ? 0u : (n + 7) / 8) : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
   for (uint32_t w = G.lane; w < tw + dw; w += LG) A.T[w * A.S] = 0;  // T and DK are contiguous
   if (MASK && LG > 1) {
 #pragma unroll
@@ -696,7 +700,7 @@ __device__ __forceinline__ uint32_t ready_count(const St &A, uint32_t nwr) {
 // score tau[prev][j] * eta1(j, LUC(j)) (R1, R4).  The step index k is the
 // Philox step (R26).  rec (leader, may be NULL) receives the order.  The
 // result is valid in the leader lane.
-template <int LG, bool MASK, bool WIDE = false, bool RLIM = false>
+template <int LG, bool MASK, bool WIDE = false, bool RLIM = false, bool LEAN = false>
 __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restrict__ tau, const St &A,
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const bool greedy, uint16_t *rec,
@@ -704,7 +708,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
                                             const uint32_t rec_stride = 1) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   constexpr bool limit = RLIM;  // R45 (rl.buf or rl.in set)
-  uint32_t wmask = init_state<1, MASK, false, false, false, LG>(V, A, G);
+  uint32_t wmask = init_state<1, MASK, false, false, LEAN, LG>(V, A, G);
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
   const uint32_t sub = lane_words<LG>(G.lane);
@@ -752,8 +756,11 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       jmax = G.bcast(jmax);
     }
     // score(j) = tau[prev][j] * eta1(j, sk(j) + d(j)) (R1, R4)
+    // (lean layout: the dynamic last-use count is derived from the state, R14)
     auto score = [&](uint32_t j) -> uint32_t {
-      return (uint32_t)trow[j] * (mix ? V.ds[j].z : (uint32_t)V.eta1[j * L1 + dk1_get(A, j)]);
+      if (mix) return (uint32_t)trow[j] * V.ds[j].z;
+      const uint32_t d = LEAN ? sum_u8x4(dyn_kills(V, A, V.ds[j].w)) : dk1_get(A, j);
+      return (uint32_t)trow[j] * (uint32_t)V.eta1[j * L1 + d];
     };
     // Lane-local argmax in ascending order: strict '>' keeps the lowest
     // index among equal scores; bs1 = best score + 1 (0 = no candidate; a
@@ -768,11 +775,20 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
         for (int u = 0; u < 4; ++u) {
           v[u] = v0[u] && (!limit || j[u] <= jmax);  // R45
           tv[u] = trow[j[u]];
-          dk[u] = A.DK[(j[u] >> 3) * A.S];
+          if constexpr (!LEAN) dk[u] = A.DK[(j[u] >> 3) * A.S];
         }
+        if constexpr (LEAN) {  // dynamic last-use counts from the state (four candidates at once)
+          uint32_t dsw[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u)
-          dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+          for (int u = 0; u < 4; ++u) dsw[u] = V.ds[j[u]].w;
+          dyn_kills4w(V, A, dsw, dk);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + sum_u8x4(dk[u])];
+        } else {
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+        }
 #if ACO_BRANCHLESS1
         // branch-free: the four candidates' chains interleave (ILP)
         uint32_t sc[4];
@@ -841,7 +857,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
       jstar = G.bcast(jstar);
     }
     if (G.leader()) {
-      commit<1, MASK, false, false>(V, A, jstar, 0, wmask, live01, live23, prp01, prp23);
+      commit<1, MASK, false, false, LEAN>(V, A, jstar, 0, wmask, live01, live23, prp01, prp23);
       if (rec) rec[(size_t)k * rec_stride] = (uint16_t)jstar;
     }
     wmask = G.bcast(wmask);
@@ -1214,9 +1230,9 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE &
       rs1 = A.cfg.ants;
     }
     if (rl.buf)
-      o = ant_pass1<LG, MASK, WIDE, true>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
+      o = ant_pass1<LG, MASK, WIDE, true, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
     else
-      o = ant_pass1<LG, MASK, WIDE>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
+      o = ant_pass1<LG, MASK, WIDE, false, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -1687,7 +1703,7 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   unsigned char *smem = (unsigned char *)smem4;
   __shared__ uint32_t s_prp[3], s_flag, s_active;
   const uint32_t n = rd->n, na = A.cfg.ants, tid = threadIdx.x;
-  const FusedLayout F = fused_layout(n, rd->nwr, rd->nremw, rd->img.bytes, na);
+  const FusedLayout F = fused_layout(n, rd->nwr, rd->nremw, rd->img.bytes, na, A.cfg.group_size);
   stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
   const unsigned char *img = smem;
   uint16_t *tau = (uint16_t *)(smem + F.o_tau);
@@ -1699,6 +1715,7 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   uint16_t *ord = (uint16_t *)(smem + F.o_ord);
   uint32_t *cyc = (uint32_t *)(smem + F.o_cyc);
   uint16_t *next = (uint16_t *)(smem + F.o_next);
+  uint32_t *coins = (uint32_t *)(smem + F.o_coins);
   tau_fill(tau, W.tau_len, A.cfg.tau0);
   __syncthreads();
   init_greedy<true>(A, rd, W, rs, img, tau, st);  // (k_init)
@@ -1715,13 +1732,27 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
       if (tid == 0) s_active = rs.active;
       __syncthreads();
       if (!s_active) break;  // block-uniform
+      // group coins (R3) of every (step, group) of this iteration, one warp per
+      // 32 steps of a group (ballot), as k_construct precomputes them
+      const uint32_t gsz = A.cfg.group_size, g0 = A.cfg.ant_base / gsz;
+      const uint32_t ng = (A.cfg.ant_base + na - 1) / gsz - g0 + 1, cw = coin_words(pass, n);
+      {
+        const uint32_t lane = tid & 31u, c2 = pass == 1 ? it : (0x80000000u | it);
+        for (uint32_t task = tid >> 5; task < ng * cw; task += blockDim.x >> 5) {
+          const uint32_t gi = task / cw, k = (task - gi * cw) * 32 + lane;
+          const uint4 x = philox(k, 0x80000000u | (g0 + gi), c2, rd->region_id, A.cfg.seed);
+          const uint32_t word = __ballot_sync(0xFFFFFFFFu, (uint64_t)x.x < A.cfg.q0_t);
+          if (lane == 0) coins[task] = word;
+        }
+      }
+      __syncthreads();
       if (tid < na) {  // (k_construct) ant tid
         const Grp<1> G(tid);
         const uint32_t ant = A.cfg.ant_base + tid;
         AntOut o;
         if (pass == 1) {
           const St S = make_st<1, false, false>(st + tid, na, V);
-          o = ant_pass1<1, true>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, nullptr,
+          o = ant_pass1<1, true>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, coins + (ant / gsz - g0) * cw,
                                  RL{nullptr, 0, 0, 0, nullptr, nullptr}, na);
         } else {
           const St S = make_st<2, false, false>(st + tid, na, V);
@@ -1730,7 +1761,7 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
           for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
           const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
           o = ant_pass2<1, true, false, false>(V, tau, S, G, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + tid,
-                                               rec_c + tid, nullptr, 0, na);
+                                               rec_c + tid, coins + (ant / gsz - g0) * cw, cw * 32, na);
         }
         costs[tid] = o.cost;
         recp[tid] = make_uint4(o.prp01, o.prp23, o.len, 0u);
@@ -1834,9 +1865,11 @@ template <int LG, typename F>
 static void reg_lg(F &f) {
   reg1<1, LG, true, false, false, false, 2, true>(f);  // large regions, image through L1
   reg1<2, LG, true, false, false, false, 2, true>(f);
-  if constexpr (LG == 1) {  // pass-2 lean layout (large regions), image staged or through L1
+  if constexpr (LG == 1) {  // lean layouts (large regions), image staged or through L1
     reg1<2, 1, true, false, false, false, 0, true, F, true>(f);
     reg1<2, 1, true, false, false, false, 2, true, F, true>(f);
+    reg1<1, 1, true, false, false, false, 0, true, F, true>(f);
+    reg1<1, 1, true, false, false, false, 2, true, F, true>(f);
   }
   reg_w<1, LG, true, true, false, false>(f);
   reg_w<1, LG, true, false, false, false>(f);
