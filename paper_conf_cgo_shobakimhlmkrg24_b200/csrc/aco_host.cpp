@@ -911,14 +911,22 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   bool lean_on = true;  // pass-2 lean layout for large regions
   if (const char *e = getenv("ACO_LEAN")) lean_on = atoi(e) != 0;
   uint32_t lean_gain = 0;  // % more resident ants the lean layout must reach (C3: 0 measured best)
-  bool lean1_on = true;    // pass-1 lean layout for large regions
+  // pass-1 lean layout for large regions: off -- measured slower than the
+  // stored last-use counts despite ~1.8x the resident ants (r02g: n = 450 /
+  // 900 pass 1 0.174 / 0.314 -> 0.186 / 0.392 ns per ant-step; C5 1819 ->
+  // 1911 ms; C3 710 -> 706 ms, noise); kept for A/B (ACO_LEAN1=1)
+  bool lean1_on = false;
   if (const char *e = getenv("ACO_LEAN1")) lean1_on = atoi(e) != 0;
   uint32_t lean1_gain = 20;
   if (const char *e = getenv("ACO_LEAN1_GAIN")) lean1_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
-  bool gs_wide = true;  // 4-wide scan in the global-state kernels
-  if (const char *e = getenv("ACO_GS_WIDE")) gs_wide = atoi(e) != 0;
+  uint32_t gs_wide[2] = {1, 1};  // 4-wide scan in the global-state kernels, per pass
+  if (const char *e = getenv("ACO_GS_WIDE")) {
+    if (sscanf(e, "%u,%u", &gs_wide[0], &gs_wide[1]) == 1) gs_wide[1] = gs_wide[0];
+  }
+  uint32_t gs_wide_lanes = 8;  // ... with at most this many lanes per ant
+  if (const char *e = getenv("ACO_GS_WIDE_LANES")) gs_wide_lanes = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
@@ -1111,7 +1119,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // <= 8 lanes per ant (not in the u32-cycle / 3-4 class instantiations).
       // Measured (r02d, ms per step): C5 (4 lanes) 1963 -> 1808; C4 (16 lanes,
       // few candidates per lane) 855 -> 872, so 16-lane classes stay 1-wide
-      const bool gwide = g && gs_wide && sh.lanes <= 8 && !(pass == 2 && (t32 || P.nc4));
+      const bool gwide = g && gs_wide[pass - 1] && sh.lanes <= gs_wide_lanes && !(pass == 2 && (t32 || P.nc4));
       const bool wk = (wide && mask) || gwide;
       const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];

@@ -1694,6 +1694,9 @@ __global__ void k_stop(KArgs A, uint32_t pass) {
 // states -- and every result -- is that of the launches it replaces (the
 // same device functions run in the same order).  One ant per thread
 // (word-mask scan, compact pass-2 layout, group coins drawn inline).
+// FW: 4-wide candidate scan (four candidates' loads overlap: the lone ants of
+// a fused run are latency-bound).
+template <bool FW>
 __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
@@ -1752,7 +1755,7 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
         AntOut o;
         if (pass == 1) {
           const St S = make_st<1, false, false>(st + tid, na, V);
-          o = ant_pass1<1, true>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, coins + (ant / gsz - g0) * cw,
+          o = ant_pass1<1, true, FW>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, coins + (ant / gsz - g0) * cw,
                                  RL{nullptr, 0, 0, 0, nullptr, nullptr}, na);
         } else {
           const St S = make_st<2, false, false>(st + tid, na, V);
@@ -1760,7 +1763,7 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
 #pragma unroll
           for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
           const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
-          o = ant_pass2<1, true, false, false>(V, tau, S, G, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + tid,
+          o = ant_pass2<1, true, false, false, FW>(V, tau, S, G, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + tid,
                                                rec_c + tid, coins + (ant / gsz - g0) * cw, cw * 32, na);
         }
         costs[tid] = o.cost;
@@ -1985,7 +1988,8 @@ int init_kernel_attrs() {
   big_smem(k_init<false>);
   big_smem(k_pass2_init);
   big_smem(k_post);
-  big_smem(k_fused);
+  big_smem(k_fused<false>);
+  big_smem(k_fused<true>);
 #define ACO_SEL(M) big_smem(k_select<1, M, false, false>); big_smem(k_select<2, M, false, false>); \
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
   ACO_SEL(true) ACO_SEL(false)
@@ -2058,7 +2062,12 @@ int launch_post(LaunchCtx &L, uint32_t smem) {
 
 int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
   if (!L.cfg.count) return 0;
-  k_fused<<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
+  static const int fw = [] {
+    const char *e = getenv("ACO_FUSED_WIDE");
+    return e ? atoi(e) : 1;
+  }();
+  if (fw) k_fused<true><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
+  else k_fused<false><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
   L.launches++;
   return check();
 }
