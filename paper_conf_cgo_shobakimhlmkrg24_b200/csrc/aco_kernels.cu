@@ -138,7 +138,7 @@ struct SV {
   const uint32_t *muse, *mk, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0, *pg_ptr;
   const uint2 *pg;
   const uint16_t *eta1, *eta2;
-  uint32_t n, nwr, nremw, region_id, L1;
+  uint32_t n, nwr, nremw, region_id, L1, nslot;
   uint32_t livein01, livein23;  // u16 x 2
 };
 
@@ -163,6 +163,7 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   V.n = rd->n;
   V.nwr = rd->nwr;
   V.nremw = rd->nremw;
+  V.nslot = rd->nslot;
   V.region_id = rd->region_id;
   V.L1 = rd->L + 1;
   V.livein01 = (rd->livein[0] & 0xFFFFu) | (rd->livein[1] << 16);
@@ -278,12 +279,19 @@ __device__ __forceinline__ uint32_t x_slide2(uint32_t w) {
 // counts: the dynamic kills of a candidate are derived from its multi-use
 // registers' remaining-use counters / partners' scheduled bits (dyn_kills).
 constexpr uint32_t kWin8 = 128;
-__device__ __forceinline__ uint32_t r8_get(const St &A, uint32_t j) {
-  return (A.T[(j >> 2) * A.S] >> ((j & 3u) * 8)) & 0xFFu;
+// Ready-time SLOTS (r02): only an instruction with an incoming edge of
+// latency > 1 can be semi-ready (a latency-0/1 edge is met in the cycle after
+// its source issues, i.e. by the time the instruction is in the ready set), so
+// only those instructions own a u8 slot; ds.z >> 16 = slot, 0xFFFF = none
+// (always latency-ready once its predecessors are placed).  Pushes skip
+// latency <= 1 edges: they never decide "ready time <= t" (see commit).
+constexpr uint32_t kNoSlot = 0xFFFFu;
+__device__ __forceinline__ uint32_t r8_get(const St &A, uint32_t slot) {
+  return slot == kNoSlot ? 0u : (A.T[(slot >> 2) * A.S] >> ((slot & 3u) * 8)) & 0xFFu;
 }
-__device__ __forceinline__ void r8_push(const St &A, uint32_t v, uint32_t rt) {
-  uint32_t *p = A.T + (v >> 2) * A.S;
-  *p = __vmaxu4(*p, rt << ((v & 3u) * 8));  // byte-wise max (push-style ready time)
+__device__ __forceinline__ void r8_push(const St &A, uint32_t slot, uint32_t rt) {
+  uint32_t *p = A.T + (slot >> 2) * A.S;
+  *p = __vmaxu4(*p, rt << ((slot & 3u) * 8));  // byte-wise max (push-style ready time)
 }
 // kills_c(j) - static kills_c(j) as packed u8 x 4: registers read by j with >= 2
 // users whose last unscheduled user j is (R14): a counter register with one
@@ -594,8 +602,13 @@ __device__ __forceinline__ void commit(const SV &V, const St &A, uint32_t j, uin
     bool ready = true;
     uint32_t rdy = t + (e >> 16);
     if (CT) {  // ready time = max over placed predecessors
-      if (LEAN) r8_push(A, v, rdy - B);
-      else x_push_rt(A, v, rdy - B);
+      if (LEAN) {
+        // (a latency <= 1 edge is met by the next cycle: no push; such a
+        // successor of a slot-less instruction cannot occur)
+        if ((e >> 16) > 1u) r8_push(A, V.ds[v].z >> 16, rdy - B);
+      } else {
+        x_push_rt(A, v, rdy - B);
+      }
     }
     if (!(e & kSuccSingle) && (PASS == 1 || CT)) {
       // v is ready iff all its predecessors are placed: one scheduled-set
@@ -643,7 +656,7 @@ __device__ __forceinline__ uint32_t init_state(const SV &V, const St &A, const G
   for (uint32_t w = G.lane; w < V.nremw; w += LG) A.REM[w * A.S] = V.rem0[w];
   const uint32_t n = V.n;
   const bool ct = PASS == 2 && !T32 && !NC4;
-  const uint32_t tw = PASS == 1 ? 0 : (LEAN ? (n + 3) / 4 : (T32 ? n : (n + 1) / 2));
+  const uint32_t tw = PASS == 1 ? 0 : (LEAN ? (V.nslot + 3) / 4 : (T32 ? n : (n + 1) / 2));
   const uint32_t dw = PASS == 1 ? (LEAN ? 0u : (n + 7) / 8) : (ct ? 0u : (NC4 ? (n + 1) / 2 : (n + 3) / 4));
   for (uint32_t w = G.lane; w < tw + dw; w += LG) A.T[w * A.S] = 0;  // T and DK are contiguous
   if (MASK && LG > 1) {
@@ -758,7 +771,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     // score(j) = tau[prev][j] * eta1(j, sk(j) + d(j)) (R1, R4)
     // (lean layout: the dynamic last-use count is derived from the state, R14)
     auto score = [&](uint32_t j) -> uint32_t {
-      if (mix) return (uint32_t)trow[j] * V.ds[j].z;
+      if (mix) return (uint32_t)trow[j] * (V.ds[j].z & 0xFFFFu);
       const uint32_t d = LEAN ? sum_u8x4(dyn_kills(V, A, V.ds[j].w)) : dk1_get(A, j);
       return (uint32_t)trow[j] * (uint32_t)V.eta1[j * L1 + d];
     };
@@ -783,11 +796,11 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
           for (int u = 0; u < 4; ++u) dsw[u] = V.ds[j[u]].w;
           dyn_kills4w(V, A, dsw, dk);
 #pragma unroll
-          for (int u = 0; u < 4; ++u) dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + sum_u8x4(dk[u])];
+          for (int u = 0; u < 4; ++u) dk[u] = mix ? (V.ds[j[u]].z & 0xFFFFu) : V.eta1[j[u] * L1 + sum_u8x4(dk[u])];
         } else {
 #pragma unroll
           for (int u = 0; u < 4; ++u)
-            dk[u] = mix ? V.ds[j[u]].z : V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
+            dk[u] = mix ? (V.ds[j[u]].z & 0xFFFFu) : V.eta1[j[u] * L1 + ((dk[u] >> ((j[u] & 7u) * 4)) & 0xFu)];
         }
 #if ACO_BRANCHLESS1
         // branch-free: the four candidates' chains interleave (ILP)
@@ -907,9 +920,10 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   // ready time and per-class last-use counts of instruction j (LEAN: the
   // counts come from dyn_kills once ds is loaded)
   auto rd_dk = [&](uint32_t j, uint32_t &rd, uint32_t &dk) {
-    if constexpr (LEAN) {
-      rd = B + r8_get(A, j);
+    if constexpr (LEAN) {  // (the ready time needs ds.z: lean_rd below)
+      rd = 0;
       dk = 0;
+      (void)j;
     } else if constexpr (CT) {
       const uint32_t x = x_get(A, j);
       rd = B + (x & 0x3FFu);
@@ -919,6 +933,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       dk = dk2_get<NC4>(A, j);
     }
   };
+  auto lean_rd = [&](uint32_t dsz) -> uint32_t { return B + r8_get(A, dsz >> 16); };
   // heuristic of a feasible candidate: eta2 (CP), or eta1 (LUC, CP) for mixed odd groups
   auto eta_of = [&](uint32_t j, uint32_t e2, uint32_t dk) -> uint32_t {
     return mix ? (uint32_t)V.eta1[j * L1 + sum_u8x4(dk)] : e2;
@@ -928,7 +943,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   o.len = kInvalid;
   while (placed < n) {
     if (LEAN && t - B >= kWin8) {  // slide the u8 window: saturating byte subtract
-      for (uint32_t q = G.lane; q < (n + 3) / 4; q += LG) A.T[q * A.S] = __vsubus4(A.T[q * A.S], 0x80808080u);
+      for (uint32_t q = G.lane; q < (V.nslot + 3) / 4; q += LG) A.T[q * A.S] = __vsubus4(A.T[q * A.S], 0x80808080u);
       B += kWin8;
       G.sync();
     } else if (!LEAN && CT && t - B >= kWin) {  // slide the ready-time window (t - B <= 2 kWin - 2 here)
@@ -970,7 +985,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       if (lat_ok && (!mi || ((avail >> (8 * (ds.w & 0xFu))) & 1u))) {
         counts += 1u;
         if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
-          const uint32_t s = tv * eta_of(j, ds.z, dk);
+          const uint32_t s = tv * eta_of(j, ds.z & 0xFFFFu, dk);
           counts += 1u << 16;
           f_not_inc |= __vcmpgtu4(ds.x, K) == 0u;           // max_c Delta_c <= 0
           if (s + 1u > bs1) {  // ascending: strict keeps the lowest index (R1, R25)
@@ -992,10 +1007,14 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           rd_dk(j[u], rd[u], dk[u]);
-          ds[u] = V.ds[j[u]];                         // defs, static kills, eta2, type
+          ds[u] = V.ds[j[u]];                         // defs, static kills, eta2 | slot, type
           tv[u] = trow[j[u]];
         }
-        if (LEAN) dyn_kills4(V, A, ds, dk);
+        if constexpr (LEAN) {
+#pragma unroll
+          for (int u = 0; u < 4; ++u) rd[u] = lean_rd(ds[u].z);
+          dyn_kills4(V, A, ds, dk);
+        }
 #pragma unroll
         for (int u = 0; u < 4; ++u)
           if (v[u]) eval(j[u], rd[u], ds[u], dk[u], tv[u]);
@@ -1005,7 +1024,10 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         uint32_t rd, dk;
         rd_dk(j, rd, dk);
         const uint4 ds = V.ds[j];
-        if (LEAN) dk = dyn_kills(V, A, ds.w);
+        if (LEAN) {
+          rd = lean_rd(ds.z);
+          dk = dyn_kills(V, A, ds.w);
+        }
         eval(j, rd, ds, dk, trow[j]);
         return false;
       });
@@ -1062,12 +1084,13 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         scan_bits<MASK>(A, nwr, wmask, 0, 1, 0xFFFFFFFFu, [&](uint32_t j) {
           uint32_t rd, dk;
           rd_dk(j, rd, dk);
-          if (rd > t) return false;
           const uint4 ds = V.ds[j];
+          if (LEAN) rd = lean_rd(ds.z);
+          if (rd > t) return false;
           if (LEAN) dk = dyn_kills(V, A, ds.w);
           if (mi && !((avail >> (8 * (ds.w & 0xFu))) & 1u)) return false;
           if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u) return false;
-          pre += (uint32_t)trow[j] * eta_of(j, ds.z, dk);
+          pre += (uint32_t)trow[j] * eta_of(j, ds.z & 0xFFFFu, dk);
           if (pre > r) {
             jstar = j;
             return true;
