@@ -444,7 +444,20 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
     ds[4 * j] = info[(size_t)j * 4 + 0];
     ds[4 * j + 1] = info[(size_t)j * 4 + 1];
   }
-  for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j];
+  // ds.z = eta2 | ready-time slot << 16: the instructions with an incoming
+  // edge of latency > 1 get consecutive slots (lean pass-2 layout); the others
+  // 0xFFFF (latency-ready as soon as their predecessors are placed)
+  uint32_t nslot = 0;
+  {
+    static const bool all_slots = [] {  // A/B: every instruction owns a slot (the r01 lean layout)
+      const char *e = getenv("ACO_SLOTS");
+      return e && atoi(e) == 0;
+    }();
+    std::vector<uint8_t> need(n, all_slots ? 1 : 0);
+    for (uint32_t q = 0; q < E; ++q)
+      if (lats[q] > 1u) need[outs[q]] = 1;
+    for (uint32_t j = 0; j < n; ++j) ds[4 * j + 2] = eta2[j] | ((need[j] ? nslot++ : 0xFFFFu) << 16);
+  }
   // ds.w = issue type (R42, bits 0-3) | multi-use register count << 4 |
   // their start in the multi-use list << 8 (the lean pass-2 layout derives
   // the dynamic kills from them)
@@ -574,6 +587,7 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   R.max_lat = max_lat;
   R.mc_max = mc_max;
   R.compact = compact ? 1u : 0u;
+  R.nslot = nslot;
   for (uint32_t c = 0; c < 4; ++c) {
     R.livein[c] = livein[c];
     R.lbvec[c] = lbvec[c];
@@ -925,8 +939,15 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_GS_WIDE")) {
     if (sscanf(e, "%u,%u", &gs_wide[0], &gs_wide[1]) == 1) gs_wide[1] = gs_wide[0];
   }
-  uint32_t gs_wide_lanes = 8;  // ... with at most this many lanes per ant
-  if (const char *e = getenv("ACO_GS_WIDE_LANES")) gs_wide_lanes = (uint32_t)atoi(e);
+  // ... with at most this many lanes per ant (pass 1, pass 2).  Measured
+  // (r02d/h, ms per step): C5 (4 lanes) 1963 -> 1808; C4 (16 lanes) both
+  // passes 855 -> 872, pass 1 only 894 -> 822 (pass 2 has ~5 ready
+  // candidates per step at n = 2,000: a 4-wide batch rarely fills, and the
+  // 64-register cap spills)
+  uint32_t gs_wide_lanes[2] = {16, 8};
+  if (const char *e = getenv("ACO_GS_WIDE_LANES")) {
+    if (sscanf(e, "%u,%u", &gs_wide_lanes[0], &gs_wide_lanes[1]) == 1) gs_wide_lanes[1] = gs_wide_lanes[0];
+  }
   if (const char *e = getenv("ACO_GS_LANES")) sscanf(e, "%u,%u", &gs_lanes[0], &gs_lanes[1]);
   if (const char *e = getenv("ACO_GS_MIN_THREADS")) sscanf(e, "%u,%u", &gs_min_threads[0], &gs_min_threads[1]);
   if (const char *e = getenv("ACO_MAX_LANES_WIDE")) sscanf(e, "%u,%u", &max_lanes_w[0], &max_lanes_w[1]);
@@ -1023,7 +1044,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // evaluation) and gains resident ants; on the mixed C3 batch it wins
       // whenever it fits at least as many ants (B200: 684 -> 645 ms/batch;
       // ACO_LEAN_GAIN = 20 / 50 %: 654 ms)
-      const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true);
+      const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true, R.nslot);
       const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[1][2], false, false, tgt_threads[1], 1, A,
                                    p->group_size, coin_words(pass, R.n), img_l1[1] != 0, 1u, spread, 1u);
       if (shl.apb && 100ull * shl.resident >= (100ull + lean_gain) * sh.resident) {
@@ -1115,11 +1136,9 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       }
       const bool mask = R.n <= 1024 && !g;
       if (g) sh.ig = false;
-      // global-state kernels: 4-wide candidate scan over strided words with
-      // <= 8 lanes per ant (not in the u32-cycle / 3-4 class instantiations).
-      // Measured (r02d, ms per step): C5 (4 lanes) 1963 -> 1808; C4 (16 lanes,
-      // few candidates per lane) 855 -> 872, so 16-lane classes stay 1-wide
-      const bool gwide = g && gs_wide[pass - 1] && sh.lanes <= gs_wide_lanes && !(pass == 2 && (t32 || P.nc4));
+      // global-state kernels: 4-wide candidate scan over strided words (not in
+      // the u32-cycle / 3-4 class instantiations), gs_wide_lanes above
+      const bool gwide = g && gs_wide[pass - 1] && sh.lanes <= gs_wide_lanes[pass - 1] && !(pass == 2 && (t32 || P.nc4));
       const bool wk = (wide && mask) || gwide;
       const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];

@@ -76,7 +76,7 @@ struct RegionDev {
   uint32_t max_lat;  // largest edge latency
   uint32_t mc_max;   // max over instructions and classes of multi-use registers read
   uint32_t compact;  // pass 2 uses the compact layout (the image has no per-predecessor list)
-  uint32_t pad1;
+  uint32_t nslot;    // instructions with an incoming edge of latency > 1 (lean pass-2 ready-time slots)
   uint64_t o_image;  // byte offset of the block image in the arena
   ImageLayout img;
 };
@@ -189,10 +189,10 @@ inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 //           DK [ceil(n/4)] u8 = 2 classes x 4 bits (or [ceil(n/2)] u16 = 4
 //                           classes x 4 bits if nc4): per-class last-use counts
 ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32_t nremw, bool t32,
-                                 bool nc4, bool lean = false) {
+                                 bool nc4, bool lean = false, uint32_t nslot = 0xFFFFFFFFu) {
   const uint32_t w = 2 * nwr + nremw;
   if (pass == 1) return w + (lean ? 0u : (n + 7) / 8);  // lean pass 1: last-use counts derived, not stored
-  if (lean) return w + (n + 3) / 4;  // lean: u8 windowed ready time (kills derived, not stored)
+  if (lean) return w + ((nslot == 0xFFFFFFFFu ? n : nslot) + 3) / 4;  // lean: u8 ready-time slots (kills derived)
   if (!t32 && !nc4) return w + (n + 1) / 2;  // compact: u16 (windowed ready time | last uses)
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }

@@ -1208,7 +1208,7 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE &
       const uint32_t gsz = A.cfg.group_size, abase = A.cfg.ant_base + bi.ant0, g0 = abase / gsz;
       const uint32_t ng = (abase + apb - 1) / gsz - g0 + 1, cw = coin_words(PASS, rd->n);
       uint32_t *cz = (uint32_t *)(smem + state_off) +
-                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4, LEAN);
+                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4, LEAN, rd->nslot);
       const uint32_t lane = threadIdx.x & 31u, c2 = PASS == 1 ? iter : (0x80000000u | iter);
       for (uint32_t task = threadIdx.x >> 5; task < ng * cw; task += blockDim.x >> 5) {
         const uint32_t gi = task / cw, k = (task - gi * cw) * 32 + lane;
@@ -1717,8 +1717,8 @@ __global__ void k_stop(KArgs A, uint32_t pass) {
 // states -- and every result -- is that of the launches it replaces (the
 // same device functions run in the same order).  One ant per thread
 // (word-mask scan, compact pass-2 layout, group coins drawn inline).
-// FW: 4-wide candidate scan (four candidates' loads overlap: the lone ants of
-// a fused run are latency-bound).
+// FW: 4-wide candidate scan (off by default: the small regions of a fused run
+// have too few candidates per step to fill a batch of four).
 template <bool FW>
 __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   const uint32_t r = blockIdx.x;
@@ -2085,9 +2085,9 @@ int launch_post(LaunchCtx &L, uint32_t smem) {
 
 int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
   if (!L.cfg.count) return 0;
-  static const int fw = [] {
+  static const int fw = [] {  // (measured, C1: 1-wide 0.654 ms, 4-wide 0.702 ms: few candidates per step)
     const char *e = getenv("ACO_FUSED_WIDE");
-    return e ? atoi(e) : 1;
+    return e ? atoi(e) : 0;
   }();
   if (fw) k_fused<true><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
   else k_fused<false><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
