@@ -1421,6 +1421,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // B200 (ms per step, r02b): C4 852 / 839, C5 1992 / 2027 -- within 2 %, [word][ant] kept
   cfg.gs_ant_major = 0;
   if (const char *e = getenv("ACO_GS_LAYOUT")) cfg.gs_ant_major = atoi(e) != 0;
+  cfg.lazy_kills = 0;
+  if (const char *e = getenv("ACO_LAZY_KILLS")) cfg.lazy_kills = atoi(e) != 0;
   cfg.record = P.record ? 1u : 0u;
   cfg.stage_img = P.stage_img ? 1u : 0u;
   cfg.dump_slice = (uint64_t)A * sum_n;

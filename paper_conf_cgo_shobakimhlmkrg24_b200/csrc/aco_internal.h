@@ -147,7 +147,7 @@ struct RunCfg {
   uint32_t stage_img;   // k_select stages the region image in shared memory (few regions)
   uint32_t mslot;       // machine slot (c_mach[mslot]) of this context
   uint32_t gs_ant_major;  // global-state kernels: per-ant state ant-major (1) or [word][ant] (0)
-  uint32_t pad_cfg2;
+  uint32_t lazy_kills;    // lean pass 2: derive kills only for candidates where they decide
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
   int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };

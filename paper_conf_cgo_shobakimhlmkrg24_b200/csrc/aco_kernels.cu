@@ -934,6 +934,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     }
   };
   auto lean_rd = [&](uint32_t dsz) -> uint32_t { return B + r8_get(A, dsz >> 16); };
+  const bool lazy = LEAN && cfg.lazy_kills && !stall_en && !mix;  // (lean: kills only where they decide)
   // heuristic of a feasible candidate: eta2 (CP), or eta1 (LUC, CP) for mixed odd groups
   auto eta_of = [&](uint32_t j, uint32_t e2, uint32_t dk) -> uint32_t {
     return mix ? (uint32_t)V.eta1[j * L1 + sum_u8x4(dk)] : e2;
@@ -1013,7 +1014,18 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
         if constexpr (LEAN) {
 #pragma unroll
           for (int u = 0; u < 4; ++u) rd[u] = lean_rd(ds[u].z);
-          dyn_kills4(V, A, ds, dk);
+          if (lazy) {
+            // kills decide nothing for a candidate of an ant that may not stall
+            // (nor mixes heuristics) unless it is latency-ready and some class
+            // has more defs than slack: its K is skipped (dk = 0; exact)
+            uint32_t dsw[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              dsw[u] = (v[u] && rd[u] <= t && __vcmpgtu4(ds[u].x, slack) != 0u) ? ds[u].w : (ds[u].w & ~0xF0u);
+            dyn_kills4w(V, A, dsw, dk);
+          } else {
+            dyn_kills4(V, A, ds, dk);
+          }
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u)
