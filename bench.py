@@ -240,18 +240,16 @@ def host_cpu():
     return {"model": model, "threads": os.cpu_count()}
 
 
-def lib_sha256():
-    """sha256 of the loaded CUDA library (matches a profile to its build)."""
-    import hashlib
-    from paper_conf_cgo_shobakimhlmkrg24_b200 import _lib
-    with open(_lib.LIB_PATH, "rb") as f:
-        return hashlib.sha256(f.read()).hexdigest()
+def build_fingerprint():
+    """sha256 of the library's sources + nvcc flags (matches a profile to its build)."""
+    from paper_conf_cgo_shobakimhlmkrg24_b200 import build as B
+    return B.source_fingerprint()
 
 
 def ncu_evidence(workload: str):
     """DRAM traffic and issue-slot figures of the construct launches from the
     committed ncu --set full capture (profiles/r02_traffic.json) -- used only
-    when that capture profiled this very build (same libaco_b200.so sha256)."""
+    when that capture profiled this very build (same source fingerprint)."""
     try:
         with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
             tj = json.load(f)
@@ -259,9 +257,9 @@ def ncu_evidence(workload: str):
         return None, None, "no committed capture"
     if workload != "c3":
         return None, None, "capture is of the c3 batch"
-    sha = lib_sha256()
-    if tj.get("so_sha256") != sha:
-        return None, None, f"committed capture is of another build ({str(tj.get('so_sha256'))[:12]} vs {sha[:12]})"
+    sha = build_fingerprint()
+    if tj.get("build_fingerprint") != sha:
+        return None, None, f"committed capture is of another build ({str(tj.get('build_fingerprint'))[:12]} vs {sha[:12]})"
     issue = {"util_pct": tj.get("issue_util_pct"), "warps_active_pct": tj.get("warps_active_pct"),
              "source": tj.get("issue_source")}
     return tj.get("dram_bytes_per_launch"), issue, tj.get("source")

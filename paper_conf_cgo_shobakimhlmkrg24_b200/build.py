@@ -16,6 +16,19 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-gencode", "arch=compute_100a,code=s
          "-Xcompiler", "-fPIC", "-Xcompiler", "-pthread", "-shared"]
 
 
+def source_fingerprint() -> str:
+    """sha256 over the library's sources, headers and nvcc flags: identifies a
+    build (nvcc output itself is not byte-reproducible).  A profile records
+    it; bench.py uses the profile's figures only for the same fingerprint."""
+    import hashlib
+    h = hashlib.sha256()
+    for f in SOURCES + HEADERS:
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    h.update(" ".join(FLAGS).encode())
+    return h.hexdigest()
+
+
 def stale() -> bool:
     if not os.path.exists(LIB):
         return True

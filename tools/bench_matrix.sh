@@ -1,12 +1,12 @@
 # Bench lines for every config and SURVEY 8(f) mode (run under gpurun, 1 GPU).
-# Each JSON line goes to gpurun_out/bench_<name>.json.
-python paper_conf_cgo_shobakimhlmkrg24_b200/build.py
+# Each JSON line goes to $BM_OUT/bench_<name>.json (default gpurun_out/).
+O=${BM_OUT:-gpurun_out}; mkdir -p $O
 run() {  # name, args...
   name=$1; shift
-  timeout 900 python bench.py --steps 3 --warmup 3 "$@" 2>gpurun_out/bench_$name.err | tail -1 > gpurun_out/bench_$name.json
-  echo "== $name: $(cut -c1-160 gpurun_out/bench_$name.json)"
+  timeout 900 python bench.py --steps ${BM_STEPS:-5} --warmup 3 "$@" 2>$O/bench_$name.err | tail -1 > $O/bench_$name.json
+  echo "== $name: $(cut -c1-160 $O/bench_$name.json)"
 }
-for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix rlmin rlmid}; do
+for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix stall50 rlmin rlmid ref}; do
   case $w in
     c1|c2|c3|c4|c5) run $w --workload $w ;;
     dual) run c3_dual --machine dual ;;
@@ -16,5 +16,6 @@ for w in ${MATRIX:-c3 c1 c2 c4 c5 dual weighted policy mix rlmin rlmid}; do
     rlmin) run c3_rl_min --rl-limit 1 ;;
     rlmid) run c3_rl_mid --rl-limit 2 ;;
     stall50) run c3_stall50 --stall-num 2 ;;
+    ref) run c3_reference --impl reference ;;
   esac
 done

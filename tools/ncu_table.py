@@ -54,11 +54,11 @@ def main(path, traffic_out=None, source="", so_sha256=None):
                    "source": source, "issue_util_pct": round(acc / tw, 1), "warps_active_pct": round(accw / tw, 1),
                    "issue_source": "time-weighted sm__inst_issued.avg.pct_of_peak_sustained_active (and "
                                    "sm__warps_active) over the same construct launches",
-                   "so_sha256": so_sha256},
+                   "build_fingerprint": so_sha256},
                   open(traffic_out, 'w'), indent=1)
 
 
 if __name__ == "__main__":
-    # ncu_table.py prof_raw.csv [traffic.json source-text [sha256 of the profiled libaco_b200.so]]
+    # ncu_table.py prof_raw.csv [traffic.json source-text [build fingerprint of the profiled library]]
     main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, sys.argv[3] if len(sys.argv) > 3 else "",
          sys.argv[4] if len(sys.argv) > 4 else None)
