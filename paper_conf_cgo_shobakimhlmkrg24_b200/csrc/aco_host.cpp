@@ -917,6 +917,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   bool fill_sms = true;  // spread passes with fewer shared-memory blocks than SMs (below)
   if (const char *e = getenv("ACO_FILL")) fill_sms = atoi(e) != 0;
   uint32_t fill_img_max = 64 * 1024;
+  uint32_t fill_lanes[2] = {0, 0};  // lanes per ant of spread shapes (0: keep the default pick's)
+  if (const char *e = getenv("ACO_FILL_LANES")) sscanf(e, "%u,%u", &fill_lanes[0], &fill_lanes[1]);
   if (const char *e = getenv("ACO_FILL_IMG")) fill_img_max = (uint32_t)atoi(e);
   uint32_t spread_lanes = 0;  // 0: lanes ~ bitset words
   if (const char *e = getenv("ACO_SPREAD_LANES")) spread_lanes = (uint32_t)atoi(e);
@@ -1116,7 +1118,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         const uint32_t need = (uint32_t)std::ceil(148.0 * nr * (nr + 16.0) / wtot);
         const uint32_t have = (A + q.sh.apb - 1) / q.sh.apb;
         if (need <= have) continue;
-        const RegionPlan f = plan_region(r, pass, std::max(1u, (A + need - 1) / need), q.sh.lanes);
+        const RegionPlan f = plan_region(r, pass, std::max(1u, (A + need - 1) / need),
+                                         fill_lanes[pass - 1] ? fill_lanes[pass - 1] : q.sh.lanes);
         if (!f.g && f.sh.apb && (A + f.sh.apb - 1) / f.sh.apb > have) q = f;
       }
     }
