@@ -522,6 +522,15 @@ __device__ __forceinline__ void scan4_any(const St &A, uint32_t m, uint32_t firs
   else scan4s(A, first, stride, nwr, visit);
 }
 
+// Prefetch the pheromone row of the next step into L1 (the row of the
+// instruction just placed; tau in global memory): one 128-byte line per lane
+// and stride, issued right after the commit so the next scan's tau reads hit.
+template <int LG>
+__device__ __forceinline__ void tau_row_prefetch(const uint16_t *tau, uint32_t row, uint32_t n, const Grp<LG> &G) {
+  const char *p = (const char *)(tau + (size_t)row * n);
+  for (uint32_t b = G.lane * 128u; b < n * 2u; b += LG * 128u) asm volatile("prefetch.global.L1 [%0];" ::"l"(p + b));
+}
+
 struct AntOut {
   uint32_t cost;
   uint32_t prp01, prp23;
@@ -718,7 +727,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
                                             const Grp<LG> &G, const uint32_t ant, const uint32_t iter,
                                             const RunCfg &cfg, const bool greedy, uint16_t *rec,
                                             const uint32_t *coins = nullptr, const RL rl = RL{nullptr, 0, 0, 0, nullptr, nullptr},
-                                            const uint32_t rec_stride = 1) {
+                                            const uint32_t rec_stride = 1, const bool pf = false) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   constexpr bool limit = RLIM;  // R45 (rl.buf or rl.in set)
   uint32_t wmask = init_state<1, MASK, false, false, LEAN, LG>(V, A, G);
@@ -876,6 +885,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
     wmask = G.bcast(wmask);
     G.sync();
     prev = jstar;
+    if (pf) tau_row_prefetch<LG>(tau, prev, n, G);
   }
   AntOut o;
   o.prp01 = prp01;
@@ -900,7 +910,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
                                             const RunCfg &cfg, const uint32_t tgt[4], uint32_t *prune_len,
                                             const bool prune, uint16_t *rec_o, uint32_t *rec_c,
                                             const uint32_t *coins = nullptr, uint32_t coin_t = 0,
-                                            const uint32_t rec_stride = 1) {
+                                            const uint32_t rec_stride = 1, const bool pf = false) {
   const uint32_t n = V.n, nwr = V.nwr, L1 = V.L1;
   uint32_t wmask = init_state<2, MASK, T32, NC4, LEAN, LG>(V, A, G);
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
@@ -1125,6 +1135,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     G.sync();
     ++placed;
     prev = jstar;
+    if (pf) tau_row_prefetch<LG>(tau, prev, n, G);
     if (mi) {  // R42: the cycle is complete after issue_width placements
       ++used;
       used_t += 1u << (8 * (V.ds[jstar].w & 0xFu));
@@ -1253,6 +1264,8 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE &
   const Grp<LG> G(threadIdx.x);
   const SV V = make_sv(img, rd);
   const St S = make_st<PASS, T32, NC4, LEAN>(stbase, stride, V);
+  // tau rows read from global memory: prefetch the next step's row into L1
+  const bool pf = !TAU_SMEM && (A.cfg.tau_prefetch & (1u << (PASS - 1 + (GS == 1 ? 2 : 0))));
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
   if (PASS == 1) {
@@ -1265,9 +1278,9 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE &
       rs1 = A.cfg.ants;
     }
     if (rl.buf)
-      o = ant_pass1<LG, MASK, WIDE, true, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
+      o = ant_pass1<LG, MASK, WIDE, true, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1, pf);
     else
-      o = ant_pass1<LG, MASK, WIDE, false, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1);
+      o = ant_pass1<LG, MASK, WIDE, false, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1, pf);
   } else {
     uint32_t tgt[4];
 #pragma unroll
@@ -1288,7 +1301,7 @@ __global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE &
       rs2 = A.cfg.ants;
     }
     o = ant_pass2<LG, MASK, T32, NC4, WIDE, LEAN>(V, tau, S, G, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o,
-                                      rec_c, coins, coin_t, rs2);
+                                      rec_c, coins, coin_t, rs2, pf);
   }
   if (G.leader()) {
     uint32_t *costs = (uint32_t *)(A.ws + W.o_cost);
