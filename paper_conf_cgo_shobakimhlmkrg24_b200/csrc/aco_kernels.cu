@@ -174,6 +174,20 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
 __device__ __forceinline__ uint32_t lo_pair(uint32_t w) { return __byte_perm(w, 0, 0x4140); }  // u8 b0,b1 -> u16x2
 __device__ __forceinline__ uint32_t hi_pair(uint32_t w) { return __byte_perm(w, 0, 0x4342); }  // u8 b2,b3 -> u16x2
 
+// Per-class comparisons of packed small counts (values < 2^15, no carry
+// between lanes).  sm_100 has no native byte-SIMD compare / saturating add
+// (each __vcmp*u4 / __vaddus4 is a chain of ~6 dependent LOP3/PRMT/IADD), so
+// with <= 2 register classes the tests run on u16 x 2 lanes with a guard
+// bit: all_le2(a, b) = every lane a_c <= b_c.
+constexpr uint32_t kGuard2 = 0x80008000u;
+__device__ __forceinline__ bool all_le2(uint32_t a2, uint32_t b2) {
+  return (((b2 | kGuard2) - a2) & kGuard2) == kGuard2;
+}
+// some lane a_c < b_c
+__device__ __forceinline__ bool any_lt2(uint32_t a2, uint32_t b2) {
+  return ((((a2 | kGuard2) - b2) & kGuard2) != kGuard2);
+}
+
 // Per-ant state (stride S words between consecutive words of one ant).
 struct St {
   uint32_t *RB, *SCH, *REM, *T, *DK;
@@ -983,6 +997,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
 #pragma unroll
       for (int c = 0; c < 4; ++c) slack |= ::min(tgt[c] - lv[c], 255u) << (8 * c);
     }
+    const uint32_t slack2 = lo_pair(slack);  // classes 0, 1 as u16 x 2 (<= 2 classes: !NC4)
     const uint16_t *trow = tau + prev * n;
     uint32_t counts = 0, min_s = 0xFFFFFFFFu;  // counts = |R| | |F| << 16
     bool f_not_inc = false, s_dec = false, any_s = false;
@@ -995,10 +1010,14 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       const bool lat_ok = rdy <= t;
       if (lat_ok && (!mi || ((avail >> (8 * (ds.w & 0xFu))) & 1u))) {
         counts += 1u;
-        if (__vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u) {  // feasible: defs_c <= slack_c + kills_c
+        // feasible: defs_c <= slack_c + kills_c in every class (R21)
+        const bool feas = NC4 ? __vcmpgtu4(ds.x, __vaddus4(slack, K)) == 0u
+                              : all_le2(lo_pair(ds.x), slack2 + lo_pair(K));
+        if (feas) {
           const uint32_t s = tv * eta_of(j, ds.z & 0xFFFFu, dk);
           counts += 1u << 16;
-          f_not_inc |= __vcmpgtu4(ds.x, K) == 0u;           // max_c Delta_c <= 0
+          // max_c Delta_c <= 0
+          f_not_inc |= NC4 ? __vcmpgtu4(ds.x, K) == 0u : all_le2(lo_pair(ds.x), lo_pair(K));
           if (s + 1u > bs1) {  // ascending: strict keeps the lowest index (R1, R25)
             bs1 = s + 1u;
             bj = j;
@@ -1008,7 +1027,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       } else {
         any_s = true;
         min_s = ::min(min_s, lat_ok ? t + 1u : rdy);        // slot-blocked: next cycle (R42)
-        s_dec |= __vcmpltu4(ds.x, K) != 0u;                 // min_c Delta_c < 0
+        // min_c Delta_c < 0
+        s_dec |= NC4 ? __vcmpltu4(ds.x, K) != 0u : any_lt2(lo_pair(ds.x), lo_pair(K));
       }
     };
     if constexpr (wide) {
@@ -1031,7 +1051,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
             uint32_t dsw[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u)
-              dsw[u] = (v[u] && rd[u] <= t && __vcmpgtu4(ds[u].x, slack) != 0u) ? ds[u].w : (ds[u].w & ~0xF0u);
+              dsw[u] = (v[u] && rd[u] <= t && !all_le2(lo_pair(ds[u].x), slack2)) ? ds[u].w : (ds[u].w & ~0xF0u);
             dyn_kills4w(V, A, dsw, dk);
           } else {
             dyn_kills4(V, A, ds, dk);
@@ -1111,7 +1131,9 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
           if (rd > t) return false;
           if (LEAN) dk = dyn_kills(V, A, ds.w);
           if (mi && !((avail >> (8 * (ds.w & 0xFu))) & 1u)) return false;
-          if (__vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u) return false;
+          if (NC4 ? __vcmpgtu4(ds.x, __vaddus4(slack, ds.y + dk)) != 0u
+                  : !all_le2(lo_pair(ds.x), slack2 + lo_pair(ds.y + dk)))
+            return false;
           pre += (uint32_t)trow[j] * eta_of(j, ds.z & 0xFFFFu, dk);
           if (pre > r) {
             jstar = j;
