@@ -140,3 +140,67 @@ def test_record_mode_workspace(lib, monkeypatch):
     assert st0 == st1 == 0
     want = p.ants * sum(r.n_insts for r in regs) * 6 + 16 * p.ants * len(regs)
     assert want <= ws1 - ws0 <= want + 3 * 256 + 3 * 16
+
+
+PLAN_SNIPPET = r'''
+import ctypes as C, json, os, sys
+sys.path.insert(0, {root!r})
+os.environ["ACO_DEBUG_PLAN"] = "1"
+import bench
+from paper_conf_cgo_shobakimhlmkrg24_b200 import _lib
+from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch, machine_struct, params_struct
+L = _lib.load()
+a = bench.parse({argv!r})
+out = []
+for b in bench.workload(a, 0, 1)[0]:
+    hb = HostBatch(b.regs, b.ids)
+    m = machine_struct(bench.machine_of(a)); ctx = C.c_void_p()
+    L.aco_create(0, C.byref(m), C.byref(ctx))
+    need = C.c_size_t(0)
+    assert L.aco_load_regions(ctx, hb.descs, len(b.regs), None, 0, C.byref(need), None) == 0
+    ps = params_struct(b.p)
+    assert L.aco_schedule_batch(ctx, C.byref(ps), None, 0, C.byref(need), None) == 0
+    cnt = C.c_uint32(0); buf = (C.c_uint32 * 64)()
+    L.aco_last_variants(ctx, buf, 64, C.byref(cnt))
+    out.append([int(buf[i]) for i in range(cnt.value)])
+print(json.dumps(out))
+'''
+
+
+def _plan(argv):
+    """Host planning of a bench line (sizing calls, no CUDA call): the
+    variants of each batch and the '[aco plan]' class lines."""
+    import json
+    import subprocess
+    import sys
+    r = subprocess.run([sys.executable, "-c", PLAN_SNIPPET.format(root=ROOT, argv=argv)], capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    classes = []
+    for line in r.stderr.splitlines():
+        mm = re.match(r"\[aco plan\] pass (\d) class \d+: blocks (\d+) ants/blk (\d+) lanes (\d+)", line)
+        if mm:
+            classes.append(tuple(int(x) for x in mm.groups()))
+    return json.loads(r.stdout.strip().splitlines()[-1]), classes
+
+
+def test_planner_fused_for_config1_only(lib):
+    """Config 1 (64 ants, one region) runs as one fused single-block launch
+    (k_fused, variant bit 13); config 2 (1,024 ants) does not."""
+    v1, c1 = _plan(["--workload", "c1"])
+    assert v1 == [[1 << 13]]
+    v2, c2 = _plan(["--workload", "c2"])
+    assert all(not (c & (1 << 13)) for c in v2[0]) and c2
+
+
+def test_planner_fill_rule_spreads_few_large_regions(lib):
+    """Config 2 (one region holding all the work): its ants spread over many
+    small blocks in both passes (the SM fill rule), pass 1 with up to 4 lanes
+    per ant; config 3 (5,000 regions) keeps its large blocks."""
+    _, c2 = _plan(["--workload", "c2"])
+    for pass_ in (1, 2):
+        blocks = sum(b for p, b, a, l in c2 if p == pass_)
+        assert blocks >= 32, c2
+    assert any(p == 1 and l == 4 for p, b, a, l in c2)
+    _, c3 = _plan(["--workload", "c3", "--regions", "400"])
+    assert max(a * l for p, b, a, l in c3) >= 256  # large blocks kept
