@@ -395,9 +395,18 @@ def main(argv=None):
     import torch.distributed as dist
     from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch, Scheduler
 
+    # (test knobs: ACO_BENCH_ONE_GPU=1 puts every rank on cuda:0 and
+    # ACO_BENCH_BACKEND=gloo lets such ranks talk -- a dry run of the N > 1
+    # path on a one-GPU box; the product runs are one rank per GPU over NCCL)
+    if os.environ.get("ACO_BENCH_ONE_GPU") == "1":
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("ACO_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     batches, cfg, scaling = workload(args, rank, world)
     machine = machine_of(args)
     colony = args.workload == "c4" and world > 1  # one region, ants split across ranks

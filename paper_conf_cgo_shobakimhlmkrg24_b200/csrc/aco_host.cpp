@@ -511,7 +511,7 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   }
   // the per-predecessor list is needed only by the u16/u32-cycle pass-2
   // layouts (ready time = max over predecessors at readiness)
-  const bool compact = mach.issue_width <= 1 && n_classes <= 2 && max_lat <= 511u && mc_max <= 7u;
+  const bool compact = n_classes <= 2 && max_lat <= 511u && mc_max <= 7u;
   if (compact) {
     pred.clear();
     pp.assign(n + 1, 0);
@@ -973,8 +973,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     for (uint32_t r = 0; r < count; ++r) {
       const RegionDev &R = ctx->regions[r];
       if (R.n <= 600) continue;  // (host time: smaller regions always fit shared memory)
-      const bool t32 = ctx->mach.issue_width > 1 ||
-                       (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
+      const bool t32 = (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
       for (uint32_t pass = 1; pass <= 2; ++pass) {
         if (!(pmask & pass)) continue;
         const bool wide = R.n >= kWideN && R.n <= 1024, rare = pass == 2 && (t32 || P.nc4);
@@ -1006,9 +1005,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // latencies < 512, 2 classes and <= 7 multi-use registers per class and
     // instruction; otherwise u16 cycles (3-4 classes), or u32 when a
     // schedule may exceed 65535 cycles (or the compact layout does not apply)
-    // the general machine model (R42) runs in the u32-cycle variants
-    const bool t32 = ctx->mach.issue_width > 1 ||
-                     (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
+    // (the general machine model, R42, runs in every layout but lean)
+    const bool t32 = (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
     q.t32 = t32;
     const bool wide = R.n >= kWideN && R.n <= 1024;
     q.wide = wide;
@@ -1355,8 +1353,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   {
     uint32_t fused_ants = 512;
     if (const char *e = getenv("ACO_FUSED_ANTS")) fused_ants = (uint32_t)atoi(e);
-    bool ok = !colony && p->rl_limit == 0 && count > 0 && A <= 512 && (uint64_t)count * A <= fused_ants &&
-              ctx->mach.issue_width <= 1 && !P.nc4;
+    bool ok = !colony && p->rl_limit == 0 && count > 0 && A <= 512 && (uint64_t)count * A <= fused_ants && !P.nc4;
     uint32_t smem = 0;
     for (uint32_t r = 0; r < count && ok; ++r) {
       const RegionDev &R = ctx->regions[r];

@@ -913,7 +913,7 @@ __device__ __forceinline__ AntOut ant_pass1(const SV &V, const uint16_t *__restr
 // ILP pass (L108, L118, L147-L164, L200-L206; R19-R24).  t is the cycle;
 // stalls skip ahead without drawing.  rec_o / rec_c (leader, may be NULL)
 // receive the order and the cycles.  Valid in the leader lane.
-// General machine model (L64; R42, T32 variants only): the ant stays in
+// General machine model (L64; R42; not the lean layout): the ant stays in
 // cycle t until issue_width instructions were placed; a latency-met
 // instruction whose slot (width / type) is full counts as semi-ready with
 // ready time t + 1; the Philox step is t * issue_width + used.
@@ -936,8 +936,10 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   constexpr bool wide = WIDE;  // 4-wide scan (word mask or strided words)
   constexpr bool CT = !T32 && !NC4;  // compact layout (x_get)
   // general machine model (R42): runtime, only in the u32-cycle variants
-  const uint32_t w = T32 ? c_mach[cfg.mslot].issue_width : 1u;
-  const bool mi = T32 && w > 1u;
+  // (every layout but lean: the lean ready-time slots assume a placement
+  // ends its cycle, so lean is planned for single issue only)
+  const uint32_t w = LEAN ? 1u : c_mach[cfg.mslot].issue_width;
+  const bool mi = w > 1u;
   const uint32_t slots = c_mach[cfg.mslot].type_slots;  // u8 x 4
   uint32_t used = 0, used_t = 0;              // placed in cycle t: total, per type (u8 x 4)
   uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0, B = 0;
