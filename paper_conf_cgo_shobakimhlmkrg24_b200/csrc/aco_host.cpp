@@ -773,7 +773,8 @@ uint32_t lane_pow2(uint32_t words) {
 
 Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bool allow_ts, bool lanes14,
                  uint32_t target_threads, uint32_t max_lanes, uint32_t A, uint32_t gsz, uint32_t coin_w,
-                 bool allow_ig = false, uint32_t apb_mult = 1, uint32_t spread_cap = 0, uint32_t lane_pref = 1) {
+                 bool allow_ig = false, uint32_t apb_mult = 1, uint32_t spread_cap = 0, uint32_t lane_pref = 1,
+                 uint32_t max_block = kMaxBlockThreads) {
   Shape bests[2] = {Shape{0, 1, 0, false}, Shape{0, 1, 0, false}};
   for (int ig = 0; ig <= (allow_ig ? 1 : 0); ++ig) {
   Shape &best = bests[ig];
@@ -789,7 +790,7 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
         continue;
       }
       for (uint32_t threads : {32u, 64u, 96u, 128u, 192u, 256u, 384u, 512u}) {
-        if (threads > kMaxBlockThreads) break;
+        if (threads > max_block) break;  // (the kernel's launch bound)
         const uint32_t apb = threads / L;
         if (apb % apb_mult) continue;  // R45: whole ant groups per block
         if (spread_cap && apb > std::max(spread_cap, 32u / L)) break;
@@ -1030,7 +1031,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       const uint32_t Wl = ant_words(1, R.n, R.nwr, R.nremw, false, P.nc4, true);
       const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[0][2], false, false, tgt_threads[0], 1, A,
                                    p->group_size, coin_words(1, R.n) + (rl1 ? 6u : 0u), img_l1[0] != 0,
-                                   rl1 ? p->group_size : 1u, rl1 ? 0u : spread, 1u);
+                                   rl1 ? p->group_size : 1u, rl1 ? 0u : spread, 1u, kLeanMaxThreads);
       const uint64_t base_ants = sh.apb ? sh.resident / sh.lanes : 0;
       if (shl.apb && 100ull * shl.resident >= (100ull + lean1_gain) * base_ants) {
         sh = shl;
@@ -1046,7 +1047,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // ACO_LEAN_GAIN = 20 / 50 %: 654 ms)
       const uint32_t Wl = ant_words(pass, R.n, R.nwr, R.nremw, false, P.nc4, true, R.nslot);
       const Shape shl = pick_shape(R.img.bytes, tau_smem_bytes(R.n), Wl, mt[1][2], false, false, tgt_threads[1], 1, A,
-                                   p->group_size, coin_words(pass, R.n), img_l1[1] != 0, 1u, spread, 1u);
+                                   p->group_size, coin_words(pass, R.n), img_l1[1] != 0, 1u, spread, 1u, kLeanMaxThreads);
       if (shl.apb && 100ull * shl.resident >= (100ull + lean_gain) * sh.resident) {
         sh = shl;
         W = Wl;

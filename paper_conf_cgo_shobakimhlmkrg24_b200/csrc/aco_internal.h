@@ -24,6 +24,13 @@ constexpr uint32_t kMaxKernelInsts = 8191;  // ids use 13 bits in successor entr
 constexpr uint32_t kFlagLiveIn = 1, kFlagLiveOut = 2;
 constexpr uint32_t kSmemPerSM = 227 * 1024;  // max dynamic shared memory per block
 constexpr uint32_t kMaxBlockThreads = 512;   // construct blocks (launch bounds)
+// Lean variants: a 384-thread launch bound leaves the compiler up to 170
+// registers (it takes ~150; at 512 it was capped at 128): measured (r02q) C3
+// 692 -> 684 ms.  The planner caps lean blocks at this size.
+#ifndef ACO_LEAN_LB
+#define ACO_LEAN_LB 384
+#endif
+constexpr uint32_t kLeanMaxThreads = ACO_LEAN_LB;
 // Regions with at least this many instructions use the 4-wide candidate scan
 // (latency-bound: few ants fit an SM); smaller ones the 1-wide scan (issue-bound).
 constexpr uint32_t kWideN = 160;

@@ -41,9 +41,6 @@
 #ifndef ACO_PREFETCH
 #define ACO_PREFETCH 0
 #endif
-#ifndef ACO_LEAN_LB  // launch bound of the lean pass-2 variants (caps registers: 65536 / bound per thread)
-#define ACO_LEAN_LB 512
-#endif
 #ifndef ACO_BRANCHLESS1  // pass-1 4-wide evaluation without branches (measured faster)
 #define ACO_BRANCHLESS1 1
 #endif
@@ -1208,7 +1205,10 @@ __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t byt
 // staged) in shared memory: more ants resident per SM.
 // LEAN: pass-2 lean per-ant layout (u8 ready times, dynamic kills).
 template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS, bool WIDE, bool LEAN = false>
-__global__ void __launch_bounds__(LEAN ? ACO_LEAN_LB : kMaxBlockThreads, (WIDE && GS != 1) ? 1 : 2)
+#ifndef ACO_NARROW_MINB  // min blocks per SM of the 1-wide variants (2: <= 64 registers)
+#define ACO_NARROW_MINB 2
+#endif
+__global__ void __launch_bounds__(LEAN ? kLeanMaxThreads : kMaxBlockThreads, (WIDE && GS != 1) ? 1 : ACO_NARROW_MINB)
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
