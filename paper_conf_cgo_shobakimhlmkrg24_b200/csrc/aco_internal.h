@@ -33,7 +33,10 @@ constexpr uint32_t kMaxBlockThreads = 512;   // construct blocks (launch bounds)
 constexpr uint32_t kLeanMaxThreads = ACO_LEAN_LB;
 // Regions with at least this many instructions use the 4-wide candidate scan
 // (latency-bound: few ants fit an SM); smaller ones the 1-wide scan (issue-bound).
-constexpr uint32_t kWideN = 160;
+#ifndef ACO_WIDE_N
+#define ACO_WIDE_N 160
+#endif
+constexpr uint32_t kWideN = ACO_WIDE_N;
 
 // Successor entry: v (13 bits) | single-predecessor flag << 13 | latency << 16.
 constexpr uint32_t kSuccSingle = 1u << 13;
