@@ -915,6 +915,12 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     if (on) spread_cap = (uint32_t)std::max<uint64_t>(1, (total + 147) / 148);
     if (const char *e = getenv("ACO_SPREAD_CAP")) spread_cap = on ? (uint32_t)atoi(e) : 0u;
   }
+  // regions with at least this many instructions take the 4-wide candidate
+  // scan (and, in pass 2, the lean layout), per pass.  Measured (r02s, ns per
+  // ant-step at n = 130): pass 1 0.052 (1-wide) vs 0.056 (4-wide); pass 2
+  // 0.077 vs 0.066
+  uint32_t wide_n[2] = {kWideN, 120};
+  if (const char *e = getenv("ACO_WIDE_N")) sscanf(e, "%u,%u", &wide_n[0], &wide_n[1]);
   bool fill_sms = true;  // spread passes with fewer shared-memory blocks than SMs (below)
   if (const char *e = getenv("ACO_FILL")) fill_sms = atoi(e) != 0;
   uint32_t fill_img_max = 64 * 1024;
@@ -977,7 +983,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       const bool t32 = (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
       for (uint32_t pass = 1; pass <= 2; ++pass) {
         if (!(pmask & pass)) continue;
-        const bool wide = R.n >= kWideN && R.n <= 1024, rare = pass == 2 && (t32 || P.nc4);
+        const bool wide = R.n >= wide_n[pass - 1] && R.n <= 1024, rare = pass == 2 && (t32 || P.nc4);
         const uint32_t W = ant_words(pass, R.n, R.nwr, R.nremw, pass == 2 && t32, P.nc4);
         const Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                                     pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1],
@@ -1009,7 +1015,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // (the general machine model, R42, runs in every layout but lean)
     const bool t32 = (P.nc4 ? R.max_cycle_bound > 65535u : (R.max_lat > 511u || R.mc_max > 7u));
     q.t32 = t32;
-    const bool wide = R.n >= kWideN && R.n <= 1024;
+    const bool wide = R.n >= wide_n[pass - 1] && R.n <= 1024;
     q.wide = wide;
     // lean pass-2 layout (u8 ready times, kills derived at evaluation):
     // large regions, single issue, 2 classes, latencies < 128
