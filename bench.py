@@ -524,6 +524,7 @@ def main(argv=None):
     if rank == 0:
         peaks = measured_peaks()
         cpu, bpas, parity = None, None, None
+        step_ratio = 1.0
         n_cmp, n_ok, bad, log = 0, 0, [], []
 
         def check(rid, n, gdig, ora):
@@ -541,12 +542,15 @@ def main(argv=None):
             # the oracle on a stratified sample (per batch; c5 has two), on all host threads
             share = max(4, args.cpu_sample if args.workload != "c5" else 24)
             parts, stats_all, secs, scheds_cpu = [], [], 0.0, 0.0
+            nominal_steps = 0.0  # A x n x iterations of the sample (what A x n per pass-iteration counts)
             for s, b in zip(scheds, batches):
                 ps, note = cpu_sample_params(args, b.p)
                 k = share if len(batches) == 1 else max(2, share // len(batches))
                 base, stats, pick, ores, dt, sc = cpu_baseline(b.regs, b.ids, ps, k, machine, note)
                 parts.append(base)
                 stats_all.append(stats)
+                nominal_steps += sum(ps.ants * b.regs[i].n_insts * (ores[q]["iters1"] + ores[q]["iters2"])
+                                     for q, i in enumerate(pick))
                 secs += dt
                 scheds_cpu += sc
                 if args.parity == "off":
@@ -565,6 +569,9 @@ def main(argv=None):
             if len(parts) > 1:
                 cpu["sample"] = " + ".join(x["sample"] for x in parts)
             bpas = bytes_per_ant_step(np.concatenate(stats_all))
+            from oracle.pyoracle import ORS
+            placed = float(np.concatenate(stats_all)[:, ORS["placements"]].sum())
+            step_ratio = placed / max(1.0, nominal_steps)  # < 1: pass-2 ants that die early
         if args.parity != "off" and (n_cmp == 0 or args.parity == "all") and args.workload not in ("c4", "c5"):
             # the oracle with the run's own parameters on a small stratified
             # sample (N > 1: every rank's results gathered to rank 0), or on
@@ -600,8 +607,13 @@ def main(argv=None):
         # over the construct launches' CUDA-event time; peak = the SM shared
         # memory crossbar, 148 SMs x 128 B/clk x the SM clock seen under load.
         construct_ms = phase_ms[0] / max(1, args.steps)
-        ant_steps = sum(b.p.ants * sum(r.n_insts * (res[i]["iters1"] + res[i]["iters2"])
-                                       for r, i in zip(b.regs, b.ids)) for b in batches)
+        # ant-steps the method performs: A x n per region and pass-iteration,
+        # scaled by the oracle sample's placements / (A x n x iterations)
+        # (an ant that dies in pass 2 stops early; the GPU's prune is not
+        # counted as work the method must do, nor subtracted)
+        ant_steps_nominal = sum(b.p.ants * sum(r.n_insts * (res[i]["iters1"] + res[i]["iters2"])
+                                               for r, i in zip(b.regs, b.ids)) for b in batches)
+        ant_steps = int(round(ant_steps_nominal * step_ratio))
         sm_mhz = clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
         smem_peak = 148 * 128 * sm_mhz * 1e6 / 1e9  # GB/s
         roof = None
@@ -614,7 +626,9 @@ def main(argv=None):
                     "traffic_source": tsrc, "issue_slots_ncu": issue,
                     "algorithmic_bytes_per_launch": round(bpas * ant_steps / max(1.0, n_launch)),
                     "kernel": "k_construct (all classes)", "bytes_per_ant_step": round(bpas, 2),
-                    "ant_steps_per_step": ant_steps, "launches_per_step": n_launch,
+                    "ant_steps_per_step": ant_steps, "ant_steps_nominal": ant_steps_nominal,
+                    "ant_steps_source": f"A x n x iterations scaled by the oracle sample's placements ratio "
+                                        f"{step_ratio:.4f}", "launches_per_step": n_launch,
                     "construct_ms_per_step": round(construct_ms, 3),
                     "ant_steps_per_s": round(ant_steps / (construct_ms / 1000.0), 1),
                     "peak_source": f"guide: 148 SM x 128 B/clk x {sm_mhz:.0f} MHz (smem crossbar, no measured peak)"}
