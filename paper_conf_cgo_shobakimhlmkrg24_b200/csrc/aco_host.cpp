@@ -944,6 +944,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_LEAN1_GAIN")) lean1_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
+  bool huge_smem = true;  // huge regions: per-ant state in shared memory when all ants fit (ACO_HUGE_SMEM)
+  if (const char *e = getenv("ACO_HUGE_SMEM")) huge_smem = atoi(e) != 0;
   uint32_t gs_wide[2] = {1, 1};  // 4-wide scan in the global-state kernels, per pass
   if (const char *e = getenv("ACO_GS_WIDE")) {
     if (sscanf(e, "%u,%u", &gs_wide[0], &gs_wide[1]) == 1) gs_wide[1] = gs_wide[0];
@@ -975,8 +977,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // ants -> 16 lanes), fewer when many do (config 5: every n >= ~1,500 region
   // -> 4 lanes): ~148 x 1,024 threads in flight.  Measured (ms): C4 16/8/4
   // lanes 423/583/827, C5 2,961/2,529/2,328.
-  if (!gs_lanes_env) {
-    uint64_t gs_ants[2] = {0, 0};
+  uint64_t gs_ants[2] = {0, 0};  // ants of the regions that leave the shared-memory kernels, per pass
+  {
     for (uint32_t r = 0; r < count; ++r) {
       const RegionDev &R = ctx->regions[r];
       if (R.n <= 600) continue;  // (host time: smaller regions always fit shared memory)
@@ -991,7 +993,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         if (sh.apb == 0 || sh.resident < gs_min_threads[pass - 1]) gs_ants[pass - 1] += A;
       }
     }
-    for (int q = 0; q < 2; ++q) {
+    for (int q = 0; q < 2 && !gs_lanes_env; ++q) {
       const uint64_t per = gs_ants[q] ? (148ull * 1024) / gs_ants[q] : 16;
       gs_lanes[q] = per >= 16 ? 16u : (per >= 8 ? 8u : 4u);
     }
@@ -1002,7 +1004,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // given lanes per ant, 0 = off).
   struct RegionPlan {
     Shape sh;
-    bool g = false, lean = false, t32 = false, wide = false, on = false;
+    bool g = false, lean = false, t32 = false, wide = false, on = false, huge = false;
     uint32_t W = 0;
   };
   auto plan_region = [&](uint32_t r, uint32_t pass, uint32_t spread, uint32_t lane_pref) {
@@ -1067,6 +1069,34 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
     // (not for a spread shape: there few resident ants per SM is the point)
     if (sh.apb != 0 && !spread && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
+    if (sh.apb == 0 && huge_smem && R.n > 1024 && !t32 && !P.nc4 && !(rl1 && pass == 1)) {
+      // Huge regions with the per-ant state in SHARED memory, the image and
+      // tau through L1, the global-state lane count and the 4-wide strided
+      // scan; pass 2 in the lean layout when its latencies allow -- taken
+      // when every ant of the path stays resident (one wave), else the
+      // global-state kernels below
+      const uint32_t gl = gs_lanes[pass - 1];
+      const bool hl = pass == 2 && lean_on && R.max_lat < 128u && ctx->mach.issue_width <= 1;
+      const uint32_t Wh = hl ? ant_words(2, R.n, R.nwr, R.nremw, false, false, true, R.nslot)
+                             : ant_words(pass, R.n, R.nwr, R.nremw, false, false);
+      const uint32_t maxb = kMaxBlockThreads;  // (huge variants: 512-thread bound, 2 blocks per SM)
+      const uint64_t need = std::max<uint64_t>(1, gs_ants[pass - 1]);
+      for (uint32_t apb : {32u, 16u, 8u, 4u, 2u}) {
+        const uint32_t thr = apb * gl;
+        if (thr > maxb || thr < 32 || thr % 32) continue;
+        const uint64_t bytes = (uint64_t)ant_stride(apb, gl) * Wh * 4 +
+                               (uint64_t)coin_groups(apb, p->group_size) * coin_words(pass, R.n) * 4;
+        if (bytes > kSmemPerSM) continue;
+        uint32_t k = std::min<uint32_t>(kSmemSM / ((uint32_t)bytes + kBlockReserve), 2u);  // (launch bound: 2 per SM)
+        while (k && smem_for_k(k) < bytes) --k;
+        if (!k || 148ull * k * apb < need) continue;
+        sh = Shape{apb, gl, smem_for_k(k), false, k * thr, true};
+        q.huge = true;
+        lean = hl;
+        W = Wh;
+        break;
+      }
+    }
     if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
       // all ants are resident (state in the workspace); 16 lanes per ant
       // and 512-thread blocks measured best (tools/probe_gs_lanes.sh:
@@ -1151,7 +1181,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // global-state kernels: 4-wide candidate scan over strided words (not in
       // the u32-cycle / 3-4 class instantiations), gs_wide_lanes above
       const bool gwide = g && gs_wide[pass - 1] && sh.lanes <= gs_wide_lanes[pass - 1] && !(pass == 2 && (t32 || P.nc4));
-      const bool wk = (wide && mask) || gwide;
+      const bool wk = (wide && mask) || gwide || q.huge;
       const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];
       c.wide = wk;

@@ -307,7 +307,7 @@ inline uint32_t class_variant(uint32_t pass, const ClassLaunch &c) {
   const bool mask = c.max_n <= 1024 && !c.gs;
   const bool rare = pass == 2 && (c.t32 || c.nc4) && !c.gs;
   return variant_code(pass, c.lanes, mask, c.tau_smem && !rare && !c.gs, pass == 2 && c.t32, pass == 2 && c.nc4,
-                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && (mask || c.gs), c.lean);
+                      c.gs ? 1 : (c.img_l1 ? 2 : 0), c.wide && (mask || c.gs || c.img_l1), c.lean);
 }
 
 int set_machine(uint32_t slot, const MachineDev &m);  // cudaMemcpyToSymbol into slot; 0 on success

@@ -1208,7 +1208,10 @@ template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS
 #ifndef ACO_NARROW_MINB  // min blocks per SM of the 1-wide variants (2: <= 64 registers)
 #define ACO_NARROW_MINB 2
 #endif
-__global__ void __launch_bounds__(LEAN ? kLeanMaxThreads : kMaxBlockThreads, (WIDE && GS != 1) ? 1 : ACO_NARROW_MINB)
+// (huge regions with shared-memory state, !MASK && GS == 2: two blocks per SM,
+// every ant of config 4 resident)
+__global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockThreads,
+                                  (WIDE && GS != 1) ? ((MASK || GS != 2) ? 1 : 2) : ACO_NARROW_MINB)
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
@@ -1961,6 +1964,12 @@ static void reg_rare(F &f) {  // pass 2 with u32 cycles and/or 3-4 classes: tau 
   reg_w<2, LG, M, false, false, true>(f);
   reg_w<2, LG, M, false, true, true>(f);
 }
+template <int LG, typename F>
+static void reg_huge(F &f) {
+  reg1<1, LG, false, false, false, false, 2, true>(f);
+  reg1<2, LG, false, false, false, false, 2, true>(f);
+  reg1<2, LG, false, false, false, false, 2, true, F, true>(f);
+}
 template <typename F>
 static void for_each_construct(F &&f) {
   reg_lg<1>(f);
@@ -1988,6 +1997,11 @@ static void for_each_construct(F &&f) {
   reg1<2, 4, false, false, true, false, 1, false>(f);
   reg1<2, 4, false, false, false, true, 1, false>(f);
   reg1<2, 4, false, false, true, true, 1, false>(f);
+  // huge regions with the per-ant state in shared memory, image and tau
+  // through L1 (GS = 2, no word mask), 4-wide strided scan; pass 2 compact or lean
+  reg_huge<4>(f);
+  reg_huge<8>(f);
+  reg_huge<16>(f);
 }
 
 static ConstructFn g_construct[8192];

@@ -29,6 +29,7 @@ def test_global_state_lanes_every_ant(torch_cuda, monkeypatch, lanes):
     per ant, both passes, every ant bit-exact (config 5 runs the 4-lane and
     config 4 the 16-lane instantiation)."""
     monkeypatch.setenv("ACO_GS_LANES", f"{lanes},{lanes}")
+    monkeypatch.setenv("ACO_HUGE_SMEM", "0")  # (the global-state kernels, not the shared-memory huge path)
     regs = [I.gen_region(n, 9100 + n + lanes) for n in (1100, 1700)]
     ids = [31, 32]
     p = I.Params(ants=48, iterations=2, seed=70 + lanes, stall_mod=2)
@@ -36,6 +37,22 @@ def test_global_state_lanes_every_ant(torch_cuda, monkeypatch, lanes):
     s.load(regs, ids).run(p, no_prune=True, dump=True)
     codes = s.variants()
     assert any(c & 2 for c in codes), codes  # the global-state kernels ran
+    dump_parity(s, regs, ids, p)
+
+
+@pytest.mark.parametrize("lanes", [4, 8, 16])
+def test_huge_shared_state_every_ant(torch_cuda, monkeypatch, lanes):
+    """Huge regions (n > 1024) whose ants all fit with their state in shared
+    memory (image and tau through L1, 4-wide strided scan, lean pass 2):
+    every ant bit-exact at 4, 8 and 16 lanes per ant (config 4 runs 16)."""
+    monkeypatch.setenv("ACO_GS_LANES", f"{lanes},{lanes}")
+    regs = [I.gen_region(n, 9200 + n + lanes) for n in (1100, 1900)]
+    ids = [35, 36]
+    p = I.Params(ants=64, iterations=2, seed=90 + lanes, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    codes = s.variants()
+    assert any((c & (1 << 11)) and not (c & (1 << 5)) for c in codes), codes  # the huge shared-state kernels ran
     dump_parity(s, regs, ids, p)
 
 
