@@ -944,7 +944,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_LEAN1_GAIN")) lean1_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
-  bool huge_smem = true;  // huge regions: per-ant state in shared memory when all ants fit (ACO_HUGE_SMEM)
+  // huge regions: per-ant state in shared memory when all ants fit -- off:
+  // measured slower (r02u: C4 832 -> 1098 ms; the two 113 KB blocks per SM
+  // leave L1 ~28 KB for the image and tau the global-state kernels cache in
+  // the full 256 KB, and the 64-register bound spills); ACO_HUGE_SMEM=1
+  bool huge_smem = false;
   if (const char *e = getenv("ACO_HUGE_SMEM")) huge_smem = atoi(e) != 0;
   uint32_t gs_wide[2] = {1, 1};  // 4-wide scan in the global-state kernels, per pass
   if (const char *e = getenv("ACO_GS_WIDE")) {
