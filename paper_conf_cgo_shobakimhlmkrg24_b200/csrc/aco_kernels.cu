@@ -1776,11 +1776,15 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
   const RegionWs &W = A.rws[r];
-  RegionState &rs = A.state[r];
+  // the region state lives in shared memory for the whole run (its serial
+  // epilogue updates stay on chip) and is written back at the end
+  __shared__ RegionState srs;
+  RegionState &rs = srs;
   extern __shared__ uint4 smem4[];
   unsigned char *smem = (unsigned char *)smem4;
   __shared__ uint32_t s_prp[3], s_flag, s_active;
   const uint32_t n = rd->n, na = A.cfg.ants, tid = threadIdx.x;
+  for (uint32_t i = tid; i < sizeof(RegionState) / 4; i += blockDim.x) ((uint32_t *)&srs)[i] = 0;
   const FusedLayout F = fused_layout(n, rd->nwr, rd->nremw, rd->img.bytes, na, A.cfg.group_size);
   stage(smem4, (const uint4 *)(A.arena + rd->o_image), rd->img.bytes);
   const unsigned char *img = smem;
@@ -1901,6 +1905,9 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   for (uint32_t i = tid; i < n; i += blockDim.x) rec_c[i] = 0;  // (k_post)
   __syncthreads();
   if (tid == 0) post_body(A, rd, W, rs, img, rec_c);
+  __syncthreads();
+  for (uint32_t i = tid; i < sizeof(RegionState) / 4; i += blockDim.x)
+    ((uint32_t *)(A.state + r))[i] = ((const uint32_t *)&srs)[i];
 }
 
 // ------------------------------------------------------------ launchers
