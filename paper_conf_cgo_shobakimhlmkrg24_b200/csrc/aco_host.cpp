@@ -744,6 +744,7 @@ struct Shape {
   bool ts;
   uint32_t resident = 0;  // resident threads per SM of this shape
   bool ig = false;        // image read through L1 instead of staged in shared memory
+  uint32_t need = 0;      // dynamic shared memory the block actually needs (bytes, 128-aligned)
 };
 
 // Shared memory per SM and per-block reservation (sm_100: 228 KB per SM,
@@ -809,7 +810,7 @@ Shape pick_shape(uint32_t img, uint32_t tb, uint32_t W, uint32_t max_threads, bo
         if (spread_cap) score = ((uint64_t)(ts ? 1 : 0) << 40) | ((uint64_t)apb << 20) | (uint64_t)(4095 - k);
         if (score > best_score) {  // strict: the staged image wins ties
           best_score = score;
-          best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads, ig != 0};
+          best = Shape{apb, L, smem_for_k(k), ts != 0, k * threads, ig != 0, ((uint32_t)bytes + 127u) & ~127u};
         }
       }
     }
@@ -921,6 +922,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // 0.077 vs 0.066
   uint32_t wide_n[2] = {kWideN, 120};
   if (const char *e = getenv("ACO_WIDE_N")) sscanf(e, "%u,%u", &wide_n[0], &wide_n[1]);
+  bool smem_exact = true;  // classes reserve the shared memory they need (ACO_SMEM_EXACT)
+  if (const char *e = getenv("ACO_SMEM_EXACT")) smem_exact = atoi(e) != 0;
   bool fill_sms = true;  // spread passes with fewer shared-memory blocks than SMs (below)
   if (const char *e = getenv("ACO_FILL")) fill_sms = atoi(e) != 0;
   uint32_t fill_img_max = 64 * 1024;
@@ -1194,7 +1197,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       c.t32 = pass == 2 && t32;
       c.gs = g;
       c.lean = lean;
-      c.smem = std::max(c.smem, sh.smem);
+      // a class reserves what its largest block needs, not 1/k of the SM:
+      // the unreserved shared memory becomes L1 (the driver picks the
+      // smallest carveout that holds the resident blocks), which caches the
+      // image and tau of the image-through-L1 and global-tau classes
+      c.smem = std::max(c.smem, smem_exact && sh.need ? sh.need : sh.smem);
       c.regs.push_back({~(uint64_t)((uint64_t)R.n * (R.n + 16)), r});
     }
     P.p2_smem = std::max(P.p2_smem, 4 * R.n + 16);  // also k_post

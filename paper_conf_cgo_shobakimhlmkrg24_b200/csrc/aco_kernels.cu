@@ -1295,7 +1295,7 @@ __global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockTh
   const bool pf = !TAU_SMEM && (A.cfg.tau_prefetch & (1u << (PASS - 1 + (GS == 1 ? 2 : 0))));
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
-  if (PASS == 1) {
+  if constexpr (PASS == 1) {
     uint16_t *rec = nullptr;
     uint32_t rs1 = 1;
     if (dump && A.dump_order) {
@@ -1690,7 +1690,7 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
     const St S = make_st<PASS, T32, NC4>(stw, 1, V);
     const Grp<32> G32(threadIdx.x);
     AntOut o;
-    if (PASS == 1) {
+    if constexpr (PASS == 1) {
       RL rl{nullptr, 0, 0, A.cfg.rl_limit, nullptr, nullptr};
       if (A.cfg.rl_limit)  // R45: the winner's group limits as recorded by the construct kernel
         rl.in = (const uint16_t *)(A.ws + W.o_rlk) + (size_t)((want - A.cfg.ant_base) / A.cfg.group_size) * n;
