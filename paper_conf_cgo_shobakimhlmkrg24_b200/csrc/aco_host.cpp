@@ -1475,6 +1475,8 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_GS_LAYOUT")) cfg.gs_ant_major = atoi(e) != 0;
   cfg.lazy_kills = 1;  // measured (r02j): C3 702 -> 695 ms, C5 and n = 200/450 neutral to -4 %
   if (const char *e = getenv("ACO_LAZY_KILLS")) cfg.lazy_kills = atoi(e) != 0;
+  cfg.prune_cp = 0;
+  if (const char *e = getenv("ACO_PRUNE_CP")) cfg.prune_cp = atoi(e) != 0;
   cfg.tau_prefetch = 0;
   if (const char *e = getenv("ACO_TAU_PREFETCH")) cfg.tau_prefetch = (uint32_t)strtoul(e, nullptr, 0);
   cfg.record = P.record ? 1u : 0u;

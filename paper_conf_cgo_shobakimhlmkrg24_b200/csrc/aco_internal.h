@@ -159,7 +159,7 @@ struct RunCfg {
   uint32_t gs_ant_major;  // global-state kernels: per-ant state ant-major (1) or [word][ant] (0)
   uint32_t lazy_kills;    // lean pass 2: derive kills only for candidates where they decide
   uint32_t tau_prefetch;  // L1 prefetch of the next tau row: bit (pass-1) for smem-state kernels, bit 2 + (pass-1) for GS
-  uint32_t pad_cfg3;
+  uint32_t prune_cp;      // R24 prune also with the critical-path bound of the scanned candidates
   uint64_t dump_slice;  // elements per (pass, iter) order slice = ants * sum n
   int64_t *keys;        // shared colony: per-region biased winner keys (NULL: local argmin)
 };

@@ -135,7 +135,7 @@ struct SV {
   const uint32_t *muse, *mk, *cu_ptr, *cu, *succ_ptr, *succ, *pred_ptr, *pred, *rb0, *rem0, *pg_ptr;
   const uint2 *pg;
   const uint16_t *eta1, *eta2;
-  uint32_t n, nwr, nremw, region_id, L1, nslot;
+  uint32_t n, nwr, nremw, region_id, L1, nslot, cpmax;
   uint32_t livein01, livein23;  // u16 x 2
 };
 
@@ -161,6 +161,7 @@ __device__ __forceinline__ SV make_sv(const unsigned char *img, const RegionDev 
   V.nwr = rd->nwr;
   V.nremw = rd->nremw;
   V.nslot = rd->nslot;
+  V.cpmax = rd->cp_max;
   V.region_id = rd->region_id;
   V.L1 = rd->L + 1;
   V.livein01 = (rd->livein[0] & 0xFFFFu) | (rd->livein[1] << 16);
@@ -370,6 +371,11 @@ struct Grp {
   __device__ __forceinline__ uint32_t sum(uint32_t v) const {
 #pragma unroll
     for (int o = LG / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, LG);
+    return v;
+  }
+  __device__ __forceinline__ uint32_t max(uint32_t v) const {
+#pragma unroll
+    for (int o = LG / 2; o > 0; o >>= 1) v = ::max(v, __shfl_xor_sync(mask, v, o, LG));
     return v;
   }
   __device__ __forceinline__ uint32_t min(uint32_t v) const {
@@ -957,6 +963,15 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     }
   };
   auto lean_rd = [&](uint32_t dsz) -> uint32_t { return B + r8_get(A, dsz >> 16); };
+  // R24 with a critical-path bound: an unplaced instruction j with ready time
+  // rd is issued at >= max(rd, t) and its longest successor chain needs CP(j)
+  // more cycles, so length >= max(rd, t) + CP(j) + 1.  CP(j) >= the floor of
+  // (eta2(j) - 1) CPmax / 65534 (eta2 = 1 + floor(CP 65534 / CPmax), R4).
+  const bool pcp = prune && cfg.prune_cp;
+  uint32_t cp_run = 0;
+  auto cp_floor = [&](uint32_t dsz) -> uint32_t {
+    return (uint32_t)(((uint64_t)((dsz & 0xFFFFu) - 1u) * V.cpmax) / 65534u);
+  };
   const bool lazy = LEAN && cfg.lazy_kills && !stall_en && !mix;  // (lean: kills only where they decide)
   // heuristic of a feasible candidate: eta2 (CP), or eta1 (LUC, CP) for mixed odd groups
   auto eta_of = [&](uint32_t j, uint32_t e2, uint32_t dk) -> uint32_t {
@@ -979,7 +994,8 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
       uint32_t bl = 0;
       if (G.leader()) bl = *(volatile uint32_t *)prune_len;
       bl = G.bcast(bl);
-      const uint32_t lbf = mi ? t + (n - placed + used + w - 1) / w : t + (n - placed);
+      uint32_t lbf = mi ? t + (n - placed + used + w - 1) / w : t + (n - placed);
+      if (pcp) lbf = ::max(lbf, G.max(cp_run) + 1u);
       if (lbf > bl) {
         if (G.leader()) atomicAdd(prune_len + 1, 1u);  // RegionState::pruned follows prune_len
         o.cost = kInvalid;
@@ -1007,6 +1023,7 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
     auto eval = [&](uint32_t j, uint32_t rdy, const uint4 &ds, uint32_t dk, uint32_t tv) {
       const uint32_t K = ds.y + dk;                   // kills per class (R14)
       const bool lat_ok = rdy <= t;
+      if (pcp) cp_run = ::max(cp_run, ::max(rdy, t) + cp_floor(ds.z));
       if (lat_ok && (!mi || ((avail >> (8 * (ds.w & 0xFu))) & 1u))) {
         counts += 1u;
         // feasible: defs_c <= slack_c + kills_c in every class (R21)
