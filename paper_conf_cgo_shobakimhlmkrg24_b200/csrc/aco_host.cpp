@@ -947,6 +947,16 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   if (const char *e = getenv("ACO_LEAN1_GAIN")) lean1_gain = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_LEAN_GAIN")) lean_gain = (uint32_t)atoi(e);
   const bool gs_lanes_env = getenv("ACO_GS_LANES") != nullptr;
+  // lane-per-instruction ants (one warp per ant, its state in registers;
+  // aco_kernels.cu lpi_pass1/2) for regions of <= 128 instructions when the
+  // whole batch has few ants, i.e. the per-ant step latency -- not issue
+  // slots -- bounds the run (config 2: one region of 1,024 ants).
+  // ACO_LPI: 0 off, 1 auto (default), 2 every eligible region (tests)
+  uint32_t lpi_mode = 1;
+  if (const char *e = getenv("ACO_LPI")) lpi_mode = (uint32_t)atoi(e);
+  uint64_t lpi_max_ants = 148ull * 16;  // ants (= warps) in the whole batch
+  if (const char *e = getenv("ACO_LPI_ANTS")) lpi_max_ants = strtoull(e, nullptr, 10);
+  const bool lpi_batch = lpi_mode == 2 || (lpi_mode == 1 && (uint64_t)A * count <= lpi_max_ants);
   // huge regions: per-ant state in shared memory when all ants fit -- off:
   // measured slower (r02u: C4 832 -> 1098 ms; the two 113 KB blocks per SM
   // leave L1 ~28 KB for the image and tau the global-state kernels cache in
@@ -1011,7 +1021,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // given lanes per ant, 0 = off).
   struct RegionPlan {
     Shape sh;
-    bool g = false, lean = false, t32 = false, wide = false, on = false, huge = false;
+    bool g = false, lean = false, t32 = false, wide = false, on = false, huge = false, lpi = false;
     uint32_t W = 0;
   };
   auto plan_region = [&](uint32_t r, uint32_t pass, uint32_t spread, uint32_t lane_pref) {
@@ -1033,6 +1043,29 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     if (getenv("ACO_DEBUG_REGIONS"))
       fprintf(stderr, "[aco region] %u n %u pass %u img %u words %u nremw %u L %u\n", r, R.n, pass, R.img.bytes, W,
               R.nremw, R.L);
+    if (lpi_batch && R.n >= 1 && R.n <= 128 && !P.nc4 && !p->heur_mix && !(rl1 && pass == 1) &&
+        (pass == 1 || (ctx->mach.issue_width <= 1 && (uint64_t)R.max_cycle_bound + R.max_lat < 65536u))) {
+      // (pass 2: single issue; ready times are u16 pairs in registers)
+      // one warp per ant: ~148 blocks over the batch's ants (<= 8 warps each)
+      const uint64_t tot = (uint64_t)A * count;
+      uint32_t apb = (uint32_t)std::min<uint64_t>(kLpiMaxThreads / 32, std::max<uint64_t>(1, (tot + 147) / 148));
+      apb = std::min(apb, std::max(1u, A));
+      const uint64_t fixed = (uint64_t)ant_stride(apb, 32) * lpi_words(R.nremw) * 4 +
+                             (uint64_t)coin_groups(apb, p->group_size) * coin_words(pass, R.n) * 4 + R.img.bytes;
+      const bool ts = fixed + tau_smem_bytes(R.n) <= kSmemPerSM;
+      const uint64_t bytes = fixed + (ts ? tau_smem_bytes(R.n) : 0u);
+      if (bytes <= kSmemPerSM) {
+        uint32_t k = std::min<uint32_t>(kSmemSM / ((uint32_t)bytes + kBlockReserve), 64u / apb);
+        k = std::max(1u, std::min(k, 32u));
+        while (k > 1 && smem_for_k(k) < bytes) --k;
+        q.sh = Shape{apb, 32, smem_for_k(k), ts, k * apb * 32, false, ((uint32_t)bytes + 127u) & ~127u};
+        q.lpi = true;
+        q.W = lpi_words(R.nremw);
+        q.wide = false;
+        q.on = true;
+        return q;
+      }
+    }
     const bool rare = pass == 2 && (t32 || P.nc4);  // variants compiled without tau staging, 1|4 lanes
     Shape sh = pick_shape(R.img.bytes, tau_smem_bytes(R.n), W, mt[pass - 1][wide], !rare, rare,
                           pass == 1 ? tgt_threads[0] : tgt_threads[1], (wide ? max_lanes_w : max_lanes)[pass - 1], A,
@@ -1155,7 +1188,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         RegionPlan &q = rp[2 * r + pass - 1];
         // (regions with a large image stay: staging it into more blocks costs
         // more than the extra SMs give -- C5 n = 1,000: 599 -> 643 ms)
-        if (q.g || wtot <= 0 || ctx->regions[r].img.bytes > fill_img_max) continue;
+        if (q.g || q.lpi || wtot <= 0 || ctx->regions[r].img.bytes > fill_img_max) continue;
         const double nr = ctx->regions[r].n;
         const uint32_t need = (uint32_t)std::ceil(148.0 * nr * (nr + 16.0) / wtot);
         const uint32_t have = (A + q.sh.apb - 1) / q.sh.apb;
@@ -1189,12 +1222,13 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // the u32-cycle / 3-4 class instantiations), gs_wide_lanes above
       const bool gwide = g && gs_wide[pass - 1] && sh.lanes <= gs_wide_lanes[pass - 1] && !(pass == 2 && (t32 || P.nc4));
       const bool wk = (wide && mask) || gwide || q.huge;
-      const Key key(pass, sh.apb, sh.lanes, sh.ts, pass == 2 && t32, mask, g, sh.smem, wk, sh.ig, lean);
+      const bool ct32 = pass == 2 && t32 && !q.lpi;  // (lane-per-instruction ants keep u32 ready times in registers)
+      const Key key(pass, sh.apb, sh.lanes, sh.ts, ct32, mask, g, sh.smem, wk, sh.ig, lean);
       Cls &c = classes[key];
       c.wide = wk;
       c.sh = sh;
       c.mask = mask;
-      c.t32 = pass == 2 && t32;
+      c.t32 = ct32;
       c.gs = g;
       c.lean = lean;
       // a class reserves what its largest block needs, not 1/k of the SM:

@@ -209,6 +209,11 @@ ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32
   return w + (t32 ? n : (n + 1) / 2) + (nc4 ? (n + 1) / 2 : (n + 3) / 4);
 }
 
+// Lane-per-instruction ants (one warp per ant, state in registers): only the
+// u16 remaining-use counters of >= 3-user registers are per-ant shared words.
+ACO_HD inline uint32_t lpi_words(uint32_t nremw) { return nremw ? nremw : 1u; }
+constexpr uint32_t kLpiMaxThreads = 256;  // (8 ants per block: up to 255 registers per thread)
+
 // Stride (in words) between consecutive state words of one ant in a block of
 // apb ants x lg lanes.  stride = 32/lg (mod 32) makes the 32 lanes of a warp
 // hit 32 distinct banks when lane l of every ant touches a word w = l (mod lg)

@@ -1195,6 +1195,375 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
   return o;
 }
 
+// ------------------------------------------------- lane-per-instruction ants
+// Latency-bound batches (few ants in total, config 2: one region of 1,024
+// ants leaves ~1 warp per SM): ONE WARP PER ANT, lane l owns instructions
+// j = 32 q + l (q < Q, n <= 32 Q).  The ant's mutable state lives in
+// registers -- ready bits, counts of unplaced predecessors, dynamic last-use
+// counts per class (R14), pass-2 ready times; the scheduled set is a
+// warp-uniform bitset -- so a step evaluates every candidate at once (one
+// lane each), selects with warp reductions (redux.sync max / min; the
+// roulette's ascending prefix with a shuffle scan) and commits with
+// warp-uniform control flow in which the owner lanes update their registers.
+// Only the remaining-use counters of >= 3-user registers stay in shared
+// memory.  The per-ant step chain drops from ~600 dependent warp
+// instructions (one ant per lane group, state in shared memory) to ~100.
+// Same decisions in the same order with the same arithmetic and Philox
+// counters as ant_pass1 / ant_pass2 (R1-R27): bit-exact with them and the
+// oracle.  Single issue, <= 2 register classes, no R43 / R45 (host planner).
+constexpr uint32_t kFull = 0xFFFFFFFFu;
+
+// The mutable per-lane state is packed into scalars (no register arrays
+// updated under a runtime index: nvcc would move those to local memory).
+struct LpiAnt {
+  uint32_t rdy;             // bit q: j_q is in the ready set RB (predecessors placed, not scheduled)
+  uint32_t npl;             // u8 x 4: predecessors of j_q not yet placed (n <= 128: in-degree < 255)
+  uint32_t dkA, dkB;        // dynamic last-use counts (R14), u8 per class (2 classes): j_0, j_1 | j_2, j_3
+  uint32_t rtA, rtB;        // pass 2: ready times u16 x 2 (max over placed predecessors of t_p + latency)
+  uint32_t s0, s1, s2, s3;  // scheduled set, words 0-3 (warp-uniform)
+};
+__device__ __forceinline__ uint32_t lpi_sch(const LpiAnt &X, uint32_t w) {
+  return w == 0 ? X.s0 : (w == 1 ? X.s1 : (w == 2 ? X.s2 : X.s3));
+}
+// (q is a constant after unrolling)
+__device__ __forceinline__ uint32_t lpi_dk(const LpiAnt &X, uint32_t q) {  // u8 x 4 per class (classes 0, 1)
+  return ((q < 2 ? X.dkA : X.dkB) >> (16 * (q & 1))) & 0xFFFFu;
+}
+__device__ __forceinline__ uint32_t lpi_rt(const LpiAnt &X, uint32_t q) {
+  return ((q < 2 ? X.rtA : X.rtB) >> (16 * (q & 1))) & 0xFFFFu;
+}
+
+template <int Q>
+__device__ __forceinline__ void lpi_init(const SV &V, uint32_t *rem, uint32_t S, uint32_t lane, LpiAnt &X) {
+  for (uint32_t w = lane; w < V.nremw; w += 32) rem[w * S] = V.rem0[w];
+  X.rdy = 0;
+  X.npl = 0xFFFFFFFFu;  // (lanes past n never become ready)
+  X.dkA = X.dkB = X.rtA = X.rtB = 0;
+  X.s0 = X.s1 = X.s2 = X.s3 = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const uint32_t j = 32u * q + lane;
+    if (j < V.n) {
+      uint32_t c = 0;
+      for (uint32_t k = V.pg_ptr[j]; k < V.pg_ptr[j + 1]; ++k) c += __popc(V.pg[k].y);
+      if (!c) X.rdy |= 1u << q;
+      X.npl = (X.npl & ~(0xFFu << (8 * q))) | (c << (8 * q));
+    }
+  }
+  __syncwarp();
+}
+
+// Commit of instruction j at cycle t (the warp-uniform counterpart of
+// commit()): scheduled / ready sets, RP update (R14, R15), last-use
+// bookkeeping of the registers j reads (the new last user's owner lane bumps
+// its count; dirty: its q bits), successors' readiness and (pass 2) ready times.
+template <int PASS, int Q>
+__device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t S, uint32_t lane, LpiAnt &X,
+                                           uint32_t j, uint32_t t, uint32_t &live01, uint32_t &live23,
+                                           uint32_t &prp01, uint32_t &prp23, uint32_t &dirty) {
+  const uint32_t qj = j >> 5, bj = 1u << (j & 31u);
+  X.s0 |= qj == 0 ? bj : 0u;
+  if (Q > 1) X.s1 |= qj == 1 ? bj : 0u;
+  if (Q > 2) {
+    X.s2 |= qj == 2 ? bj : 0u;
+    X.s3 |= qj == 3 ? bj : 0u;
+  }
+  if (lane == (j & 31u)) X.rdy &= ~(1u << qj);
+  const uint4 inf = V.info[j];
+  uint32_t K = inf.y;  // static kills (single-use registers)
+  const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;
+  for (uint32_t q = 0; q < mc; ++q) {
+    const uint32_t e = V.muse[m0 + q];
+    const uint32_t c = (e >> 16) & 3u;
+    uint32_t u = kInvalid;  // the instruction that becomes the register's last user
+    if (e & kMuseCounter) {  // >= 3 users: remaining-use counter
+      const uint32_t m = e & 0xFFFFu, sh = (m & 1u) * 16;
+      uint32_t *p = rem + (m >> 1) * S;
+      const uint32_t w = *p;
+      const uint32_t left = (w >> sh) & 0xFFFFu;  // users left including j
+      __syncwarp();
+      if (lane == 0) *p = w - (1u << sh);
+      __syncwarp();
+      if (left == 1u) {
+        K += 1u << (8 * c);
+      } else if (left == 2u) {  // the first unscheduled user (in the list's order) remains
+        const uint32_t k0 = V.cu_ptr[m], k1 = V.cu_ptr[m + 1];
+        for (uint32_t b = k0; b < k1; b += 32) {
+          const uint32_t kk = b + lane;
+          const uint32_t x = kk < k1 ? V.cu[kk] : 0u;
+          const bool un = kk < k1 && !((lpi_sch(X, x >> 5) >> (x & 31u)) & 1u);
+          const uint32_t bal = __ballot_sync(kFull, un);
+          if (bal) {
+            u = __shfl_sync(kFull, x, __ffs(bal) - 1);
+            break;
+          }
+        }
+      }
+    } else {  // 2 users: the partner
+      const uint32_t pa = e & 0x1FFFu;
+      if ((lpi_sch(X, pa >> 5) >> (pa & 31u)) & 1u) K += 1u << (8 * c);
+      else u = pa;
+    }
+    if (u != kInvalid && lane == (u & 31u)) {
+      const uint32_t qu = u >> 5, bump = 1u << (8 * c + 16 * (qu & 1u));
+      if (qu < 2) X.dkA += bump;
+      else X.dkB += bump;
+      dirty |= 1u << qu;
+    }
+  }
+  live01 = __vsub2(live01, lo_pair(K));
+  live23 = __vsub2(live23, hi_pair(K));
+  live01 = __vadd2(live01, lo_pair(inf.x));
+  live23 = __vadd2(live23, hi_pair(inf.x));
+  prp01 = __vmaxu2(prp01, live01);
+  prp23 = __vmaxu2(prp23, live23);
+  live01 = __vsub2(live01, lo_pair(inf.z));
+  live23 = __vsub2(live23, hi_pair(inf.z));
+  const uint32_t s0 = V.succ_ptr[j], s1 = V.succ_ptr[j + 1];
+  for (uint32_t q = s0; q < s1; ++q) {
+    const uint32_t e = V.succ[q];
+    const uint32_t v = e & 0x1FFFu;
+    if (lane == (v & 31u)) {
+      const uint32_t qv = v >> 5;
+      if (PASS == 2) {  // ready time = max over placed predecessors (t + latency < 2^16: host)
+        const uint32_t r = (t + (e >> 16)) << (16 * (qv & 1u));
+        if (qv < 2) X.rtA = __vmaxu2(X.rtA, r);
+        else X.rtB = __vmaxu2(X.rtB, r);
+      }
+      X.npl -= 1u << (8 * qv);
+      if (((X.npl >> (8 * qv)) & 0xFFu) == 0u) X.rdy |= 1u << qv;
+    }
+  }
+}
+
+// Roulette over the lanes' candidates (R27): the first candidate in
+// ascending j = 32 q + lane whose inclusive prefix of scores exceeds
+// r = floor(R64 * sum / 2^64).  Scores are scanned as 16-bit halves (no
+// carries within a 32-lane chunk).  Returns kInvalid if none exceeds r.
+template <int Q>
+__device__ __forceinline__ uint32_t lpi_roulette(const uint32_t (&sc)[Q], uint32_t valid, uint32_t lane,
+                                                 uint64_t r64) {
+  uint32_t plo[Q], phi[Q];
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const uint32_t s = ((valid >> q) & 1u) ? sc[q] : 0u;
+    plo[q] = s & 0xFFFFu;
+    phi[q] = s >> 16;
+  }
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const uint32_t a = __shfl_up_sync(kFull, plo[q], o), b = __shfl_up_sync(kFull, phi[q], o);
+      if (lane >= (uint32_t)o) {
+        plo[q] += a;
+        phi[q] += b;
+      }
+    }
+  }
+  uint64_t pre[Q], base = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    pre[q] = base + ((uint64_t)phi[q] << 16) + plo[q];
+    base += ((uint64_t)__shfl_sync(kFull, phi[q], 31) << 16) + __shfl_sync(kFull, plo[q], 31);
+  }
+  const uint64_t r = __umul64hi(r64, base);
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const uint32_t b = __ballot_sync(kFull, ((valid >> q) & 1u) && pre[q] > r);
+    if (b) return 32u * q + (__ffs(b) - 1);
+  }
+  return kInvalid;
+}
+
+// Warp argmax over (key desc, j asc): key = score + 1 of a candidate, 0 = none.
+template <int Q>
+__device__ __forceinline__ uint32_t lpi_argmax(const uint32_t (&key)[Q], uint32_t lane) {
+  uint32_t bk = 0, bq = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q)
+    if (key[q] > bk) {  // ascending q: strict keeps the lane's lowest j
+      bk = key[q];
+      bq = q;
+    }
+  const uint32_t mx = __reduce_max_sync(kFull, bk);
+  return __reduce_min_sync(kFull, (bk == mx && mx) ? 32u * bq + lane : kInvalid);
+}
+
+// RP pass, one ant per warp (as ant_pass1: R1, R4, R19, R25-R27).
+template <int Q>
+__device__ __forceinline__ AntOut lpi_pass1(const SV &V, const uint16_t *__restrict__ tau, uint32_t *rem, uint32_t S,
+                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg, uint16_t *rec,
+                                            const uint32_t *coins, const uint32_t rec_stride) {
+  const uint32_t lane = threadIdx.x & 31u, n = V.n, L1 = V.L1;
+  LpiAnt X;
+  lpi_init<Q>(V, rem, S, lane, X);
+  uint32_t e1[Q];  // eta1(j, sk(j) + d(j)) at the current d (R4)
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const uint32_t j = ::min(32u * q + lane, n - 1);
+    e1[q] = V.eta1[j * L1];
+  }
+  uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
+  uint32_t prev = n;
+  for (uint32_t k = 0; k < n; ++k) {
+    const bool exploit = (coins[k >> 5] >> (k & 31u)) & 1u;  // group coin (R3)
+    const uint16_t *trow = tau + prev * n;
+    uint32_t sc[Q], key[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const uint32_t j = ::min(32u * q + lane, n - 1);
+      sc[q] = (uint32_t)trow[j] * e1[q];
+      key[q] = ((X.rdy >> q) & 1u) ? sc[q] + 1u : 0u;
+    }
+    uint32_t jstar = lpi_argmax<Q>(key, lane);
+    if (!exploit) {
+      const uint4 x = philox(k, ant, iter, V.region_id, cfg.seed);
+      const uint32_t jr = lpi_roulette<Q>(sc, X.rdy, lane, ((uint64_t)x.y << 32) | x.x);
+      if (jr != kInvalid) jstar = jr;
+    }
+    uint32_t dirty = 0;
+    lpi_commit<1, Q>(V, rem, S, lane, X, jstar, 0, live01, live23, prp01, prp23, dirty);
+    if (dirty) {
+#pragma unroll
+      for (int q = 0; q < Q; ++q)
+        if ((dirty >> q) & 1u) e1[q] = V.eta1[(32u * q + lane) * L1 + sum_u8x4(lpi_dk(X, q))];
+    }
+    if (rec && lane == 0) rec[(size_t)k * rec_stride] = (uint16_t)jstar;
+    prev = jstar;
+  }
+  AntOut o;
+  o.prp01 = prp01;
+  o.prp23 = prp23;
+  o.len = 0;
+  o.cost = cost_of(cfg.mslot, cfg.cost_mode, prp01, prp23);
+  return o;
+}
+
+// ILP pass, one ant per warp (as ant_pass2 on the single-issue machine:
+// R19-R24, R41; stalls, the RP-feasible set, the prune).
+template <int Q>
+__device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restrict__ tau, uint32_t *rem, uint32_t S,
+                                            const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
+                                            const uint32_t tgt[4], uint32_t *prune_len, const bool prune,
+                                            uint16_t *rec_o, uint32_t *rec_c, const uint32_t *coins,
+                                            const uint32_t coin_t, const uint32_t rec_stride) {
+  const uint32_t lane = threadIdx.x & 31u, n = V.n;
+  LpiAnt X;
+  lpi_init<Q>(V, rem, S, lane, X);
+  uint32_t dx2[Q], dy[Q], e2[Q];  // defs (u16 x 2), static kills (u8 x 4), eta2
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const uint4 ds = V.ds[::min(32u * q + lane, n - 1)];
+    dx2[q] = lo_pair(ds.x);
+    dy[q] = ds.y;
+    e2[q] = ds.z & 0xFFFFu;
+  }
+  uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
+  const uint32_t group = ant / cfg.group_size;
+  const bool stall_en = stall_group(cfg, group);  // R23, R44
+  const uint32_t c2 = 0x80000000u | iter;
+  uint32_t t = 0, placed = 0, kopt = 0, prev = n, turn = 0;
+  AntOut o;
+  o.prp01 = o.prp23 = 0;
+  o.len = kInvalid;
+  while (placed < n) {
+    if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune
+      uint32_t bl = 0;
+      if (lane == 0) bl = *(volatile uint32_t *)prune_len;
+      bl = __shfl_sync(kFull, bl, 0);
+      if (t + (n - placed) > bl) {
+        if (lane == 0) atomicAdd(prune_len + 1, 1u);
+        o.cost = kInvalid;
+        return o;
+      }
+    }
+    uint32_t slack = 0;  // slack_c = target_c - live_c, saturated to a byte (R21)
+    {
+      const uint32_t lv[4] = {live01 & 0xFFFFu, live01 >> 16, live23 & 0xFFFFu, live23 >> 16};
+#pragma unroll
+      for (int c = 0; c < 4; ++c) slack |= ::min(tgt[c] - lv[c], 255u) << (8 * c);
+    }
+    const uint32_t slack2 = lo_pair(slack);
+    const uint16_t *trow = tau + prev * n;
+    uint32_t sc[Q], key[Q], lat = 0, feas = 0, semi = 0, mins = kInvalid;
+    bool fni = false, sdec = false;
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const bool inr = (X.rdy >> q) & 1u;
+      const uint32_t K2 = lo_pair(dy[q] + lpi_dk(X, q));  // kills per class (R14)
+      const uint32_t rtq = lpi_rt(X, q);
+      const bool l = inr && rtq <= t;
+      const bool s = inr && rtq > t;
+      const bool f = l && all_le2(dx2[q], slack2 + K2);  // defs_c <= slack_c + kills_c (R21)
+      sc[q] = (uint32_t)trow[::min(32u * q + lane, n - 1)] * e2[q];
+      key[q] = f ? sc[q] + 1u : 0u;
+      fni |= f && all_le2(dx2[q], K2);    // max_c Delta_c <= 0
+      sdec |= s && any_lt2(dx2[q], K2);   // min_c Delta_c < 0
+      if (s) mins = ::min(mins, rtq);
+      lat |= (uint32_t)l << q;
+      feas |= (uint32_t)f << q;
+      semi |= (uint32_t)s << q;
+    }
+    const uint32_t min_s = __reduce_min_sync(kFull, mins);
+    if (!__any_sync(kFull, lat != 0u)) {  // necessary stall (L153): skip to the next ready time
+      t = min_s;
+      continue;
+    }
+    const bool any_s = __any_sync(kFull, semi != 0u);
+    if (!__any_sync(kFull, feas != 0u)) {
+      if (stall_en && any_s) {  // forced optional stall (L155, R22)
+        kopt += min_s - t;
+        t = min_s;
+        continue;
+      }
+      o.cost = kInvalid;  // the ant is terminated (L149)
+      return o;
+    }
+    uint4 x = make_uint4(0, 0, 0, 0);
+    bool have_x = false;
+    if (stall_en && any_s && !__any_sync(kFull, fni) && __any_sync(kFull, sdec)) {  // discretionary (L157-L164)
+      x = philox(t, ant, c2, V.region_id, cfg.seed);
+      have_x = true;
+      const uint32_t thr = (kopt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (kopt + 1));
+      if (x.z < thr) {
+        ++kopt;
+        ++t;
+        continue;
+      }
+    }
+    bool exploit;
+    if (t < coin_t) {
+      exploit = (coins[t >> 5] >> (t & 31u)) & 1u;
+    } else {
+      const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
+      exploit = (uint64_t)g.x < cfg.q0_t;
+    }
+    uint32_t jstar = lpi_argmax<Q>(key, lane);
+    if (!exploit) {
+      if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
+      const uint32_t jr = lpi_roulette<Q>(sc, feas, lane, ((uint64_t)x.y << 32) | x.x);
+      if (jr != kInvalid) jstar = jr;
+    }
+    uint32_t dirty = 0;
+    lpi_commit<2, Q>(V, rem, S, lane, X, jstar, t, live01, live23, prp01, prp23, dirty);
+    if (rec_o && lane == 0) {
+      rec_o[(size_t)placed * rec_stride] = (uint16_t)jstar;
+      rec_c[(size_t)placed * rec_stride] = t;
+    }
+    ++placed;
+    prev = jstar;
+    ++t;
+  }
+  if (prune && lane == 0) atomicMin(prune_len, t);
+  o.prp01 = prp01;
+  o.prp23 = prp23;
+  o.len = t;
+  o.cost = t;
+  if (cfg.weighted) o.cost = t + cfg.ws_weight * cost_of(cfg.mslot, cfg.cost_mode, prp01, prp23);  // R41
+  return o;
+}
+
 // ------------------------------------------------------------ kernels
 struct KArgs {
   const unsigned char *arena;
@@ -1227,8 +1596,10 @@ template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS
 #endif
 // (huge regions with shared-memory state, !MASK && GS == 2: two blocks per SM,
 // every ant of config 4 resident)
-__global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockThreads,
-                                  (WIDE && GS != 1) ? ((MASK || GS != 2) ? 1 : 2) : ACO_NARROW_MINB)
+// (LG == 32: lane-per-instruction ants, one warp each: latency-bound
+// batches with few warps per SM, registers unconstrained)
+__global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockThreads),
+                                  LG == 32 ? 1 : ((WIDE && GS != 1) ? ((MASK || GS != 2) ? 1 : 2) : ACO_NARROW_MINB))
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
@@ -1275,7 +1646,8 @@ __global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockTh
       const uint32_t gsz = A.cfg.group_size, abase = A.cfg.ant_base + bi.ant0, g0 = abase / gsz;
       const uint32_t ng = (abase + apb - 1) / gsz - g0 + 1, cw = coin_words(PASS, rd->n);
       uint32_t *cz = (uint32_t *)(smem + state_off) +
-                     stride * ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4, LEAN, rd->nslot);
+                     stride * (LG == 32 ? lpi_words(rd->nremw)
+                                        : ant_words(PASS, rd->n, rd->nwr, rd->nremw, T32, NC4, LEAN, rd->nslot));
       const uint32_t lane = threadIdx.x & 31u, c2 = PASS == 1 ? iter : (0x80000000u | iter);
       for (uint32_t task = threadIdx.x >> 5; task < ng * cw; task += blockDim.x >> 5) {
         const uint32_t gi = task / cw, k = (task - gi * cw) * 32 + lane;
@@ -1307,12 +1679,56 @@ __global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockTh
   }
   const Grp<LG> G(threadIdx.x);
   const SV V = make_sv(img, rd);
-  const St S = make_st<PASS, T32, NC4, LEAN>(stbase, stride, V);
   // tau rows read from global memory: prefetch the next step's row into L1
   const bool pf = !TAU_SMEM && (A.cfg.tau_prefetch & (1u << (PASS - 1 + (GS == 1 ? 2 : 0))));
   const bool dump = (A.cfg.flags & ACO_FLAG_DUMP) != 0;
   AntOut o;
-  if constexpr (PASS == 1) {
+  if constexpr (LG == 32) {  // lane-per-instruction ant (n <= 128): only its >= 3-user counters in stbase
+    static_assert(MASK && !T32 && !NC4 && GS == 0 && !WIDE && !LEAN, "LPI variants");
+    const uint32_t qn = (V.n + 31) / 32;
+    if constexpr (PASS == 1) {
+      uint16_t *rec = nullptr;
+      uint32_t rs1 = 1;
+      if (dump && A.dump_order) {
+        rec = A.dump_order + (size_t)iter * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
+      } else if (A.cfg.record) {
+        rec = (uint16_t *)(A.ws + W.o_rec) + ai;
+        rs1 = A.cfg.ants;
+      }
+      if (qn <= 1) o = lpi_pass1<1>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+      else if (qn <= 2) o = lpi_pass1<2>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+      else o = lpi_pass1<4>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+    } else {
+      uint32_t tgt[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
+      const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
+      uint16_t *rec_o = nullptr;
+      uint32_t *rec_c = nullptr;
+      if (dump && A.dump_order && A.dump_cycle) {
+        const size_t base =
+            ((size_t)A.cfg.iterations + iter) * A.cfg.dump_slice + W.o_dump + (size_t)ai * V.n;
+        rec_o = A.dump_order + base;
+        rec_c = A.dump_cycle + base;
+      }
+      uint32_t rs2 = 1;
+      if (!rec_o && A.cfg.record) {
+        rec_o = (uint16_t *)(A.ws + W.o_rec) + ai;
+        rec_c = (uint32_t *)(A.ws + W.o_recc) + ai;
+        rs2 = A.cfg.ants;
+      }
+      if (qn <= 1)
+        o = lpi_pass2<1>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+                         coin_t, rs2);
+      else if (qn <= 2)
+        o = lpi_pass2<2>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+                         coin_t, rs2);
+      else
+        o = lpi_pass2<4>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+                         coin_t, rs2);
+    }
+  } else if constexpr (PASS == 1) {
+    const St S = make_st<PASS, T32, NC4, LEAN>(stbase, stride, V);
     uint16_t *rec = nullptr;
     uint32_t rs1 = 1;
     if (dump && A.dump_order) {
@@ -1326,6 +1742,7 @@ __global__ void __launch_bounds__((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockTh
     else
       o = ant_pass1<LG, MASK, WIDE, false, LEAN>(V, tau, S, G, ant, iter, A.cfg, false, rec, coins, rl, rs1, pf);
   } else {
+    const St S = make_st<PASS, T32, NC4, LEAN>(stbase, stride, V);
     uint32_t tgt[4];
 #pragma unroll
     for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
@@ -1996,6 +2413,11 @@ static void reg_huge(F &f) {
 }
 template <typename F>
 static void for_each_construct(F &&f) {
+  // lane-per-instruction ants (one warp per ant, n <= 128), tau staged or not
+  reg1<1, 32, true, true, false, false, 0, false>(f);
+  reg1<1, 32, true, false, false, false, 0, false>(f);
+  reg1<2, 32, true, true, false, false, 0, false>(f);
+  reg1<2, 32, true, false, false, false, 0, false>(f);
   reg_lg<1>(f);
   reg_lg<2>(f);
   reg_lg<4>(f);
@@ -2055,6 +2477,7 @@ int construct_max_threads(int device, uint32_t out[2][3]) {
       ok = false;
       return;
     }
+    if (code & (1u << 10)) return;  // (lane-per-instruction variants: planned separately)
     const uint32_t p = (code >> 8) & 1u, w = ((code >> 12) & 1u) ? 2u : (code & 1u);
     regs[p][w] = std::max(regs[p][w], (uint32_t)fa.numRegs);
   });

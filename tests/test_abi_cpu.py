@@ -196,11 +196,28 @@ def test_planner_fused_for_config1_only(lib):
 def test_planner_fill_rule_spreads_few_large_regions(lib):
     """Config 2 (one region holding all the work): its ants spread over many
     small blocks in both passes (the SM fill rule), pass 1 with up to 4 lanes
-    per ant; config 3 (5,000 regions) keeps its large blocks."""
-    _, c2 = _plan(["--workload", "c2"])
+    per ant; config 3 (5,000 regions) keeps its large blocks.  (Config 2
+    runs on the lane-per-instruction ants by default: ACO_LPI=0 here.)"""
+    os.environ["ACO_LPI"] = "0"
+    try:
+        _, c2 = _plan(["--workload", "c2"])
+    finally:
+        del os.environ["ACO_LPI"]
     for pass_ in (1, 2):
         blocks = sum(b for p, b, a, l in c2 if p == pass_)
         assert blocks >= 32, c2
     assert any(p == 1 and l == 4 for p, b, a, l in c2)
     _, c3 = _plan(["--workload", "c3", "--regions", "400"])
     assert max(a * l for p, b, a, l in c3) >= 256  # large blocks kept
+
+
+def test_planner_lane_per_instruction_for_config2(lib):
+    """Config 2 (one n = 100 region, 1,024 ants: the per-ant step latency
+    bounds it) takes the lane-per-instruction ants in both passes: one warp
+    per ant, ~148 blocks; config 3's batch never does."""
+    v2, c2 = _plan(["--workload", "c2"])
+    assert v2[0] and all(c & (1 << 10) for c in v2[0]), v2
+    for pass_ in (1, 2):
+        assert sum(b for p, b, a, l in c2 if p == pass_ and l == 32) >= 128, c2
+    v3, _ = _plan(["--workload", "c3", "--regions", "400"])
+    assert not any(c & (1 << 10) for c in v3[0])
