@@ -957,12 +957,25 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint64_t lpi_max_ants = 148ull * 16;  // ants (= warps) in the whole batch
   if (const char *e = getenv("ACO_LPI_ANTS")) lpi_max_ants = strtoull(e, nullptr, 10);
   const bool lpi_batch = lpi_mode == 2 || (lpi_mode == 1 && (uint64_t)A * count <= lpi_max_ants);
-  // huge regions: per-ant state in shared memory when all ants fit -- off:
-  // measured slower (r02u: C4 832 -> 1098 ms; the two 113 KB blocks per SM
-  // leave L1 ~28 KB for the image and tau the global-state kernels cache in
-  // the full 256 KB, and the 64-register bound spills); ACO_HUGE_SMEM=1
-  bool huge_smem = false;
+  // huge regions (n > 1024): per-ant state in shared memory, image and tau
+  // through L1/L2, 8 lanes per ant, 32-ant blocks, as many waves as needed.
+  // Round 2 ran them on the global-state kernels: the first shared-state
+  // version (every ant resident in one wave, 2 blocks reserving 113 KB each,
+  // 64 registers) left L1 28 KB and spilled: C4 832 -> 1098 ms.  r03: the
+  // blocks reserve exactly their state (L1 keeps ~120 KB for the image), 128
+  // registers (launch bound ACO_HUGE_MINB = 1), waves allowed:
+  // C4 842 -> 738 ms, C5 1927 -> 1813 ms (tools/gpu_r03e.sh, r03f.sh)
+  bool huge_smem = true;
   if (const char *e = getenv("ACO_HUGE_SMEM")) huge_smem = atoi(e) != 0;
+  // ... resident blocks per SM its kernels allow, several waves of ants
+  // allowed, shared memory per SM capped (0: no cap), exact reservation, lanes
+  uint32_t huge_k = 2, huge_waves = 1, huge_exact = 1, huge_lanes[2] = {8, 8};
+  uint64_t huge_smem_max = 0;
+  if (const char *e = getenv("ACO_HUGE_LANES")) sscanf(e, "%u,%u", &huge_lanes[0], &huge_lanes[1]);
+  if (const char *e = getenv("ACO_HUGE_K")) huge_k = (uint32_t)atoi(e);
+  if (const char *e = getenv("ACO_HUGE_WAVES")) huge_waves = (uint32_t)atoi(e);
+  if (const char *e = getenv("ACO_HUGE_EXACT")) huge_exact = (uint32_t)atoi(e);
+  if (const char *e = getenv("ACO_HUGE_SMEM_KB")) huge_smem_max = 1024ull * strtoull(e, nullptr, 10);
   uint32_t gs_wide[2] = {1, 1};  // 4-wide scan in the global-state kernels, per pass
   if (const char *e = getenv("ACO_GS_WIDE")) {
     if (sscanf(e, "%u,%u", &gs_wide[0], &gs_wide[1]) == 1) gs_wide[1] = gs_wide[0];
@@ -1115,11 +1128,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       // scan; pass 2 in the lean layout when its latencies allow -- taken
       // when every ant of the path stays resident (one wave), else the
       // global-state kernels below
-      const uint32_t gl = gs_lanes[pass - 1];
+      const uint32_t gl = huge_lanes[pass - 1];
       const bool hl = pass == 2 && lean_on && R.max_lat < 128u && ctx->mach.issue_width <= 1;
       const uint32_t Wh = hl ? ant_words(2, R.n, R.nwr, R.nremw, false, false, true, R.nslot)
                              : ant_words(pass, R.n, R.nwr, R.nremw, false, false);
-      const uint32_t maxb = kMaxBlockThreads;  // (huge variants: 512-thread bound, 2 blocks per SM)
+      const uint32_t maxb = kMaxBlockThreads;  // (huge variants: 512-thread bound, ACO_HUGE_MINB blocks per SM)
       const uint64_t need = std::max<uint64_t>(1, gs_ants[pass - 1]);
       for (uint32_t apb : {32u, 16u, 8u, 4u, 2u}) {
         const uint32_t thr = apb * gl;
@@ -1127,10 +1140,14 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         const uint64_t bytes = (uint64_t)ant_stride(apb, gl) * Wh * 4 +
                                (uint64_t)coin_groups(apb, p->group_size) * coin_words(pass, R.n) * 4;
         if (bytes > kSmemPerSM) continue;
-        uint32_t k = std::min<uint32_t>(kSmemSM / ((uint32_t)bytes + kBlockReserve), 2u);  // (launch bound: 2 per SM)
+        uint32_t k = std::min<uint32_t>(kSmemSM / ((uint32_t)bytes + kBlockReserve), huge_k);  // (launch bound)
+        k = std::min<uint32_t>(k, std::max<uint32_t>(1, 65536u / (thr * 128u)));  // (<= 128 registers per thread)
         while (k && smem_for_k(k) < bytes) --k;
-        if (!k || 148ull * k * apb < need) continue;
-        sh = Shape{apb, gl, smem_for_k(k), false, k * thr, true};
+        if (k && huge_smem_max && k * bytes > huge_smem_max) k = std::max<uint64_t>(1, huge_smem_max / bytes);
+        if (!k || (!huge_waves && 148ull * k * apb < need)) continue;
+        // (exact: the block reserves what it needs; the rest of the SM's
+        // 256 KB stays L1 for the image and tau read through it)
+        sh = Shape{apb, gl, smem_for_k(k), false, k * thr, true, huge_exact ? (((uint32_t)bytes + 127u) & ~127u) : 0u};
         q.huge = true;
         lean = hl;
         W = Wh;
@@ -1622,8 +1639,11 @@ int run_finalize(aco_ctx ctx, uint32_t pass, uint32_t it, int64_t *keys) {
   Plan &P = ctx->plan;
   Bracket b(ctx, 1);
   P.L.cfg.keys = keys;
+  // few regions with small tables: select + update + stop in one launch (ACO_FIN1=0: three launches)
+  static const bool fin1_on = !getenv("ACO_FIN1") || atoi(getenv("ACO_FIN1")) != 0;
+  const bool fin1 = fin1_on && P.L.cfg.count <= kFin1MaxRegions && P.max_n <= kFin1MaxN;
   const int err = launch_finalize(P.L, pass, it, P.fin_smem[pass], P.max_n, pass == 2 && P.any_t32, P.nc4,
-                                  (const UpdItem *)(P.L.ws + P.o_upd), P.n_upd);
+                                  (const UpdItem *)(P.L.ws + P.o_upd), P.n_upd, fin1);
   P.L.cfg.keys = nullptr;
   return err;
 }

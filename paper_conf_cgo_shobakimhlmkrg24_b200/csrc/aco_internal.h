@@ -212,6 +212,9 @@ ACO_HD inline uint32_t ant_words(uint32_t pass, uint32_t n, uint32_t nwr, uint32
 // Lane-per-instruction ants (one warp per ant, state in registers): only the
 // u16 remaining-use counters of >= 3-user registers are per-ant shared words.
 ACO_HD inline uint32_t lpi_words(uint32_t nremw) { return nremw ? nremw : 1u; }
+// The end of an iteration as one launch per region block (k_finalize1) for
+// batches of at most this many regions of at most this many instructions.
+constexpr uint32_t kFin1MaxRegions = 148, kFin1MaxN = 256;
 constexpr uint32_t kLpiMaxThreads = 256;  // (8 ants per block: up to 255 registers per thread)
 
 // Stride (in words) between consecutive state words of one ant in a block of
@@ -324,7 +327,7 @@ int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n);
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c);
 int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
-                    bool nc4, const UpdItem *upd, uint32_t n_upd);
+                    bool nc4, const UpdItem *upd, uint32_t n_upd, bool fin1);  // fin1: k_finalize1
 int launch_local_keys(LaunchCtx &L, int64_t *keys);
 int launch_post(LaunchCtx &L, uint32_t smem);
 int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem);  // the whole run, one block per region  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys

@@ -31,6 +31,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <stdint.h>
 
 #include "aco_internal.h"
@@ -40,6 +42,9 @@
 // are the product configuration.
 #ifndef ACO_PREFETCH
 #define ACO_PREFETCH 0
+#endif
+#ifndef ACO_BULK_STAGE  // k_construct stages image / tau with cp.async.bulk (else 16-byte copies by every thread)
+#define ACO_BULK_STAGE 1
 #endif
 #ifndef ACO_BRANCHLESS1  // pass-1 4-wide evaluation without branches (measured faster)
 #define ACO_BRANCHLESS1 1
@@ -1581,6 +1586,36 @@ struct KArgs {
 __device__ __forceinline__ void stage(uint4 *dst, const uint4 *src, uint32_t bytes) {
   for (uint32_t i = threadIdx.x; i < bytes / 16; i += blockDim.x) dst[i] = src[i];
 }
+// ... by one warp (the select body, also run by warp 0 of k_finalize1's block)
+__device__ __forceinline__ void stage_warp(uint4 *dst, const uint4 *src, uint32_t bytes) {
+  for (uint32_t i = threadIdx.x & 31u; i < bytes / 16; i += 32) dst[i] = src[i];
+}
+
+// Bulk-async staging (sm_90+ bulk-copy / TMA engine, cp.async.bulk with an
+// mbarrier transaction count).  Sources, destinations and sizes are 16-byte
+// aligned multiples (block images and tau tables are padded to 16 bytes).
+constexpr uint32_t kBulkChunk = 32768;
+__device__ __forceinline__ void bulk_arm(uint32_t mbar, uint32_t bytes) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_copy(void *dst, const void *src, uint32_t bytes, uint32_t mbar) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(dst);
+  for (uint32_t off = 0; off < bytes; off += kBulkChunk) {
+    const uint32_t b = ::min(kBulkChunk, bytes - off);
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d + off),
+                 "l"((const char *)src + off), "r"(b), "r"(mbar)
+                 : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_wait_inval(uint32_t mbar) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n @!p bra WAIT_%=;\n}" ::"r"(mbar)
+      : "memory");
+  asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(mbar) : "memory");
+}
 
 // Launch bounds: the 1-wide variants keep <= 64 registers (2 x 512 threads per
 // SM); the 4-wide ones (large regions, few ants per SM by shared memory) may
@@ -1594,12 +1629,15 @@ template <int PASS, int LG, bool MASK, bool TAU_SMEM, bool T32, bool NC4, int GS
 #ifndef ACO_NARROW_MINB  // min blocks per SM of the 1-wide variants (2: <= 64 registers)
 #define ACO_NARROW_MINB 2
 #endif
+#ifndef ACO_HUGE_MINB  // min blocks per SM of the huge shared-state variants (1: up to 128 registers)
+#define ACO_HUGE_MINB 1
+#endif
 // (huge regions with shared-memory state, !MASK && GS == 2: two blocks per SM,
 // every ant of config 4 resident)
 // (LG == 32: lane-per-instruction ants, one warp each: latency-bound
 // batches with few warps per SM, registers unconstrained)
 __global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? kLeanMaxThreads : kMaxBlockThreads),
-                                  LG == 32 ? 1 : ((WIDE && GS != 1) ? ((MASK || GS != 2) ? 1 : 2) : ACO_NARROW_MINB))
+                                  LG == 32 ? 1 : ((WIDE && GS != 1) ? ((MASK || GS != 2) ? 1 : ACO_HUGE_MINB) : ACO_NARROW_MINB))
     k_construct(KArgs A, const BlockItem *__restrict__ items, uint32_t iter) {
   const BlockItem bi = items[blockIdx.x];
   RegionState &rs = A.state[bi.region];
@@ -1630,14 +1668,24 @@ __global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? 
     }
   } else {
     const uint32_t img_bytes = GS == 0 ? rd->img.bytes : 0u;
-    if (GS == 0) stage(smem4, (const uint4 *)img, img_bytes);
-    uint32_t state_off = img_bytes;
-    if (TAU_SMEM) {
-      const uint32_t tb = tau_smem_bytes(rd->n);
-      stage((uint4 *)(smem + img_bytes), (const uint4 *)(A.ws + W.o_tau), tb);
-      tau = (const uint16_t *)(smem + img_bytes);
-      state_off += tb;
+    const uint32_t tb = TAU_SMEM ? tau_smem_bytes(rd->n) : 0u;
+    uint32_t state_off = img_bytes + tb;
+#if ACO_BULK_STAGE
+    // image and tau by the bulk-copy (TMA) engine: thread 0 arms an mbarrier
+    // (in the first per-ant state words, unused until the ants initialise
+    // them) with the byte count and issues 1-D bulk copies; the block builds
+    // its coin table meanwhile; thread 0 waits, then the block barrier
+    const uint32_t mbar = (uint32_t)__cvta_generic_to_shared(smem + state_off);
+    if (threadIdx.x == 0 && img_bytes + tb) {
+      bulk_arm(mbar, img_bytes + tb);
+      if (GS == 0) bulk_copy(smem, img, img_bytes, mbar);
+      if (TAU_SMEM) bulk_copy(smem + img_bytes, A.ws + W.o_tau, tb, mbar);
     }
+#else
+    if (GS == 0) stage(smem4, (const uint4 *)img, img_bytes);
+    if (TAU_SMEM) stage((uint4 *)(smem + img_bytes), (const uint4 *)(A.ws + W.o_tau), tb);
+#endif
+    if (TAU_SMEM) tau = (const uint16_t *)(smem + img_bytes);
     const uint32_t apb = blockDim.x / LG;
     stride = ant_stride(apb, LG);
     // Group coins (R3) of every (step, group) of this block, one warp per
@@ -1668,6 +1716,9 @@ __global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? 
         if (ai < A.cfg.ants && ai % gsz == 0) rl.out = (uint16_t *)(A.ws + W.o_rlk) + (size_t)(ai / gsz) * rd->n;
       }
     }
+#if ACO_BULK_STAGE
+    if (threadIdx.x == 0 && img_bytes + tb) bulk_wait_inval(mbar);
+#endif
     __syncthreads();
     if (ai >= A.cfg.ants) {  // whole lane group
       if (PASS == 1 && rl.buf)  // the block's lockstep steps need every thread at the barrier (R45)
@@ -1799,18 +1850,17 @@ __device__ void tau_fill(uint16_t *tau, uint32_t len, uint32_t tau0) {
 // Evaporate + deposit + clamp (R6-R9) over all active regions' tables, 8
 // entries per 16-byte access.  One block = kUpdVec vectors of one region;
 // next[i] = the winner's successor of row i (0xFFFF: no deposit).
-__global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restrict__ items) {
-  const UpdItem it = items[blockIdx.x];
-  if (!A.state[it.region].active) return;  // the pass ended: tau is not used again
-  const RegionDev *rd = A.regions + it.region;
-  const RegionWs &W = A.rws[it.region];
+__device__ __forceinline__ void update_vecs(const KArgs &A, uint32_t region, uint32_t v0, uint32_t v1, uint32_t tid,
+                                            uint32_t nthr) {
+  const RegionDev *rd = A.regions + region;
+  const RegionWs &W = A.rws[region];
   const uint32_t n = rd->n;
   const uint32_t total = (n + 1) * n;
   const uint16_t *next = (const uint16_t *)(A.ws + W.o_next);
   uint4 *t4 = (uint4 *)(A.ws + W.o_tau);
-  const uint32_t vend = min(it.v0 + kUpdVec, W.tau_len / 8);
+  const uint32_t vend = min(v1, W.tau_len / 8);
   const uint32_t rho = A.cfg.rho_q16, dl = A.cfg.delta, lo = A.cfg.tau_min, hi = A.cfg.tau_max;
-  for (uint32_t v = it.v0 + threadIdx.x; v < vend; v += blockDim.x) {
+  for (uint32_t v = v0 + tid; v < vend; v += nthr) {
     const uint4 q = t4[v];
     uint32_t w[4] = {q.x, q.y, q.z, q.w};
     const uint32_t e0 = v * 8;
@@ -1834,6 +1884,11 @@ __global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restri
     }
     t4[v] = make_uint4(w[0], w[1], w[2], w[3]);
   }
+}
+__global__ void __launch_bounds__(256) k_update(KArgs A, const UpdItem *__restrict__ items) {
+  const UpdItem it = items[blockIdx.x];
+  if (!A.state[it.region].active) return;  // the pass ended: tau is not used again
+  update_vecs(A, it.region, it.v0, it.v0 + kUpdVec, threadIdx.x, blockDim.x);
 }
 
 // Per-region initialisation: tau0, the greedy pass-1 heuristic schedule
@@ -2082,7 +2137,7 @@ __device__ __forceinline__ void select_body(const KArgs &A, uint32_t iter, unsig
     // shared memory, so many replays are resident per SM; with few regions
     // the image is staged as well (latency-bound serial replay)
     if (A.cfg.stage_img) {
-      stage((uint4 *)smem, (const uint4 *)img, rd->img.bytes);
+      stage_warp((uint4 *)smem, (const uint4 *)img, rd->img.bytes);
       img = smem;
       stw = (uint32_t *)(smem + rd->img.bytes);
       __syncwarp();
@@ -2180,9 +2235,7 @@ __global__ void __launch_bounds__(32) k_local_keys(KArgs A, int64_t *keys) {
 }
 
 // Termination (L110, L139, L226; R12), after the pheromone update.
-__global__ void k_stop(KArgs A, uint32_t pass) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= A.cfg.count) return;
+__device__ __forceinline__ void stop_body(const KArgs &A, uint32_t r, uint32_t pass) {
   RegionState &rs = A.state[r];
   if (!rs.active) return;
   const RegionDev *rd = A.regions + r;
@@ -2191,6 +2244,40 @@ __global__ void k_stop(KArgs A, uint32_t pass) {
   if ((A.cfg.stop_at_lb && rs.best[pass - 1] == lb) || (lim > 0 && rs.no_imp >= lim) ||
       rs.iters[pass - 1] >= A.cfg.iterations)
     rs.active = 0;
+}
+__global__ void k_stop(KArgs A, uint32_t pass) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.cfg.count) return;
+  stop_body(A, r, pass);
+}
+
+// Few regions with small tables (config 2): the end of an iteration in ONE
+// launch, one block per region -- select (warp 0: argmin, winner copy or
+// replay, epilogue), the block's evaporate + deposit over the region's table,
+// the termination test: the bodies of k_select, k_update and k_stop in their
+// per-region order (regions are independent), two launches fewer per
+// iteration.
+template <int PASS, bool MASK, bool T32, bool NC4>
+__global__ void __launch_bounds__(256) k_finalize1(KArgs A, uint32_t iter) {
+  const uint32_t r = blockIdx.x;
+  if (!A.state[r].active) return;  // block-uniform
+  extern __shared__ uint4 smem4[];
+  __shared__ uint32_t s_prp[3], s_flag;
+  if (threadIdx.x < 32) {
+    const bool ct = PASS == 2 && T32 && !NC4 && A.regions[r].compact;
+    if (A.rws[r].gs) {
+      if (ct) select_body<PASS, false, false, false, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+      else select_body<PASS, false, T32, NC4, true>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    } else if (ct) {
+      select_body<PASS, MASK, false, false, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    } else {
+      select_body<PASS, MASK, T32, NC4, false>(A, iter, (unsigned char *)smem4, s_prp, s_flag);
+    }
+  }
+  __syncthreads();
+  update_vecs(A, r, 0, A.rws[r].tau_len / 8, threadIdx.x, blockDim.x);
+  __syncthreads();
+  if (threadIdx.x == 0) stop_body(A, r, PASS);
 }
 
 // ------------------------------------------------------------ fused run
@@ -2359,8 +2446,15 @@ static KArgs kargs(const LaunchCtx &L) {
   return a;
 }
 
-static int check() {
+// ACO_SYNC_DEBUG=1: synchronise after every launch and name the failing one
+// (debugging aid; compute-sanitizer is not available on every pool).
+static int check(const char *tag = "", uint32_t code = 0) {
+  static const bool sync_debug = getenv("ACO_SYNC_DEBUG") != nullptr;
   cudaError_t e = cudaGetLastError();
+  if (sync_debug && e == cudaSuccess) {
+    e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) fprintf(stderr, "[aco sync] %s (variant %u): %s\n", tag, code, cudaGetErrorString(e));
+  }
   return e == cudaSuccess ? 0 : (int)e;
 }
 
@@ -2512,7 +2606,7 @@ static void big_smem(K kernel) {
 int set_machine(uint32_t slot, const MachineDev &m) {
   if (slot >= kMachSlots) return 1;
   if (cudaMemcpyToSymbol(c_mach, &m, sizeof(m), sizeof(m) * slot) != cudaSuccess) return 1;
-  return check();
+  return check(__func__);
 }
 
 int init_kernel_attrs() {
@@ -2520,6 +2614,11 @@ int init_kernel_attrs() {
   big_smem(k_init<true>);
   big_smem(k_init<false>);
   big_smem(k_pass2_init);
+  big_smem(k_finalize1<1, true, false, false>);
+  big_smem(k_finalize1<2, true, false, false>);
+  big_smem(k_finalize1<2, true, true, false>);
+  big_smem(k_finalize1<2, true, false, true>);
+  big_smem(k_finalize1<2, true, true, true>);
   big_smem(k_post);
   big_smem(k_fused<false>);
   big_smem(k_fused<true>);
@@ -2540,7 +2639,7 @@ int launch_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   else
     k_init<false><<<L.cfg.count, 128, smem, s>>>(kargs(L));
   L.launches++;
-  return check();
+  return check(__func__);
 }
 
 int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
@@ -2548,7 +2647,7 @@ int launch_pass2_init(LaunchCtx &L, uint32_t smem, uint32_t max_n) {
   if (!L.cfg.count) return 0;
   k_pass2_init<<<L.cfg.count, 128, smem, (cudaStream_t)L.stream>>>(kargs(L));
   L.launches++;
-  return check();
+  return check(__func__);
 }
 
 int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaunch &c) {
@@ -2560,7 +2659,7 @@ int launch_construct(LaunchCtx &L, uint32_t pass, uint32_t iter, const ClassLaun
   if (!f) return (int)cudaErrorInvalidDeviceFunction;
   f<<<c.n_blocks, c.ants_pb * lg, c.smem_bytes, (cudaStream_t)L.stream>>>(kargs(L), c.items, iter);
   L.launches++;
-  return check();
+  return check("k_construct", code);
 }
 
 template <bool M>
@@ -2574,23 +2673,32 @@ static void sel(uint32_t pass, bool t32, bool nc4, uint32_t grid, uint32_t smem,
 }
 
 int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, uint32_t max_n, bool t32,
-                    bool nc4, const UpdItem *upd, uint32_t n_upd) {
+                    bool nc4, const UpdItem *upd, uint32_t n_upd, bool fin1) {
   if (!L.cfg.count) return 0;
   cudaStream_t s = (cudaStream_t)L.stream;
   KArgs a = kargs(L);
+  if (fin1) {  // few small regions: one launch (k_finalize1)
+    if (pass == 1) k_finalize1<1, true, false, false><<<L.cfg.count, 256, smem, s>>>(a, iter);
+    else if (!t32 && !nc4) k_finalize1<2, true, false, false><<<L.cfg.count, 256, smem, s>>>(a, iter);
+    else if (t32 && !nc4) k_finalize1<2, true, true, false><<<L.cfg.count, 256, smem, s>>>(a, iter);
+    else if (!t32 && nc4) k_finalize1<2, true, false, true><<<L.cfg.count, 256, smem, s>>>(a, iter);
+    else k_finalize1<2, true, true, true><<<L.cfg.count, 256, smem, s>>>(a, iter);
+    L.launches += 1;
+    return check("k_finalize1", pass);
+  }
   if (max_n <= 1024) sel<true>(pass, t32, nc4, L.cfg.count, smem, s, a, iter);
   else sel<false>(pass, t32, nc4, L.cfg.count, smem, s, a, iter);
   if (n_upd) k_update<<<n_upd, 256, 0, s>>>(a, upd);
   k_stop<<<(L.cfg.count + 255) / 256, 256, 0, s>>>(a, pass);
   L.launches += 2 + (n_upd ? 1 : 0);
-  return check();
+  return check("k_select/k_update/k_stop", pass);
 }
 
 int launch_post(LaunchCtx &L, uint32_t smem) {
   if (!L.cfg.count) return 0;
   k_post<<<L.cfg.count, 32, smem, (cudaStream_t)L.stream>>>(kargs(L));
   L.launches++;
-  return check();
+  return check(__func__);
 }
 
 int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
@@ -2602,14 +2710,14 @@ int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
   if (fw) k_fused<true><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
   else k_fused<false><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
   L.launches++;
-  return check();
+  return check(__func__);
 }
 
 int launch_local_keys(LaunchCtx &L, int64_t *keys) {
   if (!L.cfg.count) return 0;
   k_local_keys<<<L.cfg.count, 32, 0, (cudaStream_t)L.stream>>>(kargs(L), keys);
   L.launches++;
-  return check();
+  return check(__func__);
 }
 
 }  // namespace aco

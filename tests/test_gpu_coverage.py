@@ -3,6 +3,7 @@ oracle comparison: the 4- and 8-lane global-state
 kernels, config 4 at its real shape, the shared colony on a global-state
 region, the discretionary-stall and size-class-termination pins on the GPU."""
 import dataclasses
+import os
 
 import pytest
 
@@ -42,11 +43,11 @@ def test_global_state_lanes_every_ant(torch_cuda, monkeypatch, lanes):
 
 @pytest.mark.parametrize("lanes", [4, 8, 16])
 def test_huge_shared_state_every_ant(torch_cuda, monkeypatch, lanes):
-    """Huge regions (n > 1024) whose ants all fit with their state in shared
-    memory (image and tau through L1, 4-wide strided scan, lean pass 2; an
-    option, ACO_HUGE_SMEM): every ant bit-exact at 4, 8 and 16 lanes per ant."""
-    monkeypatch.setenv("ACO_GS_LANES", f"{lanes},{lanes}")
-    monkeypatch.setenv("ACO_HUGE_SMEM", "1")  # (off by default: measured slower on config 4)
+    """Huge regions (n > 1024) with their per-ant state in shared memory
+    (image and tau through L1, 4-wide strided scan, lean pass 2; configs 4
+    and 5 at 8 lanes): every ant bit-exact at 4, 8 and 16 lanes per ant."""
+    monkeypatch.setenv("ACO_HUGE_LANES", f"{lanes},{lanes}")
+    monkeypatch.setenv("ACO_HUGE_SMEM", "1")  # (the default for n > 1024 since r03)
     regs = [I.gen_region(n, 9200 + n + lanes) for n in (1100, 1900)]
     ids = [35, 36]
     p = I.Params(ants=64, iterations=2, seed=90 + lanes, stall_mod=2)
@@ -74,6 +75,20 @@ def test_shared_colony_on_global_state_region(torch_cuda):
     """The shared colony (4 emulated ranks x 64 ants) on a region whose state
     needs the global-state kernels: every rank replays the winner from its
     workspace scratch; results equal the oracle with 256 ants."""
+    os.environ["ACO_HUGE_SMEM"] = "0"
+    try:
+        _colony_check()
+    finally:
+        del os.environ["ACO_HUGE_SMEM"]
+
+
+def test_shared_colony_on_huge_shared_state_region(torch_cuda):
+    """The same with the default huge-region kernels (per-ant state in shared
+    memory): what config 4 runs at N > 1."""
+    _colony_check()
+
+
+def _colony_check():
     regs = [I.gen_region(1600, 9400)]
     ids = [3]
     p_all = I.Params(ants=256, iterations=2, seed=81)
