@@ -81,7 +81,7 @@ struct Plan {
   uint32_t pass_mask = 0, iterations = 0;
   bool any_t32 = false, nc4 = false, timing = false, p2_done = false, stage_img = false, record = false;
   bool fused = false;  // the whole run in one k_fused launch (one block per region)
-  uint32_t fused_threads = 0, fused_smem = 0;
+  uint32_t fused_threads = 0, fused_smem = 0, fused_wl = 0;  // fused_wl: lanes per lane-per-instruction ant (0: one thread per ant)
   uint64_t o_state = 0, o_rws = 0, o_upd = 0, o_gb2 = 0, o_gb2c = 0, o_keys = 0;
   LaunchCtx L{};
 };
@@ -490,8 +490,10 @@ aco_status prep_region(const aco_region_desc &d, const MachineDev &mach, Prepped
   // predecessor groups: per instruction, {bitset word, mask of its
   // predecessors in that word} (readiness test of pass 1 / compact pass 2)
   std::vector<uint32_t> pgp(n + 1, 0), pgv;
+  pgv.reserve(2 * (size_t)E);
+  std::vector<std::pair<uint32_t, uint32_t>> gr;  // (reused: one allocation per region)
   for (uint32_t v = 0; v < n; ++v) {
-    std::vector<std::pair<uint32_t, uint32_t>> gr;
+    gr.clear();
     for (uint32_t q = pp[v]; q < pp[v + 1]; ++q) {
       const uint32_t p = pred[q] & 0xFFFFu;
       bool found = false;
@@ -1463,10 +1465,29 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
       P.fused = true;
       P.fused_threads = std::max(32u, (A + 31u) & ~31u);
       P.fused_smem = smem;
+      P.fused_wl = 0;
+      // lane-per-instruction ants inside the fused run (WL lanes per ant, the
+      // smallest of 8 / 16 / 32 with n <= 4 WL; WL x A <= 512 threads): only
+      // when forced (ACO_LPI=2 or ACO_FUSED_LPI=1) -- measured slower on
+      // config 1 (0.641 -> 0.898 ms: with n = 10 a thread-per-ant step scans
+      // ~3 candidates, less than the group's reductions and uniform commit)
+      uint32_t nmax = 0;
+      const bool fused_lpi = lpi_mode == 2 || (getenv("ACO_FUSED_LPI") && atoi(getenv("ACO_FUSED_LPI")) != 0);
+      bool lok = fused_lpi && ctx->mach.issue_width <= 1 && !p->heur_mix;
+      for (uint32_t r = 0; r < count; ++r) {
+        const RegionDev &R = ctx->regions[r];
+        nmax = std::max(nmax, R.n);
+        lok = lok && (uint64_t)R.max_cycle_bound + R.max_lat < 65536u;
+      }
+      const uint32_t wl = nmax <= 32 ? 8u : (nmax <= 64 ? 16u : 32u);
+      if (lok && nmax >= 1 && nmax <= 128 && (uint64_t)A * wl <= 512) {
+        P.fused_wl = wl;
+        P.fused_threads = std::max(32u, (A * wl + 31u) & ~31u);  // (whole warps: the select body is warp 0)
+      }
     }
   }
   ctx->variants.clear();  // construct-kernel variants of this plan (aco_last_variants)
-  if (P.fused) ctx->variants.push_back(kFusedVariant);
+  if (P.fused) ctx->variants.push_back(kFusedVariant | (P.fused_wl ? kFusedLpi * (31 - __builtin_clz(P.fused_wl) - 2) : 0u));
   for (int pass = 1; pass <= 2 && !P.fused; ++pass)
     for (const ClassLaunch &cl : P.launches[pass]) {
       const uint32_t code = class_variant((uint32_t)pass, cl);
@@ -1677,7 +1698,7 @@ aco_status aco_schedule_batch(aco_ctx ctx, const aco_params *p, void *d_workspac
   }
   if (ctx->plan.fused) {  // the whole run in one launch (no graph needed)
     Bracket b(ctx, 0);
-    const int e = launch_fused(ctx->plan.L, ctx->plan.fused_threads, ctx->plan.fused_smem);
+    const int e = launch_fused(ctx->plan.L, ctx->plan.fused_threads, ctx->plan.fused_smem, ctx->plan.fused_wl);
     ctx->launches = ctx->plan.L.launches;
     return e ? ACO_E_CUDA : ACO_OK;
   }

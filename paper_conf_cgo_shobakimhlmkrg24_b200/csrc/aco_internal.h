@@ -267,6 +267,7 @@ ACO_HD inline FusedLayout fused_layout(uint32_t n, uint32_t nwr, uint32_t nremw,
   return L;
 }
 constexpr uint32_t kFusedVariant = 1u << 13;  // variant code of k_fused (aco_last_variants)
+constexpr uint32_t kFusedLpi = 1u << 14;       // ... x 1 / 2 / 3: lane-per-instruction ants of 8 / 16 / 32 lanes
 
 // ---- launch interface implemented in aco_kernels.cu ----
 struct LaunchCtx {
@@ -330,7 +331,7 @@ int launch_finalize(LaunchCtx &L, uint32_t pass, uint32_t iter, uint32_t smem, u
                     bool nc4, const UpdItem *upd, uint32_t n_upd, bool fin1);  // fin1: k_finalize1
 int launch_local_keys(LaunchCtx &L, int64_t *keys);
 int launch_post(LaunchCtx &L, uint32_t smem);
-int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem);  // the whole run, one block per region  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys
+int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem, uint32_t wl);  // the whole run, one block per region  // heuristic length + revert filter (R40)  // shared colony: per-region local argmin keys
 
 // Biased winner key: (cost << 32 | global ant) XOR 2^63, so that a signed
 // int64 MIN (NCCL / torch) orders keys like the unsigned (cost, ant) pair.

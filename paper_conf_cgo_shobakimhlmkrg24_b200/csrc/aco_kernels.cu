@@ -1218,6 +1218,24 @@ __device__ __forceinline__ AntOut ant_pass2(const SV &V, const uint16_t *__restr
 // oracle.  Single issue, <= 2 register classes, no R43 / R45 (host planner).
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 
+// The lanes of one ant: WL = 32 (a warp, k_construct) or 8 / 16 (a fused
+// single-block run of a small region, k_fused): lane l of the group owns
+// instructions j = WL q + l; mask = the group's lanes for the .sync
+// collectives (redux / ballot / shuffle with width WL).
+template <int WL>
+struct LpiGrp {
+  uint32_t lane, base, mask;
+  __device__ __forceinline__ LpiGrp() {
+    const uint32_t l = threadIdx.x & 31u;
+    lane = l & (WL - 1);
+    base = l - lane;
+    mask = WL == 32 ? kFull : (((1u << WL) - 1u) << base);
+  }
+  __device__ __forceinline__ uint32_t ballot(bool p) const {  // the group's bits, lane 0 = bit 0
+    return WL == 32 ? __ballot_sync(kFull, p) : (__ballot_sync(mask, p) >> base) & ((1u << WL) - 1u);
+  }
+};
+
 // The mutable per-lane state is packed into scalars (no register arrays
 // updated under a runtime index: nvcc would move those to local memory).
 struct LpiAnt {
@@ -1238,16 +1256,16 @@ __device__ __forceinline__ uint32_t lpi_rt(const LpiAnt &X, uint32_t q) {
   return ((q < 2 ? X.rtA : X.rtB) >> (16 * (q & 1))) & 0xFFFFu;
 }
 
-template <int Q>
-__device__ __forceinline__ void lpi_init(const SV &V, uint32_t *rem, uint32_t S, uint32_t lane, LpiAnt &X) {
-  for (uint32_t w = lane; w < V.nremw; w += 32) rem[w * S] = V.rem0[w];
+template <int WL, int Q>
+__device__ __forceinline__ void lpi_init(const SV &V, uint32_t *rem, uint32_t S, const LpiGrp<WL> &G, LpiAnt &X) {
+  for (uint32_t w = G.lane; w < V.nremw; w += WL) rem[w * S] = V.rem0[w];
   X.rdy = 0;
   X.npl = 0xFFFFFFFFu;  // (lanes past n never become ready)
   X.dkA = X.dkB = X.rtA = X.rtB = 0;
   X.s0 = X.s1 = X.s2 = X.s3 = 0;
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const uint32_t j = 32u * q + lane;
+    const uint32_t j = (uint32_t)WL * q + G.lane;
     if (j < V.n) {
       uint32_t c = 0;
       for (uint32_t k = V.pg_ptr[j]; k < V.pg_ptr[j + 1]; ++k) c += __popc(V.pg[k].y);
@@ -1255,25 +1273,25 @@ __device__ __forceinline__ void lpi_init(const SV &V, uint32_t *rem, uint32_t S,
       X.npl = (X.npl & ~(0xFFu << (8 * q))) | (c << (8 * q));
     }
   }
-  __syncwarp();
+  __syncwarp(G.mask);
 }
 
 // Commit of instruction j at cycle t (the warp-uniform counterpart of
 // commit()): scheduled / ready sets, RP update (R14, R15), last-use
 // bookkeeping of the registers j reads (the new last user's owner lane bumps
 // its count; dirty: its q bits), successors' readiness and (pass 2) ready times.
-template <int PASS, int Q>
-__device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t S, uint32_t lane, LpiAnt &X,
+template <int PASS, int WL, int Q>
+__device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t S, const LpiGrp<WL> &G, LpiAnt &X,
                                            uint32_t j, uint32_t t, uint32_t &live01, uint32_t &live23,
                                            uint32_t &prp01, uint32_t &prp23, uint32_t &dirty) {
-  const uint32_t qj = j >> 5, bj = 1u << (j & 31u);
+  const uint32_t qj = j >> 5, bj = 1u << (j & 31u);  // (the scheduled set's word and bit)
   X.s0 |= qj == 0 ? bj : 0u;
   if (Q > 1) X.s1 |= qj == 1 ? bj : 0u;
   if (Q > 2) {
     X.s2 |= qj == 2 ? bj : 0u;
     X.s3 |= qj == 3 ? bj : 0u;
   }
-  if (lane == (j & 31u)) X.rdy &= ~(1u << qj);
+  if (G.lane == j % WL) X.rdy &= ~(1u << (j / WL));
   const uint4 inf = V.info[j];
   uint32_t K = inf.y;  // static kills (single-use registers)
   const uint32_t m0 = inf.w >> 8, mc = inf.w & 0xFFu;
@@ -1286,20 +1304,20 @@ __device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t 
       uint32_t *p = rem + (m >> 1) * S;
       const uint32_t w = *p;
       const uint32_t left = (w >> sh) & 0xFFFFu;  // users left including j
-      __syncwarp();
-      if (lane == 0) *p = w - (1u << sh);
-      __syncwarp();
+      __syncwarp(G.mask);
+      if (G.lane == 0) *p = w - (1u << sh);
+      __syncwarp(G.mask);
       if (left == 1u) {
         K += 1u << (8 * c);
       } else if (left == 2u) {  // the first unscheduled user (in the list's order) remains
         const uint32_t k0 = V.cu_ptr[m], k1 = V.cu_ptr[m + 1];
-        for (uint32_t b = k0; b < k1; b += 32) {
-          const uint32_t kk = b + lane;
+        for (uint32_t b = k0; b < k1; b += WL) {
+          const uint32_t kk = b + G.lane;
           const uint32_t x = kk < k1 ? V.cu[kk] : 0u;
           const bool un = kk < k1 && !((lpi_sch(X, x >> 5) >> (x & 31u)) & 1u);
-          const uint32_t bal = __ballot_sync(kFull, un);
+          const uint32_t bal = G.ballot(un);
           if (bal) {
-            u = __shfl_sync(kFull, x, __ffs(bal) - 1);
+            u = __shfl_sync(G.mask, x, __ffs(bal) - 1, WL);
             break;
           }
         }
@@ -1309,8 +1327,8 @@ __device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t 
       if ((lpi_sch(X, pa >> 5) >> (pa & 31u)) & 1u) K += 1u << (8 * c);
       else u = pa;
     }
-    if (u != kInvalid && lane == (u & 31u)) {
-      const uint32_t qu = u >> 5, bump = 1u << (8 * c + 16 * (qu & 1u));
+    if (u != kInvalid && G.lane == u % WL) {
+      const uint32_t qu = u / WL, bump = 1u << (8 * c + 16 * (qu & 1u));
       if (qu < 2) X.dkA += bump;
       else X.dkB += bump;
       dirty |= 1u << qu;
@@ -1328,8 +1346,8 @@ __device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t 
   for (uint32_t q = s0; q < s1; ++q) {
     const uint32_t e = V.succ[q];
     const uint32_t v = e & 0x1FFFu;
-    if (lane == (v & 31u)) {
-      const uint32_t qv = v >> 5;
+    if (G.lane == v % WL) {
+      const uint32_t qv = v / WL;
       if (PASS == 2) {  // ready time = max over placed predecessors (t + latency < 2^16: host)
         const uint32_t r = (t + (e >> 16)) << (16 * (qv & 1u));
         if (qv < 2) X.rtA = __vmaxu2(X.rtA, r);
@@ -1345,8 +1363,8 @@ __device__ __forceinline__ void lpi_commit(const SV &V, uint32_t *rem, uint32_t 
 // ascending j = 32 q + lane whose inclusive prefix of scores exceeds
 // r = floor(R64 * sum / 2^64).  Scores are scanned as 16-bit halves (no
 // carries within a 32-lane chunk).  Returns kInvalid if none exceeds r.
-template <int Q>
-__device__ __forceinline__ uint32_t lpi_roulette(const uint32_t (&sc)[Q], uint32_t valid, uint32_t lane,
+template <int WL, int Q>
+__device__ __forceinline__ uint32_t lpi_roulette(const uint32_t (&sc)[Q], uint32_t valid, const LpiGrp<WL> &G,
                                                  uint64_t r64) {
   uint32_t plo[Q], phi[Q];
 #pragma unroll
@@ -1356,11 +1374,11 @@ __device__ __forceinline__ uint32_t lpi_roulette(const uint32_t (&sc)[Q], uint32
     phi[q] = s >> 16;
   }
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
+  for (int o = 1; o < WL; o <<= 1) {
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const uint32_t a = __shfl_up_sync(kFull, plo[q], o), b = __shfl_up_sync(kFull, phi[q], o);
-      if (lane >= (uint32_t)o) {
+      const uint32_t a = __shfl_up_sync(G.mask, plo[q], o, WL), b = __shfl_up_sync(G.mask, phi[q], o, WL);
+      if (G.lane >= (uint32_t)o) {
         plo[q] += a;
         phi[q] += b;
       }
@@ -1370,20 +1388,20 @@ __device__ __forceinline__ uint32_t lpi_roulette(const uint32_t (&sc)[Q], uint32
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     pre[q] = base + ((uint64_t)phi[q] << 16) + plo[q];
-    base += ((uint64_t)__shfl_sync(kFull, phi[q], 31) << 16) + __shfl_sync(kFull, plo[q], 31);
+    base += ((uint64_t)__shfl_sync(G.mask, phi[q], WL - 1, WL) << 16) + __shfl_sync(G.mask, plo[q], WL - 1, WL);
   }
   const uint64_t r = __umul64hi(r64, base);
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const uint32_t b = __ballot_sync(kFull, ((valid >> q) & 1u) && pre[q] > r);
-    if (b) return 32u * q + (__ffs(b) - 1);
+    const uint32_t b = G.ballot(((valid >> q) & 1u) && pre[q] > r);
+    if (b) return (uint32_t)WL * q + (__ffs(b) - 1);
   }
   return kInvalid;
 }
 
 // Warp argmax over (key desc, j asc): key = score + 1 of a candidate, 0 = none.
-template <int Q>
-__device__ __forceinline__ uint32_t lpi_argmax(const uint32_t (&key)[Q], uint32_t lane) {
+template <int WL, int Q>
+__device__ __forceinline__ uint32_t lpi_argmax(const uint32_t (&key)[Q], const LpiGrp<WL> &G) {
   uint32_t bk = 0, bq = 0;
 #pragma unroll
   for (int q = 0; q < Q; ++q)
@@ -1391,22 +1409,23 @@ __device__ __forceinline__ uint32_t lpi_argmax(const uint32_t (&key)[Q], uint32_
       bk = key[q];
       bq = q;
     }
-  const uint32_t mx = __reduce_max_sync(kFull, bk);
-  return __reduce_min_sync(kFull, (bk == mx && mx) ? 32u * bq + lane : kInvalid);
+  const uint32_t mx = __reduce_max_sync(G.mask, bk);
+  return __reduce_min_sync(G.mask, (bk == mx && mx) ? (uint32_t)WL * bq + G.lane : kInvalid);
 }
 
 // RP pass, one ant per warp (as ant_pass1: R1, R4, R19, R25-R27).
-template <int Q>
+template <int WL, int Q>
 __device__ __forceinline__ AntOut lpi_pass1(const SV &V, const uint16_t *__restrict__ tau, uint32_t *rem, uint32_t S,
                                             const uint32_t ant, const uint32_t iter, const RunCfg &cfg, uint16_t *rec,
                                             const uint32_t *coins, const uint32_t rec_stride) {
-  const uint32_t lane = threadIdx.x & 31u, n = V.n, L1 = V.L1;
+  const LpiGrp<WL> G;
+  const uint32_t n = V.n, L1 = V.L1;
   LpiAnt X;
-  lpi_init<Q>(V, rem, S, lane, X);
+  lpi_init<WL, Q>(V, rem, S, G, X);
   uint32_t e1[Q];  // eta1(j, sk(j) + d(j)) at the current d (R4)
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const uint32_t j = ::min(32u * q + lane, n - 1);
+    const uint32_t j = ::min((uint32_t)WL * q + G.lane, n - 1);
     e1[q] = V.eta1[j * L1];
   }
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
@@ -1417,24 +1436,24 @@ __device__ __forceinline__ AntOut lpi_pass1(const SV &V, const uint16_t *__restr
     uint32_t sc[Q], key[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const uint32_t j = ::min(32u * q + lane, n - 1);
+      const uint32_t j = ::min((uint32_t)WL * q + G.lane, n - 1);
       sc[q] = (uint32_t)trow[j] * e1[q];
       key[q] = ((X.rdy >> q) & 1u) ? sc[q] + 1u : 0u;
     }
-    uint32_t jstar = lpi_argmax<Q>(key, lane);
+    uint32_t jstar = lpi_argmax<WL, Q>(key, G);
     if (!exploit) {
       const uint4 x = philox(k, ant, iter, V.region_id, cfg.seed);
-      const uint32_t jr = lpi_roulette<Q>(sc, X.rdy, lane, ((uint64_t)x.y << 32) | x.x);
+      const uint32_t jr = lpi_roulette<WL, Q>(sc, X.rdy, G, ((uint64_t)x.y << 32) | x.x);
       if (jr != kInvalid) jstar = jr;
     }
     uint32_t dirty = 0;
-    lpi_commit<1, Q>(V, rem, S, lane, X, jstar, 0, live01, live23, prp01, prp23, dirty);
+    lpi_commit<1, WL, Q>(V, rem, S, G, X, jstar, 0, live01, live23, prp01, prp23, dirty);
     if (dirty) {
 #pragma unroll
       for (int q = 0; q < Q; ++q)
-        if ((dirty >> q) & 1u) e1[q] = V.eta1[(32u * q + lane) * L1 + sum_u8x4(lpi_dk(X, q))];
+        if ((dirty >> q) & 1u) e1[q] = V.eta1[((uint32_t)WL * q + G.lane) * L1 + sum_u8x4(lpi_dk(X, q))];
     }
-    if (rec && lane == 0) rec[(size_t)k * rec_stride] = (uint16_t)jstar;
+    if (rec && G.lane == 0) rec[(size_t)k * rec_stride] = (uint16_t)jstar;
     prev = jstar;
   }
   AntOut o;
@@ -1447,19 +1466,20 @@ __device__ __forceinline__ AntOut lpi_pass1(const SV &V, const uint16_t *__restr
 
 // ILP pass, one ant per warp (as ant_pass2 on the single-issue machine:
 // R19-R24, R41; stalls, the RP-feasible set, the prune).
-template <int Q>
+template <int WL, int Q>
 __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restrict__ tau, uint32_t *rem, uint32_t S,
                                             const uint32_t ant, const uint32_t iter, const RunCfg &cfg,
                                             const uint32_t tgt[4], uint32_t *prune_len, const bool prune,
                                             uint16_t *rec_o, uint32_t *rec_c, const uint32_t *coins,
                                             const uint32_t coin_t, const uint32_t rec_stride) {
-  const uint32_t lane = threadIdx.x & 31u, n = V.n;
+  const LpiGrp<WL> G;
+  const uint32_t n = V.n;
   LpiAnt X;
-  lpi_init<Q>(V, rem, S, lane, X);
+  lpi_init<WL, Q>(V, rem, S, G, X);
   uint32_t dx2[Q], dy[Q], e2[Q];  // defs (u16 x 2), static kills (u8 x 4), eta2
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const uint4 ds = V.ds[::min(32u * q + lane, n - 1)];
+    const uint4 ds = V.ds[::min((uint32_t)WL * q + G.lane, n - 1)];
     dx2[q] = lo_pair(ds.x);
     dy[q] = ds.y;
     e2[q] = ds.z & 0xFFFFu;
@@ -1475,10 +1495,10 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
   while (placed < n) {
     if (prune && ((++turn & 7u) == 0u)) {  // R24: winner-invariant prune
       uint32_t bl = 0;
-      if (lane == 0) bl = *(volatile uint32_t *)prune_len;
-      bl = __shfl_sync(kFull, bl, 0);
+      if (G.lane == 0) bl = *(volatile uint32_t *)prune_len;
+      bl = __shfl_sync(G.mask, bl, 0, WL);
       if (t + (n - placed) > bl) {
-        if (lane == 0) atomicAdd(prune_len + 1, 1u);
+        if (G.lane == 0) atomicAdd(prune_len + 1, 1u);
         o.cost = kInvalid;
         return o;
       }
@@ -1501,7 +1521,7 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
       const bool l = inr && rtq <= t;
       const bool s = inr && rtq > t;
       const bool f = l && all_le2(dx2[q], slack2 + K2);  // defs_c <= slack_c + kills_c (R21)
-      sc[q] = (uint32_t)trow[::min(32u * q + lane, n - 1)] * e2[q];
+      sc[q] = (uint32_t)trow[::min((uint32_t)WL * q + G.lane, n - 1)] * e2[q];
       key[q] = f ? sc[q] + 1u : 0u;
       fni |= f && all_le2(dx2[q], K2);    // max_c Delta_c <= 0
       sdec |= s && any_lt2(dx2[q], K2);   // min_c Delta_c < 0
@@ -1510,13 +1530,13 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
       feas |= (uint32_t)f << q;
       semi |= (uint32_t)s << q;
     }
-    const uint32_t min_s = __reduce_min_sync(kFull, mins);
-    if (!__any_sync(kFull, lat != 0u)) {  // necessary stall (L153): skip to the next ready time
+    const uint32_t min_s = __reduce_min_sync(G.mask, mins);
+    if (!__any_sync(G.mask, lat != 0u)) {  // necessary stall (L153): skip to the next ready time
       t = min_s;
       continue;
     }
-    const bool any_s = __any_sync(kFull, semi != 0u);
-    if (!__any_sync(kFull, feas != 0u)) {
+    const bool any_s = __any_sync(G.mask, semi != 0u);
+    if (!__any_sync(G.mask, feas != 0u)) {
       if (stall_en && any_s) {  // forced optional stall (L155, R22)
         kopt += min_s - t;
         t = min_s;
@@ -1527,7 +1547,7 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
     }
     uint4 x = make_uint4(0, 0, 0, 0);
     bool have_x = false;
-    if (stall_en && any_s && !__any_sync(kFull, fni) && __any_sync(kFull, sdec)) {  // discretionary (L157-L164)
+    if (stall_en && any_s && !__any_sync(G.mask, fni) && __any_sync(G.mask, sdec)) {  // discretionary (L157-L164)
       x = philox(t, ant, c2, V.region_id, cfg.seed);
       have_x = true;
       const uint32_t thr = (kopt + 1 >= 32) ? 0u : (0xFFFFFFFFu >> (kopt + 1));
@@ -1544,15 +1564,15 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
       const uint4 g = philox(t, 0x80000000u | group, c2, V.region_id, cfg.seed);
       exploit = (uint64_t)g.x < cfg.q0_t;
     }
-    uint32_t jstar = lpi_argmax<Q>(key, lane);
+    uint32_t jstar = lpi_argmax<WL, Q>(key, G);
     if (!exploit) {
       if (!have_x) x = philox(t, ant, c2, V.region_id, cfg.seed);
-      const uint32_t jr = lpi_roulette<Q>(sc, feas, lane, ((uint64_t)x.y << 32) | x.x);
+      const uint32_t jr = lpi_roulette<WL, Q>(sc, feas, G, ((uint64_t)x.y << 32) | x.x);
       if (jr != kInvalid) jstar = jr;
     }
     uint32_t dirty = 0;
-    lpi_commit<2, Q>(V, rem, S, lane, X, jstar, t, live01, live23, prp01, prp23, dirty);
-    if (rec_o && lane == 0) {
+    lpi_commit<2, WL, Q>(V, rem, S, G, X, jstar, t, live01, live23, prp01, prp23, dirty);
+    if (rec_o && G.lane == 0) {
       rec_o[(size_t)placed * rec_stride] = (uint16_t)jstar;
       rec_c[(size_t)placed * rec_stride] = t;
     }
@@ -1560,7 +1580,7 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
     prev = jstar;
     ++t;
   }
-  if (prune && lane == 0) atomicMin(prune_len, t);
+  if (prune && G.lane == 0) atomicMin(prune_len, t);
   o.prp01 = prp01;
   o.prp23 = prp23;
   o.len = t;
@@ -1746,9 +1766,9 @@ __global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? 
         rec = (uint16_t *)(A.ws + W.o_rec) + ai;
         rs1 = A.cfg.ants;
       }
-      if (qn <= 1) o = lpi_pass1<1>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
-      else if (qn <= 2) o = lpi_pass1<2>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
-      else o = lpi_pass1<4>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+      if (qn <= 1) o = lpi_pass1<32, 1>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+      else if (qn <= 2) o = lpi_pass1<32, 2>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
+      else o = lpi_pass1<32, 4>(V, tau, stbase, stride, ant, iter, A.cfg, rec, coins, rs1);
     } else {
       uint32_t tgt[4];
 #pragma unroll
@@ -1769,13 +1789,13 @@ __global__ void __launch_bounds__(LG == 32 ? kLpiMaxThreads : ((LEAN && MASK) ? 
         rs2 = A.cfg.ants;
       }
       if (qn <= 1)
-        o = lpi_pass2<1>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+        o = lpi_pass2<32, 1>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
                          coin_t, rs2);
       else if (qn <= 2)
-        o = lpi_pass2<2>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+        o = lpi_pass2<32, 2>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
                          coin_t, rs2);
       else
-        o = lpi_pass2<4>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
+        o = lpi_pass2<32, 4>(V, tau, stbase, stride, ant, iter, A.cfg, tgt, &rs.prune_len, prune, rec_o, rec_c, coins,
                          coin_t, rs2);
     }
   } else if constexpr (PASS == 1) {
@@ -2292,7 +2312,9 @@ __global__ void __launch_bounds__(256) k_finalize1(KArgs A, uint32_t iter) {
 // (word-mask scan, compact pass-2 layout, group coins drawn inline).
 // FW: 4-wide candidate scan (off by default: the small regions of a fused run
 // have too few candidates per step to fill a batch of four).
-template <bool FW>
+// WL > 0: every ant is a group of WL lanes (lane-per-instruction ants,
+// lpi_pass1/2; n <= 4 WL); else one thread per ant.
+template <bool FW, int WL = 0>
 __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
   const uint32_t r = blockIdx.x;
   const RegionDev *rd = A.regions + r;
@@ -2349,11 +2371,34 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
         }
       }
       __syncthreads();
-      if (tid < na) {  // (k_construct) ant tid
+      const uint32_t ai = WL ? tid / WL : tid;  // the ant of this thread
+      if (ai < na) {  // (k_construct) ant ai
         const Grp<1> G(tid);
-        const uint32_t ant = A.cfg.ant_base + tid;
+        const uint32_t ant = A.cfg.ant_base + ai;
         AntOut o;
-        if (pass == 1) {
+        if constexpr (WL > 0) {
+          const uint32_t qn = (n + WL - 1) / WL;
+          const uint32_t *cz = coins + (ant / gsz - g0) * cw;
+          if (pass == 1) {
+            if (qn <= 1) o = lpi_pass1<WL, 1>(V, tau, st + ai, na, ant, it, A.cfg, rec_o + ai, cz, na);
+            else if (qn <= 2) o = lpi_pass1<WL, 2>(V, tau, st + ai, na, ant, it, A.cfg, rec_o + ai, cz, na);
+            else o = lpi_pass1<WL, 4>(V, tau, st + ai, na, ant, it, A.cfg, rec_o + ai, cz, na);
+          } else {
+            uint32_t tgt[4];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) tgt[c] = rs.target[c];
+            const bool prune = !dump && !(A.cfg.flags & ACO_FLAG_NO_PRUNE) && !A.cfg.keys && !A.cfg.weighted;
+            if (qn <= 1)
+              o = lpi_pass2<WL, 1>(V, tau, st + ai, na, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + ai,
+                                   rec_c + ai, cz, cw * 32, na);
+            else if (qn <= 2)
+              o = lpi_pass2<WL, 2>(V, tau, st + ai, na, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + ai,
+                                   rec_c + ai, cz, cw * 32, na);
+            else
+              o = lpi_pass2<WL, 4>(V, tau, st + ai, na, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + ai,
+                                   rec_c + ai, cz, cw * 32, na);
+          }
+        } else if (pass == 1) {
           const St S = make_st<1, false, false>(st + tid, na, V);
           o = ant_pass1<1, true, FW>(V, tau, S, G, ant, it, A.cfg, false, rec_o + tid, coins + (ant / gsz - g0) * cw,
                                  RL{nullptr, 0, 0, 0, nullptr, nullptr}, na);
@@ -2366,15 +2411,18 @@ __global__ void __launch_bounds__(512, 1) k_fused(KArgs A) {
           o = ant_pass2<1, true, false, false, FW>(V, tau, S, G, ant, it, A.cfg, tgt, &rs.prune_len, prune, rec_o + tid,
                                                rec_c + tid, coins + (ant / gsz - g0) * cw, cw * 32, na);
         }
-        costs[tid] = o.cost;
-        recp[tid] = make_uint4(o.prp01, o.prp23, o.len, 0u);
-        if (dump && A.dump_cost) {
-          A.dump_cost[(((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.count + r) * na + tid] = o.cost;
-          const size_t base = ((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.dump_slice + W.o_dump + (size_t)tid * n;
-          if (A.dump_order && o.cost != kInvalid)
-            for (uint32_t k = 0; k < n; ++k) A.dump_order[base + k] = rec_o[k * na + tid];
-          if (A.dump_cycle && pass == 2 && o.cost != kInvalid)
-            for (uint32_t k = 0; k < n; ++k) A.dump_cycle[base + k] = rec_c[k * na + tid];
+        if (!WL || tid % WL == 0) {  // (the group's lane 0 recorded the schedule)
+          costs[ai] = o.cost;
+          recp[ai] = make_uint4(o.prp01, o.prp23, o.len, 0u);
+          if (dump && A.dump_cost) {
+            A.dump_cost[(((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.count + r) * na + ai] = o.cost;
+            const size_t base =
+                ((size_t)(pass - 1) * A.cfg.iterations + it) * A.cfg.dump_slice + W.o_dump + (size_t)ai * n;
+            if (A.dump_order && o.cost != kInvalid)
+              for (uint32_t k = 0; k < n; ++k) A.dump_order[base + k] = rec_o[k * na + ai];
+            if (A.dump_cycle && pass == 2 && o.cost != kInvalid)
+              for (uint32_t k = 0; k < n; ++k) A.dump_cycle[base + k] = rec_c[k * na + ai];
+          }
         }
       }
       __syncthreads();
@@ -2621,6 +2669,9 @@ int init_kernel_attrs() {
   big_smem(k_finalize1<2, true, true, true>);
   big_smem(k_post);
   big_smem(k_fused<false>);
+  big_smem(k_fused<false, 8>);
+  big_smem(k_fused<false, 16>);
+  big_smem(k_fused<false, 32>);
   big_smem(k_fused<true>);
 #define ACO_SEL(M) big_smem(k_select<1, M, false, false>); big_smem(k_select<2, M, false, false>); \
   big_smem(k_select<2, M, true, false>); big_smem(k_select<2, M, false, true>); big_smem(k_select<2, M, true, true>);
@@ -2701,8 +2752,15 @@ int launch_post(LaunchCtx &L, uint32_t smem) {
   return check(__func__);
 }
 
-int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem) {
+int launch_fused(LaunchCtx &L, uint32_t threads, uint32_t smem, uint32_t wl) {
   if (!L.cfg.count) return 0;
+  if (wl) {  // lane-per-instruction ants of wl lanes
+    if (wl == 8) k_fused<false, 8><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
+    else if (wl == 16) k_fused<false, 16><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
+    else k_fused<false, 32><<<L.cfg.count, threads, smem, (cudaStream_t)L.stream>>>(kargs(L));
+    L.launches++;
+    return check(__func__);
+  }
   static const int fw = [] {  // (measured, C1: 1-wide 0.654 ms, 4-wide 0.702 ms: few candidates per step)
     const char *e = getenv("ACO_FUSED_WIDE");
     return e ? atoi(e) : 0;

@@ -132,3 +132,37 @@ def test_lpi_equals_group_kernels(lpi_forced):
         for k in ("length", "prp", "trace_hash", "iters1", "iters2", "cost_rp"):
             assert x[k] == y[k], k
         assert np.array_equal(x["order"], y["order"]) and np.array_equal(x["cycle"], y["cycle"])
+
+
+FUSED, FUSED_LPI = 1 << 13, 1 << 14
+
+
+@pytest.mark.parametrize("wl,sizes,ants", [(8, (10, 25, 32), 21), (16, (40, 64), 16), (32, (100, 128), 8), (8, (7,), 2)])
+def test_lpi_fused_every_ant(lpi_forced, wl, sizes, ants):
+    """The fused single-block run with lane-per-instruction ants of WL lanes
+    (the smallest of 8 / 16 / 32 with n <= 4 WL; an option, ACO_FUSED_LPI,
+    forced here): every ant bit-exact in dump mode."""
+    regs = [I.gen_region(n, 7900 + n + wl, "mixed" if i % 2 else "unit") for i, n in enumerate(sizes)]
+    ids = [60 + i for i in range(len(regs))]
+    # (the fused run: <= 512 ants in the batch, WL x ants <= 512 threads; 2 x 8 lanes: a partial warp)
+    p = I.Params(ants=ants, iterations=4, seed=wl, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    assert s.variants() == [FUSED | FUSED_LPI * {8: 1, 16: 2, 32: 3}[wl]], s.variants()
+    dump_parity(s, regs, ids, p)
+
+
+@pytest.mark.parametrize("kind", ["both", "paper", "weighted", "pass1", "pass2"])
+def test_lpi_fused_modes(lpi_forced, kind):
+    """Config 1's shape (FIX10-A, 64 ants, 20 iterations) through the fused
+    lane-per-instruction run in every pass mode and policy: final results
+    equal the oracle's (production mode: record, prune)."""
+    import dataclasses
+    x = I.fix10a()
+    base = I.Params(ants=64, iterations=20, seed=3, cost_mode=0)
+    p = {"both": base, "paper": I.paper_policy(base), "weighted": dataclasses.replace(base, passes=4, ws_weight=2),
+         "pass1": dataclasses.replace(base, passes=1), "pass2": dataclasses.replace(base, passes=2)}[kind]
+    s = _sched()
+    s.load([x], [7]).run(p)
+    assert s.variants() == [FUSED | FUSED_LPI], s.variants()
+    compare_results(s.results()[0], O.schedule(x, 7, I.GFX906, p), kind)
