@@ -14,6 +14,11 @@
 // Exploit/explore is a coin per group of 64 ants (L198): a warp takes one
 // branch in pass 1.  Candidates are scored four at a time so that their
 // shared-memory loads overlap (ILP).
+// Latency-bound batches (few ants in total: config 2) instead run
+// lane-per-instruction ants (lpi_pass1/2): one warp per ant, every candidate
+// on its own lane, the ant's state in registers.  Huge regions (n > 1024)
+// keep the per-ant state in shared memory and read the image and tau through
+// L1 (or, when even that does not fit, through L1/L2 from the workspace).
 //
 // Per pass and iteration (L135-L139):
 //   k_construct : every ant builds a schedule and writes its cost (K1a); in
