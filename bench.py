@@ -248,12 +248,18 @@ def build_fingerprint():
 
 def ncu_evidence(workload: str):
     """DRAM traffic and issue-slot figures of the construct launches from the
-    committed ncu --set full capture (profiles/r02_traffic.json) -- used only
-    when that capture profiled this very build (same source fingerprint)."""
-    try:
-        with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
-            tj = json.load(f)
-    except Exception:
+    committed ncu --set full capture (profiles/r03_traffic.json, else the
+    round-2 one) -- used only when that capture profiled this very build
+    (same source fingerprint)."""
+    tj = None
+    for name in ("r03_traffic.json", "r02_traffic.json"):
+        try:
+            with open(os.path.join(ROOT, "profiles", name)) as f:
+                tj = json.load(f)
+            break
+        except Exception:
+            continue
+    if tj is None:
         return None, None, "no committed capture"
     if workload != "c3":
         return None, None, "capture is of the c3 batch"
@@ -494,17 +500,21 @@ def main(argv=None):
     sum_n = sum(int(h.offsets[-1]) for h in hosts)
     outs = [(np.zeros(max(1, int(h.offsets[-1])), np.uint32), np.zeros(max(1, int(h.offsets[-1])), np.uint32))
             for h in hosts]
+    e2e_phase = []  # (load, run, results) host wall-clock ms per step (diagnostic split of e2e)
     for _ in range(max(1, args.e2e_steps)):
         barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for s, b, h in zip(scheds, batches, hosts):
             s.load(b.regs, b.ids, batch=h)
+        t1 = time.perf_counter()
         run()
+        t2 = time.perf_counter()
         for s, b, (o, c) in zip(scheds, batches, outs):
             if b.regs:
                 s.results_raw(0, len(b.regs), o, c)
         e2e_ms.append((time.perf_counter() - t0) * 1000.0)
+        e2e_phase.append(((t1 - t0) * 1000.0, (t2 - t1) * 1000.0, (time.perf_counter() - t2) * 1000.0))
     h2d = sum(int(s.arena.numel()) for s in scheds if s.arena is not None)
     n_regs = sum(len(b.regs) for b in batches)
     d2h = int(n_regs * 72 + 4 * 2 * sum_n)  # aco_result + orders + cycles
@@ -650,7 +660,12 @@ def main(argv=None):
             "pruned_pass2_ant_frac": round(prune_frac, 4),
             "gpu_launches": int(launches),
             "e2e": {"value": round(e2e_value, 1), "unit": METRIC, "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "ms_per_step": round(float(e.item()), 3)},
+                    "d2h_bytes_per_step": d2h, "ms_per_step": round(float(e.item()), 3),
+                    "host_split_ms": dict(zip(("load", "run", "results"),
+                                              [round(float(x), 3) for x in np.median(np.array(e2e_phase), axis=0)])),
+                    "host_split_note": "rank 0 wall clock around the public calls (load: host preprocessing + "
+                                       "H2D; run: planning + launch enqueue (asynchronous); results: waits for "
+                                       "the device, then D2H)"},
             "clocks": clocks, "roofline": roof, "cpu_baseline": cpu, "parity": parity,
             "schedule_quality": schedule_quality(res) if args.workload != "c4" or not colony else None,
         }
