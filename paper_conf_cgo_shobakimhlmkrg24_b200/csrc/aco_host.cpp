@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <atomic>
 #include <cmath>
 #include <cstdio>
@@ -185,8 +186,8 @@ struct aco_ctx_s {
     }
   }
   // Copy `bytes` from host `src` to device `dst` through pinned staging slot k.
-  aco_status staged_h2d(int k, void *dst, const void *src, size_t bytes, cudaStream_t s) {
-    if (!bytes) return ACO_OK;
+  // Pinned staging slot k with at least `bytes` (after its previous copy completed).
+  aco_status pinned(int k, size_t bytes, unsigned char **out) {
     if (pin_ev[k]) {
       if (cudaEventSynchronize(pin_ev[k]) != cudaSuccess) return ACO_E_CUDA;
     } else if (cudaEventCreateWithFlags(&pin_ev[k], cudaEventDisableTiming) != cudaSuccess) {
@@ -200,10 +201,21 @@ struct aco_ctx_s {
       if (cudaMallocHost(&pin[k], want) != cudaSuccess) return ACO_E_CUDA;
       pin_bytes[k] = want;
     }
-    std::memcpy(pin[k], src, bytes);
+    *out = (unsigned char *)pin[k];
+    return ACO_OK;
+  }
+  // H2D of the first `bytes` of pinned slot k (filled by the caller)
+  aco_status pinned_h2d(int k, void *dst, size_t bytes, cudaStream_t s) {
     if (cudaMemcpyAsync(dst, pin[k], bytes, cudaMemcpyHostToDevice, s) != cudaSuccess) return ACO_E_CUDA;
     if (cudaEventRecord(pin_ev[k], s) != cudaSuccess) return ACO_E_CUDA;
     return ACO_OK;
+  }
+  aco_status staged_h2d(int k, void *dst, const void *src, size_t bytes, cudaStream_t s) {
+    if (!bytes) return ACO_OK;
+    unsigned char *p = nullptr;
+    if (aco_status st = pinned(k, bytes, &p)) return st;
+    std::memcpy(p, src, bytes);
+    return pinned_h2d(k, dst, bytes, s);
   }
   cudaEvent_t next_event() {
     if (ev_used == ev_pool.size()) {
@@ -662,6 +674,8 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
       if (ids[i] == ids[i - 1]) return ACO_E_ARG;
   }
   // host preprocessing of the regions in parallel (independent per region)
+  static const bool dbg_load = getenv("ACO_DEBUG_LOAD") != nullptr;
+  const auto t_0 = std::chrono::steady_clock::now();
   std::vector<Prepped> P(count);
   std::vector<aco_status> stv(count, ACO_OK);
   {
@@ -682,15 +696,15 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   }
   for (uint32_t i = 0; i < count; ++i)
     if (stv[i] != ACO_OK) return stv[i];
-  std::vector<unsigned char> blob(align16(sizeof(RegionDev) * (size_t)count + 16), 0);
+  const auto t_1 = std::chrono::steady_clock::now();
+  // arena layout: RegionDev[count], then every image at a 16-byte aligned offset
+  const size_t table = align16(sizeof(RegionDev) * (size_t)count + 16);
+  size_t total = table;
   for (uint32_t i = 0; i < count; ++i) {
-    RegionDev &R = P[i].rd;
-    R.o_image = align16(blob.size());
-    blob.resize(R.o_image + P[i].image.size(), 0);
-    std::memcpy(blob.data() + R.o_image, P[i].image.data(), P[i].image.size());
-    std::memcpy(blob.data() + sizeof(RegionDev) * (size_t)i, &R, sizeof(RegionDev));
+    P[i].rd.o_image = align16(total);
+    total = P[i].rd.o_image + P[i].image.size();
   }
-  const size_t need = align256(blob.size());
+  const size_t need = align256(total);
   if (arena_needed) *arena_needed = need;
   if (!d_arena && getenv("ACO_DEBUG_PLAN")) {  // debug: keep host metadata for a sizing-only plan
     ctx->count = count;
@@ -705,8 +719,32 @@ aco_status aco_load_regions(aco_ctx ctx, const aco_region_desc *regions, uint32_
   if (!d_arena) return ACO_OK;
   if (arena_bytes < need) return ACO_E_WORKSPACE;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return ACO_E_CUDA;
-  aco_status hs = ctx->staged_h2d(0, d_arena, blob.data(), blob.size(), (cudaStream_t)cuda_stream);
-  if (hs != ACO_OK) return hs;
+  {  // assemble the arena directly in the pinned staging buffer (threads), one H2D
+    unsigned char *pin = nullptr;
+    if (aco_status st = ctx->pinned(0, total, &pin)) return st;
+    std::memset(pin, 0, table);
+    for (uint32_t i = 0; i < count; ++i) std::memcpy(pin + sizeof(RegionDev) * (size_t)i, &P[i].rd, sizeof(RegionDev));
+    const uint32_t hw = std::max(1u, std::thread::hardware_concurrency());
+    const uint32_t nt = std::min<uint32_t>(hw, std::max<uint32_t>(1, count / 64));
+    auto fill = [&](uint32_t t) {
+      for (uint32_t i = t; i < count; i += nt) {
+        const size_t o = P[i].rd.o_image, e = i + 1 < count ? P[i + 1].rd.o_image : total;
+        std::memcpy(pin + o, P[i].image.data(), P[i].image.size());
+        std::memset(pin + o + P[i].image.size(), 0, e - o - P[i].image.size());  // (alignment padding)
+      }
+    };
+    std::vector<std::thread> th;
+    for (uint32_t t = 1; t < nt; ++t) th.emplace_back(fill, t);
+    fill(0);
+    for (auto &t : th) t.join();
+    if (aco_status st = ctx->pinned_h2d(0, d_arena, total, (cudaStream_t)cuda_stream)) return st;
+  }
+  if (dbg_load) {
+    const auto t_2 = std::chrono::steady_clock::now();
+    fprintf(stderr, "[aco load] prep %.2f ms, arena assembly + H2D enqueue %.2f ms (%zu bytes)\n",
+            std::chrono::duration<double, std::milli>(t_1 - t_0).count(),
+            std::chrono::duration<double, std::milli>(t_2 - t_1).count(), total);
+  }
   ctx->count = count;
   ctx->regions.resize(count);
   ctx->inst_off.assign(count + 1, 0);

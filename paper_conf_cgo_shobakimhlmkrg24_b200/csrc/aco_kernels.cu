@@ -1481,13 +1481,20 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
   const uint32_t n = V.n;
   LpiAnt X;
   lpi_init<WL, Q>(V, rem, S, G, X);
-  uint32_t dx2[Q], dy[Q], e2[Q];  // defs (u16 x 2), static kills (u8 x 4), eta2
+  uint32_t dx2[Q], dy[Q], e2[Q], K2[Q];  // defs (u16 x 2), static kills (u8 x 4), eta2, kills (u16 x 2)
+  uint32_t fnim = 0, sdm = 0;  // bit q: max_c Delta_c <= 0 / min_c Delta_c < 0 for j_q (change only with its kills)
+  auto kill_tests = [&](int q) {
+    K2[q] = lo_pair(dy[q] + lpi_dk(X, q));  // kills per class (R14)
+    fnim = (fnim & ~(1u << q)) | ((all_le2(dx2[q], K2[q]) ? 1u : 0u) << q);
+    sdm = (sdm & ~(1u << q)) | ((any_lt2(dx2[q], K2[q]) ? 1u : 0u) << q);
+  };
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     const uint4 ds = V.ds[::min((uint32_t)WL * q + G.lane, n - 1)];
     dx2[q] = lo_pair(ds.x);
     dy[q] = ds.y;
     e2[q] = ds.z & 0xFFFFu;
+    kill_tests(q);
   }
   uint32_t live01 = V.livein01, live23 = V.livein23, prp01 = live01, prp23 = live23;
   const uint32_t group = ant / cfg.group_size;
@@ -1508,33 +1515,26 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
         return o;
       }
     }
-    uint32_t slack = 0;  // slack_c = target_c - live_c, saturated to a byte (R21)
-    {
-      const uint32_t lv[4] = {live01 & 0xFFFFu, live01 >> 16, live23 & 0xFFFFu, live23 >> 16};
-#pragma unroll
-      for (int c = 0; c < 4; ++c) slack |= ::min(tgt[c] - lv[c], 255u) << (8 * c);
-    }
-    const uint32_t slack2 = lo_pair(slack);
+    // slack_c = target_c - live_c saturated to a byte (R21), classes 0 and 1 as u16 x 2
+    const uint32_t slack2 = ::min(tgt[0] - (live01 & 0xFFFFu), 255u) | (::min(tgt[1] - (live01 >> 16), 255u) << 16);
     const uint16_t *trow = tau + prev * n;
     uint32_t sc[Q], key[Q], lat = 0, feas = 0, semi = 0, mins = kInvalid;
-    bool fni = false, sdec = false;
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       const bool inr = (X.rdy >> q) & 1u;
-      const uint32_t K2 = lo_pair(dy[q] + lpi_dk(X, q));  // kills per class (R14)
       const uint32_t rtq = lpi_rt(X, q);
       const bool l = inr && rtq <= t;
       const bool s = inr && rtq > t;
-      const bool f = l && all_le2(dx2[q], slack2 + K2);  // defs_c <= slack_c + kills_c (R21)
+      const bool f = l && all_le2(dx2[q], slack2 + K2[q]);  // defs_c <= slack_c + kills_c (R21)
       sc[q] = (uint32_t)trow[::min((uint32_t)WL * q + G.lane, n - 1)] * e2[q];
       key[q] = f ? sc[q] + 1u : 0u;
-      fni |= f && all_le2(dx2[q], K2);    // max_c Delta_c <= 0
-      sdec |= s && any_lt2(dx2[q], K2);   // min_c Delta_c < 0
       if (s) mins = ::min(mins, rtq);
       lat |= (uint32_t)l << q;
       feas |= (uint32_t)f << q;
       semi |= (uint32_t)s << q;
     }
+    const bool fni = (feas & fnim) != 0u;   // a feasible candidate with max_c Delta_c <= 0
+    const bool sdec = (semi & sdm) != 0u;   // a semi-ready one with min_c Delta_c < 0
     const uint32_t min_s = __reduce_min_sync(G.mask, mins);
     if (!__any_sync(G.mask, lat != 0u)) {  // necessary stall (L153): skip to the next ready time
       t = min_s;
@@ -1577,6 +1577,11 @@ __device__ __forceinline__ AntOut lpi_pass2(const SV &V, const uint16_t *__restr
     }
     uint32_t dirty = 0;
     lpi_commit<2, WL, Q>(V, rem, S, G, X, jstar, t, live01, live23, prp01, prp23, dirty);
+    if (dirty) {
+#pragma unroll
+      for (int q = 0; q < Q; ++q)
+        if ((dirty >> q) & 1u) kill_tests(q);
+    }
     if (rec_o && G.lane == 0) {
       rec_o[(size_t)placed * rec_stride] = (uint16_t)jstar;
       rec_c[(size_t)placed * rec_stride] = t;
