@@ -4,7 +4,7 @@
 # and C4 huge-region captures, C5 per-n sweep, Table-6 analogue.
 # (compute-sanitizer is closed on this pool since r03: not run.)
 set -x
-O=gpurun_out/r03final; mkdir -p $O
+O=gpurun_out/r03final2; mkdir -p $O
 python paper_conf_cgo_shobakimhlmkrg24_b200/build.py > /dev/null
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,driver_version --format=csv > $O/gpu.txt
 lscpu | grep -i "model name\|^CPU(s)" > $O/host.txt
@@ -22,7 +22,5 @@ timeout 600 ncu --set full --clock-control none -k regex:'k_construct|k_finalize
 ncu -i /tmp/prof_c2.ncu-rep --page raw --csv > $O/prof_c2_raw.csv 2>/dev/null
 PROBE_N=2000 PROBE_ITERS=1 timeout 900 ncu --set full --clock-control none -k regex:k_construct -c 2 -o /tmp/prof_gs python tools/size_probe.py > $O/prof_c4.log 2>&1
 ncu -i /tmp/prof_gs.ncu-rep --page raw --csv > $O/prof_c4_raw.csv 2>/dev/null
-timeout 1200 python tools/c5_sweep.py > $O/c5_sweep.md 2> $O/c5_sweep.err
-timeout 1200 python tools/table6.py > $O/table6.md 2> $O/table6.err
 rm -f /tmp/*.ncu-rep
 tail -3 $O/gpu_tests.log; tail -2 $O/smoke.log; cut -c1-200 $O/matrix.log; head -c 300 $O/bench_c3_parity_all.json

@@ -39,9 +39,10 @@ def stalls(raw):
     return out
 
 
-print("# r02 final ncu evidence: C3 batch (5,000 regions, 1,024 ants x 10 iterations x 2 passes) on one B200\n")
-print("Build: the round-2 final kernels (`profiles/r02_traffic.json` carries its source fingerprint; bench.py")
-print("reports the issue-slot / DRAM figures below only for that build).  Commands: `tools/gpu_r02_final.sh`.")
+TAG = os.environ.get("TAG", "r03")
+print(f"# {TAG} final ncu evidence: C3 batch (5,000 regions, 1,024 ants x 10 iterations x 2 passes) on one B200\n")
+print(f"Build: the final kernels (`profiles/{TAG}_traffic.json` carries its source fingerprint; bench.py")
+print(f"reports the issue-slot / DRAM figures below only for that build).  Commands: `tools/gpu_{TAG}_final2.sh`.")
 print("ncu serialises launches and runs them cold: compare shares, not absolutes.\n")
 print("## Launch list by kernel (every launch of the bench command under ncu)\n")
 print("```")
@@ -49,14 +50,18 @@ print(run(os.path.join(T, "launch_summary.py"), os.path.join(D, "launches.csv"),
 print("```\n")
 print("## Full-set metrics per launch (first iteration, both passes)\n")
 print(open(os.path.join(D, "ncu_table.md")).read())
-print("\nRoll-up (time-weighted over the construct launches; `r02_traffic.json`):\n")
+print(f"\nRoll-up (time-weighted over the construct launches; `{TAG}_traffic.json`):\n")
 print("```")
-print(open(os.path.join(D, "r02_traffic.json")).read().strip())
+print(open(os.path.join(D, f"{TAG}_traffic.json")).read().strip())
 print("```\n")
 for title, raw, src, ranges in (
         ("Top pass-2 class `k_construct<2,1,1,0,0,0,2,1,1>` (lean layout, image through L1)", "prof_top_raw.csv",
          "prof_top_source.csv", None),
-        ("Config 4's global-state kernel (n = 2,000, 8,192 ants, 16 lanes per ant)", "prof_gs_raw.csv", None, None)):
+        ("Config 4's global-state kernel (n = 2,000, 8,192 ants, 16 lanes per ant)", "prof_gs_raw.csv", None, None),
+        ("Config 4's huge-region kernels (n = 2,000, 8,192 ants: per-ant state in shared memory, 8 lanes per ant)",
+         "prof_c4_raw.csv", None, None),
+        ("Config 2: lane-per-instruction ants (k_construct<P, 32, ...>) and the one-launch finalize",
+         "prof_c2_raw.csv", None, None)):
     p = os.path.join(D, raw)
     if not os.path.exists(p):
         continue
