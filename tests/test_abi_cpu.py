@@ -221,3 +221,56 @@ def test_planner_lane_per_instruction_for_config2(lib):
         assert sum(b for p, b, a, l in c2 if p == pass_ and l == 32) >= 128, c2
     v3, _ = _plan(["--workload", "c3", "--regions", "400"])
     assert not any(c & (1 << 10) for c in v3[0])
+
+
+def _variants_of(lib, machine, regions, p):
+    """Construct variants a run would launch (sizing calls only, no CUDA)."""
+    from paper_conf_cgo_shobakimhlmkrg24_b200.api import HostBatch, machine_struct, params_struct
+    os.environ["ACO_DEBUG_PLAN"] = "1"
+    try:
+        m = machine_struct(machine)
+        ctx = C.c_void_p()
+        assert lib.aco_create(0, C.byref(m), C.byref(ctx)) == 0
+        b = HostBatch(regions, list(range(len(regions))))
+        need = C.c_size_t(0)
+        assert lib.aco_load_regions(ctx, b.descs, len(regions), None, 0, C.byref(need), None) == 0
+        ps = params_struct(p)
+        ws = C.c_size_t(0)
+        assert lib.aco_schedule_batch(ctx, C.byref(ps), None, 0, C.byref(ws), None) == 0
+        cnt = C.c_uint32(0)
+        assert lib.aco_last_variants(ctx, None, 0, C.byref(cnt)) == 0
+        buf = (C.c_uint32 * max(1, cnt.value))()
+        assert lib.aco_last_variants(ctx, buf, cnt.value, C.byref(cnt)) == 0
+        lib.aco_destroy(ctx)
+        return [int(buf[i]) for i in range(cnt.value)]
+    finally:
+        del os.environ["ACO_DEBUG_PLAN"]
+
+
+def test_planner_lane_per_instruction_eligibility(lib):
+    """Lane-per-instruction ants (variant bit 10) only where their
+    arithmetic holds: n <= 128, <= 2 register classes, single issue in pass 2
+    (pass 1 ignores the machine model, R19), no mixed heuristics (R43), a
+    batch with few ants in total."""
+    import dataclasses
+    lpi = 1 << 10
+    p = I.Params(ants=1024, iterations=3, seed=1)
+    r100 = [I.gen_region(100, 11)]
+    v = _variants_of(lib, I.GFX906, r100, p)
+    assert v and all(c & lpi for c in v), v
+    # dual issue: pass 1 keeps the lane-per-instruction ants, pass 2 does not
+    v = _variants_of(lib, I.DUAL_ISSUE, r100, p)
+    assert any(c & lpi and not c & 256 for c in v) and not any(c & lpi and c & 256 for c in v), v
+    # three register classes, mixed heuristics, n = 129, many ants: never
+    m3 = I.Machine(n_classes=3, steps=I.GFX906.steps + ((10, 20),), perp_limit=(24, 80, 10, 0))
+    assert not any(c & lpi for c in _variants_of(lib, m3, r100, p))
+    assert not any(c & lpi for c in _variants_of(lib, I.GFX906, r100, dataclasses.replace(p, heur_mix=1)))
+    assert not any(c & lpi for c in _variants_of(lib, I.GFX906, [I.gen_region(129, 12)], p))
+    assert not any(c & lpi for c in _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(4)], p))
+    # ... unless forced (tests), which still respects eligibility
+    os.environ["ACO_LPI"] = "2"
+    try:
+        v = _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(4)] + [I.gen_region(300, 20)], p)
+    finally:
+        del os.environ["ACO_LPI"]
+    assert any(c & lpi for c in v) and any(not c & lpi for c in v), v
