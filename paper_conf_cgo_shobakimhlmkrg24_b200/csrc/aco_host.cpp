@@ -994,7 +994,11 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   // ACO_LPI: 0 off, 1 auto (default), 2 every eligible region (tests)
   uint32_t lpi_mode = 1;
   if (const char *e = getenv("ACO_LPI")) lpi_mode = (uint32_t)atoi(e);
-  uint64_t lpi_max_ants = 148ull * 16;  // ants (= warps) in the whole batch
+  // ants (= warps) in the whole batch; measured crossover (tools/lpi_crossover.py,
+  // profiles/r03_lpi_crossover.md): k regions of n = 30-128 with 1,024 ants
+  // each, lane-per-instruction faster at 4,096 ants (n = 100: 6.4 vs 7.7 ms),
+  // slower at 8,192 (11.2 vs 8.0 ms)
+  uint64_t lpi_max_ants = 148ull * 32;
   if (const char *e = getenv("ACO_LPI_ANTS")) lpi_max_ants = strtoull(e, nullptr, 10);
   const bool lpi_batch = lpi_mode == 2 || (lpi_mode == 1 && (uint64_t)A * count <= lpi_max_ants);
   // huge regions (n > 1024): per-ant state in shared memory, image and tau

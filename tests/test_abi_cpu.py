@@ -266,11 +266,11 @@ def test_planner_lane_per_instruction_eligibility(lib):
     assert not any(c & lpi for c in _variants_of(lib, m3, r100, p))
     assert not any(c & lpi for c in _variants_of(lib, I.GFX906, r100, dataclasses.replace(p, heur_mix=1)))
     assert not any(c & lpi for c in _variants_of(lib, I.GFX906, [I.gen_region(129, 12)], p))
-    assert not any(c & lpi for c in _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(4)], p))
+    assert not any(c & lpi for c in _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(5)], p))
     # ... unless forced (tests), which still respects eligibility
     os.environ["ACO_LPI"] = "2"
     try:
-        v = _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(4)] + [I.gen_region(300, 20)], p)
+        v = _variants_of(lib, I.GFX906, [I.gen_region(100, 13 + k) for k in range(5)] + [I.gen_region(300, 20)], p)
     finally:
         del os.environ["ACO_LPI"]
     assert any(c & lpi for c in v) and any(not c & lpi for c in v), v
