@@ -1016,6 +1016,17 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
   uint32_t huge_k = 2, huge_waves = 1, huge_exact = 1, huge_lanes[2] = {8, 8};
   uint64_t huge_smem_max = 0;
   if (const char *e = getenv("ACO_HUGE_LANES")) sscanf(e, "%u,%u", &huge_lanes[0], &huge_lanes[1]);
+  // In a batch with few ants in total (<= 148 x 512: config 5, not config 3)
+  // regions above huge_min_n instructions take the huge-region kernels even
+  // when a shared-memory shape exists: with few regions in flight the
+  // standard blocks leave the SMs latency-starved (tools/gpu_r03s.sh / r03t.sh:
+  // C5 1773 -> 1363 ms, its n = 500 row 155 -> 75 ms and n = 1,000 row
+  // 602 -> 225 ms; forcing it on config 3 costs 690 -> 1104 ms)
+  uint32_t huge_min_n = 400;
+  if (const char *e = getenv("ACO_HUGE_MIN_N")) huge_min_n = (uint32_t)atoi(e);
+  uint64_t huge_few_ants = 148ull * 512;
+  if (const char *e = getenv("ACO_HUGE_FEW_ANTS")) huge_few_ants = strtoull(e, nullptr, 10);
+  const bool huge_few = (uint64_t)A * count <= huge_few_ants;
   if (const char *e = getenv("ACO_HUGE_K")) huge_k = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_HUGE_WAVES")) huge_waves = (uint32_t)atoi(e);
   if (const char *e = getenv("ACO_HUGE_EXACT")) huge_exact = (uint32_t)atoi(e);
@@ -1166,7 +1177,10 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
     // (measured: n = 2,000 pass 1, 1 warp/SM in smem, 9x slower).
     // (not for a spread shape: there few resident ants per SM is the point)
     if (sh.apb != 0 && !spread && sh.resident < gs_min_threads[pass - 1]) sh.apb = 0;
-    if (sh.apb == 0 && huge_smem && R.n > 1024 && !t32 && !P.nc4 && !(rl1 && pass == 1)) {
+    const bool force_huge = huge_few && huge_min_n < 1024u && R.n > huge_min_n;
+    const Shape sh_std = sh;
+    if ((sh.apb == 0 || force_huge) && huge_smem && (R.n > 1024 || force_huge) && !t32 && !P.nc4 &&
+        !(rl1 && pass == 1)) {
       // Huge regions with the per-ant state in SHARED memory, the image and
       // tau through L1, the global-state lane count and the 4-wide strided
       // scan; pass 2 in the lean layout when its latencies allow -- taken
@@ -1197,6 +1211,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         W = Wh;
         break;
       }
+      if (!q.huge) sh = sh_std;
     }
     if (sh.apb == 0) {  // does not fit shared memory: global-state kernels
       // all ants are resident (state in the workspace); 16 lanes per ant
@@ -1277,7 +1292,7 @@ aco_status make_plan(aco_ctx ctx, const aco_params *p, uint32_t ant_base, void *
         gs[r] = 1;
         gs_words[r] = std::max(gs_words[r], (q.W + 3u) & ~3u);  // (ant-major rows padded to 16 B)
       }
-      const bool mask = R.n <= 1024 && !g;
+      const bool mask = R.n <= 1024 && !g && !q.huge;  // (the huge-region variants scan strided words)
       if (g) sh.ig = false;
       // global-state kernels: 4-wide candidate scan over strided words (not in
       // the u32-cycle / 3-4 class instantiations), gs_wide_lanes above

@@ -147,3 +147,18 @@ def test_fused_run_equals_oracle_and_multilaunch(torch_cuda, monkeypatch, kind):
     assert (1 << 13) not in m.variants()
     for k, g in enumerate(m.results()):
         compare_results(g, O.schedule(regs[k], ids[k], I.GFX906, p), f"{kind} multi-launch region {k}")
+
+
+def test_huge_kernels_for_mid_size_regions_of_few_ant_batches(torch_cuda, monkeypatch):
+    """Batches with few ants in total (config 5) run regions above 400
+    instructions on the huge-region kernels (strided-word scan, n <= 1024
+    included): every ant bit-exact."""
+    monkeypatch.setenv("ACO_HUGE_MIN_N", "400")
+    regs = [I.gen_region(n, 9500 + n, "mixed" if n % 2 else "unit") for n in (450, 800, 1000)]
+    ids = [41, 42, 43]
+    p = I.Params(ants=64, iterations=2, seed=17, stall_mod=2)
+    s = _sched()
+    s.load(regs, ids).run(p, no_prune=True, dump=True)
+    codes = s.variants()
+    assert any((c & (1 << 11)) and not (c & (1 << 5)) for c in codes), codes  # huge (image via L1, no word mask)
+    dump_parity(s, regs, ids, p)
