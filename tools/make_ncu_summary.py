@@ -42,7 +42,7 @@ def stalls(raw):
 TAG = os.environ.get("TAG", "r03")
 print(f"# {TAG} final ncu evidence: C3 batch (5,000 regions, 1,024 ants x 10 iterations x 2 passes) on one B200\n")
 print(f"Build: the final kernels (`profiles/{TAG}_traffic.json` carries its source fingerprint; bench.py")
-print(f"reports the issue-slot / DRAM figures below only for that build).  Commands: `tools/gpu_{TAG}_final3.sh`.")
+print(f"reports the issue-slot / DRAM figures below only for that build).  Commands: `tools/gpu_{TAG}_final4.sh`.")
 print("ncu serialises launches and runs them cold: compare shares, not absolutes.\n")
 print("## Launch list by kernel (every launch of the bench command under ncu)\n")
 print("```")
